@@ -1,0 +1,181 @@
+"""CPU oracle for the incremental-flattening hot path -- TEST INFRASTRUCTURE.
+
+Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s
+``cpu_baseline`` / ``--impl reference`` legs may import this package.  The
+product path (``paper_conf_ppopp_henriksenteo19_b200``) never does, and the
+two share no code: this wrapper loads ``libifl_oracle.so`` built from
+``oracle/ifl_oracle.c`` (plain C, -O2, no fast-math, single thread).
+
+Every function cites the PAPER.md passage it follows (``P:<line>``, the
+line of /root/reference/PAPER.md).  Pins live in ``tests/test_oracle.py``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "ifl_oracle.c")
+_LIB = os.path.join(_HERE, "libifl_oracle.so")
+
+OPS = {"sum": 0, "prod": 1, "min": 2, "max": 3, "and": 4, "or": 5, "xor": 6}
+MAPS = {"id": 0, "sq": 1, "abs": 2}
+
+_c_i64 = ctypes.c_int64
+_c_int = ctypes.c_int
+_vp = ctypes.c_void_p
+
+
+def build(force: bool = False) -> str:
+    """Compile libifl_oracle.so with gcc (plain C, no fast-math)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(
+            ["gcc", "-O2", "-std=c11", "-fPIC", "-shared", "-fno-fast-math",
+             "-ffp-contract=off", "-o", _LIB, _SRC, "-lm"])
+    return _LIB
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    global _lib
+    if _lib is None:
+        build()
+        L = ctypes.CDLL(_LIB)
+        for name, argt in {
+            "oracle_segred_i32": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_int32],
+            "oracle_segscan_i32": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_int32, _c_int],
+            "oracle_colred_i32": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_int32],
+            "oracle_segred_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double],
+            "oracle_segscan_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double, _c_int],
+            "oracle_colred_f32": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double],
+            "oracle_segred_f32_literal": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_float],
+            "oracle_redomap2": [_vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int],
+            "oracle_tridag": [_vp, _vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _vp],
+        }.items():
+            fn = getattr(L, name)
+            fn.argtypes = argt
+            fn.restype = _c_int
+        _lib = L
+    return _lib
+
+
+def _ptr(a: np.ndarray):
+    return a.ctypes.data_as(_vp)
+
+
+def _i32(v) -> int:
+    """Wrap a Python int to the int32 range (two's complement)."""
+    return ((int(v) + 2**31) % 2**32) - 2**31
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise ValueError(f"oracle returned {rc}")
+
+
+# Canonical neutral elements 0_(+) (reading C6a).
+def canonical_ne(op: str, dtype: str):
+    if dtype == "i32":
+        return {"sum": 0, "prod": 1, "min": 2**31 - 1, "max": -2**31,
+                "and": -1, "or": 0, "xor": 0}[op]
+    return {"sum": 0.0, "prod": 1.0, "min": float("inf"), "max": float("-inf")}[op]
+
+
+def segred(x: np.ndarray, op: str = "sum", f: str = "id", d=None, with_absum=False):
+    """P:79/P:85/P:109: out[i] = d (+) f(x[i,0]) (+) ... (+) f(x[i,m-1]).
+
+    int32 -> int32 (wrapping); float32 -> float64 (exact-ish reference)."""
+    x = np.ascontiguousarray(x)
+    n, m = x.shape
+    if x.dtype == np.int32:
+        d = canonical_ne(op, "i32") if d is None else int(d)
+        out = np.empty(n, np.int32)
+        _check(lib().oracle_segred_i32(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f],
+                                       _i32(d)))
+        return (out, None) if with_absum else out
+    if x.dtype == np.float32:
+        d = canonical_ne(op, "f32") if d is None else float(np.float32(d))
+        out = np.empty(n, np.float64)
+        ab = np.empty(n, np.float64)
+        _check(lib().oracle_segred_f32(_ptr(x), _ptr(out), _ptr(ab), n, m, OPS[op], MAPS[f], d))
+        return (out, ab) if with_absum else out
+    raise TypeError(x.dtype)
+
+
+def segscan(x: np.ndarray, op: str = "sum", f: str = "id", d=None, reverse=False, with_absum=False):
+    """P:79 (inclusive, pinned by P:116) / P:113: per-row scanomap."""
+    x = np.ascontiguousarray(x)
+    n, m = x.shape
+    if x.dtype == np.int32:
+        d = canonical_ne(op, "i32") if d is None else int(d)
+        out = np.empty((n, m), np.int32)
+        _check(lib().oracle_segscan_i32(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f],
+                                        _i32(d), int(reverse)))
+        return (out, None) if with_absum else out
+    if x.dtype == np.float32:
+        d = canonical_ne(op, "f32") if d is None else float(np.float32(d))
+        out = np.empty((n, m), np.float64)
+        ab = np.empty((n, m), np.float64)
+        _check(lib().oracle_segscan_f32(_ptr(x), _ptr(out), _ptr(ab), n, m, OPS[op], MAPS[f],
+                                        d, int(reverse)))
+        return (out, ab) if with_absum else out
+    raise TypeError(x.dtype)
+
+
+def colred(x: np.ndarray, op: str = "sum", f: str = "id", d=None):
+    """P:156 (G4 left-hand side): column reduction of an [n][m] matrix."""
+    x = np.ascontiguousarray(x)
+    n, m = x.shape
+    if x.dtype == np.int32:
+        d = canonical_ne(op, "i32") if d is None else int(d)
+        out = np.empty(m, np.int32)
+        _check(lib().oracle_colred_i32(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f],
+                                       _i32(d)))
+        return out
+    d = canonical_ne(op, "f32") if d is None else float(np.float32(d))
+    out = np.empty(m, np.float64)
+    _check(lib().oracle_colred_f32(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f], d))
+    return out
+
+
+def segred_f32_literal(x: np.ndarray, op: str = "sum", f: str = "id", d=None):
+    """Information only: P:79 left-to-right in f32 (not a parity reference)."""
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    n, m = x.shape
+    d = canonical_ne(op, "f32") if d is None else float(d)
+    out = np.empty(n, np.float32)
+    _check(lib().oracle_segred_f32_literal(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f], d))
+    return out
+
+
+def redomap2(A: np.ndarray, B: np.ndarray, b_kmajor: bool = True, with_abs=False):
+    """C = xss x yss with B given as transpose yss ([p][m], b_kmajor)
+    or as yss ([m][p]).  A/B float32, or uint16 holding bf16 bits."""
+    A = np.ascontiguousarray(A)
+    B = np.ascontiguousarray(B)
+    n, m = A.shape
+    p = B.shape[0] if b_kmajor else B.shape[1]
+    assert (B.shape[1] if b_kmajor else B.shape[0]) == m
+    in_dt = 0 if A.dtype == np.float32 else 1
+    assert A.dtype == B.dtype and A.dtype in (np.float32, np.uint16)
+    C = np.empty((n, p), np.float64)
+    ab = np.empty((n, p), np.float64)
+    _check(lib().oracle_redomap2(_ptr(A), _ptr(B), _ptr(C), _ptr(ab), n, m, p, in_dt, int(b_kmajor)))
+    return (C, ab) if with_abs else C
+
+
+def tridag(a, b, c, y, coef_rows: int):
+    """Thomas algorithm in double (textbook; reading R8)."""
+    a, b, c, y = (np.ascontiguousarray(v, dtype=np.float32) for v in (a, b, c, y))
+    S, L = y.shape
+    assert a.shape == b.shape == c.shape == (coef_rows, L)
+    x = np.empty((S, L), np.float64)
+    work = np.empty(max(L, 1), np.float64)
+    rc = lib().oracle_tridag(_ptr(a), _ptr(b), _ptr(c), _ptr(y), _ptr(x), S, L, coef_rows, _ptr(work))
+    _check(rc)
+    return x

@@ -1,0 +1,328 @@
+"""Pins for the CPU oracle (oracle/ifl_oracle.c) against things other than
+itself: the paper's worked example, closed forms, brute force with
+an independent formulation (Python ints / numpy / math.fsum), algebraic
+invariants, and textbook/library routines (scipy banded solver).
+
+A plausible mistake anywhere in the oracle -- a dropped term, an exclusive
+instead of inclusive scan, a wrong index, a transposed operand, a missing
+neutral element, non-wrapping overflow -- fails at least one test here.
+"""
+import functools
+import math
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import ifl_inputs as gen
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+INT_OPS = ["sum", "prod", "min", "max", "and", "or", "xor"]
+F32_OPS = ["sum", "prod", "min", "max"]
+MAPS = ["id", "sq", "abs"]
+
+
+def load_golden():
+    rows = {}
+    for line in open(os.path.join(HERE, "golden", "p116_worked_example.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        name, val = (s.strip() for s in line.split("|"))
+        rows[name] = np.array([[int(v) for v in r.split(",")] for r in val.split(";")])
+    return rows
+
+
+# ----------------------------------------------------------------- P:116
+
+
+def test_p116_worked_example(orc):
+    g = load_golden()
+    x = g["input"].astype(np.int32)
+    np.testing.assert_array_equal(orc.segscan(x, "sum", "id", 0), g["segscan_sum"])
+    np.testing.assert_array_equal(orc.segred(x, "sum", "id", 0), g["segred_sum"][:, 0])
+    xf = x.astype(np.float32)
+    np.testing.assert_array_equal(orc.segscan(xf, "sum", "id", 0.0), g["segscan_sum"])
+    np.testing.assert_array_equal(orc.segred(xf, "sum", "id", 0.0), g["segred_sum"][:, 0])
+
+
+# ----------------------------------------------------- empty / neutral
+
+
+@pytest.mark.parametrize("op", INT_OPS)
+def test_empty_segment_is_neutral(orc, op):
+    # reduce (+) 0 [] = 0 (empty list => the neutral element alone).
+    x = np.zeros((5, 0), np.int32)
+    np.testing.assert_array_equal(orc.segred(x, op, "id", 1234), np.full(5, 1234))
+    assert orc.segscan(x, op).shape == (5, 0)
+    if op in F32_OPS:
+        xf = np.zeros((3, 0), np.float32)
+        np.testing.assert_array_equal(orc.segred(xf, op, "id", 2.5), np.full(3, 2.5))
+
+
+def test_neutral_element_applied_once(orc):
+    # d (+) a1 (+) ... : with d = 7 and sum, the result is 7 + sum (not 7*m + sum).
+    x = np.ones((2, 5), np.int32)
+    np.testing.assert_array_equal(orc.segred(x, "sum", "id", 7), [12, 12])
+    np.testing.assert_array_equal(orc.segscan(x, "sum", "id", 7), [[8, 9, 10, 11, 12]] * 2)
+
+
+# ---------------------------------------------------------- closed forms
+
+
+def test_closed_form_sum_0_to_k_config1(orc):
+    n = m = 1024  # BASELINE.json configs[0]
+    j = np.arange(m, dtype=np.int64)
+    x = np.broadcast_to(j, (n, m)).astype(np.int32)
+    np.testing.assert_array_equal(orc.segred(x, "sum"), np.full(n, m * (m - 1) // 2))
+    i = np.arange(n, dtype=np.int64)[:, None]
+    x2 = (i * m + j).astype(np.int32)
+    want = m * m * np.arange(n, dtype=np.int64) + m * (m - 1) // 2
+    assert want.max() < 2**31
+    np.testing.assert_array_equal(orc.segred(x2, "sum"), want)
+
+
+def test_closed_form_wraparound(orc):
+    # sum of 0..k-1 with k = 2^17 exceeds 2^31: must wrap mod 2^32.
+    k = 1 << 17
+    x = np.arange(k, dtype=np.int64).astype(np.int32)[None, :]
+    want = (k * (k - 1) // 2) % 2**32
+    want = want - 2**32 if want >= 2**31 else want
+    assert orc.segred(x, "sum")[0] == want
+    # product of 2's: 2^40 mod 2^32 = 0
+    assert orc.segred(np.full((1, 40), 2, np.int32), "prod")[0] == 0
+    assert orc.segred(np.full((1, 31), 2, np.int32), "prod")[0] == -2**31
+
+
+@pytest.mark.parametrize("m", [1, 7, 64, 1000])
+def test_closed_form_scans(orc, m):
+    ones = np.ones((3, m), np.int32)
+    np.testing.assert_array_equal(orc.segscan(ones, "sum"), np.tile(np.arange(1, m + 1), (3, 1)))
+    j = np.tile(np.arange(m, dtype=np.int32), (2, 1))
+    np.testing.assert_array_equal(orc.segscan(j, "sum"), np.tile(np.arange(m) * (np.arange(m) + 1) // 2, (2, 1)))
+    np.testing.assert_array_equal(orc.segscan(j, "max"), j)             # increasing row
+    np.testing.assert_array_equal(orc.segscan(j[:, ::-1].copy(), "min"), j[:, ::-1])
+    # reverse scan of ones: m - j
+    np.testing.assert_array_equal(orc.segscan(ones, "sum", reverse=True), np.tile(np.arange(m, 0, -1), (3, 1)))
+    jf = j.astype(np.float32)
+    np.testing.assert_array_equal(orc.segscan(jf, "sum"), np.tile(np.arange(m) * (np.arange(m) + 1) / 2, (2, 1)))
+
+
+def test_closed_form_min_max_permutation(orc):
+    rng = np.random.default_rng(0)
+    m = 513
+    x = np.stack([rng.permutation(m) for _ in range(8)]).astype(np.int32)
+    np.testing.assert_array_equal(orc.segred(x, "min"), np.zeros(8))
+    np.testing.assert_array_equal(orc.segred(x, "max"), np.full(8, m - 1))
+    np.testing.assert_array_equal(orc.segred(x.astype(np.float32) - 256, "min"), np.full(8, -256.0))
+
+
+def test_maps(orc):
+    x = np.array([[-3, 2, -2**31]], np.int32)
+    assert orc.segred(x[:, :2], "sum", "sq")[0] == 13
+    assert orc.segred(x[:, :2], "sum", "abs")[0] == 5
+    assert orc.segred(x[:, 2:], "sum", "abs")[0] == -2**31  # |INT_MIN| wraps
+    xf = np.array([[-1.5, 0.5]], np.float32)
+    assert orc.segred(xf, "sum", "sq")[0] == 2.5
+    assert orc.segred(xf, "max", "abs")[0] == 1.5
+
+
+# ------------------------------------------- brute force, independent forms
+
+
+def _ref_op(op):
+    M = 1 << 32
+    if op == "sum":
+        return lambda a, b: (a + b) % M
+    if op == "prod":
+        return lambda a, b: (a * b) % M
+    if op == "min":
+        return lambda a, b: a if _s(a) <= _s(b) else b
+    if op == "max":
+        return lambda a, b: a if _s(a) >= _s(b) else b
+    if op == "and":
+        return lambda a, b: a & b
+    if op == "or":
+        return lambda a, b: a | b
+    return lambda a, b: a ^ b
+
+
+def _s(u):
+    return u - (1 << 32) if u >= (1 << 31) else u
+
+
+def _ref_map(f):
+    M = 1 << 32
+    return {"id": lambda v: v % M, "sq": lambda v: (v * v) % M, "abs": lambda v: abs(v) % M}[f]
+
+
+@pytest.mark.parametrize("seed", [1, 2, 3])
+@pytest.mark.parametrize("op", INT_OPS)
+def test_brute_force_int(orc, seed, op):
+    """All (n, m) in [0..8]^2: the O(m) running oracle against an O(m^2)
+    re-definition in Python ints (each scan element a fresh reduce)."""
+    fn = _ref_op(op)
+    d = int(gen.generate("I32_FULL", seed + 100, 1)[0])
+    for f in MAPS:
+        mp = _ref_map(f)
+        for n in range(9):
+            for m in range(9):
+                x = gen.matrix("I32_SMALL" if op == "prod" else "I32_FULL", seed, n, m).numpy()
+                red = orc.segred(x, op, f, d)
+                scn = orc.segscan(x, op, f, d)
+                for i in range(n):
+                    row = [mp(int(v)) for v in x[i]]
+                    want = functools.reduce(fn, row, d % (1 << 32))
+                    assert red[i] == _s(want)
+                    for j in range(m):
+                        assert scn[i, j] == _s(functools.reduce(fn, row[: j + 1], d % (1 << 32)))
+
+
+def test_against_numpy_int(orc):
+    x = gen.matrix("I32_FULL", 1, 64, 300).numpy()
+    s = (x.astype(np.int64).sum(1) % 2**32)
+    s = np.where(s >= 2**31, s - 2**32, s)
+    np.testing.assert_array_equal(orc.segred(x, "sum"), s)
+    np.testing.assert_array_equal(orc.segred(x, "xor"), np.bitwise_xor.reduce(x, axis=1))
+    np.testing.assert_array_equal(orc.segred(x, "and"), np.bitwise_and.reduce(x, axis=1))
+    np.testing.assert_array_equal(orc.segred(x, "or"), np.bitwise_or.reduce(x, axis=1))
+    np.testing.assert_array_equal(orc.segred(x, "min"), x.min(1))
+    np.testing.assert_array_equal(orc.segred(x, "max"), x.max(1))
+    c = np.cumsum(x.astype(np.int64), 1) % 2**32
+    np.testing.assert_array_equal(orc.segscan(x, "sum"), np.where(c >= 2**31, c - 2**32, c))
+    np.testing.assert_array_equal(orc.segscan(x, "max"), np.maximum.accumulate(x, 1))
+
+
+@pytest.mark.parametrize("f", MAPS)
+def test_f32_against_fsum(orc, f):
+    """f32 sums: the double-accumulating oracle vs the exactly-rounded
+    math.fsum of the same f32 terms; |err| <= m * 2^-53 * sum|f(x)|."""
+    x = gen.matrix("F32_SIGNED", 2, 16, 4096).numpy()
+    fx = {"id": x, "sq": (x * x).astype(np.float32), "abs": np.abs(x)}[f]
+    out, ab = orc.segred(x, "sum", f, 0.0, with_absum=True)
+    for i in range(x.shape[0]):
+        exact = math.fsum(fx[i].astype(np.float64))
+        assert abs(out[i] - exact) <= x.shape[1] * 2**-53 * ab[i]
+        assert ab[i] == pytest.approx(np.abs(fx[i].astype(np.float64)).sum(), rel=1e-12)
+    np.testing.assert_array_equal(orc.segred(x, "max", f), fx.max(1))
+    np.testing.assert_array_equal(orc.segred(x, "min", f), fx.min(1))
+    sc, sab = orc.segscan(x[:2, :300], "sum", f, 0.0, with_absum=True)
+    np.testing.assert_allclose(sc, np.cumsum(fx[:2, :300].astype(np.float64), 1), rtol=0, atol=1e-9)
+    np.testing.assert_allclose(sab, np.cumsum(np.abs(fx[:2, :300].astype(np.float64)), 1), rtol=1e-12)
+
+
+def test_f32_prod_against_numpy(orc):
+    x = (0.5 + gen.matrix("F32_UNIT", 9, 8, 50).numpy()).astype(np.float32)
+    np.testing.assert_allclose(orc.segred(x, "prod"), np.prod(x.astype(np.float64), 1), rtol=1e-12)
+
+
+def test_f32_exact_distribution_any_order(orc):
+    """F32_EXACT: |partial sums| stay < 2^24, so every association is exact;
+    the literal f32 left-to-right oracle equals the double one bit for bit."""
+    x = gen.matrix("F32_EXACT", 3, 4, 1 << 20).numpy()
+    pre = np.cumsum(x.astype(np.int64), 1)
+    assert (pre.max(1) - np.minimum(pre.min(1), 0)).max() < 2**24
+    np.testing.assert_array_equal(orc.segred_f32_literal(x), orc.segred(x).astype(np.float32))
+    np.testing.assert_array_equal(orc.segred(x), x.astype(np.int64).sum(1))
+
+
+# ------------------------------------------------------------ invariants
+
+
+@pytest.mark.parametrize("op", INT_OPS)
+def test_associativity_and_identity(orc, op):
+    t = gen.matrix("I32_FULL", 11, 200, 3).numpy()
+    whole = orc.segred(t, op)
+    left = orc.segred(t[:, :2], op)
+    two = np.stack([left, t[:, 2]], 1).astype(np.int32)
+    np.testing.assert_array_equal(orc.segred(two, op), whole)             # (a+b)+c
+    right = orc.segred(t[:, 1:], op)
+    np.testing.assert_array_equal(orc.segred(np.stack([t[:, 0], right], 1).astype(np.int32), op), whole)
+    # canonical d is neutral: d (+) x = x
+    np.testing.assert_array_equal(orc.segred(t[:, :1], op), t[:, 0])
+
+
+@pytest.mark.parametrize("op", INT_OPS)
+def test_scan_last_column_and_split(orc, op):
+    x = gen.matrix("I32_FULL", 12, 37, 129).numpy()
+    np.testing.assert_array_equal(orc.segscan(x, op)[:, -1], orc.segred(x, op))
+    for k in (0, 1, 64, 128, 129):  # split invariance (multi-GPU inner split relies on it)
+        parts = np.stack([orc.segred(x[:, :k], op), orc.segred(x[:, k:], op)], 1).astype(np.int32)
+        np.testing.assert_array_equal(orc.segred(parts, op), orc.segred(x, op))
+
+
+def test_g4_column_identity(orc):
+    # reduce (map (+)) (replicate m 0) M == map (reduce (+) 0) (transpose M)
+    M = gen.matrix("I32_FULL", 13, 33, 70).numpy()
+    np.testing.assert_array_equal(orc.colred(M), orc.segred(np.ascontiguousarray(M.T)))
+    np.testing.assert_array_equal(orc.colred(M), (M.astype(np.int64).sum(0) + 2**31) % 2**32 - 2**31)
+    Mf = gen.matrix("F32_EXACT", 13, 33, 70).numpy()
+    np.testing.assert_array_equal(orc.colred(Mf), Mf.astype(np.float64).sum(0))
+
+
+# --------------------------------------------------------------- redomap2
+
+
+def _bf16_bits(t: torch.Tensor) -> np.ndarray:
+    return t.contiguous().view(torch.int16).numpy().view(np.uint16)
+
+
+def test_redomap2_closed_forms(orc):
+    n, m, p = 5, 37, 6
+    C = orc.redomap2(np.ones((n, m), np.float32), np.ones((p, m), np.float32))
+    np.testing.assert_array_equal(C, np.full((n, p), m))
+    # A = 1, B[k][j] = k mod 16 (B given as [m][p])  ->  C[i][j] = sum_k (k mod 16)
+    B = np.tile((np.arange(m) % 16)[:, None], (1, p)).astype(np.float32)
+    C = orc.redomap2(np.ones((n, m), np.float32), B, b_kmajor=False)
+    np.testing.assert_array_equal(C, np.full((n, p), (np.arange(m) % 16).sum()))
+    # A = I (n = m) -> C = B  (B as [m][p], and as transpose [p][m])
+    Bm = gen.matrix("F32_SIGNED", 6, m, p).numpy()
+    I = np.eye(m, dtype=np.float32)
+    np.testing.assert_array_equal(orc.redomap2(I, Bm, b_kmajor=False), Bm)
+    np.testing.assert_array_equal(orc.redomap2(I, np.ascontiguousarray(Bm.T), b_kmajor=True), Bm)
+
+
+def test_redomap2_against_numpy(orc):
+    A = gen.matrix("F32_SIGNED", 6, 17, 45).numpy()
+    Bt = gen.matrix("F32_SIGNED", 7, 23, 45).numpy()
+    C, ab = orc.redomap2(A, Bt, b_kmajor=True, with_abs=True)
+    np.testing.assert_allclose(C, A.astype(np.float64) @ Bt.T.astype(np.float64), rtol=0, atol=1e-12)
+    np.testing.assert_allclose(ab, np.abs(A.astype(np.float64)) @ np.abs(Bt.T.astype(np.float64)), rtol=1e-12)
+    Ab = gen.matrix("BF16_SIGNED", 6, 9, 40)
+    Bb = gen.matrix("BF16_SIGNED", 7, 40, 11)
+    C = orc.redomap2(_bf16_bits(Ab), _bf16_bits(Bb), b_kmajor=False)
+    np.testing.assert_allclose(C, Ab.double().numpy() @ Bb.double().numpy(), rtol=0, atol=1e-12)
+
+
+# ----------------------------------------------------------------- tridag
+
+
+def test_tridag_poisson_closed_form(orc):
+    # tridiag(-1, 2, -1) x = 1  ->  x_j = (j+1)(L-j)/2  (j = 0..L-1)
+    for L in (1, 2, 5, 32):
+        a = np.full((1, L), -1, np.float32)
+        b = np.full((1, L), 2, np.float32)
+        c = np.full((1, L), -1, np.float32)
+        y = np.ones((3, L), np.float32)
+        x = orc.tridag(a, b, c, y, 1)
+        j = np.arange(L)
+        np.testing.assert_allclose(x, np.tile((j + 1) * (L - j) / 2.0, (3, 1)), rtol=1e-12)
+
+
+def test_tridag_against_scipy_and_residual(orc):
+    from scipy.linalg import solve_banded
+    S, L, R = 12, 33, 4
+    a, b, c, y = (t.numpy() for t in gen.tridag_system(7, S, L, R))
+    x = orc.tridag(a, b, c, y, R)
+    for s in range(S):
+        r = s % R  # coefficient row shared every R systems
+        ab = np.zeros((3, L))
+        ab[0, 1:] = c[r, :-1]
+        ab[1] = b[r]
+        ab[2, :-1] = a[r, 1:]
+        want = solve_banded((1, 1), ab, y[s].astype(np.float64))
+        np.testing.assert_allclose(x[s], want, rtol=1e-10, atol=1e-12)
+        Ax = b[r] * x[s]
+        Ax[1:] += a[r, 1:] * x[s, :-1]
+        Ax[:-1] += c[r, :-1] * x[s, 1:]
+        assert np.abs(Ax - y[s]).max() < 1e-12
