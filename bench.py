@@ -1,0 +1,454 @@
+#!/usr/bin/env python
+"""Benchmark of the incremental-flattening hot path on B200 (BASELINE.json).
+
+Workload (BASELINE.json configs[1]): the fp32 segmented redomap sweep at
+n*m = 2^26 -- n = 2^k, m = 2^(26-k), k = 0..26 -- running segred and segscan
+(op +, f = id) through the AUTO selector with thresholds set by the offline
+tuner (ifl_tune, trained on the n*m = 2^22 and 2^24 sweeps).
+
+One "step" = one pass of the whole sweep (27 shapes x {segred, segscan}).
+value = algorithmic bytes of the step (segred 4(nm+n), segscan 8nm) / time,
+GB/s, whole job (all ranks).  Inputs (256 MiB, > 126 MB L2) alternate between
+two resident copies.  Also measured and reported on the same line:
+  * every forced single version (top / middle / flat) per shape, and the
+    tuned program's speed against the best single version (the metric's
+    second half),
+  * the roofline of the dominant kernel (CUDA events on its stream),
+  * e2e: the same metric through the public API with pinned HOST buffers
+    (H2D of the input and D2H of every result inside the timed region),
+  * cpu_baseline: the CPU oracle on a bounded sample, on this host,
+  * SM clocks sampled by nvidia-smi during the timed region.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+LOG2_N = 26
+METRIC = "segred/segscan GB/s vs HBM peak over n×m sweep; speedup vs best single version"
+NOMINAL_HBM_GBS = 8000.0
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": float(d["hbm_gbs"]), "source": "measured (MEASURED_PEAKS.json)"}
+    return {"hbm_gbs": 6650.0, "source": "fallback (B200_PROFILING.md)"}
+
+
+def shapes(log2n=LOG2_N):
+    return [(1 << k, 1 << (log2n - k)) for k in range(log2n + 1)]
+
+
+def bytes_segred(n, m):
+    return 4 * (n * m + n)
+
+
+def bytes_segscan(n, m):
+    return 8 * n * m
+
+
+# ---------------------------------------------------------------- clocks
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                       "--format=csv,noheader,nounits", "-lms", "100"],
+                                      stdout=self.f, stderr=subprocess.DEVNULL)
+        except OSError:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.p.kill()
+        self.f.flush()
+        rows = [r.split(",") for r in open(self.f.name).read().strip().splitlines() if r.strip()]
+        os.unlink(self.f.name)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in rows:
+            r = [c.strip() for c in r]
+            try:
+                sm.append(float(r[1]))
+                mx.append(float(r[2]))
+            except (ValueError, IndexError):
+                continue
+            for nm, v in zip(names, r[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        # samples under load: the top 80% by clock (idle gaps excluded)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# -------------------------------------------------------------- our arm
+
+
+def run_ours(args, rank, world, device):
+    import numpy as np
+    import torch
+
+    import ifl_inputs as gen
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+
+    torch.cuda.set_device(device)
+    dist = world > 1
+    if dist:
+        import torch.distributed as td
+
+    ifl.reset_thresholds()
+    N = 1 << LOG2_N
+    sh = shapes()
+    stream = torch.cuda.current_stream()
+
+    # ---- offline tuning (untimed): train on the 2^22 and 2^24 sweeps
+    tuned = {}
+    if not args.no_tune:
+        t0 = time.time()
+        for site in ("segred.b4", "segscan.b4"):
+            train = [s for lg in (22, 24) for s in shapes(lg)]
+            scratch_bytes = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data,
+                                                             len(train))
+            scratch = torch.empty(scratch_bytes, dtype=torch.uint8, device=device)
+            scratch.view(-1)[: (scratch_bytes // 4) * 4].view(torch.float32).copy_(
+                gen.generate("F32_UNIT", 4, scratch_bytes // 4, device=device))
+            a, b, tbl = ifl.tune(site, train, reps=3, cost=1, scratch=scratch)
+            tuned[site] = {"t_top": a, "t_intra": b}
+            del scratch
+        log(f"[bench] tuned in {time.time() - t0:.1f}s: {tuned}")
+    if args.thresholds:
+        ifl.load_thresholds(args.thresholds)
+
+    # ---- resident inputs: two copies > L2, alternate per step
+    xs = [gen.generate("F32_UNIT", 2 + rank * 101, N, device=device),
+          gen.generate("F32_UNIT", 3 + rank * 101, N, device=device)]
+    out_red = torch.empty(N, dtype=torch.float32, device=device)
+    out_scan = torch.empty(N, dtype=torch.float32, device=device)
+    ws = ifl.workspace(ifl.workspace_bytes("segscan", 1, N), device)
+    torch.cuda.synchronize()
+
+    def call(kind, x, n, m, version="auto"):
+        xv = x.view(n, m)
+        if kind == "segred":
+            return ifl.segred(xv, out=out_red[:n], ws=ws, version=version, return_choice=True)[1]
+        return ifl.segscan(xv, out=out_scan.view(n, m), ws=ws, version=version, return_choice=True)[1]
+
+    calls = [(kind, n, m) for (n, m) in sh for kind in ("segred", "segscan")]
+    step_bytes = sum(bytes_segred(n, m) if k == "segred" else bytes_segscan(n, m) for k, n, m in calls)
+    choices = {}
+
+    def step(i, evs=None):
+        x = xs[i % 2]
+        for j, (kind, n, m) in enumerate(calls):
+            if evs is not None:
+                evs[j][0].record(stream)
+            c = call(kind, x, n, m)
+            if evs is not None:
+                evs[j][1].record(stream)
+            choices[(kind, n)] = c.version
+
+    # ---- warm-up, then exactly K timed steps (contract)
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    if dist:
+        td.barrier()
+    torch.cuda.synchronize()
+    clocks = Clocks(device)
+    clocks.start()
+    time.sleep(0.3)
+    ev_step = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    ev_call = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in calls]
+               for _ in range(args.steps)]
+    for i in range(args.steps):
+        ev_step[i][0].record(stream)
+        step(i, ev_call[i])
+        ev_step[i][1].record(stream)
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    if dist:
+        td.barrier()
+    torch.cuda.synchronize()
+    step_ms = [a.elapsed_time(b) for a, b in ev_step]
+    total_ms = sum(step_ms)
+    if dist:
+        t = torch.tensor([total_ms], dtype=torch.float64, device=device)
+        td.all_reduce(t, op=td.ReduceOp.MAX)
+        total_ms = float(t.item())
+    value = world * step_bytes * args.steps / (total_ms / 1e3) / 1e9
+    per_call_ms = [statistics.median(ev_call[i][j][0].elapsed_time(ev_call[i][j][1]) for i in range(args.steps))
+                   for j in range(len(calls))]
+    auto_ms = {(k, n): t for (k, n, m), t in zip(calls, per_call_ms)}
+
+    # ---- every forced single version, per shape (the metric's second half)
+    forced = {}
+    reps = max(1, min(args.steps, 3))
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    for kind, n, m in calls:
+        for v in ("top", "middle", "flat"):
+            x = xs[0]
+            e0.record(stream)
+            call(kind, x, n, m, v)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            first = e0.elapsed_time(e1)
+            ts = [first]
+            if first < 50 * auto_ms[(kind, n)]:  # hopeless shapes: one run is evidence enough
+                ts = []
+                for r in range(reps):
+                    e0.record(stream)
+                    call(kind, xs[(r + 1) % 2], n, m, v)
+                    e1.record(stream)
+                    torch.cuda.synchronize()
+                    ts.append(e0.elapsed_time(e1))
+            forced[(kind, n, v)] = statistics.median(ts)
+    table = []
+    ratios = []
+    fixed_tot = {v: 0.0 for v in ("top", "middle", "flat")}
+    auto_tot = 0.0
+    for kind, n, m in calls:
+        tv = {v: forced[(kind, n, v)] for v in ("top", "middle", "flat")}
+        best = min(tv.values())
+        ta = auto_ms[(kind, n)]
+        b = bytes_segred(n, m) if kind == "segred" else bytes_segscan(n, m)
+        ratios.append(best / ta)
+        for v in tv:
+            fixed_tot[v] += tv[v]
+        auto_tot += ta
+        table.append({"op": kind, "n": n, "m": m, "chosen": choices[(kind, n)], "auto_us": ta * 1e3,
+                      "top_us": tv["top"] * 1e3, "middle_us": tv["middle"] * 1e3, "flat_us": tv["flat"] * 1e3,
+                      "best_single": min(tv, key=tv.get), "best_over_auto": best / ta,
+                      "auto_GBps": b / (ta / 1e3) / 1e9, "frac_of_8TBps": b / (ta / 1e3) / 1e9 / NOMINAL_HBM_GBS})
+
+    # ---- dominant kernel roofline (CUDA-event durations of the timed steps)
+    groups = {}
+    for (kind, n, m), t in zip(calls, per_call_ms):
+        key = f"{kind}_{choices[(kind, n)]}"
+        b = bytes_segred(n, m) if kind == "segred" else bytes_segscan(n, m)
+        g = groups.setdefault(key, [0.0, 0, 0])
+        g[0] += t
+        g[1] += b
+        g[2] += 1
+    dom = max(groups, key=lambda k: groups[k][0])
+    pk = peaks()
+    achieved = groups[dom][1] / (groups[dom][0] / 1e3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(dom)
+
+    # ---- e2e through the public API with pinned host buffers
+    e2e = None
+    if not args.no_e2e:
+        import torch as _t
+        hx = _t.empty(N, dtype=_t.float32, pin_memory=True)
+        hx.copy_(xs[0])
+        hred = _t.empty(N, dtype=_t.float32, pin_memory=True)
+        hscan = _t.empty(N, dtype=_t.float32, pin_memory=True)
+        dx = _t.empty(N, dtype=_t.float32, device=device)
+        h2d = d2h = 0
+        esteps = max(1, min(args.steps, 3))
+        s0, s1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        s0.record(stream)
+        for i in range(esteps):
+            for (n, m) in sh:
+                dx.copy_(hx, non_blocking=True)
+                ifl.segred(dx.view(n, m), out=out_red[:n], ws=ws)
+                hred[:n].copy_(out_red[:n], non_blocking=True)
+                ifl.segscan(dx.view(n, m), out=out_scan.view(n, m), ws=ws)
+                hscan.copy_(out_scan, non_blocking=True)
+                if i == 0:
+                    h2d += N * 4
+                    d2h += n * 4 + N * 4
+        s1.record(stream)
+        torch.cuda.synchronize()
+        ems = s0.elapsed_time(s1)
+        e2e = {"value": round(world * step_bytes * esteps / (ems / 1e3) / 1e9, 2), "unit": "GB/s",
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+               "note": "pinned host input copied in once per shape and shared by segred+segscan"}
+
+    res = {
+        "value": value, "total_ms": total_ms, "step_ms": step_ms, "step_bytes": step_bytes, "table": table,
+        "ratios": ratios, "fixed_tot": fixed_tot, "auto_tot": auto_tot, "tuned": tuned, "clocks": ck,
+        "dom": dom, "achieved": achieved, "peak": pk, "traffic": traffic, "e2e": e2e, "groups": groups,
+        "launches": len(calls) * args.steps,
+    }
+    return res
+
+
+# ------------------------------------------------------------ CPU oracle
+
+
+def oracle_sample(step_index: int = 0):
+    """The CPU oracle (single thread) on a bounded sample of the workload:
+    7 of the 27 shapes (k = 0, 4, ..., 24) at full size, segred + segscan."""
+    import torch
+
+    import ifl_inputs as gen
+    import oracle
+
+    N = 1 << LOG2_N
+    x = gen.generate("F32_UNIT", 2, N).numpy()
+    ks = list(range(0, LOG2_N + 1, 4))
+    nbytes = 0
+    t0 = time.perf_counter()
+    for k in ks:
+        n, m = 1 << k, 1 << (LOG2_N - k)
+        xv = x.reshape(n, m)
+        oracle.segred(xv, "sum")
+        oracle.segscan(xv, "sum")
+        nbytes += bytes_segred(n, m) + bytes_segscan(n, m)
+    dt = time.perf_counter() - t0
+    return nbytes / dt / 1e9, dt, f"segred+segscan f32 sum on shapes n=2^k, k in {ks}, n*m=2^26 (full size)"
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle as it stands, timed on host cores."""
+    if rank != 0:
+        return None
+    import oracle
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle_sample()
+    vals, secs = [], 0.0
+    sample = ""
+    for _ in range(args.steps):
+        v, dt, sample = oracle_sample()
+        vals.append(v)
+        secs += dt
+    value = statistics.median(vals)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 4), "unit": "GB/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(secs / args.steps * 1e3, 2),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": "configs[1] fp32 segmented redomap sweep n*m=2^26 (bounded sample, CPU oracle)"},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    return line
+
+
+# ------------------------------------------------------------------- main
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-tune", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--thresholds", default=None)
+    ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"))
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        line = run_reference(args, rank, world)
+        if line is not None:
+            print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    if world > 1:
+        import torch.distributed as td
+        torch.cuda.set_device(local)
+        td.init_process_group("nccl", device_id=torch.device("cuda", local))
+    r = run_ours(args, rank, world, local)
+    if rank == 0:
+        import numpy as np
+        pk = r["peak"]
+        cpu = None
+        if not args.no_cpu and world == 1:
+            v, dt, sample = oracle_sample()
+            cpu = {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
+                   "seconds": round(dt, 2)}
+        best_fixed = min(r["fixed_tot"].values())
+        line = {
+            "metric": METRIC,
+            "value": round(r["value"], 2),
+            "unit": "GB/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": round(r["total_ms"] / args.steps, 4),
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "f32",
+            "data": "synthetic",
+            "config": {
+                "workload": "configs[1]: fp32 segmented redomap sweep, n*m=2^26, n=2^0..2^26; segred+segscan "
+                            "(+, f=id), AUTO selector with tuned thresholds",
+                "n_times_m": 1 << LOG2_N, "shapes": LOG2_N + 1,
+                "l2": "inputs 256 MiB > 126 MB L2; two resident copies alternate per step",
+                "thresholds": r["tuned"] or "default 2^15 (P:370)",
+                "parallelism": f"weak: {world} independent sweeps, one per GPU",
+            },
+            "frac_of_8TBps": round(r["value"] / world / NOMINAL_HBM_GBS, 4),
+            "frac_of_measured_hbm": round(r["value"] / world / pk["hbm_gbs"], 4),
+            "speedup_vs_best_single_version": round(best_fixed / r["auto_tot"], 4),
+            "min_shape_best_over_auto": round(min(r["ratios"]), 4),
+            "roofline": {"bound": "hbm", "kernel": r["dom"], "achieved": round(r["achieved"], 1),
+                         "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": round(r["achieved"] / pk["hbm_gbs"], 4),
+                         "traffic": r["traffic"], "peak_source": pk["source"]},
+            "cpu_baseline": cpu,
+            "e2e": r["e2e"],
+            "gpu_launches": r["launches"],
+            "clocks": r["clocks"],
+        }
+        os.makedirs(os.path.dirname(args.detail), exist_ok=True)
+        with open(args.detail, "w") as fp:
+            json.dump({"line": line, "table": r["table"], "groups": r["groups"], "fixed_tot_ms": r["fixed_tot"],
+                       "auto_tot_ms": r["auto_tot"], "step_ms": r["step_ms"]}, fp, indent=1)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as td
+        td.barrier()
+        td.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

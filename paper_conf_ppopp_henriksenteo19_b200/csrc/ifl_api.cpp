@@ -1,0 +1,356 @@
+// ifl_api.cpp -- the C ABI of include/ifl.h: argument validation, the G3
+// version selector, the per-site threshold table (P:201,
+// default 2^15 per P:370), workspace sizing and error reporting.
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <map>
+#include <mutex>
+#include <string>
+
+#include "../../include/ifl.h"
+#include "ifl_internal.h"
+
+namespace {
+
+thread_local std::string g_err;
+
+int fail(int code, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return code;
+}
+
+int cuda_status(cudaError_t e, const char* what) {
+    if (e == cudaSuccess) return IFL_OK;
+    if (e == cudaErrorNotSupported) return fail(IFL_EUNSUPPORTED, "%s: not supported", what);
+    return fail(IFL_ECUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+constexpr int64_t kDefaultThreshold = 1 << 15;
+constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE kernel (reading R3)
+
+const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag"};
+
+struct Table {
+    std::mutex mu;
+    std::map<std::string, std::pair<int64_t, int64_t>> thr;
+    int par_mode = 1;
+    Table() { reset(); }
+    void reset() {
+        thr.clear();
+        for (const char* s : kSites) thr[s] = {kDefaultThreshold, kDefaultThreshold};
+        par_mode = 1;
+    }
+};
+Table& table() {
+    static Table t;
+    return t;
+}
+
+bool known_site(const char* s) {
+    if (!s) return false;
+    for (const char* k : kSites)
+        if (strcmp(s, k) == 0) return true;
+    return false;
+}
+
+int64_t sat_mul(int64_t a, int64_t b) {
+    if (a <= 0 || b <= 0) return 0;
+    if (a > INT64_MAX / b) return INT64_MAX;
+    return a * b;
+}
+
+bool mul_overflows(int64_t a, int64_t b) { return a > 0 && b > 0 && a > INT64_MAX / b; }
+
+// Par(Sigma') and Par(e_middle) of rule G3 for a site and shape.
+void par_values(const char* site, int64_t n, int64_t m, int64_t p, int mode, int64_t* ptop, int64_t* pmid) {
+    int64_t outer = n;
+    if (strncmp(site, "redomap2", 8) == 0) outer = sat_mul(n, p);
+    *ptop = outer;
+    *pmid = mode == 1 ? sat_mul(outer, std::min(m, kBmax)) : sat_mul(outer, m);
+}
+
+int select_version(const char* site, int64_t n, int64_t m, int64_t p, bool mid_fits, ifl_choice* c) {
+    Table& T = table();
+    int64_t tt, ti;
+    int mode;
+    {
+        std::lock_guard<std::mutex> g(T.mu);
+        auto it = T.thr.find(site);
+        tt = it->second.first;
+        ti = it->second.second;
+        mode = T.par_mode;
+    }
+    int64_t ptop, pmid;
+    par_values(site, n, m, p, mode, &ptop, &pmid);
+    int v;
+    if (ptop >= tt) v = IFL_V_TOP;  // G3 guard 1 (reading R1: >=)
+    else if (pmid >= ti && mid_fits) v = IFL_V_MIDDLE;  // guard 2 + fit clause (R4)
+    else v = IFL_V_FLAT;
+    if (c) {
+        c->version = v;
+        c->par_top = ptop;
+        c->par_mid = pmid;
+        c->t_top = tt;
+        c->t_intra = ti;
+    }
+    return v;
+}
+
+uint32_t canonical_bits(int dt, int op) {
+    if (dt == IFL_I32) {
+        switch (op) {
+        case IFL_SUM: return 0u;
+        case IFL_PROD: return 1u;
+        case IFL_MIN: return 0x7fffffffu;
+        case IFL_MAX: return 0x80000000u;
+        case IFL_AND: return 0xffffffffu;
+        default: return 0u;
+        }
+    }
+    switch (op) {
+    case IFL_SUM: return 0x00000000u;  // 0.0f
+    case IFL_PROD: return 0x3f800000u; // 1.0f
+    case IFL_MIN: return 0x7f800000u;  // +inf
+    case IFL_MAX: return 0xff800000u;  // -inf
+    default: return 0u;
+    }
+}
+
+bool overlap(const void* a, size_t an, const void* b, size_t bn) {
+    const char* x = (const char*)a;
+    const char* y = (const char*)b;
+    return x < y + bn && y < x + an;
+}
+
+int validate_seg(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, int version,
+                 const char* what) {
+    if (n < 0 || m < 0) return fail(IFL_EINVAL, "%s: negative size n=%lld m=%lld", what, (long long)n, (long long)m);
+    if (mul_overflows(n, m) || mul_overflows(n * m, 4))
+        return fail(IFL_EINVAL, "%s: n*m overflows int64", what);
+    if (dt != IFL_I32 && dt != IFL_F32) return fail(IFL_EUNSUPPORTED, "%s: dtype %d unsupported", what, dt);
+    if (op < IFL_SUM || op > IFL_XOR) return fail(IFL_EINVAL, "%s: bad op %d", what, op);
+    if (dt == IFL_F32 && op > IFL_MAX) return fail(IFL_EUNSUPPORTED, "%s: bitwise op on f32", what);
+    if (f < IFL_F_ID || f > IFL_F_ABS) return fail(IFL_EINVAL, "%s: bad map %d", what, f);
+    if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "%s: bad version %d", what, version);
+    if (n > 0 && m > 0 && in == nullptr) return fail(IFL_EINVAL, "%s: in is NULL", what);
+    if (n > 0 && out == nullptr) return fail(IFL_EINVAL, "%s: out is NULL", what);
+    if (((uintptr_t)in % 4) || ((uintptr_t)out % 4)) return fail(IFL_EINVAL, "%s: pointers not element-aligned", what);
+    return IFL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* ifl_last_error(void) { return g_err.c_str(); }
+
+const char* ifl_build_info(void) {
+    return "ifl " __DATE__ " sm_100a; versions: top/middle/flat; segred segscan redomap2 tridag tune";
+}
+
+int ifl_select(const char* site, int64_t n, int64_t m, int64_t p, ifl_choice* choice) {
+    if (!known_site(site)) return fail(IFL_EINVAL, "ifl_select: unknown site '%s'", site ? site : "(null)");
+    if (n < 0 || m < 0 || p < 0) return fail(IFL_EINVAL, "ifl_select: negative size");
+    bool fits = true;
+    if (strcmp(site, "tridag") == 0) fits = ifl::tridag_mid_fits(m);
+    return select_version(site, n, m, p, fits, choice) >= 0 ? IFL_OK : IFL_EINVAL;
+}
+
+int ifl_set_thresholds(const char* site, int64_t t_top, int64_t t_intra) {
+    if (!known_site(site)) return fail(IFL_EINVAL, "unknown site '%s'", site ? site : "(null)");
+    if (t_top < 0 || t_intra < 0) return fail(IFL_EINVAL, "negative threshold");
+    Table& T = table();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.thr[site] = {t_top, t_intra};
+    return IFL_OK;
+}
+
+int ifl_get_thresholds(const char* site, int64_t* t_top, int64_t* t_intra) {
+    if (!known_site(site)) return fail(IFL_EINVAL, "unknown site '%s'", site ? site : "(null)");
+    Table& T = table();
+    std::lock_guard<std::mutex> g(T.mu);
+    auto& v = T.thr[site];
+    if (t_top) *t_top = v.first;
+    if (t_intra) *t_intra = v.second;
+    return IFL_OK;
+}
+
+int ifl_reset_thresholds(void) {
+    Table& T = table();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.reset();
+    return IFL_OK;
+}
+
+int ifl_set_par_mode(int mode) {
+    if (mode != 0 && mode != 1) return fail(IFL_EINVAL, "par mode must be 0 or 1");
+    Table& T = table();
+    std::lock_guard<std::mutex> g(T.mu);
+    T.par_mode = mode;
+    return IFL_OK;
+}
+
+int ifl_get_par_mode(void) {
+    Table& T = table();
+    std::lock_guard<std::mutex> g(T.mu);
+    return T.par_mode;
+}
+
+int ifl_save_thresholds(const char* path) {
+    if (!path) return fail(IFL_EINVAL, "NULL path");
+    FILE* fp = fopen(path, "w");
+    if (!fp) return fail(IFL_EINVAL, "cannot open %s", path);
+    Table& T = table();
+    {
+        std::lock_guard<std::mutex> g(T.mu);
+        fprintf(fp, "# ifl thresholds: site t_top t_intra (par_mode %d)\n", T.par_mode);
+        for (auto& kv : T.thr)
+            fprintf(fp, "%s %lld %lld\n", kv.first.c_str(), (long long)kv.second.first, (long long)kv.second.second);
+    }
+    fclose(fp);
+    return IFL_OK;
+}
+
+int ifl_load_thresholds(const char* path) {
+    if (!path) return fail(IFL_EINVAL, "NULL path");
+    FILE* fp = fopen(path, "r");
+    if (!fp) return fail(IFL_EINVAL, "cannot open %s", path);
+    char line[256];
+    int rc = IFL_OK;
+    while (fgets(line, sizeof line, fp)) {
+        if (line[0] == '#' || line[0] == '\n') continue;
+        char site[64];
+        long long a, b;
+        if (sscanf(line, "%63s %lld %lld", site, &a, &b) != 3) {
+            rc = fail(IFL_EINVAL, "malformed line in %s: %s", path, line);
+            break;
+        }
+        if ((rc = ifl_set_thresholds(site, a, b)) != IFL_OK) break;
+    }
+    fclose(fp);
+    return rc;
+}
+
+size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, int dt, int version) {
+    (void)dt;
+    if (!entry || n < 0 || m < 0 || p < 0 || mul_overflows(n, m)) return 0;
+    if (strcmp(entry, "segred") == 0 || strcmp(entry, "segscan") == 0) {
+        if (version == IFL_V_FLAT || version == IFL_AUTO) return n * m > 0 ? ifl::flat_ws_bytes(n * m) : 0;
+        return 0;
+    }
+    if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
+    if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(n, m, version);
+    return 0;
+}
+
+int ifl_workspace_init(void* ws, size_t ws_bytes, void* stream) {
+    if (ws_bytes == 0) return IFL_OK;
+    if (!ws) return fail(IFL_EINVAL, "workspace is NULL");
+    return cuda_status(cudaMemsetAsync(ws, 0, ws_bytes, (cudaStream_t)stream), "ifl_workspace_init");
+}
+
+static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f,
+                   const void* ne, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    const char* what = scan ? "ifl_segscan" : "ifl_segred";
+    int rc = validate_seg(in, out, n, m, dt, op, f, version, what);
+    if (rc) return rc;
+    const size_t ob = (size_t)(scan ? n * m : n) * 4, ib = (size_t)(n * m) * 4;
+    if (scan) {
+        if (in != out && overlap(in, ib, out, ob)) return fail(IFL_EINVAL, "%s: in/out partially overlap", what);
+    } else if (overlap(in, ib, out, ob)) {
+        return fail(IFL_EINVAL, "%s: out overlaps in", what);
+    }
+    uint32_t bits = canonical_bits(dt, op);
+    if (ne) memcpy(&bits, ne, 4);
+    const char* site = scan ? "segscan.b4" : "segred.b4";
+    ifl_choice c;
+    const int v = select_version(site, n, m, 0, true, &c);
+    if (version != IFL_AUTO) c.version = version;
+    if (choice) *choice = c;
+    if (n == 0) return IFL_OK;
+    if (m == 0) {  // reduce of an empty list is d; scan of it is empty
+        if (scan) return IFL_OK;
+        return cuda_status(ifl::launch_fill(out, n, bits, (cudaStream_t)stream), what);
+    }
+    (void)v;
+    ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream};
+    cudaError_t e;
+    switch (c.version) {
+    case IFL_V_TOP: e = scan ? ifl::launch_segscan_top(a) : ifl::launch_segred_top(a); break;
+    case IFL_V_MIDDLE: e = scan ? ifl::launch_segscan_mid(a) : ifl::launch_segred_mid(a); break;
+    default: {
+        const size_t need = ifl::flat_ws_bytes(n * m);
+        if (!ws || ws_bytes < need)
+            return fail(IFL_EWORKSPACE, "%s: V_FLAT needs %zu workspace bytes, got %zu", what, need, ws_bytes);
+        e = ifl::launch_flat(a, scan);
+    }
+    }
+    return cuda_status(e, what);
+}
+
+int ifl_segred(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int version,
+               void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    return run_seg(false, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+}
+
+int ifl_segscan(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int reverse,
+                int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    if (reverse) return fail(IFL_EUNSUPPORTED, "ifl_segscan: reverse scans are not exposed");
+    return run_seg(true, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+}
+
+int ifl_redomap2(const void* A, const void* B, float* C, int64_t n, int64_t m, int64_t p, int in_dt, int b_kmajor,
+                 int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    if (n < 0 || m < 0 || p < 0) return fail(IFL_EINVAL, "ifl_redomap2: negative size");
+    if (mul_overflows(n, m) || mul_overflows(m, p) || mul_overflows(n, p) || mul_overflows(sat_mul(n, p), m))
+        return fail(IFL_EINVAL, "ifl_redomap2: size overflow");
+    if (in_dt != IFL_F32 && in_dt != IFL_BF16) return fail(IFL_EUNSUPPORTED, "ifl_redomap2: dtype %d", in_dt);
+    if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "ifl_redomap2: bad version");
+    if (n * p > 0 && !C) return fail(IFL_EINVAL, "ifl_redomap2: C is NULL");
+    if (n * m > 0 && !A) return fail(IFL_EINVAL, "ifl_redomap2: A is NULL");
+    if (m * p > 0 && !B) return fail(IFL_EINVAL, "ifl_redomap2: B is NULL");
+    const char* site = in_dt == IFL_BF16 ? "redomap2.bf16" : "redomap2.f32";
+    ifl_choice c;
+    select_version(site, n, m, p, true, &c);
+    if (version != IFL_AUTO) c.version = version;
+    if (choice) *choice = c;
+    if (n * p == 0) return IFL_OK;
+    ifl::MmArgs a{A, B, C, n, m, p, in_dt, b_kmajor ? 1 : 0, ws, ws_bytes, (cudaStream_t)stream};
+    const size_t need = ifl::redomap2_ws_bytes(n, m, p, c.version);
+    if (need && (!ws || ws_bytes < need))
+        return fail(IFL_EWORKSPACE, "ifl_redomap2: needs %zu workspace bytes, got %zu", need, ws_bytes);
+    return cuda_status(ifl::launch_redomap2(c.version, a), "ifl_redomap2");
+}
+
+int ifl_tridag(const float* a, const float* b, const float* c, const float* y, float* x, int64_t S, int64_t L,
+               int64_t coef_rows, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    if (S < 0 || L < 0 || coef_rows <= 0) return fail(IFL_EINVAL, "ifl_tridag: bad sizes");
+    if (mul_overflows(S, L) || mul_overflows(coef_rows, L)) return fail(IFL_EINVAL, "ifl_tridag: size overflow");
+    if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "ifl_tridag: bad version");
+    if (S * L > 0 && (!a || !b || !c || !y || !x)) return fail(IFL_EINVAL, "ifl_tridag: NULL pointer");
+    const bool fits = ifl::tridag_mid_fits(L);
+    ifl_choice ch;
+    select_version("tridag", S, L, 0, fits, &ch);
+    if (version != IFL_AUTO) ch.version = version;
+    if (choice) *choice = ch;
+    if (ch.version == IFL_V_MIDDLE && !fits)
+        return fail(IFL_ENOTFIT, "ifl_tridag: V_MIDDLE does not fit L=%lld in shared memory", (long long)L);
+    if (S * L == 0) return IFL_OK;
+    const size_t need = ifl::tridag_ws_bytes(S, L, ch.version);
+    if (need && (!ws || ws_bytes < need))
+        return fail(IFL_EWORKSPACE, "ifl_tridag: needs %zu workspace bytes, got %zu", need, ws_bytes);
+    ifl::TriArgs t{a, b, c, y, x, S, L, coef_rows, ws, ws_bytes, (cudaStream_t)stream};
+    return cuda_status(ifl::launch_tridag(ch.version, t), "ifl_tridag");
+}
+
+}  // extern "C"

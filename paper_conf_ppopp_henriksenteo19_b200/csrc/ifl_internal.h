@@ -1,0 +1,68 @@
+// ifl_internal.h -- launch entry points between the C ABI (ifl_api.cpp) and
+// the kernel translation units.  Not installed; not part of the ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+namespace ifl {
+
+// Arguments of one segred/segscan call after validation and version choice.
+struct SegArgs {
+    const void* in;
+    void* out;
+    int64_t n, m;
+    int dt, op, f;
+    uint32_t ne_bits;  // neutral element d as raw 32-bit pattern
+    void* ws;
+    size_t ws_bytes;
+    cudaStream_t stream;
+};
+
+// Flat engine tile geometry (flat.cu).  ws layout: 256-byte header then one
+// 64-bit status word per tile.
+constexpr int kFlatThreads = 256;
+constexpr int kFlatItems = 28;
+constexpr int64_t kFlatTile = (int64_t)kFlatThreads * kFlatItems;
+size_t flat_ws_bytes(int64_t total_elems);
+
+// Version kernels: return the launch error (cudaSuccess on success).
+cudaError_t launch_segred_top(const SegArgs& a);
+cudaError_t launch_segred_mid(const SegArgs& a);
+cudaError_t launch_segscan_top(const SegArgs& a);
+cudaError_t launch_segscan_mid(const SegArgs& a);
+cudaError_t launch_flat(const SegArgs& a, bool scan);
+cudaError_t launch_fill(void* out, int64_t count, uint32_t bits, cudaStream_t s);
+
+// Group size (threads per segment) used by the V_MIDDLE kernels.
+int mid_group_size(int64_t m);
+int midscan_group_size(int64_t m);
+
+// redomap2 (redomap2.cu) and tridag (tridag.cu)
+struct MmArgs {
+    const void* A;
+    const void* B;
+    float* C;
+    int64_t n, m, p;
+    int in_dt, b_kmajor;
+    void* ws;
+    size_t ws_bytes;
+    cudaStream_t stream;
+};
+size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version);
+cudaError_t launch_redomap2(int version, const MmArgs& a);
+bool redomap2_tc_ok(const MmArgs& a);
+
+struct TriArgs {
+    const float *a, *b, *c, *y;
+    float* x;
+    int64_t S, L, coef_rows;
+    void* ws;
+    size_t ws_bytes;
+    cudaStream_t stream;
+};
+size_t tridag_ws_bytes(int64_t S, int64_t L, int version);
+bool tridag_mid_fits(int64_t L);
+cudaError_t launch_tridag(int version, const TriArgs& a);
+
+}  // namespace ifl

@@ -1,0 +1,220 @@
+// segred.cu -- the V_TOP and V_MIDDLE versions of segred (rule G3's e_top and
+// e_middle) for an [n][m] row-major array.
+//
+//   V_TOP    segmap^1 <xs in xss> (redomap (+) f d xs)
+//            one thread per segment; the CTA's 256 rows are staged through
+//            shared memory in [256][32] column tiles with coalesced 128-bit
+//            loads, then each thread walks its own row sequentially
+//            (bank-conflict-free: one pad word per 32).
+//   V_MIDDLE segmap^1 <xs in xss> (segred^0 <x in xs> (+) d (f x))
+//            one thread group of G threads per segment (G = m/16 rounded to a
+//            power of two in [2, 1024]); 128-bit loads with per-row scalar
+//            head/tail for any alignment, then a warp-shuffle / shared-memory
+//            tree -- the level-0 reduction of P:346-358.
+#include <string.h>
+
+#include "common.cuh"
+#include "dispatch.cuh"
+#include "ifl_internal.h"
+
+namespace ifl {
+
+// ------------------------------------------------------------------ V_TOP
+
+constexpr int kTopRows = 256;  // threads = segments per CTA
+constexpr int kTopKT = 32;     // columns per smem tile (128 B of f32 per row)
+constexpr int kTopWords = kTopRows * kTopKT + kTopRows * kTopKT / 32;
+
+__device__ __forceinline__ int padq(int q) { return q + (q >> 5); }
+
+// Stage the CTA's tile into shared memory.  Whole-row mode (m <= 32): the
+// region [r0*m, (r0+rows)*m) is contiguous and copied linearly.  Column-tile
+// mode: columns [k0, k0+kt) of `rows` rows.  Padded index padq(q) with
+// q = row*KT + col (KT = m in whole-row mode, 32 otherwise).
+template <typename T>
+__device__ __forceinline__ void top_load_tile(T* tile, const T* __restrict__ in, int64_t r0, int rows,
+                                              int64_t m, int64_t k0, int kt, bool whole, bool vec) {
+    const int t = threadIdx.x;
+    using V = typename Vec4<T>::type;
+    if (whole) {
+        const int cnt = rows * (int)m;
+        const T* src = in + r0 * m;
+        int p0 = 0;
+        if (vec) {
+            const int nv = cnt >> 2;
+            for (int v = t; v < nv; v += kTopRows) {
+                V q = ldg_stream4(src + 4 * v);
+                T e[4];
+                unpack4<T>(q, e);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) tile[padq(4 * v + u)] = e[u];
+            }
+            p0 = nv << 2;
+        }
+        for (int p = p0 + t; p < cnt; p += kTopRows) tile[padq(p)] = ldg1(src + p);
+    } else if (vec && kt == kTopKT) {
+        // rows x 8 float4 per tile; a warp covers 4 rows x 128 B per load.
+        for (int v = t; v < rows * 8; v += kTopRows) {
+            const int row = v >> 3, c4 = v & 7;
+            V q = ldg_stream4(in + (r0 + row) * m + k0 + 4 * c4);
+            T e[4];
+            unpack4<T>(q, e);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) tile[padq(row * kTopKT + 4 * c4 + u)] = e[u];
+        }
+    } else {
+        for (int p = t; p < rows * kTopKT; p += kTopRows) {
+            const int row = p >> 5, col = p & 31;
+            if (col < kt) tile[padq(p)] = ldg1(in + (r0 + row) * m + k0 + col);
+        }
+    }
+}
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(kTopRows) segred_top_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                              int64_t n, int64_t m, T d, bool vec) {
+    __shared__ T tile[kTopWords];
+    const int t = threadIdx.x;
+    const int64_t r0 = (int64_t)blockIdx.x * kTopRows;
+    const int rows = (int)min((int64_t)kTopRows, n - r0);
+    T acc[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+    if (m <= kTopKT) {
+        top_load_tile(tile, in, r0, rows, m, 0, (int)m, true, vec);
+        __syncthreads();
+        if (t < rows) {
+            const int mm = (int)m;
+            for (int k = 0; k < mm; ++k) acc[k & 3] = combine<OP>(acc[k & 3], apply_map<F>(tile[padq(t * mm + k)]));
+        }
+    } else {
+        for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
+            const int kt = (int)min((int64_t)kTopKT, m - k0);
+            top_load_tile(tile, in, r0, rows, m, k0, kt, false, vec);
+            __syncthreads();
+            if (t < rows) {
+                if (kt == kTopKT) {
+#pragma unroll
+                    for (int k = 0; k < kTopKT; ++k)
+                        acc[k & 3] = combine<OP>(acc[k & 3], apply_map<F>(tile[padq(t * kTopKT + k)]));
+                } else {
+                    for (int k = 0; k < kt; ++k)
+                        acc[k & 3] = combine<OP>(acc[k & 3], apply_map<F>(tile[padq(t * kTopKT + k)]));
+                }
+            }
+            __syncthreads();
+        }
+    }
+    if (t < rows) {
+        T r = combine<OP>(combine<OP>(acc[0], acc[1]), combine<OP>(acc[2], acc[3]));
+        out[r0 + t] = combine<OP>(d, r);
+    }
+}
+
+cudaError_t launch_segred_top(const SegArgs& a) {
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        const bool vec = ((uintptr_t)a.in % 16 == 0) && (a.m <= kTopKT || a.m % 4 == 0);
+        const int64_t grid = ceil_div(a.n, kTopRows);
+        segred_top_kernel<T, OP, F><<<(unsigned)grid, kTopRows, 0, a.stream>>>(
+            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
+        return cudaGetLastError();
+    });
+}
+
+// --------------------------------------------------------------- V_MIDDLE
+
+int mid_group_size(int64_t m) {
+    int64_t g = 2;
+    while (g < 1024 && g * 16 < m) g <<= 1;
+    return (int)g;
+}
+
+// Reduce `acc` over the G threads of a group.  G <= 32: shuffles inside the
+// warp; G > 32: warp shuffles, then the group's warp totals via shared memory.
+template <int OP, typename T>
+__device__ __forceinline__ T group_reduce(T acc, int G, T* red) {
+    if (G <= 32) {
+        for (int off = G >> 1; off > 0; off >>= 1) acc = combine<OP>(acc, __shfl_xor_sync(0xffffffffu, acc, off));
+        return acc;
+    }
+    acc = warp_reduce<OP>(acc);
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane == 0) red[w] = acc;
+    __syncthreads();
+    const int wpg = G >> 5, w0 = (threadIdx.x / G) * wpg;
+    T r = identity<OP, T>();
+    for (int k = 0; k < wpg; ++k) r = combine<OP>(r, red[w0 + k]);
+    return r;
+}
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(1024) segred_mid_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                          int64_t n, int64_t m, T d, int G) {
+    __shared__ T red[32];
+    using V = typename Vec4<T>::type;
+    const int g = threadIdx.x % G;
+    const int64_t i = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
+    T acc = identity<OP, T>();
+    if (i < n) {
+        const T* row = in + i * m;
+        int64_t h = (int64_t)(((16u - ((uint32_t)(uintptr_t)row & 15u)) & 15u) / sizeof(T));
+        if (h > m) h = m;
+        const int64_t nvec = (m - h) >> 2;
+        for (int64_t k = g; k < h; k += G) acc = combine<OP>(acc, apply_map<F>(ldg1(row + k)));
+        const T* body = row + h;
+        T a4[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+        int64_t v = g;
+        for (; v + 3 * (int64_t)G < nvec; v += 4 * (int64_t)G) {
+            V q[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) q[u] = ldg_stream4(body + 4 * (v + u * (int64_t)G));
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+                T e[4];
+                unpack4<T>(q[u], e);
+#pragma unroll
+                for (int c = 0; c < 4; ++c) a4[c] = combine<OP>(a4[c], apply_map<F>(e[c]));
+            }
+        }
+        for (; v < nvec; v += G) {
+            T e[4];
+            unpack4<T>(ldg_stream4(body + 4 * v), e);
+#pragma unroll
+            for (int c = 0; c < 4; ++c) a4[c] = combine<OP>(a4[c], apply_map<F>(e[c]));
+        }
+        const int64_t t0 = h + 4 * nvec;
+        for (int64_t k = t0 + g; k < m; k += G) acc = combine<OP>(acc, apply_map<F>(ldg1(row + k)));
+        acc = combine<OP>(acc, combine<OP>(combine<OP>(a4[0], a4[1]), combine<OP>(a4[2], a4[3])));
+    }
+    acc = group_reduce<OP>(acc, G, red);
+    if (g == 0 && i < n) out[i] = combine<OP>(d, acc);
+}
+
+cudaError_t launch_segred_mid(const SegArgs& a) {
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        const int G = mid_group_size(a.m);
+        const int B = G > 256 ? G : 256;
+        const int64_t grid = ceil_div(a.n, B / G);
+        segred_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, a.m,
+                                                                        bits_to<T>(a.ne_bits), G);
+        return cudaGetLastError();
+    });
+}
+
+// ------------------------------------------------------------ m == 0 fill
+
+__global__ void fill_kernel(uint32_t* out, int64_t count, uint32_t bits) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < count; i += (int64_t)gridDim.x * blockDim.x)
+        out[i] = bits;
+}
+
+cudaError_t launch_fill(void* out, int64_t count, uint32_t bits, cudaStream_t s) {
+    if (count <= 0) return cudaSuccess;
+    const int64_t grid = min(ceil_div(count, 256), (int64_t)148 * 16);
+    fill_kernel<<<(unsigned)grid, 256, 0, s>>>((uint32_t*)out, count, bits);
+    return cudaGetLastError();
+}
+
+}  // namespace ifl

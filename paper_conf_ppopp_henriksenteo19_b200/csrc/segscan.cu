@@ -1,0 +1,250 @@
+// segscan.cu -- the V_TOP and V_MIDDLE versions of segscan (Fig 6c
+// versions 1 and 2) for an [n][m] row-major array.
+//
+//   V_TOP    segmap^1 <xs in xss> (scanomap (+) f d xs): one thread per row,
+//            [256][32] column tiles staged through padded shared memory
+//            (coalesced 128-bit loads and stores), each thread scans its row
+//            sequentially in place with a running carry.
+//   V_MIDDLE segmap^1 <xs in xss> (segscan^0 <x in xs> (+) d (f x)): a group
+//            of G threads per row; per round each thread scans 8 consecutive
+//            elements in registers, the group scans the thread totals with
+//            warp shuffles (+ shared memory when G > 32) and carries the
+//            round total to the next round.
+#include <string.h>
+
+#include "common.cuh"
+#include "dispatch.cuh"
+#include "ifl_internal.h"
+
+namespace ifl {
+
+constexpr int kTopRows = 256;
+constexpr int kTopKT = 32;
+constexpr int kTopWords = kTopRows * kTopKT + kTopRows * kTopKT / 32;
+
+__device__ __forceinline__ int spadq(int q) { return q + (q >> 5); }
+
+// Copy between a global [rows][kt] window and the padded smem tile.  LOAD:
+// global -> smem (applying nothing); STORE: smem -> global.
+template <bool LOAD, typename T>
+__device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* __restrict__ out, int64_t r0,
+                                         int rows, int64_t m, int64_t k0, int kt, bool whole, bool vec) {
+    const int t = threadIdx.x;
+    using V = typename Vec4<T>::type;
+    if (whole) {
+        const int cnt = rows * (int)m;
+        int p0 = 0;
+        if (vec) {
+            const int nv = cnt >> 2;
+            for (int v = t; v < nv; v += kTopRows) {
+                if (LOAD) {
+                    T e[4];
+                    unpack4<T>(ldg_stream4(in + r0 * m + 4 * v), e);
+#pragma unroll
+                    for (int u = 0; u < 4; ++u) tile[spadq(4 * v + u)] = e[u];
+                } else {
+                    V q;
+                    q.x = tile[spadq(4 * v)];
+                    q.y = tile[spadq(4 * v + 1)];
+                    q.z = tile[spadq(4 * v + 2)];
+                    q.w = tile[spadq(4 * v + 3)];
+                    *reinterpret_cast<V*>(out + r0 * m + 4 * v) = q;
+                }
+            }
+            p0 = nv << 2;
+        }
+        for (int p = p0 + t; p < cnt; p += kTopRows) {
+            if (LOAD) tile[spadq(p)] = ldg1(in + r0 * m + p);
+            else out[r0 * m + p] = tile[spadq(p)];
+        }
+    } else if (vec && kt == kTopKT) {
+        for (int v = t; v < rows * 8; v += kTopRows) {
+            const int row = v >> 3, c4 = v & 7;
+            const int64_t gi = (r0 + row) * m + k0 + 4 * c4;
+            const int q0 = row * kTopKT + 4 * c4;
+            if (LOAD) {
+                T e[4];
+                unpack4<T>(ldg_stream4(in + gi), e);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) tile[spadq(q0 + u)] = e[u];
+            } else {
+                V q;
+                q.x = tile[spadq(q0)];
+                q.y = tile[spadq(q0 + 1)];
+                q.z = tile[spadq(q0 + 2)];
+                q.w = tile[spadq(q0 + 3)];
+                *reinterpret_cast<V*>(out + gi) = q;
+            }
+        }
+    } else {
+        for (int p = t; p < rows * kTopKT; p += kTopRows) {
+            const int row = p >> 5, col = p & 31;
+            if (col < kt) {
+                const int64_t gi = (r0 + row) * m + k0 + col;
+                if (LOAD) tile[spadq(p)] = ldg1(in + gi);
+                else out[gi] = tile[spadq(p)];
+            }
+        }
+    }
+}
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(kTopRows) segscan_top_kernel(const T* in, T* out, int64_t n, int64_t m, T d,
+                                                               bool vec) {
+    __shared__ T tile[kTopWords];
+    const int t = threadIdx.x;
+    const int64_t r0 = (int64_t)blockIdx.x * kTopRows;
+    const int rows = (int)min((int64_t)kTopRows, n - r0);
+    T acc = d;  // d (+) f(x0) (+) ... : d applied once, at the row start
+    if (m <= kTopKT) {
+        top_xfer<true>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
+        __syncthreads();
+        if (t < rows) {
+            const int mm = (int)m;
+            for (int k = 0; k < mm; ++k) {
+                acc = combine<OP>(acc, apply_map<F>(tile[spadq(t * mm + k)]));
+                tile[spadq(t * mm + k)] = acc;
+            }
+        }
+        __syncthreads();
+        top_xfer<false>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
+    } else {
+        for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
+            const int kt = (int)min((int64_t)kTopKT, m - k0);
+            top_xfer<true>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+            __syncthreads();
+            if (t < rows) {
+                if (kt == kTopKT) {
+#pragma unroll
+                    for (int k = 0; k < kTopKT; ++k) {
+                        acc = combine<OP>(acc, apply_map<F>(tile[spadq(t * kTopKT + k)]));
+                        tile[spadq(t * kTopKT + k)] = acc;
+                    }
+                } else {
+                    for (int k = 0; k < kt; ++k) {
+                        acc = combine<OP>(acc, apply_map<F>(tile[spadq(t * kTopKT + k)]));
+                        tile[spadq(t * kTopKT + k)] = acc;
+                    }
+                }
+            }
+            __syncthreads();
+            top_xfer<false>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+            __syncthreads();
+        }
+    }
+}
+
+cudaError_t launch_segscan_top(const SegArgs& a) {
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) &&
+                         (a.m <= kTopKT || a.m % 4 == 0);
+        const int64_t grid = ceil_div(a.n, kTopRows);
+        segscan_top_kernel<T, OP, F><<<(unsigned)grid, kTopRows, 0, a.stream>>>(
+            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
+        return cudaGetLastError();
+    });
+}
+
+// --------------------------------------------------------------- V_MIDDLE
+
+constexpr int kMidItems = 8;  // consecutive elements per thread per round
+
+int midscan_group_size(int64_t m) {
+    int64_t g = 2;
+    while (g < 1024 && g * kMidItems < m) g <<= 1;
+    return (int)g;
+}
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, int64_t n, int64_t m, T d, int G,
+                                                           bool vec) {
+    __shared__ T wtot[2][32];
+    using V = typename Vec4<T>::type;
+    const int g = threadIdx.x % G;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t i = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
+    const bool live = i < n;
+    const T* row = in + (live ? i * m : 0);
+    T* orow = out + (live ? i * m : 0);
+    T carry = d;
+    int par = 0;
+    for (int64_t base = 0; base < m; base += (int64_t)G * kMidItems, par ^= 1) {
+        const int64_t k0 = base + (int64_t)g * kMidItems;
+        T v[kMidItems];
+        if (live && vec && k0 + kMidItems <= m) {
+            T e[4];
+            unpack4<T>(ldg_stream4(row + k0), e);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) v[u] = apply_map<F>(e[u]);
+            unpack4<T>(ldg_stream4(row + k0 + 4), e);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) v[4 + u] = apply_map<F>(e[u]);
+        } else {
+#pragma unroll
+            for (int u = 0; u < kMidItems; ++u)
+                v[u] = (live && k0 + u < m) ? apply_map<F>(ldg1(row + k0 + u)) : identity<OP, T>();
+        }
+#pragma unroll
+        for (int u = 1; u < kMidItems; ++u) v[u] = combine<OP>(v[u - 1], v[u]);
+        // inclusive scan of thread totals across the group
+        T s = v[kMidItems - 1];
+        const int width = G < 32 ? G : 32;
+        const int gl = threadIdx.x % width;  // lane within the (sub)warp group
+        for (int off = 1; off < width; off <<= 1) {
+            T o = __shfl_up_sync(0xffffffffu, s, off, width);
+            if (gl >= off) s = combine<OP>(o, s);
+        }
+        T ex = __shfl_up_sync(0xffffffffu, s, 1, width);
+        if (gl == 0) ex = identity<OP, T>();
+        T total;
+        if (G <= 32) {
+            total = __shfl_sync(0xffffffffu, s, width - 1, width);
+        } else {
+            if (lane == 31) wtot[par][w] = s;
+            __syncthreads();
+            const int wpg = G >> 5, w0 = (threadIdx.x / G) * wpg;
+            T before = identity<OP, T>();
+            total = identity<OP, T>();
+            for (int k = 0; k < wpg; ++k) {
+                if (w0 + k < w) before = combine<OP>(before, wtot[par][w0 + k]);
+                total = combine<OP>(total, wtot[par][w0 + k]);
+            }
+            ex = combine<OP>(before, ex);
+        }
+        const T pre = combine<OP>(carry, ex);
+#pragma unroll
+        for (int u = 0; u < kMidItems; ++u) v[u] = combine<OP>(pre, v[u]);
+        if (live) {
+            if (vec && k0 + kMidItems <= m) {
+                V q0, q1;
+                q0.x = v[0]; q0.y = v[1]; q0.z = v[2]; q0.w = v[3];
+                q1.x = v[4]; q1.y = v[5]; q1.z = v[6]; q1.w = v[7];
+                *reinterpret_cast<V*>(orow + k0) = q0;
+                *reinterpret_cast<V*>(orow + k0 + 4) = q1;
+            } else {
+#pragma unroll
+                for (int u = 0; u < kMidItems; ++u)
+                    if (k0 + u < m) orow[k0 + u] = v[u];
+            }
+        }
+        carry = combine<OP>(carry, total);
+    }
+}
+
+cudaError_t launch_segscan_mid(const SegArgs& a) {
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        const int G = midscan_group_size(a.m);
+        const int B = G > 256 ? G : 256;
+        const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) && (a.m % 4 == 0);
+        const int64_t grid = ceil_div(a.n, B / G);
+        segscan_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, a.m,
+                                                                         bits_to<T>(a.ne_bits), G, vec);
+        return cudaGetLastError();
+    });
+}
+
+}  // namespace ifl

@@ -1,0 +1,254 @@
+// tune.cpp -- the offline threshold tuner.
+//
+// The paper tunes one LogIntegerParameter per threshold with OpenTuner,
+// summing runtimes over user datasets, and memoises repeated paths
+// through the branching tree; it suggests using the tree to avoid
+// redundant settings altogether.  That is what this does, exactly:
+//   1. measure: run every forced version on every training shape, R reps,
+//      CUDA events on the caller's stream, median -> cost_table[s][v];
+//   2. search: the only thresholds that matter are those between adjacent
+//      training Par values (anything in between gives the same path), so
+//      enumerate t_top over {min Par_top, geometric midpoints, +inf} and
+//      t_intra likewise, map each pair to its path (one version per shape),
+//      evaluate each DISTINCT path once (memoised), keep the cheapest.
+#include <cuda_runtime.h>
+#include <string.h>
+
+#include <algorithm>
+#include <cmath>
+#include <limits>
+#include <map>
+#include <vector>
+
+#include "../../include/ifl.h"
+#include "ifl_internal.h"
+
+namespace {
+
+std::vector<int64_t> candidates(std::vector<int64_t> v) {
+    std::sort(v.begin(), v.end());
+    v.erase(std::unique(v.begin(), v.end()), v.end());
+    std::vector<int64_t> c;
+    if (v.empty()) return {INT64_MAX};
+    c.push_back(v.front());  // every shape passes the guard
+    for (size_t i = 0; i + 1 < v.size(); ++i) {
+        // geometric midpoint, strictly above v[i] and at most v[i+1] (reading q)
+        double g = std::ceil(std::sqrt((double)v[i] * (double)v[i + 1]));
+        int64_t t = (int64_t)g;
+        if (t <= v[i]) t = v[i] + 1;
+        if (t > v[i + 1]) t = v[i + 1];
+        c.push_back(t);
+    }
+    c.push_back(INT64_MAX);  // no shape passes the guard
+    return c;
+}
+
+}  // namespace
+
+extern "C" int ifl_tune_search(const int64_t* par_top, const int64_t* par_mid, const double* cost_table, int nshapes,
+                               int cost, int64_t* t_top, int64_t* t_intra, int* n_paths) {
+    if (nshapes <= 0 || !par_top || !par_mid || !cost_table || (cost != 0 && cost != 1)) return IFL_EINVAL;
+    std::vector<int64_t> pt(par_top, par_top + nshapes), pm(par_mid, par_mid + nshapes);
+    const std::vector<int64_t> ct = candidates(pt), ci = candidates(pm);
+    std::vector<double> best(nshapes, std::numeric_limits<double>::infinity());
+    for (int s = 0; s < nshapes; ++s)
+        for (int v = 0; v < 3; ++v) best[s] = std::min(best[s], cost_table[s * 3 + v]);
+
+    std::map<std::vector<int>, std::pair<double, double>> memo;  // path -> (primary, sum)
+    double bp = std::numeric_limits<double>::infinity(), bs = bp;
+    int64_t btop = ct.back(), bintra = ci.back();
+    for (int64_t a : ct) {
+        for (int64_t b : ci) {
+            std::vector<int> path(nshapes);
+            for (int s = 0; s < nshapes; ++s)
+                path[s] = pt[s] >= a ? IFL_V_TOP : (pm[s] >= b ? IFL_V_MIDDLE : IFL_V_FLAT);
+            auto it = memo.find(path);
+            if (it == memo.end()) {
+                double sum = 0, worst = 0;
+                for (int s = 0; s < nshapes; ++s) {
+                    const double c = cost_table[s * 3 + path[s]];
+                    sum += c;
+                    worst = std::max(worst, c / best[s]);
+                }
+                it = memo.emplace(path, std::make_pair(cost == 0 ? sum : worst, sum)).first;
+            }
+            const double p = it->second.first, s = it->second.second;
+            if (p < bp || (p == bp && s < bs)) {
+                bp = p;
+                bs = s;
+                btop = a;
+                bintra = b;
+            }
+        }
+    }
+    if (t_top) *t_top = btop;
+    if (t_intra) *t_intra = bintra;
+    if (n_paths) *n_paths = (int)memo.size();
+    return std::isfinite(bp) ? IFL_OK : IFL_ENOTFIT;
+}
+
+namespace {
+
+enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_BAD };
+
+Kind kind_of(const char* site) {
+    if (!site) return K_BAD;
+    if (!strcmp(site, "segred.b4")) return K_SEGRED;
+    if (!strcmp(site, "segscan.b4")) return K_SEGSCAN;
+    if (!strcmp(site, "redomap2.f32")) return K_MM_F32;
+    if (!strcmp(site, "redomap2.bf16")) return K_MM_BF16;
+    if (!strcmp(site, "tridag")) return K_TRIDAG;
+    return K_BAD;
+}
+
+int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN) ? 2 : 3; }
+
+size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
+
+size_t ws_bytes_of(Kind k, const int64_t* s) {
+    switch (k) {
+    case K_SEGRED: return ifl_workspace_bytes("segred", s[0], s[1], 0, IFL_F32, -1);
+    case K_SEGSCAN: return ifl_workspace_bytes("segscan", s[0], s[1], 0, IFL_F32, -1);
+    case K_MM_F32: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_F32, -1);
+    case K_MM_BF16: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_BF16, -1);
+    case K_TRIDAG: return ifl_workspace_bytes("tridag", s[0], s[1], 0, IFL_F32, -1);
+    default: return 0;
+    }
+}
+
+// Scratch layout per shape: [in/A/...][out][ws], each 256-byte aligned.
+size_t shape_bytes(Kind k, const int64_t* s) {
+    switch (k) {
+    case K_SEGRED: {
+        const int64_t n = s[0], m = s[1];
+        return align256(n * m * 4) + align256(n * 4) + align256(ifl_workspace_bytes("segred", n, m, 0, IFL_F32, -1));
+    }
+    case K_SEGSCAN: {
+        const int64_t n = s[0], m = s[1];
+        return 2 * align256(n * m * 4) + align256(ifl_workspace_bytes("segscan", n, m, 0, IFL_F32, -1));
+    }
+    case K_MM_F32:
+    case K_MM_BF16: {
+        const int64_t n = s[0], m = s[1], p = s[2], e = k == K_MM_F32 ? 4 : 2;
+        return align256(n * m * e) + align256(m * p * e) + align256(n * p * 4) +
+               align256(ifl_workspace_bytes("redomap2", n, m, p, k == K_MM_F32 ? IFL_F32 : IFL_BF16, -1));
+    }
+    case K_TRIDAG: {
+        const int64_t S = s[0], L = s[1], R = s[2];
+        return 3 * align256(R * L * 4) + 2 * align256(S * L * 4) +
+               align256(ifl_workspace_bytes("tridag", S, L, 0, IFL_F32, -1));
+    }
+    default: return 0;
+    }
+}
+
+int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_t st) {
+    switch (k) {
+    case K_SEGRED: {
+        const int64_t n = s[0], m = s[1];
+        char* in = scratch;
+        char* out = in + align256(n * m * 4);
+        char* ws = out + align256(n * 4);
+        return ifl_segred(in, out, n, m, IFL_F32, IFL_SUM, IFL_F_ID, nullptr, version, ws,
+                          ifl_workspace_bytes("segred", n, m, 0, IFL_F32, -1), st, nullptr);
+    }
+    case K_SEGSCAN: {
+        const int64_t n = s[0], m = s[1];
+        char* in = scratch;
+        char* out = in + align256(n * m * 4);
+        char* ws = out + align256(n * m * 4);
+        return ifl_segscan(in, out, n, m, IFL_F32, IFL_SUM, IFL_F_ID, nullptr, 0, version, ws,
+                           ifl_workspace_bytes("segscan", n, m, 0, IFL_F32, -1), st, nullptr);
+    }
+    case K_MM_F32:
+    case K_MM_BF16: {
+        const int64_t n = s[0], m = s[1], p = s[2], e = k == K_MM_F32 ? 4 : 2;
+        const int dt = k == K_MM_F32 ? IFL_F32 : IFL_BF16;
+        char* A = scratch;
+        char* B = A + align256(n * m * e);
+        char* C = B + align256(m * p * e);
+        char* ws = C + align256(n * p * 4);
+        return ifl_redomap2(A, B, (float*)C, n, m, p, dt, 1, version, ws,
+                            ifl_workspace_bytes("redomap2", n, m, p, dt, -1), st, nullptr);
+    }
+    case K_TRIDAG: {
+        const int64_t S = s[0], L = s[1], R = s[2];
+        char* a = scratch;
+        char* b = a + align256(R * L * 4);
+        char* c = b + align256(R * L * 4);
+        char* y = c + align256(R * L * 4);
+        char* x = y + align256(S * L * 4);
+        char* ws = x + align256(S * L * 4);
+        return ifl_tridag((float*)a, (float*)b, (float*)c, (float*)y, (float*)x, S, L, R, version, ws,
+                          ifl_workspace_bytes("tridag", S, L, 0, IFL_F32, -1), st, nullptr);
+    }
+    default: return IFL_EINVAL;
+    }
+}
+
+}  // namespace
+
+extern "C" size_t ifl_tune_scratch_bytes(const char* site, const int64_t* shapes, int nshapes) {
+    const Kind k = kind_of(site);
+    if (k == K_BAD || !shapes || nshapes <= 0) return 0;
+    size_t mx = 0;
+    for (int i = 0; i < nshapes; ++i) mx = std::max(mx, shape_bytes(k, shapes + i * arity(k)));
+    return mx;
+}
+
+extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, int reps, int cost, void* scratch,
+                        size_t scratch_bytes, void* stream, int64_t* t_top, int64_t* t_intra, double* cost_table) {
+    const Kind k = kind_of(site);
+    if (k == K_BAD || !shapes || nshapes <= 0 || reps <= 0 || !scratch) return IFL_EINVAL;
+    if (scratch_bytes < ifl_tune_scratch_bytes(site, shapes, nshapes)) return IFL_EWORKSPACE;
+    const int ar = arity(k);
+    cudaStream_t st = (cudaStream_t)stream;
+    std::vector<double> table(nshapes * 3, std::numeric_limits<double>::infinity());
+    std::vector<int64_t> ptop(nshapes), pmid(nshapes);
+    cudaEvent_t e0, e1;
+    if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess) return IFL_ECUDA;
+    int rc = IFL_OK;
+    for (int i = 0; i < nshapes && rc == IFL_OK; ++i) {
+        const int64_t* s = shapes + i * ar;
+        ifl_choice c;
+        ifl_select(site, s[0], s[1], ar == 3 && k != K_TRIDAG ? s[2] : 0, &c);
+        ptop[i] = c.par_top;
+        pmid[i] = c.par_mid;
+        // zero this shape's workspace (the tail of its scratch layout); the
+        // input region keeps the caller's data
+        const size_t tot = shape_bytes(k, s), wsb = ws_bytes_of(k, s);
+        if (wsb && cudaMemsetAsync((char*)scratch + (tot - align256(wsb)), 0, align256(wsb), st) != cudaSuccess) {
+            rc = IFL_ECUDA;
+            break;
+        }
+        for (int v = 0; v < 3; ++v) {
+            int r = run_forced(k, s, v, (char*)scratch, st);  // warm-up; also feasibility (ENOTFIT)
+            if (r == IFL_ENOTFIT || r == IFL_EUNSUPPORTED) continue;
+            if (r != IFL_OK) {
+                rc = r;
+                break;
+            }
+            std::vector<float> ms(reps);
+            for (int q = 0; q < reps; ++q) {
+                cudaEventRecord(e0, st);
+                run_forced(k, s, v, (char*)scratch, st);
+                cudaEventRecord(e1, st);
+                cudaEventSynchronize(e1);
+                cudaEventElapsedTime(&ms[q], e0, e1);
+            }
+            std::sort(ms.begin(), ms.end());
+            table[i * 3 + v] = ms[reps / 2];
+        }
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    if (rc != IFL_OK) return rc;
+    if (cost_table) std::copy(table.begin(), table.end(), cost_table);
+    int64_t a, b;
+    int np;
+    rc = ifl_tune_search(ptop.data(), pmid.data(), table.data(), nshapes, cost, &a, &b, &np);
+    if (rc != IFL_OK) return rc;
+    if (t_top) *t_top = a;
+    if (t_intra) *t_intra = b;
+    return ifl_set_thresholds(site, a, b);
+}
