@@ -109,6 +109,30 @@ __device__ __forceinline__ typename Vec4<T>::type ldg_stream4(const T* p) {
 template <typename T>
 __device__ __forceinline__ T ldg1(const T* p) { return __ldg(p); }
 
+// Running (+)-accumulator.  For f32 sums it is Kahan-compensated, so a long
+// sequential chain (a thread-per-segment walk over m ~ 2^26 elements) stays
+// within the 1e-5 relative parity bound; every other (+) is exact or
+// associative already.
+template <int OP, typename T>
+struct Acc {
+    T s;
+    __device__ __forceinline__ explicit Acc(T init) : s(init) {}
+    __device__ __forceinline__ void add(T x) { s = combine<OP>(s, x); }
+    __device__ __forceinline__ T get() const { return s; }
+};
+template <>
+struct Acc<OP_SUM, float> {
+    float s, c;
+    __device__ __forceinline__ explicit Acc(float init) : s(init), c(0.0f) {}
+    __device__ __forceinline__ void add(float x) {
+        const float y = __fsub_rn(x, c);
+        const float t = __fadd_rn(s, y);
+        c = __fsub_rn(__fsub_rn(t, s), y);
+        s = t;
+    }
+    __device__ __forceinline__ float get() const { return s; }
+};
+
 // ------------------------------------------------------- warp primitives
 
 template <int OP, typename T>
@@ -174,6 +198,9 @@ __device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t by
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() {
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read1() {
+    asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
 }
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 

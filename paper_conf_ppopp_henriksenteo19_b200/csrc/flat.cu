@@ -1,27 +1,37 @@
 // flat.cu -- V_FLAT: the fully flattened segred^1 / segscan^1 over all n*m
 // elements (rule G3's e_flat; Fig 6c version 3).
 //
-// One single-pass kernel serves both (SCAN writes every prefix, RED writes
-// only the segment ends).  The flat index space [0, n*m) is cut into tiles of
-// kFlatTile = 256 x 28 elements.  Per tile (one CTA, dynamic tile id):
-//   1. the TMA engine copies the contiguous tile into shared memory
-//      (cp.async.bulk, completion on an mbarrier);
-//   2. thread t takes 28 consecutive elements (7 conflict-free LDS.128: the
-//      112-byte stride is an odd multiple of 16 B) and runs a sequential
-//      segmented scan; segment starts are arithmetic (multiples of m), so no
-//      flag array is read -- d is combined into every segment's first element;
-//   3. the CTA scans the (flag, value) thread aggregates with the segmented
-//      operator (f1,v1).(f2,v2) = (f1|f2, f2 ? v2 : v1 (+) v2);
-//   4. decoupled look-back over predecessor tiles' 64-bit status words
-//      (aggregate / inclusive prefix, with the segment flag) gives the carry
-//      into the tile; a tile that starts with a segment start skips it;
-//   5. SCAN: results go back to shared memory and the TMA engine stores the
-//      tile (cp.async.bulk shared -> global); RED: each segment end writes
-//      out[segment].
-// The workspace header carries a dynamic tile counter, a completion counter
-// and an epoch; the last CTA resets the counters and bumps the epoch, and
-// status words carry the epoch as a tag, so no memset is needed per call.
+// The flat index space [0, n*m) is cut into tiles of kFlatTile = 256 x 20
+// elements.  Segment starts are arithmetic (multiples of m): no flag array is
+// read, and d is combined into every segment's first element.  Both kernels
+// are persistent (grid = resident CTAs) and stream tiles through a ring of
+// kSlots shared-memory slots filled by the TMA engine (cp.async.bulk +
+// mbarrier), so loads for the next tiles are in flight while a tile is
+// processed.  Per tile:
+//   * thread t takes its 20 consecutive elements (5 conflict-free LDS.128: the
+//     80-byte stride is an odd multiple of 16 B).  A thread whose items hold
+//     no segment boundary (the common case once m exceeds a few dozen) takes a
+//     branch-free fast path; otherwise a sequential segmented scan;
+//   * the CTA scans the (flag, value) thread aggregates with the segmented
+//     operator (f1,v1).(f2,v2) = (f1|f2, f2 ? v2 : v1 (+) v2).
+// segred (two passes, no inter-CTA waiting):
+//   pass 1  complete segments are written to out directly; each tile leaves
+//           head[t] (partial of the segment it starts inside) and tail[t]
+//           (the open segment at its end, or the whole tile) in the workspace;
+//   pass 2  every segment that crosses tiles ta < tb is
+//           out = tail[ta] (+) tail[ta+1..tb-1] (+) head[tb]   (a tree reduce).
+// segscan (single pass, decoupled look-back):
+//   tiles are claimed dynamically; each publishes a 64-bit status word
+//   (aggregate / inclusive prefix, segment flag, epoch tag) and looks back for
+//   its carry only if it does not begin with a segment start; results return to
+//   the slot and the TMA engine stores the tile (cp.async.bulk shared->global).
+//   The workspace is re-armed by the last CTA (counter reset, epoch bump), so no
+//   per-call memset is needed.
+// Workspace: [header 256 B][status: 8 B/tile][head: 4 B/tile][tail: 4 B/tile].
 #include <string.h>
+
+#include <algorithm>
+#include <unordered_map>
 
 #include "common.cuh"
 #include "dispatch.cuh"
@@ -32,6 +42,7 @@ namespace ifl {
 constexpr int FB = kFlatThreads;
 constexpr int FI = kFlatItems;
 constexpr int FT = (int)kFlatTile;
+constexpr int kSlots = 4;
 static_assert(FI % 4 == 0 && (FI / 4) % 2 == 1, "odd number of 16-byte chunks per thread");
 
 struct FlatHdr {
@@ -44,7 +55,7 @@ static_assert(sizeof(FlatHdr) == 256, "header size");
 
 size_t flat_ws_bytes(int64_t total) {
     const int64_t tiles = ceil_div(total, kFlatTile);
-    return sizeof(FlatHdr) + (size_t)tiles * 8;
+    return sizeof(FlatHdr) + (size_t)tiles * 16;
 }
 
 // status word: [63:35] tag, [34:33] status (1 aggregate, 2 inclusive), [32] flag, [31:0] value
@@ -53,85 +64,80 @@ __device__ __forceinline__ uint64_t pack_status(uint32_t tag, uint64_t st, uint3
     return ((uint64_t)tag << 35) | (st << 33) | ((uint64_t)flag << 32) | (uint64_t)val;
 }
 
-template <typename T, int OP, int F, bool SCAN>
-__global__ void __launch_bounds__(FB) flat_kernel(const T* in, T* out, int64_t N, int64_t m, T d, uint8_t* ws,
-                                                  int num_tiles, bool tma_in, bool tma_out) {
-    __shared__ alignas(128) T buf[FT];
-    __shared__ alignas(8) uint64_t mbar;
-    __shared__ int s_tile;
-    __shared__ uint32_t s_tag;
-    __shared__ T s_wval[FB / 32];
-    __shared__ uint32_t s_wflag[FB / 32];
-    __shared__ T s_carry;
+// Per-slot tile metadata, written by the producer thread when it claims a tile.
+struct SlotMeta {
+    int tile;
+    int cnt;
+    int64_t pos;  // (tile*FT) % m
+    int64_t seg;  // (tile*FT) / m
+};
 
-    FlatHdr* hdr = reinterpret_cast<FlatHdr*>(ws);
-    uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-
-    if (t == 0) {
-        s_tile = (int)atomicAdd(&hdr->tile_ctr, 1u);
-        s_tag = ld_relaxed_u32(&hdr->epoch) & 0x1FFFFFFFu;
-        mbar_init(&mbar, 1);
-        fence_mbar_init();
-    }
-    __syncthreads();
-    const int tile = s_tile;
-    const uint32_t tag = s_tag;
+__device__ __forceinline__ void fill_meta(SlotMeta& sm, int tile, int64_t N, int64_t m) {
     const int64_t base = (int64_t)tile * FT;
-    const int cnt = (int)min((int64_t)FT, N - base);
-    const bool full = (cnt == FT);
+    sm.tile = tile;
+    sm.cnt = (int)std::min((int64_t)FT, N - base);
+    sm.pos = base % m;
+    sm.seg = base / m;
+}
 
-    // ---- 1. stage the tile in shared memory
-    if (full && tma_in) {
-        if (t == 0) {
-            mbar_arrive_expect_tx(&mbar, FT * sizeof(T));
-            bulk_g2s(buf, in + base, FT * sizeof(T), &mbar);
+// Thread view of a tile: position of its first item inside its segment.
+struct ThreadPos {
+    int nvalid, nx0, mi;
+    int64_t seg;  // segment of the thread's first item
+};
+
+__device__ __forceinline__ ThreadPos thread_pos(const SlotMeta& sm, int64_t m) {
+    ThreadPos p;
+    const int off = threadIdx.x * FI;
+    p.nvalid = max(0, min(FI, sm.cnt - off));
+    int64_t pos;
+    if (m > FT) {  // at most one boundary inside the tile: no division
+        pos = sm.pos + off;
+        p.seg = sm.seg;
+        if (pos >= m) {
+            pos -= m;
+            p.seg += 1;
         }
-        mbar_wait(&mbar, 0);
-    } else {
-        for (int p = t; p < cnt; p += FB) buf[p] = in[base + p];
-        __syncthreads();
+    } else {  // m fits 32 bits
+        const uint32_t q = (uint32_t)sm.pos + (uint32_t)off, mm = (uint32_t)m;
+        pos = q % mm;
+        p.seg = sm.seg + q / mm;
     }
+    p.mi = (int)std::min(m, (int64_t)FI + 1);
+    p.nx0 = (int)std::min(pos == 0 ? (int64_t)0 : m - pos, (int64_t)FI + 1);
+    return p;
+}
 
-    // ---- 2. thread-local segmented scan over FI consecutive elements
-    const int o = t * FI;
-    T v[FI];
-    {
-        using V = typename Vec4<T>::type;
+template <typename T>
+__device__ __forceinline__ void load_items(const T* buf, T (&v)[FI]) {
+    using V = typename Vec4<T>::type;
+    const int o = threadIdx.x * FI;
 #pragma unroll
-        for (int c = 0; c < FI / 4; ++c) {
-            V q = *reinterpret_cast<const V*>(&buf[o + 4 * c]);
-            v[4 * c] = q.x; v[4 * c + 1] = q.y; v[4 * c + 2] = q.z; v[4 * c + 3] = q.w;
-        }
+    for (int c = 0; c < FI / 4; ++c) {
+        V q = *reinterpret_cast<const V*>(&buf[o + 4 * c]);
+        v[4 * c] = q.x; v[4 * c + 1] = q.y; v[4 * c + 2] = q.z; v[4 * c + 3] = q.w;
     }
-    const int nvalid = max(0, min(FI, cnt - o));
-    const int64_t g0 = base + o;
-    const int64_t pos = (nvalid > 0) ? (g0 % m) : 0;
-    const int mi = (int)min(m, (int64_t)FI + 1);                      // step between starts (capped)
-    const int nx0 = (int)min(pos == 0 ? (int64_t)0 : m - pos, (int64_t)FI + 1);  // first start in thread
-    bool has_start = false;
-    T acc = identity<OP, T>();
-    {
-        int nx = nx0;
-#pragma unroll
-        for (int k = 0; k < FI; ++k) {
-            if (k < nvalid) {
-                const T x = apply_map<F>(v[k]);
-                if (k == nx) {
-                    acc = combine<OP>(d, x);
-                    has_start = true;
-                    nx += mi;
-                } else {
-                    acc = combine<OP>(acc, x);
-                }
-                v[k] = acc;
-            }
-        }
-    }
+}
 
-    // ---- 3. CTA-wide exclusive segmented scan of (has_start, acc)
-    uint32_t fl = has_start ? 1u : 0u;
-    T sv = acc;
+template <typename T>
+__device__ __forceinline__ void store_items(T* buf, const T (&v)[FI]) {
+    using V = typename Vec4<T>::type;
+    const int o = threadIdx.x * FI;
+#pragma unroll
+    for (int c = 0; c < FI / 4; ++c) {
+        V q;
+        q.x = v[4 * c]; q.y = v[4 * c + 1]; q.z = v[4 * c + 2]; q.w = v[4 * c + 3];
+        *reinterpret_cast<V*>(&buf[o + 4 * c]) = q;
+    }
+}
+
+// CTA-wide exclusive scan of the thread aggregates (fl, sv) under the
+// segmented operator.  Returns the thread's exclusive prefix (exf, exv) and
+// the tile aggregate (aggf, aggv).  Contains one __syncthreads.
+template <typename T, int OP>
+__device__ __forceinline__ void cta_seg_scan(uint32_t fl, T sv, uint32_t& exf, T& exv, uint32_t& aggf, T& aggv,
+                                             T* s_wval, uint32_t* s_wflag) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
 #pragma unroll
     for (int off = 1; off < 32; off <<= 1) {
         const T ov = __shfl_up_sync(0xffffffffu, sv, off);
@@ -145,18 +151,17 @@ __global__ void __launch_bounds__(FB) flat_kernel(const T* in, T* out, int64_t N
         s_wval[w] = sv;
         s_wflag[w] = fl;
     }
-    T exv = __shfl_up_sync(0xffffffffu, sv, 1);
-    uint32_t exf = __shfl_up_sync(0xffffffffu, fl, 1);
+    exv = __shfl_up_sync(0xffffffffu, sv, 1);
+    exf = __shfl_up_sync(0xffffffffu, fl, 1);
     if (lane == 0) {
         exv = identity<OP, T>();
         exf = 0;
     }
     __syncthreads();
-    // prefix of the preceding warps, and the tile aggregate
     T pw = identity<OP, T>();
     uint32_t pf = 0;
-    T aggv = identity<OP, T>();
-    uint32_t aggf = 0;
+    aggv = identity<OP, T>();
+    aggf = 0;
 #pragma unroll
     for (int k = 0; k < FB / 32; ++k) {
         const T wv = s_wval[k];
@@ -168,134 +173,444 @@ __global__ void __launch_bounds__(FB) flat_kernel(const T* in, T* out, int64_t N
         aggv = wf ? wv : combine<OP>(aggv, wv);
         aggf |= wf;
     }
-    // thread exclusive = (warp prefix) . (in-warp exclusive)
     if (!exf) exv = combine<OP>(pw, exv);
     exf |= pf;
+}
 
-    // ---- 4. decoupled look-back (warp 0)
-    const bool tile_starts = (base % m) == 0;  // first element starts a segment
-    if (w == 0) {
-        T carry = identity<OP, T>();
-        if (tile == 0) {
-            if (lane == 0) st_release_u64(&status[0], pack_status(tag, ST_P, aggf, to_bits(aggv)));
-        } else {
-            if (lane == 0)
-                st_release_u64(&status[tile], pack_status(tag, aggf ? ST_P : ST_A, aggf, to_bits(aggv)));
-            if (!tile_starts || !aggf) {
-                int pred = tile - 1;
-                T run = identity<OP, T>();
-                while (true) {
-                    const int idx = pred - lane;
-                    uint64_t word = 0;
-                    if (idx >= 0) {
-                        do {
-                            word = ld_acquire_u64(&status[idx]);
-                        } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
-                    }
-                    const bool term = idx < 0 || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
-                    const uint32_t tm = __ballot_sync(0xffffffffu, term);
-                    const int stop = tm ? (__ffs(tm) - 1) : 31;
-                    T val = (lane <= stop && idx >= 0) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
-                    // ordered reduce: lane l+k is older than lane l
-#pragma unroll
-                    for (int off = 1; off < 32; off <<= 1) {
-                        const T older = __shfl_down_sync(0xffffffffu, val, off);
-                        if (lane + off < 32) val = combine<OP>(older, val);
-                    }
-                    val = __shfl_sync(0xffffffffu, val, 0);
-                    run = combine<OP>(val, run);
-                    if (tm) break;
-                    pred -= 32;
-                }
-                carry = run;
-                if (!aggf && lane == 0)
-                    st_release_u64(&status[tile], pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, aggv))));
+// ------------------------------------------------------------ ring helpers
+
+template <typename T>
+__device__ __forceinline__ void issue_tile_load(T* slot, const T* in, int tile, uint64_t* bar) {
+    mbar_arrive_expect_tx(bar, FT * sizeof(T));
+    bulk_g2s(slot, in + (int64_t)tile * FT, FT * sizeof(T), bar);
+}
+
+// Make tile data available in `slot`: wait for its TMA load (full tiles with
+// an aligned input) or copy it cooperatively.
+template <typename T>
+__device__ __forceinline__ void acquire_tile(T* slot, const T* in, const SlotMeta& sm, bool tma, uint64_t* bar,
+                                             uint32_t& phase_bits, int s) {
+    if (tma && sm.cnt == FT) {
+        mbar_wait(bar, (phase_bits >> s) & 1u);
+        phase_bits ^= 1u << s;
+    } else {
+        const int64_t base = (int64_t)sm.tile * FT;
+        for (int p = threadIdx.x; p < sm.cnt; p += FB) slot[p] = in[base + p];
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------ segred pass 1
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(FB, 2) flat_red_kernel(const T* in, T* out, int64_t N, int64_t m, T d, T* head,
+                                                         T* tail, int num_tiles, bool tma) {
+    extern __shared__ __align__(128) uint8_t smem_raw[];
+    T* ring = reinterpret_cast<T*>(smem_raw);
+    __shared__ alignas(8) uint64_t full[kSlots];
+    __shared__ SlotMeta meta[kSlots];
+    __shared__ T s_wval[FB / 32];
+    __shared__ uint32_t s_wflag[FB / 32];
+    const int t = threadIdx.x;
+    const int G = gridDim.x;
+    if (t == 0) {
+        for (int s = 0; s < kSlots; ++s) mbar_init(&full[s], 1);
+        fence_mbar_init();
+        for (int s = 0; s < kSlots; ++s) {
+            const int tile = blockIdx.x + s * G;
+            if (tile < num_tiles) {
+                fill_meta(meta[s], tile, N, m);
+                if (tma && meta[s].cnt == FT) issue_tile_load(ring + s * FT, in, tile, &full[s]);
+            } else {
+                meta[s].tile = num_tiles;
             }
         }
-        if (lane == 0) s_carry = carry;
     }
     __syncthreads();
-    const T carry_t = exf ? exv : combine<OP>(s_carry, exv);
-
-    // ---- 5. apply the carry to the elements before the thread's first start
-    {
-#pragma unroll
-        for (int k = 0; k < FI; ++k)
-            if (k < nx0 && k < nvalid) v[k] = combine<OP>(carry_t, v[k]);
-    }
-    if constexpr (SCAN) {
-        using V = typename Vec4<T>::type;
-#pragma unroll
-        for (int c = 0; c < FI / 4; ++c) {
-            V q;
-            q.x = v[4 * c]; q.y = v[4 * c + 1]; q.z = v[4 * c + 2]; q.w = v[4 * c + 3];
-            *reinterpret_cast<V*>(&buf[o + 4 * c]) = q;
+    uint32_t phase_bits = 0;
+    for (int i = 0;; ++i) {
+        const int s = i % kSlots;
+        const SlotMeta sm = meta[s];
+        if (sm.tile >= num_tiles) break;
+        T* buf = ring + s * FT;
+        acquire_tile(buf, in, sm, tma, &full[s], phase_bits, s);
+        const ThreadPos tp = thread_pos(sm, m);
+        T v[FI];
+        load_items(buf, v);
+        __syncthreads();  // slot s fully read: refill it right away
+        if (t == 0) {
+            const int nt = sm.tile + kSlots * G;
+            if (nt < num_tiles) {
+                fill_meta(meta[s], nt, N, m);
+                if (tma && meta[s].cnt == FT) issue_tile_load(buf, in, nt, &full[s]);
+            } else {
+                meta[s].tile = num_tiles;
+            }
         }
-        if (full && tma_out) {
-            fence_proxy_async_smem();
+        bool has_start = false, stash = false;
+        T acc, stash_v = identity<OP, T>();
+        if (tp.nx0 > tp.nvalid) {
+            // no boundary among this thread's items: plain reduction, 4 chains
+            T a4[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+#pragma unroll
+            for (int k = 0; k < FI; ++k)
+                if (k < tp.nvalid) a4[k & 3] = combine<OP>(a4[k & 3], apply_map<F>(v[k]));
+            acc = combine<OP>(combine<OP>(a4[0], a4[1]), combine<OP>(a4[2], a4[3]));
+        } else {
+            acc = identity<OP, T>();
+            int nx = tp.nx0;
+            int64_t sg = tp.seg;
+#pragma unroll
+            for (int k = 0; k < FI; ++k) {
+                if (k < tp.nvalid) {
+                    const T x = apply_map<F>(v[k]);
+                    if (k == nx) {
+                        acc = combine<OP>(d, x);
+                        has_start = true;
+                        nx += tp.mi;
+                    } else {
+                        acc = combine<OP>(acc, x);
+                    }
+                    if (k + 1 == nx) {  // item k ends segment sg
+                        if (k < tp.nx0) {
+                            stash = true;
+                            stash_v = acc;
+                        } else {
+                            out[sg] = acc;
+                        }
+                        ++sg;
+                    }
+                }
+            }
+        }
+        uint32_t exf, aggf;
+        T exv, aggv;
+        cta_seg_scan<T, OP>(has_start ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+        if (stash) {
+            const T val = combine<OP>(exv, stash_v);
+            if (exf) out[tp.seg] = val;  // began earlier in this tile: complete
+            else head[sm.tile] = val;    // began before this tile: head partial
+        }
+        if (t == 0) tail[sm.tile] = aggv;
+        __syncthreads();  // s_wval reuse
+    }
+}
+
+// Pass 2: finish every segment that crosses a tile boundary,
+//   out = tail[ta] (+) tail[ta+1..tb-1] (+) head[tb],   ta < tb.
+// m < FT: a crossing segment spans exactly two tiles; one thread per tile
+// boundary b (it is crossed iff b*FT is not a segment start).
+template <typename T, int OP>
+__global__ void __launch_bounds__(256) flat_red_fix_short(T* out, int64_t m, const T* head, const T* tail,
+                                                          int num_tiles) {
+    for (int b = 1 + blockIdx.x * blockDim.x + threadIdx.x; b < num_tiles; b += gridDim.x * blockDim.x) {
+        const uint32_t rem = (uint32_t)(((uint64_t)b * FT) % (uint64_t)m);
+        if (rem == 0) continue;
+        const int64_t seg = ((int64_t)b * FT) / m;
+        out[seg] = combine<OP>(tail[b - 1], head[b]);
+    }
+}
+
+// m >= FT: one CTA per segment; the middle range of whole-tile partials is
+// reduced with independent loads (8 in flight per thread) and a CTA tree.
+template <typename T, int OP>
+__global__ void __launch_bounds__(512) flat_red_fix_long(T* out, int64_t n, int64_t m, const T* head, const T* tail) {
+    __shared__ T red[16];
+    for (int64_t sgi = blockIdx.x; sgi < n; sgi += gridDim.x) {
+        const int ta = (int)((sgi * m) / FT);
+        const int tb = (int)(((sgi + 1) * m - 1) / FT);
+        if (ta == tb) continue;  // segment inside one tile: pass 1 wrote it
+        T a8[8];
+#pragma unroll
+        for (int q = 0; q < 8; ++q) a8[q] = identity<OP, T>();
+        const int stride = blockDim.x;
+        int u = ta + 1 + threadIdx.x;
+        for (; u + 7 * stride < tb; u += 8 * stride) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q) a8[q] = combine<OP>(a8[q], tail[u + q * stride]);
+        }
+        for (; u < tb; u += stride) a8[0] = combine<OP>(a8[0], tail[u]);
+        T acc = a8[0];
+#pragma unroll
+        for (int q = 1; q < 8; ++q) acc = combine<OP>(acc, a8[q]);
+        acc = warp_reduce<OP>(acc);
+        if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = acc;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            T r = tail[ta];
+            for (int k = 0; k < (int)(blockDim.x >> 5); ++k) r = combine<OP>(r, red[k]);
+            out[sgi] = combine<OP>(r, head[tb]);
+        }
+        __syncthreads();
+    }
+}
+
+// ------------------------------------------------------------------ segscan
+
+// Thread-local segmented inclusive scan of the thread's items (in registers).
+template <typename T, int OP, int F>
+__device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, T d, bool& has_start, T& acc) {
+    has_start = false;
+    acc = identity<OP, T>();
+    if (tp.nx0 > tp.nvalid) {  // no boundary: plain inclusive scan
+#pragma unroll
+        for (int k = 0; k < FI; ++k) {
+            acc = combine<OP>(acc, apply_map<F>(v[k]));
+            v[k] = acc;
+        }
+    } else {
+        int nx = tp.nx0;
+#pragma unroll
+        for (int k = 0; k < FI; ++k) {
+            if (k < tp.nvalid) {
+                const T x = apply_map<F>(v[k]);
+                if (k == nx) {
+                    acc = combine<OP>(d, x);
+                    has_start = true;
+                    nx += tp.mi;
+                } else {
+                    acc = combine<OP>(acc, x);
+                }
+                v[k] = acc;
+            }
+        }
+    }
+}
+
+// Chunked single-kernel reduce-then-scan.  Each persistent CTA claims one
+// contiguous chunk of tiles (the claim counter and the status epoch share one
+// 64-bit word; the last claimer re-arms both in a single atomic), then
+//   phase 1  streams its chunk through the TMA ring and folds the tile
+//            aggregates into the chunk aggregate (flag, value), published
+//            with a release store;
+//   look-back  reduces the aggregates of the preceding chunks, CTA-wide, up to
+//            the nearest one containing a segment start -- chunk aggregates are
+//            published after a single streaming pass, so nobody waits on a
+//            chain of inclusive prefixes;
+//   phase 3  streams the chunk again and scans it with the running carry; the
+//            TMA engine stores each finished tile from its ring slot.
+// The ring runs over the virtual sequence phase-1 tiles ++ phase-3 tiles, so
+// the first phase-3 loads are already in flight during the look-back.
+// Traffic: 2 reads + 1 write per element (12 B for f32) -- the price of not
+// serialising on look-back chains across ~10^4 tiles.
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
+                                                          uint8_t* ws, int num_tiles, int tiles_per_chunk,
+                                                          int num_chunks, bool tma_in, bool tma_out) {
+    extern __shared__ __align__(128) uint8_t smem_raw[];
+    T* ring = reinterpret_cast<T*>(smem_raw);
+    __shared__ alignas(8) uint64_t full[kSlots];
+    __shared__ SlotMeta meta[kSlots];
+    __shared__ int s_chunk;
+    __shared__ uint32_t s_tag;
+    __shared__ T s_wval[FB / 32];
+    __shared__ uint32_t s_wflag[FB / 32];
+    __shared__ int s_lbterm[FB / 32];
+    __shared__ T s_lbval[FB / 32];
+    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | chunk:32}
+    uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+
+    if (t == 0) {
+        const unsigned long long old = atomicAdd(ctr, 1ull);
+        s_chunk = (int)(uint32_t)old;
+        s_tag = (uint32_t)(old >> 32) & 0x1FFFFFFFu;
+        if (s_chunk == num_chunks - 1) atomicAdd(ctr, (1ull << 32) - (unsigned long long)num_chunks);
+        for (int q = 0; q < kSlots; ++q) mbar_init(&full[q], 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    const int chunk = s_chunk;
+    const uint32_t tag = s_tag;
+    const int t0 = chunk * tiles_per_chunk;
+    const int L = min(tiles_per_chunk, num_tiles - t0);
+    const int V = 2 * L;  // virtual sequence: phase 1 then phase 3
+    int next_w = 0;       // producer state (thread 0 only)
+    auto produce = [&](int wv) {  // thread 0: stage virtual index wv in slot wv % kSlots
+        const int sl = wv % kSlots;
+        const int tile = t0 + (wv < L ? wv : wv - L);
+        fill_meta(meta[sl], tile, N, m);
+        if (tma_in && meta[sl].cnt == FT) issue_tile_load(ring + sl * FT, in, tile, &full[sl]);
+    };
+    if (t == 0)
+        for (; next_w < min(kSlots, V); ++next_w) produce(next_w);
+    __syncthreads();
+    uint32_t phase_bits = 0;
+
+    // ---- phase 1: chunk aggregate
+    uint32_t run_f = 0;
+    T run_v = identity<OP, T>();
+    for (int vi = 0; vi < L; ++vi) {
+        const int sl = vi % kSlots;
+        const SlotMeta sm = meta[sl];
+        T* buf = ring + sl * FT;
+        acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
+        const ThreadPos tp = thread_pos(sm, m);
+        T v[FI];
+        load_items(buf, v);
+        __syncthreads();  // slot read by everyone: refill it
+        if (t == 0 && next_w < V && next_w == vi + kSlots) produce(next_w++);
+        bool hs;
+        T acc;
+        local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
+        uint32_t exf, aggf;
+        T exv, aggv;
+        cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+        run_v = aggf ? aggv : combine<OP>(run_v, aggv);
+        run_f |= aggf;
+        __syncthreads();  // s_wval reuse
+    }
+    if (t == 0) st_release_u64(&status[chunk], pack_status(tag, ST_A, run_f, to_bits(run_v)));
+
+    // ---- look-back over preceding chunk aggregates (CTA-wide windows)
+    T carry = identity<OP, T>();
+    if (chunk > 0 && ((int64_t)t0 * FT) % m != 0) {
+        int pred = chunk - 1;
+        while (true) {
+            const int idx = pred - t;
+            uint64_t word = 0;
+            if (idx >= 0) {
+                do {
+                    word = ld_acquire_u64(&status[idx]);
+                } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
+            }
+            const bool term = idx < 0 || ((word >> 32) & 1u);
+            const uint32_t tb = __ballot_sync(0xffffffffu, term);
+            if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
             __syncthreads();
+            int stop = FB;
+#pragma unroll
+            for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
+            T val = (t <= stop && idx >= 0) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
+#pragma unroll
+            for (int off = 1; off < 32; off <<= 1) {  // ordered: higher lane = older chunk
+                const T older = __shfl_down_sync(0xffffffffu, val, off);
+                if (lane + off < 32) val = combine<OP>(older, val);
+            }
+            if (lane == 0) s_lbval[w] = val;
+            __syncthreads();
+            T win = identity<OP, T>();
+#pragma unroll
+            for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
+            carry = combine<OP>(win, carry);
+            __syncthreads();
+            if (stop < FB) break;
+            pred -= FB;
+        }
+    }
+
+    // ---- phase 3: scan the chunk with the running carry
+    for (int vi = L; vi < V; ++vi) {
+        const int sl = vi % kSlots;
+        const SlotMeta sm = meta[sl];
+        T* buf = ring + sl * FT;
+        const int64_t base = (int64_t)sm.tile * FT;
+        acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
+        const ThreadPos tp = thread_pos(sm, m);
+        T v[FI];
+        load_items(buf, v);
+        bool hs;
+        T acc;
+        local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
+        uint32_t exf, aggf;
+        T exv, aggv;
+        cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+        {
+            const T carry_t = exf ? exv : combine<OP>(carry, exv);
+            const int lim = min(tp.nx0, tp.nvalid);
+#pragma unroll
+            for (int k = 0; k < FI; ++k)
+                if (k < lim) v[k] = combine<OP>(carry_t, v[k]);
+        }
+        carry = aggf ? aggv : combine<OP>(carry, aggv);
+        store_items(buf, v);
+        const bool bulk = tma_out && sm.cnt == FT;
+        if (bulk) fence_proxy_async_smem();
+        __syncthreads();
+        if (bulk) {
             if (t == 0) {
                 bulk_s2g(out + base, buf, FT * sizeof(T));
                 bulk_commit();
-                bulk_wait_read0();
             }
         } else {
-            __syncthreads();
-            for (int p = t; p < cnt; p += FB) out[base + p] = buf[p];
+            for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
         }
-    } else {
-        // segment ends: global index g with (g + 1) % m == 0
-        if (nvalid > 0) {
-            int64_t seg = g0 / m;
-            int nx = nx0;
-#pragma unroll
-            for (int k = 0; k < FI; ++k) {
-                if (k < nvalid) {
-                    if (k == nx) {
-                        nx += mi;
-                    }
-                    if (k + 1 == nx) {
-                        // the element ends segment `seg` (segment that contains g0 + k)
-                        out[seg] = v[k];
-                        ++seg;
-                    }
-                }
-            }
+        // refill the slot of the previous iteration once its store has read smem
+        if (t == 0 && next_w < V && next_w == vi - 1 + kSlots) {
+            if (bulk) bulk_wait_read1();
+            else bulk_wait_read0();
+            produce(next_w++);
         }
+        __syncthreads();
     }
+    if (t == 0) bulk_wait0();
+}
 
-    // ---- completion: the last CTA re-arms the workspace for the next call
-    __syncthreads();
-    if (t == 0) {
-        __threadfence();
-        const uint32_t old = atomicAdd(&hdr->done_ctr, 1u);
-        if (old == (uint32_t)num_tiles - 1) {
-            hdr->tile_ctr = 0;
-            hdr->done_ctr = 0;
-            hdr->epoch = hdr->epoch + 1;
-            __threadfence();
-        }
+// ------------------------------------------------------------------ launch
+
+static int sm_count() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
     }
+    return n;
+}
+
+template <typename K>
+static int resident_ctas(K kernel, size_t smem) {
+    static thread_local std::unordered_map<const void*, int> cache;
+    auto it = cache.find((const void*)kernel);
+    if (it != cache.end()) return it->second;
+    cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, FB, smem);
+    if (per_sm < 1) per_sm = 1;
+    const int n = per_sm * sm_count();
+    cache[(const void*)kernel] = n;
+    return n;
 }
 
 cudaError_t launch_flat(const SegArgs& a, bool scan) {
     const int64_t N = a.n * a.m;
     const int64_t tiles = ceil_div(N, kFlatTile);
-    if (tiles > 0x7fffffffLL) return cudaErrorInvalidValue;
+    if (tiles > 0x3fffffffLL) return cudaErrorInvalidValue;
     const bool tma_in = ((uintptr_t)a.in % 16) == 0;
     const bool tma_out = ((uintptr_t)a.out % 16) == 0;
+    const size_t smem = (size_t)kSlots * FT * 4;
+    uint8_t* ws = (uint8_t*)a.ws;
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
-        if (scan)
-            flat_kernel<T, OP, F, true><<<(unsigned)tiles, FB, 0, a.stream>>>(
-                (const T*)a.in, (T*)a.out, N, a.m, bits_to<T>(a.ne_bits), (uint8_t*)a.ws, (int)tiles, tma_in,
-                tma_out);
-        else
-            flat_kernel<T, OP, F, false><<<(unsigned)tiles, FB, 0, a.stream>>>(
-                (const T*)a.in, (T*)a.out, N, a.m, bits_to<T>(a.ne_bits), (uint8_t*)a.ws, (int)tiles, tma_in,
-                tma_out);
-        return cudaGetLastError();
+        const T d = bits_to<T>(a.ne_bits);
+        if (scan) {
+            auto k = flat_scan_kernel<T, OP, F>;
+            const int64_t g = std::min<int64_t>(tiles, resident_ctas(k, smem));
+            const int per = (int)ceil_div(tiles, g);
+            const int chunks = (int)ceil_div(tiles, per);
+            k<<<chunks, FB, smem, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, per, chunks, tma_in,
+                                              tma_out);
+            return cudaGetLastError();
+        }
+        T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
+        T* tail = head + tiles;
+        auto k = flat_red_kernel<T, OP, F>;
+        const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem));
+        k<<<grid, FB, smem, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, head, tail, (int)tiles, tma_in);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+        if (a.m > FT) {
+            const int g2 = (int)std::min<int64_t>(a.n, (int64_t)sm_count() * 4);
+            flat_red_fix_long<T, OP><<<g2, 512, 0, a.stream>>>((T*)a.out, a.n, a.m, head, tail);
+            e = cudaGetLastError();
+        } else if (FT % a.m != 0 && tiles > 1) {
+            const int g2 = (int)std::min<int64_t>(ceil_div(tiles, 256), (int64_t)sm_count() * 4);
+            flat_red_fix_short<T, OP><<<g2, 256, 0, a.stream>>>((T*)a.out, a.m, head, tail, (int)tiles);
+            e = cudaGetLastError();
+        }
+        return e;
     });
 }
 

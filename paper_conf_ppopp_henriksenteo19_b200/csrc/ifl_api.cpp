@@ -132,7 +132,7 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
     return x < y + bn && y < x + an;
 }
 
-int validate_seg(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, int version,
+int validate_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, int version,
                  const char* what) {
     if (n < 0 || m < 0) return fail(IFL_EINVAL, "%s: negative size n=%lld m=%lld", what, (long long)n, (long long)m);
     if (mul_overflows(n, m) || mul_overflows(n * m, 4))
@@ -143,7 +143,7 @@ int validate_seg(const void* in, void* out, int64_t n, int64_t m, int dt, int op
     if (f < IFL_F_ID || f > IFL_F_ABS) return fail(IFL_EINVAL, "%s: bad map %d", what, f);
     if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "%s: bad version %d", what, version);
     if (n > 0 && m > 0 && in == nullptr) return fail(IFL_EINVAL, "%s: in is NULL", what);
-    if (n > 0 && out == nullptr) return fail(IFL_EINVAL, "%s: out is NULL", what);
+    if ((scan ? n * m : n) > 0 && out == nullptr) return fail(IFL_EINVAL, "%s: out is NULL", what);
     if (((uintptr_t)in % 4) || ((uintptr_t)out % 4)) return fail(IFL_EINVAL, "%s: pointers not element-aligned", what);
     return IFL_OK;
 }
@@ -262,7 +262,7 @@ int ifl_workspace_init(void* ws, size_t ws_bytes, void* stream) {
 static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f,
                    const void* ne, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
     const char* what = scan ? "ifl_segscan" : "ifl_segred";
-    int rc = validate_seg(in, out, n, m, dt, op, f, version, what);
+    int rc = validate_seg(scan, in, out, n, m, dt, op, f, version, what);
     if (rc) return rc;
     const size_t ob = (size_t)(scan ? n * m : n) * 4, ib = (size_t)(n * m) * 4;
     if (scan) {

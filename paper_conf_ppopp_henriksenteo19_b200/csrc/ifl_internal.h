@@ -22,7 +22,7 @@ struct SegArgs {
 // Flat engine tile geometry (flat.cu).  ws layout: 256-byte header then one
 // 64-bit status word per tile.
 constexpr int kFlatThreads = 256;
-constexpr int kFlatItems = 28;
+constexpr int kFlatItems = 20;
 constexpr int64_t kFlatTile = (int64_t)kFlatThreads * kFlatItems;
 size_t flat_ws_bytes(int64_t total_elems);
 

@@ -21,16 +21,21 @@ namespace ifl {
 
 // ------------------------------------------------------------------ V_TOP
 
-constexpr int kTopRows = 256;  // threads = segments per CTA
-constexpr int kTopKT = 32;     // columns per smem tile (128 B of f32 per row)
-constexpr int kTopWords = kTopRows * kTopKT + kTopRows * kTopKT / 32;
+constexpr int kTopThreads = 256;  // threads per CTA
+constexpr int kTopKT = 32;        // columns per smem tile (128 B of f32 per row)
+constexpr int kTopElems = kTopThreads * kTopKT;          // 8192 staged elements
+constexpr int kTopWords = kTopElems + kTopElems / 32;    // + one pad word per 32
 
 __device__ __forceinline__ int padq(int q) { return q + (q >> 5); }
 
-// Stage the CTA's tile into shared memory.  Whole-row mode (m <= 32): the
-// region [r0*m, (r0+rows)*m) is contiguous and copied linearly.  Column-tile
-// mode: columns [k0, k0+kt) of `rows` rows.  Padded index padq(q) with
-// q = row*KT + col (KT = m in whole-row mode, 32 otherwise).
+// Rows per thread in whole-row mode (m <= 32): rpt rows of m elements each,
+// so a CTA stages 256*rpt*m <= 8192 contiguous elements.
+__host__ __device__ __forceinline__ int top_rpt(int64_t m) { return m <= kTopKT ? (int)(kTopKT / m) : 1; }
+
+// Stage the CTA's tile into shared memory.  Whole-row mode: the region
+// [r0*m, (r0+rows)*m) is contiguous and copied linearly.  Column-tile mode:
+// columns [k0, k0+kt) of `rows` rows.  Padded index padq(q), q = row*KT + col
+// (KT = m in whole-row mode, 32 otherwise): walking a row is conflict-free.
 template <typename T>
 __device__ __forceinline__ void top_load_tile(T* tile, const T* __restrict__ in, int64_t r0, int rows,
                                               int64_t m, int64_t k0, int kt, bool whole, bool vec) {
@@ -42,28 +47,26 @@ __device__ __forceinline__ void top_load_tile(T* tile, const T* __restrict__ in,
         int p0 = 0;
         if (vec) {
             const int nv = cnt >> 2;
-            for (int v = t; v < nv; v += kTopRows) {
-                V q = ldg_stream4(src + 4 * v);
+            for (int v = t; v < nv; v += kTopThreads) {
                 T e[4];
-                unpack4<T>(q, e);
+                unpack4<T>(ldg_stream4(src + 4 * v), e);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) tile[padq(4 * v + u)] = e[u];
             }
             p0 = nv << 2;
         }
-        for (int p = p0 + t; p < cnt; p += kTopRows) tile[padq(p)] = ldg1(src + p);
+        for (int p = p0 + t; p < cnt; p += kTopThreads) tile[padq(p)] = ldg1(src + p);
     } else if (vec && kt == kTopKT) {
         // rows x 8 float4 per tile; a warp covers 4 rows x 128 B per load.
-        for (int v = t; v < rows * 8; v += kTopRows) {
+        for (int v = t; v < rows * 8; v += kTopThreads) {
             const int row = v >> 3, c4 = v & 7;
-            V q = ldg_stream4(in + (r0 + row) * m + k0 + 4 * c4);
             T e[4];
-            unpack4<T>(q, e);
+            unpack4<T>(ldg_stream4(in + (r0 + row) * m + k0 + 4 * c4), e);
 #pragma unroll
             for (int u = 0; u < 4; ++u) tile[padq(row * kTopKT + 4 * c4 + u)] = e[u];
         }
     } else {
-        for (int p = t; p < rows * kTopKT; p += kTopRows) {
+        for (int p = t; p < rows * kTopKT; p += kTopThreads) {
             const int row = p >> 5, col = p & 31;
             if (col < kt) tile[padq(p)] = ldg1(in + (r0 + row) * m + k0 + col);
         }
@@ -71,42 +74,69 @@ __device__ __forceinline__ void top_load_tile(T* tile, const T* __restrict__ in,
 }
 
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kTopRows) segred_top_kernel(const T* __restrict__ in, T* __restrict__ out,
-                                                              int64_t n, int64_t m, T d, bool vec) {
+__global__ void __launch_bounds__(kTopThreads) segred_top_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                                 int64_t n, int64_t m, T d, bool vec) {
     __shared__ T tile[kTopWords];
     const int t = threadIdx.x;
-    const int64_t r0 = (int64_t)blockIdx.x * kTopRows;
-    const int rows = (int)min((int64_t)kTopRows, n - r0);
-    T acc[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
-    if (m <= kTopKT) {
-        top_load_tile(tile, in, r0, rows, m, 0, (int)m, true, vec);
-        __syncthreads();
-        if (t < rows) {
-            const int mm = (int)m;
-            for (int k = 0; k < mm; ++k) acc[k & 3] = combine<OP>(acc[k & 3], apply_map<F>(tile[padq(t * mm + k)]));
-        }
-    } else {
-        for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
-            const int kt = (int)min((int64_t)kTopKT, m - k0);
-            top_load_tile(tile, in, r0, rows, m, k0, kt, false, vec);
+    const int rpt = top_rpt(m);
+    const int64_t rows_blk = (int64_t)kTopThreads * rpt;
+    const int64_t nblk = ceil_div(n, rows_blk);
+    for (int64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
+        const int64_t r0 = b * rows_blk;
+        const int rows = (int)min(rows_blk, n - r0);
+        if (m <= kTopKT) {
+            top_load_tile(tile, in, r0, rows, m, 0, (int)m, true, vec);
             __syncthreads();
-            if (t < rows) {
-                if (kt == kTopKT) {
-#pragma unroll
-                    for (int k = 0; k < kTopKT; ++k)
-                        acc[k & 3] = combine<OP>(acc[k & 3], apply_map<F>(tile[padq(t * kTopKT + k)]));
-                } else {
-                    for (int k = 0; k < kt; ++k)
-                        acc[k & 3] = combine<OP>(acc[k & 3], apply_map<F>(tile[padq(t * kTopKT + k)]));
+            const int mm = (int)m;
+            for (int j = 0; j < rpt; ++j) {
+                const int r = t + j * kTopThreads;
+                if (r < rows) {
+                    Acc<OP, T> a(d);
+                    for (int k = 0; k < mm; ++k) a.add(apply_map<F>(tile[padq(r * mm + k)]));
+                    out[r0 + r] = a.get();
                 }
             }
             __syncthreads();
+        } else {
+            Acc<OP, T> a0(d), a1(identity<OP, T>()), a2(identity<OP, T>()), a3(identity<OP, T>());
+            for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
+                const int kt = (int)min((int64_t)kTopKT, m - k0);
+                top_load_tile(tile, in, r0, rows, m, k0, kt, false, vec);
+                __syncthreads();
+                if (t < rows) {
+                    if (kt == kTopKT) {
+#pragma unroll
+                        for (int k = 0; k < kTopKT; k += 4) {
+                            a0.add(apply_map<F>(tile[padq(t * kTopKT + k)]));
+                            a1.add(apply_map<F>(tile[padq(t * kTopKT + k + 1)]));
+                            a2.add(apply_map<F>(tile[padq(t * kTopKT + k + 2)]));
+                            a3.add(apply_map<F>(tile[padq(t * kTopKT + k + 3)]));
+                        }
+                    } else {
+                        for (int k = 0; k < kt; ++k) a0.add(apply_map<F>(tile[padq(t * kTopKT + k)]));
+                    }
+                }
+                __syncthreads();
+            }
+            if (t < rows) {
+                a0.add(a1.get());
+                a2.add(a3.get());
+                a0.add(a2.get());
+                out[r0 + t] = a0.get();
+            }
         }
     }
-    if (t < rows) {
-        T r = combine<OP>(combine<OP>(acc[0], acc[1]), combine<OP>(acc[2], acc[3]));
-        out[r0 + t] = combine<OP>(d, r);
+}
+
+static int top_grid(int64_t nblk) {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
     }
+    return (int)min(nblk, (int64_t)sms * 6);
 }
 
 cudaError_t launch_segred_top(const SegArgs& a) {
@@ -114,8 +144,8 @@ cudaError_t launch_segred_top(const SegArgs& a) {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && (a.m <= kTopKT || a.m % 4 == 0);
-        const int64_t grid = ceil_div(a.n, kTopRows);
-        segred_top_kernel<T, OP, F><<<(unsigned)grid, kTopRows, 0, a.stream>>>(
+        const int64_t nblk = ceil_div(a.n, (int64_t)kTopThreads * top_rpt(a.m));
+        segred_top_kernel<T, OP, F><<<top_grid(nblk), kTopThreads, 0, a.stream>>>(
             (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
         return cudaGetLastError();
     });

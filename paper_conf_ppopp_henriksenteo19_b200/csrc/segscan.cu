@@ -18,14 +18,16 @@
 
 namespace ifl {
 
-constexpr int kTopRows = 256;
+constexpr int kTopThreads = 256;
 constexpr int kTopKT = 32;
-constexpr int kTopWords = kTopRows * kTopKT + kTopRows * kTopKT / 32;
+constexpr int kTopElems = kTopThreads * kTopKT;
+constexpr int kTopWords = kTopElems + kTopElems / 32;
 
 __device__ __forceinline__ int spadq(int q) { return q + (q >> 5); }
+__host__ __device__ __forceinline__ int stop_rpt(int64_t m) { return m <= kTopKT ? (int)(kTopKT / m) : 1; }
 
-// Copy between a global [rows][kt] window and the padded smem tile.  LOAD:
-// global -> smem (applying nothing); STORE: smem -> global.
+// Copy between a global window and the padded smem tile (see segred.cu).
+// LOAD: global -> smem; STORE: smem -> global.
 template <bool LOAD, typename T>
 __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* __restrict__ out, int64_t r0,
                                          int rows, int64_t m, int64_t k0, int kt, bool whole, bool vec) {
@@ -36,7 +38,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
         int p0 = 0;
         if (vec) {
             const int nv = cnt >> 2;
-            for (int v = t; v < nv; v += kTopRows) {
+            for (int v = t; v < nv; v += kTopThreads) {
                 if (LOAD) {
                     T e[4];
                     unpack4<T>(ldg_stream4(in + r0 * m + 4 * v), e);
@@ -53,12 +55,12 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
             }
             p0 = nv << 2;
         }
-        for (int p = p0 + t; p < cnt; p += kTopRows) {
+        for (int p = p0 + t; p < cnt; p += kTopThreads) {
             if (LOAD) tile[spadq(p)] = ldg1(in + r0 * m + p);
             else out[r0 * m + p] = tile[spadq(p)];
         }
     } else if (vec && kt == kTopKT) {
-        for (int v = t; v < rows * 8; v += kTopRows) {
+        for (int v = t; v < rows * 8; v += kTopThreads) {
             const int row = v >> 3, c4 = v & 7;
             const int64_t gi = (r0 + row) * m + k0 + 4 * c4;
             const int q0 = row * kTopKT + 4 * c4;
@@ -77,7 +79,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
             }
         }
     } else {
-        for (int p = t; p < rows * kTopKT; p += kTopRows) {
+        for (int p = t; p < rows * kTopKT; p += kTopThreads) {
             const int row = p >> 5, col = p & 31;
             if (col < kt) {
                 const int64_t gi = (r0 + row) * m + k0 + col;
@@ -89,49 +91,70 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
 }
 
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kTopRows) segscan_top_kernel(const T* in, T* out, int64_t n, int64_t m, T d,
-                                                               bool vec) {
+__global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T* out, int64_t n, int64_t m, T d,
+                                                                  bool vec) {
     __shared__ T tile[kTopWords];
     const int t = threadIdx.x;
-    const int64_t r0 = (int64_t)blockIdx.x * kTopRows;
-    const int rows = (int)min((int64_t)kTopRows, n - r0);
-    T acc = d;  // d (+) f(x0) (+) ... : d applied once, at the row start
-    if (m <= kTopKT) {
-        top_xfer<true>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
-        __syncthreads();
-        if (t < rows) {
-            const int mm = (int)m;
-            for (int k = 0; k < mm; ++k) {
-                acc = combine<OP>(acc, apply_map<F>(tile[spadq(t * mm + k)]));
-                tile[spadq(t * mm + k)] = acc;
-            }
-        }
-        __syncthreads();
-        top_xfer<false>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
-    } else {
-        for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
-            const int kt = (int)min((int64_t)kTopKT, m - k0);
-            top_xfer<true>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+    const int rpt = stop_rpt(m);
+    const int64_t rows_blk = (int64_t)kTopThreads * rpt;
+    const int64_t nblk = ceil_div(n, rows_blk);
+    for (int64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
+        const int64_t r0 = b * rows_blk;
+        const int rows = (int)min(rows_blk, n - r0);
+        if (m <= kTopKT) {
+            top_xfer<true>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
             __syncthreads();
-            if (t < rows) {
-                if (kt == kTopKT) {
-#pragma unroll
-                    for (int k = 0; k < kTopKT; ++k) {
-                        acc = combine<OP>(acc, apply_map<F>(tile[spadq(t * kTopKT + k)]));
-                        tile[spadq(t * kTopKT + k)] = acc;
-                    }
-                } else {
-                    for (int k = 0; k < kt; ++k) {
-                        acc = combine<OP>(acc, apply_map<F>(tile[spadq(t * kTopKT + k)]));
-                        tile[spadq(t * kTopKT + k)] = acc;
+            const int mm = (int)m;
+            for (int j = 0; j < rpt; ++j) {
+                const int r = t + j * kTopThreads;
+                if (r < rows) {
+                    Acc<OP, T> a(d);  // d (+) f(x0) (+) ...: d applied once, at the row start
+                    for (int k = 0; k < mm; ++k) {
+                        a.add(apply_map<F>(tile[spadq(r * mm + k)]));
+                        tile[spadq(r * mm + k)] = a.get();
                     }
                 }
             }
             __syncthreads();
-            top_xfer<false>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+            top_xfer<false>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
             __syncthreads();
+        } else {
+            Acc<OP, T> a(d);
+            for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
+                const int kt = (int)min((int64_t)kTopKT, m - k0);
+                top_xfer<true>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+                __syncthreads();
+                if (t < rows) {
+                    if (kt == kTopKT) {
+#pragma unroll
+                        for (int k = 0; k < kTopKT; ++k) {
+                            a.add(apply_map<F>(tile[spadq(t * kTopKT + k)]));
+                            tile[spadq(t * kTopKT + k)] = a.get();
+                        }
+                    } else {
+                        for (int k = 0; k < kt; ++k) {
+                            a.add(apply_map<F>(tile[spadq(t * kTopKT + k)]));
+                            tile[spadq(t * kTopKT + k)] = a.get();
+                        }
+                    }
+                }
+                __syncthreads();
+                top_xfer<false>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+                __syncthreads();
+            }
         }
     }
+}
+
+static int stop_grid(int64_t nblk) {
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    return (int)min(nblk, (int64_t)sms * 6);
 }
 
 cudaError_t launch_segscan_top(const SegArgs& a) {
@@ -140,8 +163,8 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) &&
                          (a.m <= kTopKT || a.m % 4 == 0);
-        const int64_t grid = ceil_div(a.n, kTopRows);
-        segscan_top_kernel<T, OP, F><<<(unsigned)grid, kTopRows, 0, a.stream>>>(
+        const int64_t nblk = ceil_div(a.n, (int64_t)kTopThreads * stop_rpt(a.m));
+        segscan_top_kernel<T, OP, F><<<stop_grid(nblk), kTopThreads, 0, a.stream>>>(
             (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
         return cudaGetLastError();
     });

@@ -1,0 +1,29 @@
+"""Run one (op, version, n, m) configuration a few times -- a small target
+for `ncu -k regex:... --set full` (not part of the product)."""
+import argparse
+import sys
+
+import torch
+
+sys.path.insert(0, ".")
+import ifl_inputs as gen  # noqa: E402
+import paper_conf_ppopp_henriksenteo19_b200 as ifl  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--op", default="segred")
+ap.add_argument("--version", default="flat")
+ap.add_argument("--n", type=int, default=1)
+ap.add_argument("--m", type=int, default=1 << 26)
+ap.add_argument("--reps", type=int, default=3)
+a = ap.parse_args()
+x = gen.generate("F32_UNIT", 2, a.n * a.m, device="cuda").view(a.n, a.m)
+fn = ifl.segred if a.op == "segred" else ifl.segscan
+for _ in range(a.reps):
+    fn(x, version=a.version)
+torch.cuda.synchronize()
+e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+e0.record()
+fn(x, version=a.version)
+e1.record()
+torch.cuda.synchronize()
+print(f"{a.op} {a.version} n={a.n} m={a.m}: {e0.elapsed_time(e1)*1e3:.1f} us")
