@@ -377,173 +377,239 @@ __device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, 
     }
 }
 
-// Chunked single-kernel reduce-then-scan.  Each persistent CTA claims one
-// contiguous chunk of tiles (the claim counter and the status epoch share one
-// 64-bit word; the last claimer re-arms both in a single atomic), then
-//   phase 1  streams its chunk through the TMA ring and folds the tile
-//            aggregates into the chunk aggregate (flag, value), published
-//            with a release store;
-//   look-back  reduces the aggregates of the preceding chunks, CTA-wide, up to
-//            the nearest one containing a segment start -- chunk aggregates are
-//            published after a single streaming pass, so nobody waits on a
-//            chain of inclusive prefixes;
-//   phase 3  streams the chunk again and scans it with the running carry; the
-//            TMA engine stores each finished tile from its ring slot.
-// The ring runs over the virtual sequence phase-1 tiles ++ phase-3 tiles, so
-// the first phase-3 loads are already in flight during the look-back.
-// Traffic: 2 reads + 1 write per element (12 B for f32) -- the price of not
-// serialising on look-back chains across ~10^4 tiles.
+// L2-blocked two-phase segscan.  Persistent CTAs, co-resident by cooperative
+// launch, own chunks of kChunkTiles consecutive tiles statically
+// (chunk c = round * grid + blockIdx).  Per chunk:
+//   phase 1  (only if the next chunk continues a segment into it) stream the
+//            chunk through the TMA ring with an L2 evict_last policy and fold
+//            the tile aggregates into the chunk aggregate; publish it;
+//   look-back (only if the chunk does not begin a segment) over the chunk
+//            aggregates, CTA-wide, to the nearest inclusive prefix or chunk
+//            containing a segment start -- that is at most one round back,
+//            and the previous round's prefixes are long final;
+//   phase 3  stream the chunk again (evict_first: the round, ~48 MB, is still
+//            in the 126 MB L2, so DRAM sees one read and one write per
+//            element), scan with the running carry, and store each tile from
+//            its ring slot with the TMA engine (evict_first).
+// The ring runs over the CTA's whole virtual item sequence, so loads for the
+// next phase / chunk are in flight during the look-back and the scans.
+// Status words carry an epoch tag; the last CTA to finish bumps the epoch
+// (one 64-bit {epoch | done} word), so no per-call memset is needed.
+constexpr int kChunkTiles = 8;
+
+struct ScanItem {
+    int chunk, j, phase;  // phase 1 = aggregate pass, 3 = scan pass
+};
+
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
-                                                          uint8_t* ws, int num_tiles, int tiles_per_chunk,
-                                                          int num_chunks, bool tma_in, bool tma_out) {
+                                                          uint8_t* ws, int num_tiles, int num_chunks, bool tma_in,
+                                                          bool tma_out) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
     __shared__ alignas(8) uint64_t full[kSlots];
     __shared__ SlotMeta meta[kSlots];
-    __shared__ int s_chunk;
     __shared__ uint32_t s_tag;
     __shared__ T s_wval[FB / 32];
     __shared__ uint32_t s_wflag[FB / 32];
     __shared__ int s_lbterm[FB / 32];
     __shared__ T s_lbval[FB / 32];
-    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | chunk:32}
+    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | done:32}
     uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int G = gridDim.x;
+    const int64_t chunk_elems = (int64_t)kChunkTiles * FT;
+    // chunk c needs its predecessors' carry / its successor needs c's aggregate
+    auto need_carry = [&](int c) { return c > 0 && ((int64_t)c * chunk_elems) % m != 0; };
+    auto need_agg = [&](int c) { return need_carry(c + 1) && c + 1 < num_chunks; };
+    auto chunk_tiles = [&](int c) { return min(kChunkTiles, num_tiles - c * kChunkTiles); };
+
+    // producer state (thread 0): walks chunk by chunk, phase 1 (if needed) then 3
+    int p_chunk = blockIdx.x, p_phase = 0, p_j = 0;
+    auto p_norm = [&]() {  // settle (p_chunk, p_phase, p_j) on a valid item or past the end
+        while (p_chunk < num_chunks) {
+            if (p_phase == 0) {
+                p_phase = need_agg(p_chunk) ? 1 : 3;
+                p_j = 0;
+            }
+            if (p_j < chunk_tiles(p_chunk)) return;
+            if (p_phase == 1) {
+                p_phase = 3;
+                p_j = 0;
+            } else {
+                p_chunk += G;
+                p_phase = 0;
+            }
+        }
+    };
+    uint32_t free_mask = (1u << kSlots) - 1;
+    int next_slot = 0, pend_slot = -1;
+    uint64_t pol_keep = 0, pol_stream = 0;
+    auto produce_all = [&]() {  // thread 0: fill every free slot, in sequence order
+        p_norm();
+        while (p_chunk < num_chunks && ((free_mask >> next_slot) & 1u)) {
+            free_mask &= ~(1u << next_slot);
+            const int tile = p_chunk * kChunkTiles + p_j;
+            SlotMeta& sm = meta[next_slot];
+            fill_meta(sm, tile, N, m);
+            if (tma_in && sm.cnt == FT) {
+                T* dst = ring + next_slot * FT;
+                mbar_arrive_expect_tx(&full[next_slot], FT * sizeof(T));
+                bulk_g2s_hint(dst, in + (int64_t)tile * FT, FT * sizeof(T), &full[next_slot],
+                              p_phase == 1 ? pol_keep : pol_stream);
+            }
+            next_slot = (next_slot + 1) % kSlots;
+            ++p_j;
+            p_norm();
+        }
+    };
 
     if (t == 0) {
-        const unsigned long long old = atomicAdd(ctr, 1ull);
-        s_chunk = (int)(uint32_t)old;
-        s_tag = (uint32_t)(old >> 32) & 0x1FFFFFFFu;
-        if (s_chunk == num_chunks - 1) atomicAdd(ctr, (1ull << 32) - (unsigned long long)num_chunks);
+        s_tag = (uint32_t)(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)) >> 32) & 0x1FFFFFFFu;
+        pol_keep = policy_evict_last();
+        pol_stream = policy_evict_first();
         for (int q = 0; q < kSlots; ++q) mbar_init(&full[q], 1);
         fence_mbar_init();
+        produce_all();
     }
     __syncthreads();
-    const int chunk = s_chunk;
     const uint32_t tag = s_tag;
-    const int t0 = chunk * tiles_per_chunk;
-    const int L = min(tiles_per_chunk, num_tiles - t0);
-    const int V = 2 * L;  // virtual sequence: phase 1 then phase 3
-    int next_w = 0;       // producer state (thread 0 only)
-    auto produce = [&](int wv) {  // thread 0: stage virtual index wv in slot wv % kSlots
-        const int sl = wv % kSlots;
-        const int tile = t0 + (wv < L ? wv : wv - L);
-        fill_meta(meta[sl], tile, N, m);
-        if (tma_in && meta[sl].cnt == FT) issue_tile_load(ring + sl * FT, in, tile, &full[sl]);
-    };
-    if (t == 0)
-        for (; next_w < min(kSlots, V); ++next_w) produce(next_w);
-    __syncthreads();
     uint32_t phase_bits = 0;
+    int vi = 0;  // consumer position in the virtual sequence
 
-    // ---- phase 1: chunk aggregate
-    uint32_t run_f = 0;
-    T run_v = identity<OP, T>();
-    for (int vi = 0; vi < L; ++vi) {
-        const int sl = vi % kSlots;
-        const SlotMeta sm = meta[sl];
-        T* buf = ring + sl * FT;
-        acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
-        const ThreadPos tp = thread_pos(sm, m);
-        T v[FI];
-        load_items(buf, v);
-        __syncthreads();  // slot read by everyone: refill it
-        if (t == 0 && next_w < V && next_w == vi + kSlots) produce(next_w++);
-        bool hs;
-        T acc;
-        local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
-        uint32_t exf, aggf;
-        T exv, aggv;
-        cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
-        run_v = aggf ? aggv : combine<OP>(run_v, aggv);
-        run_f |= aggf;
-        __syncthreads();  // s_wval reuse
-    }
-    if (t == 0) st_release_u64(&status[chunk], pack_status(tag, ST_A, run_f, to_bits(run_v)));
-
-    // ---- look-back over preceding chunk aggregates (CTA-wide windows)
-    T carry = identity<OP, T>();
-    if (chunk > 0 && ((int64_t)t0 * FT) % m != 0) {
-        int pred = chunk - 1;
-        while (true) {
-            const int idx = pred - t;
-            uint64_t word = 0;
-            if (idx >= 0) {
-                do {
-                    word = ld_acquire_u64(&status[idx]);
-                } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
+    // consume one item: returns with the tile's values scanned in registers
+    for (int c = blockIdx.x; c < num_chunks; c += G) {
+        const int L = chunk_tiles(c);
+        const bool agg_needed = need_agg(c), carry_needed = need_carry(c);
+        // ---- phase 1
+        uint32_t run_f = 0;
+        T run_v = identity<OP, T>();
+        if (agg_needed) {
+            for (int j = 0; j < L; ++j, ++vi) {
+                const int sl = vi % kSlots;
+                const SlotMeta sm = meta[sl];
+                T* buf = ring + sl * FT;
+                acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
+                const ThreadPos tp = thread_pos(sm, m);
+                T v[FI];
+                load_items(buf, v);
+                bool hs;
+                T acc;
+                local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
+                uint32_t exf, aggf;
+                T exv, aggv;
+                cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+                run_v = aggf ? aggv : combine<OP>(run_v, aggv);
+                run_f |= aggf;
+                __syncthreads();  // slot consumed, s_wval reusable
+                if (t == 0) {
+                    free_mask |= 1u << sl;
+                    if (pend_slot >= 0) {
+                        bulk_wait_read0();
+                        free_mask |= 1u << pend_slot;
+                        pend_slot = -1;
+                    }
+                    produce_all();
+                }
             }
-            const bool term = idx < 0 || ((word >> 32) & 1u);
-            const uint32_t tb = __ballot_sync(0xffffffffu, term);
-            if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
-            __syncthreads();
-            int stop = FB;
+            if (t == 0)
+                st_release_u64(&status[c], pack_status(tag, (run_f || !carry_needed) ? ST_P : ST_A, run_f,
+                                                       to_bits(run_v)));
+        }
+        // ---- look-back over preceding chunk aggregates.  The carry spans the
+        // chunks from cs (holding the last segment start before this chunk) to
+        // c-1; every one of them publishes (its successor continues a segment),
+        // and nothing older is ever waited on.
+        T carry = identity<OP, T>();
+        if (carry_needed) {
+            const int64_t cstart = (int64_t)c * chunk_elems;
+            const int cs = (int)((((cstart - 1) / m) * m) / chunk_elems);
+            int pred = c - 1;
+            while (true) {
+                const int idx = pred - t;
+                uint64_t word = 0;
+                if (idx >= cs) {
+                    do {
+                        word = ld_acquire_u64(&status[idx]);
+                    } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
+                }
+                const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
+                const uint32_t tb = __ballot_sync(0xffffffffu, term);
+                if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
+                __syncthreads();
+                int stop = FB;
 #pragma unroll
-            for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
-            T val = (t <= stop && idx >= 0) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
+                for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
+                T val = (t <= stop && idx >= cs) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
 #pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {  // ordered: higher lane = older chunk
-                const T older = __shfl_down_sync(0xffffffffu, val, off);
-                if (lane + off < 32) val = combine<OP>(older, val);
+                for (int off = 1; off < 32; off <<= 1) {  // ordered: higher lane = older chunk
+                    const T older = __shfl_down_sync(0xffffffffu, val, off);
+                    if (lane + off < 32) val = combine<OP>(older, val);
+                }
+                if (lane == 0) s_lbval[w] = val;
+                __syncthreads();
+                T win = identity<OP, T>();
+#pragma unroll
+                for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
+                carry = combine<OP>(win, carry);
+                __syncthreads();
+                if (stop < FB) break;
+                pred -= FB;
             }
-            if (lane == 0) s_lbval[w] = val;
-            __syncthreads();
-            T win = identity<OP, T>();
-#pragma unroll
-            for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
-            carry = combine<OP>(win, carry);
-            __syncthreads();
-            if (stop < FB) break;
-            pred -= FB;
+            if (agg_needed && !run_f && t == 0)
+                st_release_u64(&status[c], pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, run_v))));
         }
-    }
-
-    // ---- phase 3: scan the chunk with the running carry
-    for (int vi = L; vi < V; ++vi) {
-        const int sl = vi % kSlots;
-        const SlotMeta sm = meta[sl];
-        T* buf = ring + sl * FT;
-        const int64_t base = (int64_t)sm.tile * FT;
-        acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
-        const ThreadPos tp = thread_pos(sm, m);
-        T v[FI];
-        load_items(buf, v);
-        bool hs;
-        T acc;
-        local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
-        uint32_t exf, aggf;
-        T exv, aggv;
-        cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
-        {
-            const T carry_t = exf ? exv : combine<OP>(carry, exv);
-            const int lim = min(tp.nx0, tp.nvalid);
+        // ---- phase 3
+        for (int j = 0; j < L; ++j, ++vi) {
+            const int sl = vi % kSlots;
+            const SlotMeta sm = meta[sl];
+            T* buf = ring + sl * FT;
+            const int64_t base = (int64_t)sm.tile * FT;
+            acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
+            const ThreadPos tp = thread_pos(sm, m);
+            T v[FI];
+            load_items(buf, v);
+            bool hs;
+            T acc;
+            local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
+            uint32_t exf, aggf;
+            T exv, aggv;
+            cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+            {
+                const T carry_t = exf ? exv : combine<OP>(carry, exv);
+                const int lim = min(tp.nx0, tp.nvalid);
 #pragma unroll
-            for (int k = 0; k < FI; ++k)
-                if (k < lim) v[k] = combine<OP>(carry_t, v[k]);
-        }
-        carry = aggf ? aggv : combine<OP>(carry, aggv);
-        store_items(buf, v);
-        const bool bulk = tma_out && sm.cnt == FT;
-        if (bulk) fence_proxy_async_smem();
-        __syncthreads();
-        if (bulk) {
+                for (int k = 0; k < FI; ++k)
+                    if (k < lim) v[k] = combine<OP>(carry_t, v[k]);
+            }
+            carry = aggf ? aggv : combine<OP>(carry, aggv);
+            store_items(buf, v);
+            const bool bulk = tma_out && sm.cnt == FT;
+            if (bulk) fence_proxy_async_smem();
+            __syncthreads();
+            if (bulk) {
+                if (t == 0) bulk_s2g_hint(out + base, buf, FT * sizeof(T), pol_stream);
+            } else {
+                for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
+                __syncthreads();
+            }
             if (t == 0) {
-                bulk_s2g(out + base, buf, FT * sizeof(T));
-                bulk_commit();
+                bulk_commit();  // one group per phase-3 item (empty for cooperative stores)
+                if (pend_slot >= 0) {
+                    bulk_wait_read1();  // all but the newest group have read their slots
+                    free_mask |= 1u << pend_slot;
+                }
+                pend_slot = sl;
+                produce_all();
             }
-        } else {
-            for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
         }
-        // refill the slot of the previous iteration once its store has read smem
-        if (t == 0 && next_w < V && next_w == vi - 1 + kSlots) {
-            if (bulk) bulk_wait_read1();
-            else bulk_wait_read0();
-            produce(next_w++);
-        }
-        __syncthreads();
     }
-    if (t == 0) bulk_wait0();
+    if (t == 0) {
+        bulk_wait0();
+        __threadfence();
+        const unsigned long long old = atomicAdd(ctr, 1ull);
+        if ((uint32_t)old == (uint32_t)G - 1) atomicAdd(ctr, (1ull << 32) - (unsigned long long)G);
+    }
 }
 
 // ------------------------------------------------------------------ launch
@@ -587,12 +653,21 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         const T d = bits_to<T>(a.ne_bits);
         if (scan) {
             auto k = flat_scan_kernel<T, OP, F>;
-            const int64_t g = std::min<int64_t>(tiles, resident_ctas(k, smem));
-            const int per = (int)ceil_div(tiles, g);
-            const int chunks = (int)ceil_div(tiles, per);
-            k<<<chunks, FB, smem, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, per, chunks, tma_in,
-                                              tma_out);
-            return cudaGetLastError();
+            const int chunks = (int)ceil_div(tiles, kChunkTiles);
+            const int grid = (int)std::min<int64_t>(chunks, resident_ctas(k, smem));
+            // cooperative launch: all CTAs co-resident (static chunk ownership + look-back)
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3((unsigned)grid);
+            cfg.blockDim = dim3(FB);
+            cfg.dynamicSmemBytes = smem;
+            cfg.stream = a.stream;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeCooperative;
+            attr[0].val.cooperative = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            int nt = (int)tiles;
+            return cudaLaunchKernelEx(&cfg, k, (const T*)a.in, (T*)a.out, N, a.m, d, ws, nt, chunks, tma_in, tma_out);
         }
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
         T* tail = head + tiles;
