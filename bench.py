@@ -4,7 +4,7 @@
 Workload (BASELINE.json configs[1]): the fp32 segmented redomap sweep at
 n*m = 2^26 -- n = 2^k, m = 2^(26-k), k = 0..26 -- running segred and segscan
 (op +, f = id) through the AUTO selector with thresholds set by the offline
-tuner (ifl_tune, trained on the n*m = 2^22 and 2^24 sweeps).
+tuner (ifl_tune, trained on the n*m = 2^25 and 2^27 sweeps, bracketing the test size).
 
 One "step" = one pass of the whole sweep (27 shapes x {segred, segscan}).
 value = algorithmic bytes of the step (segred 4(nm+n), segscan 8nm) / time,
@@ -136,12 +136,12 @@ def run_ours(args, rank, world, device):
     sh = shapes()
     stream = torch.cuda.current_stream()
 
-    # ---- offline tuning (untimed): train on the 2^22 and 2^24 sweeps
+    # ---- offline tuning (untimed): train on the 2^25 and 2^27 sweeps (L2 flushed; bracket 2^26)
     tuned = {}
     if not args.no_tune:
         t0 = time.time()
         for site in ("segred.b4", "segscan.b4"):
-            train = [s for lg in (22, 24) for s in shapes(lg)]
+            train = [s for lg in (25, 27) for s in shapes(lg)]
             scratch_bytes = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data,
                                                              len(train))
             scratch = torch.empty(scratch_bytes, dtype=torch.uint8, device=device)

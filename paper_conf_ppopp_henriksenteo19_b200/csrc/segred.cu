@@ -73,7 +73,7 @@ __device__ __forceinline__ void top_load_tile(T* tile, const T* __restrict__ in,
     }
 }
 
-template <typename T, int OP, int F>
+template <typename T, int OP, int F, bool COLS>
 __global__ void __launch_bounds__(kTopThreads) segred_top_kernel(const T* __restrict__ in, T* __restrict__ out,
                                                                  int64_t n, int64_t m, T d, bool vec) {
     __shared__ T tile[kTopWords];
@@ -84,7 +84,7 @@ __global__ void __launch_bounds__(kTopThreads) segred_top_kernel(const T* __rest
     for (int64_t b = blockIdx.x; b < nblk; b += gridDim.x) {
         const int64_t r0 = b * rows_blk;
         const int rows = (int)min(rows_blk, n - r0);
-        if (m <= kTopKT) {
+        if constexpr (!COLS) {
             top_load_tile(tile, in, r0, rows, m, 0, (int)m, true, vec);
             __syncthreads();
             const int mm = (int)m;
@@ -99,9 +99,37 @@ __global__ void __launch_bounds__(kTopThreads) segred_top_kernel(const T* __rest
             __syncthreads();
         } else {
             Acc<OP, T> a0(d), a1(identity<OP, T>()), a2(identity<OP, T>()), a3(identity<OP, T>());
-            for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
+            using V = typename Vec4<T>::type;
+            const int64_t nfull = vec ? (m / kTopKT) : 0;  // full 32-column tiles on the vector path
+            // software pipeline over the full column tiles: the next tile's eight
+            // 128-bit loads per thread are in flight while this tile is summed
+            V pre[8];
+            auto issue = [&](int64_t k0) {
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    const int v = t + j * kTopThreads, row = v >> 3, c4 = v & 7;
+                    if (row < rows) pre[j] = ldg_stream4(in + (r0 + row) * m + k0 + 4 * c4);
+                }
+            };
+            if (nfull > 0) issue(0);
+            for (int64_t ti = 0; ti * kTopKT < m; ++ti) {
+                const int64_t k0 = ti * kTopKT;
                 const int kt = (int)min((int64_t)kTopKT, m - k0);
-                top_load_tile(tile, in, r0, rows, m, k0, kt, false, vec);
+                if (ti < nfull) {
+#pragma unroll
+                    for (int j = 0; j < 8; ++j) {
+                        const int v = t + j * kTopThreads, row = v >> 3, c4 = v & 7;
+                        if (row < rows) {
+                            T e[4];
+                            unpack4<T>(pre[j], e);
+#pragma unroll
+                            for (int u = 0; u < 4; ++u) tile[padq(row * kTopKT + 4 * c4 + u)] = e[u];
+                        }
+                    }
+                    if (ti + 1 < nfull) issue(k0 + kTopKT);
+                } else {
+                    top_load_tile(tile, in, r0, rows, m, k0, kt, false, false);
+                }
                 __syncthreads();
                 if (t < rows) {
                     if (kt == kTopKT) {
@@ -128,6 +156,127 @@ __global__ void __launch_bounds__(kTopThreads) segred_top_kernel(const T* __rest
     }
 }
 
+// V_TOP for m in {1, 2, 4} with 16-byte-aligned input: every 128-bit load
+// holds 4/m whole rows, so each thread reduces its rows straight from
+// registers -- fully coalesced warp-striped loads, no shared memory.
+template <typename T, int OP, int F, int M>
+__global__ void __launch_bounds__(256) segred_top_small_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                               int64_t n, T d) {
+    using V = typename Vec4<T>::type;
+    const int64_t N = n * M, nv = N >> 2;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < nv; v0 += 4 * stride) {
+        V q[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (v0 + u * stride < nv) q[u] = ldg_stream4(in + 4 * (v0 + u * stride));
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int64_t v = v0 + u * stride;
+            if (v >= nv) break;
+            T e[4];
+            unpack4<T>(q[u], e);
+            if constexpr (M == 1) {
+                V r;
+                r.x = combine<OP>(d, apply_map<F>(e[0]));
+                r.y = combine<OP>(d, apply_map<F>(e[1]));
+                r.z = combine<OP>(d, apply_map<F>(e[2]));
+                r.w = combine<OP>(d, apply_map<F>(e[3]));
+                *reinterpret_cast<V*>(out + 4 * v) = r;
+            } else if constexpr (M == 2) {
+                out[2 * v] = combine<OP>(combine<OP>(d, apply_map<F>(e[0])), apply_map<F>(e[1]));
+                out[2 * v + 1] = combine<OP>(combine<OP>(d, apply_map<F>(e[2])), apply_map<F>(e[3]));
+            } else {
+                T a = combine<OP>(d, apply_map<F>(e[0]));
+                a = combine<OP>(a, apply_map<F>(e[1]));
+                a = combine<OP>(a, apply_map<F>(e[2]));
+                out[v] = combine<OP>(a, apply_map<F>(e[3]));
+            }
+        }
+    }
+    // rows not covered by whole 128-bit words (N % 4 != 0)
+    const int64_t r0 = (nv * 4) / M;
+    for (int64_t r = r0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += stride) {
+        T a = d;
+        for (int k = 0; k < M; ++k) a = combine<OP>(a, apply_map<F>(in[r * M + k]));
+        out[r] = a;
+    }
+}
+
+// V_TOP for m in {8, 16, 32}, 16-byte-aligned: each warp takes 32 consecutive
+// rows (a contiguous 32*m-element block), loads and stores it with fully
+// coalesced 128-bit accesses through a padded per-warp tile, and every lane
+// walks its own row sequentially (conflict-free: one pad word per 32).
+template <typename T, int OP, int F, int M, bool SCAN>
+__global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int64_t n, T d) {
+    using V = typename Vec4<T>::type;
+    constexpr int W4 = M / 4;
+    __shared__ T sm[8][32 * M + M];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    T* s = sm[warp];
+    const int64_t nw = (int64_t)gridDim.x * 8;
+    for (int64_t wc = (int64_t)blockIdx.x * 8 + warp; wc * 32 < n; wc += nw) {
+        const int64_t r0 = wc * 32;
+        const int rows = (int)min((int64_t)32, n - r0);
+        const T* src = in + r0 * M;
+#pragma unroll
+        for (int u = 0; u < W4; ++u) {
+            const int q4 = lane + 32 * u;
+            if (q4 < rows * W4) {
+                T e[4];
+                unpack4<T>(ldg_stream4(src + 4 * q4), e);
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int q = 4 * q4 + k;
+                    s[q + (q >> 5)] = e[k];
+                }
+            }
+        }
+        __syncwarp();
+        if (lane < rows) {  // rows of <= 32 elements: plain chains (no compensation needed)
+            if constexpr (SCAN) {
+                T a = d;
+#pragma unroll
+                for (int k = 0; k < M; ++k) {
+                    const int q = lane * M + k;
+                    a = combine<OP>(a, apply_map<F>(s[q + (q >> 5)]));
+                    s[q + (q >> 5)] = a;
+                }
+            } else {
+                T a0 = d, a1 = identity<OP, T>();
+#pragma unroll
+                for (int k = 0; k < M; k += 2) {
+                    const int q = lane * M + k;
+                    a0 = combine<OP>(a0, apply_map<F>(s[q + (q >> 5)]));
+                    a1 = combine<OP>(a1, apply_map<F>(s[q + 1 + ((q + 1) >> 5)]));
+                }
+                out[r0 + lane] = combine<OP>(a0, a1);
+            }
+        }
+        if (SCAN) {
+            __syncwarp();
+            T* dst = out + r0 * M;
+#pragma unroll
+            for (int u = 0; u < W4; ++u) {
+                const int q4 = lane + 32 * u;
+                if (q4 < rows * W4) {
+                    V v;
+                    int q = 4 * q4;
+                    v.x = s[q + (q >> 5)];
+                    ++q;
+                    v.y = s[q + (q >> 5)];
+                    ++q;
+                    v.z = s[q + (q >> 5)];
+                    ++q;
+                    v.w = s[q + (q >> 5)];
+                    *reinterpret_cast<V*>(dst + 4 * q4) = v;
+                }
+            }
+        }
+        __syncwarp();
+    }
+}
+
 static int top_grid(int64_t nblk) {
     static int sms = 0;
     if (!sms) {
@@ -144,9 +293,36 @@ cudaError_t launch_segred_top(const SegArgs& a) {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && (a.m <= kTopKT || a.m % 4 == 0);
+        if (vec && (a.m == 1 || a.m == 2 || a.m == 4) && ((uintptr_t)a.out % 16 == 0)) {
+            const int64_t nv = ceil_div(a.n * a.m, 4);
+            const int grid = top_grid(ceil_div(nv, 256 * 4)) * 2;
+            const T d = bits_to<T>(a.ne_bits);
+            if (a.m == 1)
+                segred_top_small_kernel<T, OP, F, 1><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else if (a.m == 2)
+                segred_top_small_kernel<T, OP, F, 2><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else
+                segred_top_small_kernel<T, OP, F, 4><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            return cudaGetLastError();
+        }
+        if (vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
+            const int grid = top_grid(ceil_div(a.n, 256));
+            const T d = bits_to<T>(a.ne_bits);
+            if (a.m == 8)
+                top_warp_kernel<T, OP, F, 8, false><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else if (a.m == 16)
+                top_warp_kernel<T, OP, F, 16, false><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else
+                top_warp_kernel<T, OP, F, 32, false><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            return cudaGetLastError();
+        }
         const int64_t nblk = ceil_div(a.n, (int64_t)kTopThreads * top_rpt(a.m));
-        segred_top_kernel<T, OP, F><<<top_grid(nblk), kTopThreads, 0, a.stream>>>(
-            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
+        if (a.m <= kTopKT)
+            segred_top_kernel<T, OP, F, false><<<top_grid(nblk), kTopThreads, 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
+        else
+            segred_top_kernel<T, OP, F, true><<<top_grid(nblk), kTopThreads, 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
         return cudaGetLastError();
     });
 }

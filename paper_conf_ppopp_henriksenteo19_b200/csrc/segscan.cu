@@ -146,6 +146,118 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
     }
 }
 
+// V_TOP for m in {1, 2, 4} with 16-byte-aligned in/out: each 128-bit word
+// holds 4/m whole rows, scanned in registers and stored back as one word.
+template <typename T, int OP, int F, int M>
+__global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* out, int64_t n, T d) {
+    using V = typename Vec4<T>::type;
+    const int64_t N = n * M, nv = N >> 2;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t v0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v0 < nv; v0 += 4 * stride) {
+        V q[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+            if (v0 + u * stride < nv) q[u] = ldg_stream4(in + 4 * (v0 + u * stride));
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const int64_t v = v0 + u * stride;
+            if (v >= nv) break;
+            T e[4];
+            unpack4<T>(q[u], e);
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+                const T x = apply_map<F>(e[k]);
+                e[k] = (k % M == 0) ? combine<OP>(d, x) : combine<OP>(e[k - 1 < 0 ? 0 : k - 1], x);
+            }
+            V r;
+            r.x = e[0]; r.y = e[1]; r.z = e[2]; r.w = e[3];
+            *reinterpret_cast<V*>(out + 4 * v) = r;
+        }
+    }
+    const int64_t r0 = (nv * 4) / M;
+    for (int64_t r = r0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += stride) {
+        T a = d;
+        for (int k = 0; k < M; ++k) {
+            a = combine<OP>(a, apply_map<F>(in[r * M + k]));
+            out[r * M + k] = a;
+        }
+    }
+}
+
+// V_TOP for m in {8, 16, 32}, 16-byte-aligned: each warp takes 32 consecutive
+// rows (a contiguous 32*m-element block), loads and stores it with fully
+// coalesced 128-bit accesses through a padded per-warp tile, and every lane
+// walks its own row sequentially (conflict-free: one pad word per 32).
+template <typename T, int OP, int F, int M, bool SCAN>
+__global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int64_t n, T d) {
+    using V = typename Vec4<T>::type;
+    constexpr int W4 = M / 4;
+    __shared__ T sm[8][32 * M + M];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    T* s = sm[warp];
+    const int64_t nw = (int64_t)gridDim.x * 8;
+    for (int64_t wc = (int64_t)blockIdx.x * 8 + warp; wc * 32 < n; wc += nw) {
+        const int64_t r0 = wc * 32;
+        const int rows = (int)min((int64_t)32, n - r0);
+        const T* src = in + r0 * M;
+#pragma unroll
+        for (int u = 0; u < W4; ++u) {
+            const int q4 = lane + 32 * u;
+            if (q4 < rows * W4) {
+                T e[4];
+                unpack4<T>(ldg_stream4(src + 4 * q4), e);
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const int q = 4 * q4 + k;
+                    s[q + (q >> 5)] = e[k];
+                }
+            }
+        }
+        __syncwarp();
+        if (lane < rows) {  // rows of <= 32 elements: plain chains (no compensation needed)
+            if constexpr (SCAN) {
+                T a = d;
+#pragma unroll
+                for (int k = 0; k < M; ++k) {
+                    const int q = lane * M + k;
+                    a = combine<OP>(a, apply_map<F>(s[q + (q >> 5)]));
+                    s[q + (q >> 5)] = a;
+                }
+            } else {
+                T a0 = d, a1 = identity<OP, T>();
+#pragma unroll
+                for (int k = 0; k < M; k += 2) {
+                    const int q = lane * M + k;
+                    a0 = combine<OP>(a0, apply_map<F>(s[q + (q >> 5)]));
+                    a1 = combine<OP>(a1, apply_map<F>(s[q + 1 + ((q + 1) >> 5)]));
+                }
+                out[r0 + lane] = combine<OP>(a0, a1);
+            }
+        }
+        if (SCAN) {
+            __syncwarp();
+            T* dst = out + r0 * M;
+#pragma unroll
+            for (int u = 0; u < W4; ++u) {
+                const int q4 = lane + 32 * u;
+                if (q4 < rows * W4) {
+                    V v;
+                    int q = 4 * q4;
+                    v.x = s[q + (q >> 5)];
+                    ++q;
+                    v.y = s[q + (q >> 5)];
+                    ++q;
+                    v.z = s[q + (q >> 5)];
+                    ++q;
+                    v.w = s[q + (q >> 5)];
+                    *reinterpret_cast<V*>(dst + 4 * q4) = v;
+                }
+            }
+        }
+        __syncwarp();
+    }
+}
+
 static int stop_grid(int64_t nblk) {
     static int sms = 0;
     if (!sms) {
@@ -163,6 +275,29 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) &&
                          (a.m <= kTopKT || a.m % 4 == 0);
+        if (vec && (a.m == 1 || a.m == 2 || a.m == 4)) {
+            const int64_t nv = ceil_div(a.n * a.m, 4);
+            const int grid = stop_grid(ceil_div(nv, 256 * 4)) * 2;
+            const T d = bits_to<T>(a.ne_bits);
+            if (a.m == 1)
+                segscan_top_small_kernel<T, OP, F, 1><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else if (a.m == 2)
+                segscan_top_small_kernel<T, OP, F, 2><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else
+                segscan_top_small_kernel<T, OP, F, 4><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            return cudaGetLastError();
+        }
+        if (vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
+            const int grid = stop_grid(ceil_div(a.n, 256));
+            const T d = bits_to<T>(a.ne_bits);
+            if (a.m == 8)
+                top_warp_kernel<T, OP, F, 8, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else if (a.m == 16)
+                top_warp_kernel<T, OP, F, 16, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else
+                top_warp_kernel<T, OP, F, 32, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            return cudaGetLastError();
+        }
         const int64_t nblk = ceil_div(a.n, (int64_t)kTopThreads * stop_rpt(a.m));
         segscan_top_kernel<T, OP, F><<<stop_grid(nblk), kTopThreads, 0, a.stream>>>(
             (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);

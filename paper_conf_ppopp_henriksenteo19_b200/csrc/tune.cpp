@@ -232,12 +232,27 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
             rc = IFL_ECUDA;
             break;
         }
-        for (int v = 0; v < 3; ++v) {
+        // versions in the order flat, middle, top; a version whose warm-up run
+        // is > 50x slower than the best timed so far is recorded from that one
+        // run (avoid spending the budget on settings that cannot win)
+        double best_ms = std::numeric_limits<double>::infinity();
+        for (int vv = 0; vv < 3; ++vv) {
+            const int v = 2 - vv;
+            cudaMemsetAsync(flush, 0, kFlushBytes, st);
+            cudaEventRecord(e0, st);
             int r = run_forced(k, s, v, (char*)scratch, st);  // warm-up; also feasibility (ENOTFIT)
+            cudaEventRecord(e1, st);
             if (r == IFL_ENOTFIT || r == IFL_EUNSUPPORTED) continue;
             if (r != IFL_OK) {
                 rc = r;
                 break;
+            }
+            cudaEventSynchronize(e1);
+            float warm = 0;
+            cudaEventElapsedTime(&warm, e0, e1);
+            if (warm > 50.0 * best_ms) {
+                table[i * 3 + v] = warm;
+                continue;
             }
             std::vector<float> ms(reps);
             for (int q = 0; q < reps; ++q) {
@@ -250,6 +265,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
             }
             std::sort(ms.begin(), ms.end());
             table[i * 3 + v] = ms[reps / 2];
+            best_ms = std::min(best_ms, (double)ms[reps / 2]);
         }
     }
     cudaEventDestroy(e0);
