@@ -326,7 +326,10 @@ int ifl_redomap2(const void* A, const void* B, float* C, int64_t n, int64_t m, i
     if (choice) *choice = c;
     if (n * p == 0) return IFL_OK;
     ifl::MmArgs a{A, B, C, n, m, p, in_dt, b_kmajor ? 1 : 0, ws, ws_bytes, (cudaStream_t)stream};
-    const size_t need = ifl::redomap2_ws_bytes(n, m, p, c.version);
+    // actual need: B transposition (b_kmajor = 0) + split-K partials (V_FLAT)
+    const size_t esz = in_dt == IFL_BF16 ? 2 : 4;
+    size_t need = ifl::redomap2_ws_bytes(n, m, p, c.version) - (((size_t)m * p * 4 + 255) & ~(size_t)255);
+    if (!b_kmajor) need += ((size_t)m * p * esz + 255) & ~(size_t)255;
     if (need && (!ws || ws_bytes < need))
         return fail(IFL_EWORKSPACE, "ifl_redomap2: needs %zu workspace bytes, got %zu", need, ws_bytes);
     return cuda_status(ifl::launch_redomap2(c.version, a), "ifl_redomap2");

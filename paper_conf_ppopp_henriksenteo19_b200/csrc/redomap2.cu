@@ -1,8 +1,372 @@
-// redomap2.cu -- placeholder, filled in below.
+// redomap2.cu -- the map-map-redomap contraction of P:122,
+//     C = map (\xs -> map (\ys -> redomap (+) (*) 0 xs ys) (transpose yss)) xss,
+// in the three code versions of P:126-134 / rule G3:
+//   V_FLAT   segred^1 <xs in xss> <ys in yss^T> <x y in xs ys> (+) 0 (x*y)
+//            (paper version 1): every (i, j, k) parallel -- the m-long dot
+//            products are split across CTAs (split-K), partials reduced in a
+//            deterministic second pass.  For degenerate shapes (n*p small).
+//   V_MIDDLE segmap^1 <i><j> (segred^0 <k> ...): a warp per output element,
+//            lanes split k, shuffle-tree reduction.
+//   V_TOP    segmap^1 <i><j> (redomap sequential in k) with block tiling and
+//            register tiling (paper versions 2 and 3): a 128x128 output tile
+//            per CTA, 8x8 per thread, k-tiles double-buffered in shared
+//            memory.  bf16 inputs take the tcgen05/TMEM/TMA tensor-core kernel
+//            (redomap2_tc.cu) when the shape allows.
+// A is [n][m]; B is yss^T as [p][m] (b_kmajor = 1, the array P:122 maps over)
+// or yss as [m][p] (b_kmajor = 0: transposed into the workspace first).
+// Inputs f32 or bf16, accumulation and C in f32.
+#include <cuda_bf16.h>
+
+#include <algorithm>
+
 #include "common.cuh"
 #include "ifl_internal.h"
+
 namespace ifl {
-size_t redomap2_ws_bytes(int64_t, int64_t, int64_t, int) { return 0; }
-bool redomap2_tc_ok(const MmArgs&) { return false; }
-cudaError_t launch_redomap2(int, const MmArgs&) { return cudaErrorNotSupported; }
+
+// ------------------------------------------------------------- helpers
+
+template <typename Tin>
+__device__ __forceinline__ float to_f(Tin v) {
+    if constexpr (std::is_same<Tin, float>::value) return v;
+    else return __bfloat162float(v);
+}
+
+// E = elements per 16-byte vector
+template <typename Tin>
+struct VecE {
+    static constexpr int E = 16 / sizeof(Tin);
+};
+
+template <typename Tin>
+__device__ __forceinline__ void load16(const Tin* p, float (&o)[VecE<Tin>::E]) {
+    const uint4 u = __ldg(reinterpret_cast<const uint4*>(p));
+    if constexpr (std::is_same<Tin, float>::value) {
+        o[0] = __uint_as_float(u.x);
+        o[1] = __uint_as_float(u.y);
+        o[2] = __uint_as_float(u.z);
+        o[3] = __uint_as_float(u.w);
+    } else {
+        const uint32_t w[4] = {u.x, u.y, u.z, u.w};
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            o[2 * q] = __uint_as_float(w[q] << 16);
+            o[2 * q + 1] = __uint_as_float(w[q] & 0xffff0000u);
+        }
+    }
+}
+
+// --------------------------------------------------------- B transpose
+// yss [m][p] -> yss^T [p][m] in the workspace (32x32 smem tiles, coalesced).
+template <typename Tin>
+__global__ void __launch_bounds__(256) transpose_kernel(const Tin* __restrict__ B, Tin* __restrict__ Bt, int64_t m,
+                                                        int64_t p) {
+    __shared__ Tin tile[32][33];
+    const int64_t k0 = (int64_t)blockIdx.y * 32, j0 = (int64_t)blockIdx.x * 32;
+    const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;
+    for (int r = ty; r < 32; r += 8)
+        if (k0 + r < m && j0 + tx < p) tile[r][tx] = B[(k0 + r) * p + j0 + tx];
+    __syncthreads();
+    for (int r = ty; r < 32; r += 8)
+        if (j0 + r < p && k0 + tx < m) Bt[(j0 + r) * m + k0 + tx] = tile[tx][r];
+}
+
+// --------------------------------------------------------------- V_FLAT
+
+constexpr int kFlatMmThreads = 256;
+
+int64_t mm_flat_splits(int64_t n, int64_t m, int64_t p) {
+    const int64_t outs = n * p;
+    const int64_t want = ceil_div((int64_t)148 * 8, outs);          // fill the GPU
+    const int64_t maxs = std::max<int64_t>(1, ceil_div(m, 4096));   // >= 4096 k per split
+    return std::max<int64_t>(1, std::min(want, maxs));
+}
+
+template <typename Tin, bool VEC>
+__global__ void __launch_bounds__(kFlatMmThreads) mm_flat_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
+                                                                 float* __restrict__ C, float* __restrict__ part,
+                                                                 int64_t n, int64_t m, int64_t p, int64_t kchunk,
+                                                                 int nsplit) {
+    __shared__ float red[kFlatMmThreads / 32];
+    constexpr int E = VecE<Tin>::E;
+    const int64_t o = (int64_t)blockIdx.y + (int64_t)blockIdx.z * gridDim.y;
+    if (o >= n * p) return;
+    const int64_t i = o / p, j = o - i * p;
+    const int split = blockIdx.x;
+    const int64_t k0 = split * kchunk, k1 = std::min(m, k0 + kchunk);
+    const Tin* a = A + i * m;
+    const Tin* b = Bt + j * m;
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+    int64_t k = k0 + (int64_t)threadIdx.x * E;
+    if (VEC) {
+        for (; k + E + (int64_t)kFlatMmThreads * E <= k1; k += 2 * (int64_t)kFlatMmThreads * E) {
+            float x0[E], y0[E], x1[E], y1[E];
+            load16(a + k, x0);
+            load16(b + k, y0);
+            load16(a + k + kFlatMmThreads * E, x1);
+            load16(b + k + kFlatMmThreads * E, y1);
+#pragma unroll
+            for (int e = 0; e < E; ++e) {
+                acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+                acc[(e + 2) & 3] = fmaf(x1[e], y1[e], acc[(e + 2) & 3]);
+            }
+        }
+        for (; k + E <= k1; k += (int64_t)kFlatMmThreads * E) {
+            float x0[E], y0[E];
+            load16(a + k, x0);
+            load16(b + k, y0);
+#pragma unroll
+            for (int e = 0; e < E; ++e) acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+        }
+        // ragged tail of the chunk (fewer than E elements per thread slot)
+        const int64_t tail0 = k1 - ((k1 - k0) % E);
+        for (int64_t kk = tail0 + threadIdx.x; kk < k1; kk += kFlatMmThreads) acc[0] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[0]);
+    } else {
+        for (int64_t kk = k0 + threadIdx.x; kk < k1; kk += kFlatMmThreads)
+            acc[kk & 3] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[kk & 3]);
+    }
+    float s = (acc[0] + acc[1]) + (acc[2] + acc[3]);
+    s = warp_reduce<OP_SUM>(s);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        float r = 0.f;
+        for (int w = 0; w < kFlatMmThreads / 32; ++w) r += red[w];
+        if (nsplit == 1) C[o] = r;
+        else part[o * nsplit + split] = r;
+    }
+}
+
+__global__ void mm_flat_finalize(const float* __restrict__ part, float* __restrict__ C, int64_t outs, int nsplit) {
+    for (int64_t o = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; o < outs; o += (int64_t)gridDim.x * blockDim.x) {
+        float r = 0.f;
+        for (int s = 0; s < nsplit; ++s) r += part[o * nsplit + s];
+        C[o] = r;
+    }
+}
+
+// ------------------------------------------------------------- V_MIDDLE
+
+template <typename Tin, bool VEC>
+__global__ void __launch_bounds__(256) mm_mid_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
+                                                     float* __restrict__ C, int64_t n, int64_t m, int64_t p) {
+    constexpr int E = VecE<Tin>::E;
+    const int lane = threadIdx.x & 31;
+    const int64_t o = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+    if (o >= n * p) return;
+    const int64_t i = o / p, j = o - i * p;
+    const Tin* a = A + i * m;
+    const Tin* b = Bt + j * m;
+    float acc[4] = {0.f, 0.f, 0.f, 0.f};
+    if (VEC) {
+        int64_t k = (int64_t)lane * E;
+        for (; k + E + 32 * E <= m; k += 64 * E) {
+            float x0[E], y0[E], x1[E], y1[E];
+            load16(a + k, x0);
+            load16(b + k, y0);
+            load16(a + k + 32 * E, x1);
+            load16(b + k + 32 * E, y1);
+#pragma unroll
+            for (int e = 0; e < E; ++e) {
+                acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+                acc[(e + 2) & 3] = fmaf(x1[e], y1[e], acc[(e + 2) & 3]);
+            }
+        }
+        for (; k + E <= m; k += 32 * E) {
+            float x0[E], y0[E];
+            load16(a + k, x0);
+            load16(b + k, y0);
+#pragma unroll
+            for (int e = 0; e < E; ++e) acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+        }
+        for (int64_t kk = m - (m % E) + lane; kk < m; kk += 32) acc[0] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[0]);
+    } else {
+        for (int64_t kk = lane; kk < m; kk += 32) acc[kk & 3] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[kk & 3]);
+    }
+    float s = (acc[0] + acc[1]) + (acc[2] + acc[3]);
+    s = warp_reduce<OP_SUM>(s);
+    if (lane == 0) C[o] = s;
+}
+
+// --------------------------------------------------------------- V_TOP (SIMT)
+
+constexpr int TBM = 128, TBN = 128, TBK = 16;
+
+template <typename Tin, bool VEC>
+__global__ void __launch_bounds__(256) mm_top_simt_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
+                                                          float* __restrict__ C, int64_t n, int64_t m, int64_t p) {
+    __shared__ __align__(16) float As[2][TBK][TBM + 4];
+    __shared__ __align__(16) float Bs[2][TBK][TBN + 4];
+    const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
+    const int64_t row0 = (int64_t)blockIdx.y * TBM, col0 = (int64_t)blockIdx.x * TBN;
+    const int lr = tid >> 1, lk = (tid & 1) * 8;  // each thread stages 8 k-values of one row of A and of Bt
+    float ra[8], rb[8];
+    const bool arow = row0 + lr < n, brow = col0 + lr < p;
+    const Tin* ap = A + (arow ? (row0 + lr) * m : 0);
+    const Tin* bp = Bt + (brow ? (col0 + lr) * m : 0);
+    auto gload = [&](int64_t k0) {
+        const int64_t kb = k0 + lk;
+        if (VEC && kb + 8 <= m) {
+            constexpr int E = VecE<Tin>::E;
+#pragma unroll
+            for (int h = 0; h < 8 / E; ++h) {
+                float x[E], y[E];
+                if (arow) load16(ap + kb + h * E, x);
+                else
+#pragma unroll
+                    for (int e = 0; e < E; ++e) x[e] = 0.f;
+                if (brow) load16(bp + kb + h * E, y);
+                else
+#pragma unroll
+                    for (int e = 0; e < E; ++e) y[e] = 0.f;
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    ra[h * E + e] = x[e];
+                    rb[h * E + e] = y[e];
+                }
+            }
+        } else {
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+                const int64_t k = kb + e;
+                ra[e] = (arow && k < m) ? to_f(ap[k]) : 0.f;
+                rb[e] = (brow && k < m) ? to_f(bp[k]) : 0.f;
+            }
+        }
+    };
+    auto sstore = [&](int buf) {
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+            As[buf][lk + e][lr] = ra[e];
+            Bs[buf][lk + e][lr] = rb[e];
+        }
+    };
+    float acc[8][8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+#pragma unroll
+        for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
+    const int64_t nk = ceil_div(m, TBK);
+    gload(0);
+    sstore(0);
+    __syncthreads();
+    for (int64_t kt = 0; kt < nk; ++kt) {
+        const int cur = (int)(kt & 1);
+        if (kt + 1 < nk) gload((kt + 1) * TBK);
+#pragma unroll
+        for (int k = 0; k < TBK; ++k) {
+            const float4 a0 = *reinterpret_cast<const float4*>(&As[cur][k][ty * 4]);
+            const float4 a1 = *reinterpret_cast<const float4*>(&As[cur][k][64 + ty * 4]);
+            const float4 b0 = *reinterpret_cast<const float4*>(&Bs[cur][k][tx * 4]);
+            const float4 b1 = *reinterpret_cast<const float4*>(&Bs[cur][k][64 + tx * 4]);
+            const float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
+            const float b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+#pragma unroll
+                for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+        }
+        if (kt + 1 < nk) sstore(cur ^ 1);
+        __syncthreads();
+    }
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+        const int64_t r = row0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
+        if (r >= n) continue;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            const int64_t c = col0 + h * 64 + tx * 4;
+            float* dst = C + r * p + c;
+            if (c + 4 <= p && ((uintptr_t)dst % 16 == 0)) {
+                *reinterpret_cast<float4*>(dst) =
+                    make_float4(acc[i][h * 4], acc[i][h * 4 + 1], acc[i][h * 4 + 2], acc[i][h * 4 + 3]);
+            } else {
+                for (int j = 0; j < 4; ++j)
+                    if (c + j < p) dst[j] = acc[i][h * 4 + j];
+            }
+        }
+    }
+}
+
+// -------------------------------------------------------------------- launch
+
+// tcgen05 bf16 kernel (redomap2_tc.cu)
+bool tc_shape_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* Bt);
+cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, int64_t n, int64_t m, int64_t p,
+                             cudaStream_t s);
+
+static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
+
+size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
+    // transposition buffer for b_kmajor = 0 (upper bound: 4-byte elements) +
+    // split-K partials of V_FLAT
+    size_t b = align256((size_t)m * p * 4);
+    if (version == 2 || version == -1) {
+        const int64_t s = mm_flat_splits(n, m, p);
+        if (s > 1) b += align256((size_t)n * p * s * 4);
+    }
+    return b;
+}
+
+bool redomap2_tc_ok(const MmArgs& a) { return a.in_dt == 2 && tc_shape_ok(a.n, a.m, a.p, a.A, a.B); }
+
+template <typename Tin>
+static cudaError_t run_mm(int version, const MmArgs& a) {
+    const Tin* A = (const Tin*)a.A;
+    const Tin* Bt = (const Tin*)a.B;
+    char* ws = (char*)a.ws;
+    size_t used = 0;
+    if (!a.b_kmajor) {  // yss [m][p] -> yss^T [p][m]
+        Tin* t = (Tin*)ws;
+        used = align256((size_t)a.m * a.p * sizeof(Tin));
+        if (a.m * a.p > 0) {
+            dim3 g((unsigned)ceil_div(a.p, 32), (unsigned)ceil_div(a.m, 32));
+            transpose_kernel<Tin><<<g, 256, 0, a.stream>>>((const Tin*)a.B, t, a.m, a.p);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return e;
+        }
+        Bt = t;
+    }
+    if (a.m == 0) return cudaMemsetAsync(a.C, 0, (size_t)a.n * a.p * sizeof(float), a.stream);
+    constexpr int E = VecE<Tin>::E;
+    const bool vec = ((uintptr_t)A % 16 == 0) && ((uintptr_t)Bt % 16 == 0) && (a.m % E == 0);
+    const int64_t outs = a.n * a.p;
+    if (version == 2) {
+        const int64_t s = mm_flat_splits(a.n, a.m, a.p);
+        int64_t kchunk = ceil_div(a.m, s);
+        kchunk = ceil_div(kchunk, (int64_t)E) * E;  // keep vector alignment of every chunk
+        const int nsplit = (int)ceil_div(a.m, kchunk);
+        float* part = (float*)(ws + used);
+        const int64_t gy = std::min<int64_t>(outs, 65535), gz = ceil_div(outs, gy);
+        dim3 g((unsigned)nsplit, (unsigned)gy, (unsigned)gz);
+        if (vec) mm_flat_kernel<Tin, true><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
+        else mm_flat_kernel<Tin, false><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess || nsplit == 1) return e;
+        mm_flat_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 8), 256, 0, a.stream>>>(part, a.C, outs,
+                                                                                                       nsplit);
+        return cudaGetLastError();
+    }
+    if (version == 1) {
+        const int64_t grid = ceil_div(outs, 8);
+        if (vec) mm_mid_kernel<Tin, true><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+        else mm_mid_kernel<Tin, false><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+        return cudaGetLastError();
+    }
+    // V_TOP
+    if constexpr (std::is_same<Tin, __nv_bfloat16>::value) {
+        if (tc_shape_ok(a.n, a.m, a.p, A, Bt)) return launch_mm_top_tc(A, Bt, a.C, a.n, a.m, a.p, a.stream);
+    }
+    dim3 g((unsigned)ceil_div(a.p, TBN), (unsigned)ceil_div(a.n, TBM));
+    if (vec) mm_top_simt_kernel<Tin, true><<<g, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+    else mm_top_simt_kernel<Tin, false><<<g, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_redomap2(int version, const MmArgs& a) {
+    if (a.in_dt == 1) return run_mm<float>(version, a);
+    if (a.in_dt == 2) return run_mm<__nv_bfloat16>(version, a);
+    return cudaErrorInvalidValue;
+}
+
 }  // namespace ifl

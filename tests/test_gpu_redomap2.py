@@ -1,0 +1,106 @@
+"""GPU parity for redomap2 (P:122 map-map-redomap contraction), every
+version x dtype x B layout, against the CPU oracle.  Bound:
+|C - C*| <= 1e-5 * sum_k |A_ik * Y_kj| + 1e-30 (bf16 products are exact in
+f32, so both dtypes share it)."""
+import numpy as np
+import pytest
+import torch
+
+import ifl_inputs as gen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ifl():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_henriksenteo19_b200 import build
+    build.build()
+    import paper_conf_ppopp_henriksenteo19_b200 as m
+    m.reset_thresholds()
+    return m
+
+
+def bits(t):
+    return t.contiguous().view(torch.int16).numpy().view(np.uint16)
+
+
+def operands(dt, n, m, p, seed=6):
+    if dt == "f32":
+        A = gen.matrix("F32_SIGNED", seed, n, m)
+        Bt = gen.matrix("F32_SIGNED", seed + 1, p, m)
+    else:
+        A = gen.matrix("BF16_SIGNED", seed, n, m)
+        Bt = gen.matrix("BF16_SIGNED", seed + 1, p, m)
+    return A, Bt
+
+
+def check(orc, A, Bt, C):
+    a = A.numpy() if A.dtype == torch.float32 else bits(A)
+    b = Bt.numpy() if Bt.dtype == torch.float32 else bits(Bt)
+    want, ab = orc.redomap2(a, b, b_kmajor=True, with_abs=True)
+    err = np.abs(C.cpu().numpy().astype(np.float64) - want)
+    bound = 1e-5 * ab + 1e-30
+    assert (err <= bound).all(), f"max err {err.max():.3g} at {np.unravel_index(err.argmax(), err.shape)}"
+
+
+SHAPES = [(1, 1, 1), (3, 5, 7), (1, 1 << 16, 1), (2, 100003, 3), (130, 77, 260), (256, 512, 256),
+          (129, 200, 257), (1000, 64, 300), (64, 4096, 1)]
+
+
+@pytest.mark.parametrize("version", ["top", "middle", "flat", "auto"])
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+def test_redomap2_versions(ifl, orc, version, dt):
+    for (n, m, p) in SHAPES:
+        A, Bt = operands(dt, n, m, p)
+        C = ifl.redomap2(A.cuda(), Bt.cuda(), b_kmajor=True, version=version)
+        check(orc, A, Bt, C)
+
+
+@pytest.mark.parametrize("version", ["top", "middle", "flat"])
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+def test_redomap2_row_major_B(ifl, orc, version, dt):
+    """B given as yss [m][p] (b_kmajor = 0): same result."""
+    for (n, m, p) in [(5, 33, 17), (200, 128, 300), (1, 5000, 2)]:
+        A, Bt = operands(dt, n, m, p, seed=9)
+        B = Bt.t().contiguous()
+        C = ifl.redomap2(A.cuda(), B.cuda(), b_kmajor=False, version=version)
+        check(orc, A, Bt, C)
+
+
+def test_redomap2_closed_forms(ifl):
+    # A = 1, B = 1 -> C = m ; A = I -> C = B  (all versions, both dtypes)
+    for dt in (torch.float32, torch.bfloat16):
+        for v in ("top", "middle", "flat"):
+            n, m, p = 130, 264, 300
+            C = ifl.redomap2(torch.ones(n, m, dtype=dt, device="cuda"), torch.ones(p, m, dtype=dt, device="cuda"),
+                             version=v)
+            assert torch.equal(C, torch.full((n, p), float(m), device="cuda"))
+            I = torch.eye(m, dtype=dt, device="cuda")
+            Bt = gen.matrix("BF16_SIGNED", 3, p, m).to(dt).cuda()
+            C = ifl.redomap2(I, Bt, version=v)
+            assert torch.equal(C, Bt.t().float()), (dt, v)
+
+
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+def test_config2_family_k20(ifl, orc, dt):
+    """BASELINE.json configs[2]: A[2^a][2^(k-2a)] x B[2^(k-2a)][2^a], k = 20,
+    tall-skinny to square, every version."""
+    k = 20
+    for a in range(0, k // 2 + 1, 2):
+        n = p = 1 << a
+        m = 1 << (k - 2 * a)
+        A, Bt = operands(dt, n, m, p, seed=6)
+        for v in ("top", "middle", "flat", "auto"):
+            C = ifl.redomap2(A.cuda(), Bt.cuda(), version=v)
+            check(orc, A, Bt, C)
+
+
+def test_tc_dense_square(ifl, orc):
+    """Dense bf16 square through the tcgen05 kernel, sampled rows vs oracle."""
+    n = m = p = 1024
+    A, Bt = operands("bf16", n, m, p, seed=11)
+    C = ifl.redomap2(A.cuda(), Bt.cuda(), version="top")
+    rows = [0, 1, 127, 128, 511, 1023]
+    check(orc, A[rows], Bt, C[rows])
