@@ -188,28 +188,40 @@ __global__ void __launch_bounds__(256) mm_mid_kernel(const Tin* __restrict__ A, 
     if (lane == 0) C[o] = s;
 }
 
-// --------------------------------------------------------------- V_TOP (SIMT)
-
-constexpr int TBM = 128, TBN = 128, TBK = 16;
-
-template <typename Tin, bool VEC>
-__global__ void __launch_bounds__(256) mm_top_simt_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
-                                                          float* __restrict__ C, int64_t n, int64_t m, int64_t p) {
-    __shared__ __align__(16) float As[2][TBK][TBM + 4];
-    __shared__ __align__(16) float Bs[2][TBK][TBN + 4];
+// -------------------------------------------------------- tiled SIMT kernel
+// A BM x BN output tile per CTA of 256 threads (16 x 16), TM x TN = BM/16 x
+// BN/16 outputs per thread in registers (register tiling), BK-deep k-tiles of
+// A and Bt staged in double-buffered shared memory (block tiling), the next
+// k-tile prefetched into registers while the current one is multiplied.
+// blockIdx.z = k-split: k-tiles [z*kps, (z+1)*kps); partial tiles go to
+// part[z] when gridDim.z > 1 (V_FLAT's split-K), else straight to C.
+template <typename Tin, int BM, int BN, int BK, bool VEC>
+__global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
+                                                           float* __restrict__ C, float* __restrict__ part, int64_t n,
+                                                           int64_t m, int64_t p, int64_t kps) {
+    constexpr int TM = BM / 16, TN = BN / 16;
+    constexpr int EPT = BM * BK / 256;  // k-values each thread stages per tile (BM == BN)
+    static_assert(BM == BN && EPT >= 1 && BK % EPT == 0, "tile config");
+    constexpr int TPR = BK / EPT;  // threads per staged row
+    __shared__ __align__(16) float As[2][BK][BM + 4];
+    __shared__ __align__(16) float Bs[2][BK][BN + 4];
     const int tid = threadIdx.x, tx = tid & 15, ty = tid >> 4;
-    const int64_t row0 = (int64_t)blockIdx.y * TBM, col0 = (int64_t)blockIdx.x * TBN;
-    const int lr = tid >> 1, lk = (tid & 1) * 8;  // each thread stages 8 k-values of one row of A and of Bt
-    float ra[8], rb[8];
+    const int64_t row0 = (int64_t)blockIdx.y * BM, col0 = (int64_t)blockIdx.x * BN;
+    const int lr = tid / TPR, lk = (tid % TPR) * EPT;
+    float ra[EPT], rb[EPT];
     const bool arow = row0 + lr < n, brow = col0 + lr < p;
     const Tin* ap = A + (arow ? (row0 + lr) * m : 0);
     const Tin* bp = Bt + (brow ? (col0 + lr) * m : 0);
+    const int64_t nk_all = ceil_div(m, BK);
+    const int64_t kt_begin = (int64_t)blockIdx.z * kps;
+    const int64_t kt_end = std::min(nk_all, kt_begin + kps);
+    float* out = gridDim.z == 1 ? C : part + (int64_t)blockIdx.z * n * p;
     auto gload = [&](int64_t k0) {
         const int64_t kb = k0 + lk;
-        if (VEC && kb + 8 <= m) {
-            constexpr int E = VecE<Tin>::E;
+        constexpr int E = VecE<Tin>::E;
+        if (VEC && (EPT % E == 0) && kb + EPT <= m) {
 #pragma unroll
-            for (int h = 0; h < 8 / E; ++h) {
+            for (int h = 0; h < EPT / E; ++h) {
                 float x[E], y[E];
                 if (arow) load16(ap + kb + h * E, x);
                 else
@@ -227,7 +239,7 @@ __global__ void __launch_bounds__(256) mm_top_simt_kernel(const Tin* __restrict_
             }
         } else {
 #pragma unroll
-            for (int e = 0; e < 8; ++e) {
+            for (int e = 0; e < EPT; ++e) {
                 const int64_t k = kb + e;
                 ra[e] = (arow && k < m) ? to_f(ap[k]) : 0.f;
                 rb[e] = (brow && k < m) ? to_f(bp[k]) : 0.f;
@@ -236,76 +248,103 @@ __global__ void __launch_bounds__(256) mm_top_simt_kernel(const Tin* __restrict_
     };
     auto sstore = [&](int buf) {
 #pragma unroll
-        for (int e = 0; e < 8; ++e) {
+        for (int e = 0; e < EPT; ++e) {
             As[buf][lk + e][lr] = ra[e];
             Bs[buf][lk + e][lr] = rb[e];
         }
     };
-    float acc[8][8];
+    float acc[TM][TN];
 #pragma unroll
-    for (int i = 0; i < 8; ++i)
+    for (int i = 0; i < TM; ++i)
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[i][j] = 0.f;
-    const int64_t nk = ceil_div(m, TBK);
-    gload(0);
-    sstore(0);
+        for (int j = 0; j < TN; ++j) acc[i][j] = 0.f;
+    if (kt_begin < kt_end) {
+        gload(kt_begin * BK);
+        sstore(0);
+    }
     __syncthreads();
-    for (int64_t kt = 0; kt < nk; ++kt) {
-        const int cur = (int)(kt & 1);
-        if (kt + 1 < nk) gload((kt + 1) * TBK);
+    for (int64_t kt = kt_begin; kt < kt_end; ++kt) {
+        const int cur = (int)((kt - kt_begin) & 1);
+        if (kt + 1 < kt_end) gload((kt + 1) * BK);
 #pragma unroll
-        for (int k = 0; k < TBK; ++k) {
-            const float4 a0 = *reinterpret_cast<const float4*>(&As[cur][k][ty * 4]);
-            const float4 a1 = *reinterpret_cast<const float4*>(&As[cur][k][64 + ty * 4]);
-            const float4 b0 = *reinterpret_cast<const float4*>(&Bs[cur][k][tx * 4]);
-            const float4 b1 = *reinterpret_cast<const float4*>(&Bs[cur][k][64 + tx * 4]);
-            const float a[8] = {a0.x, a0.y, a0.z, a0.w, a1.x, a1.y, a1.z, a1.w};
-            const float b[8] = {b0.x, b0.y, b0.z, b0.w, b1.x, b1.y, b1.z, b1.w};
+        for (int k = 0; k < BK; ++k) {
+            // each thread's rows/cols are two halves {t*TM/2 ..} and {BM/2 + t*TM/2 ..}
+            float a[TM], b[TN];
+            if constexpr (TM == 1) {
+                a[0] = As[cur][k][ty];
+                b[0] = Bs[cur][k][tx];
+            } else {
 #pragma unroll
-            for (int i = 0; i < 8; ++i)
+                for (int i = 0; i < TM / 2; ++i) {
+                    a[i] = As[cur][k][ty * (TM / 2) + i];
+                    a[TM / 2 + i] = As[cur][k][BM / 2 + ty * (TM / 2) + i];
+                }
 #pragma unroll
-                for (int j = 0; j < 8; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+                for (int j = 0; j < TN / 2; ++j) {
+                    b[j] = Bs[cur][k][tx * (TN / 2) + j];
+                    b[TN / 2 + j] = Bs[cur][k][BN / 2 + tx * (TN / 2) + j];
+                }
+            }
+#pragma unroll
+            for (int i = 0; i < TM; ++i)
+#pragma unroll
+                for (int j = 0; j < TN; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
         }
-        if (kt + 1 < nk) sstore(cur ^ 1);
+        if (kt + 1 < kt_end) sstore(cur ^ 1);
         __syncthreads();
     }
 #pragma unroll
-    for (int i = 0; i < 8; ++i) {
-        const int64_t r = row0 + (i < 4 ? ty * 4 + i : 64 + ty * 4 + i - 4);
+    for (int i = 0; i < TM; ++i) {
+        const int64_t r = row0 + (TM == 1 ? ty : (i < TM / 2 ? ty * (TM / 2) + i : BM / 2 + ty * (TM / 2) + i - TM / 2));
         if (r >= n) continue;
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            const int64_t c = col0 + h * 64 + tx * 4;
-            float* dst = C + r * p + c;
-            if (c + 4 <= p && ((uintptr_t)dst % 16 == 0)) {
-                *reinterpret_cast<float4*>(dst) =
-                    make_float4(acc[i][h * 4], acc[i][h * 4 + 1], acc[i][h * 4 + 2], acc[i][h * 4 + 3]);
-            } else {
-                for (int j = 0; j < 4; ++j)
-                    if (c + j < p) dst[j] = acc[i][h * 4 + j];
-            }
+        for (int j = 0; j < TN; ++j) {
+            const int64_t c =
+                col0 + (TN == 1 ? tx : (j < TN / 2 ? tx * (TN / 2) + j : BN / 2 + tx * (TN / 2) + j - TN / 2));
+            if (c < p) out[r * p + c] = acc[i][j];
         }
     }
 }
 
 // -------------------------------------------------------------------- launch
 
-// tcgen05 bf16 kernel (redomap2_tc.cu)
+// tcgen05 bf16 kernel and the split-K finalize (redomap2_tc.cu)
+__global__ void mm_splitk_finalize(const float* __restrict__ part, float* __restrict__ C, int64_t outs, int splits);
 bool tc_shape_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* Bt);
-cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, int64_t n, int64_t m, int64_t p,
-                             cudaStream_t s);
+int tc_splits(int64_t n, int64_t m, int64_t p, bool flat);
+cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* part, int64_t n, int64_t m, int64_t p,
+                             int splits, cudaStream_t s);
 
 static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 
+// V_FLAT's SIMT form: tiny n*p -> one CTA per (output, k-chunk) dot product;
+// otherwise 32x32 output tiles split along k until the GPU is full.
+constexpr int kFlatTileBM = 32, kFlatTileBK = 32;
+static bool flat_use_dot(int64_t n, int64_t p) { return n * p <= 16; }
+static int64_t simt_flat_splits(int64_t n, int64_t m, int64_t p) {
+    const int64_t tiles = ceil_div(n, kFlatTileBM) * ceil_div(p, kFlatTileBM);
+    const int64_t nk = ceil_div(m, kFlatTileBK);
+    return std::max<int64_t>(1, std::min(ceil_div((int64_t)148 * 6, tiles), nk));
+}
+
 size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
     // transposition buffer for b_kmajor = 0 (upper bound: 4-byte elements) +
-    // split-K partials of V_FLAT
+    // split-K partials (V_FLAT always may split; V_TOP's tensor-core kernel
+    // splits k to fill idle SMs)
     size_t b = align256((size_t)m * p * 4);
+    size_t part = 0;
     if (version == 2 || version == -1) {
-        const int64_t s = mm_flat_splits(n, m, p);
-        if (s > 1) b += align256((size_t)n * p * s * 4);
+        part = std::max(part, (size_t)n * p * mm_flat_splits(n, m, p) * 4);
+        part = std::max(part, (size_t)n * p * simt_flat_splits(n, m, p) * 4);
+        part = std::max(part, (size_t)n * p * tc_splits(n, m, p, true) * 4);
     }
-    return b;
+    if (version == 0 || version == -1) {
+        part = std::max(part, (size_t)n * p * tc_splits(n, m, p, false) * 4);
+        const int64_t tiles = ceil_div(n, 128) * ceil_div(p, 128), nk = ceil_div(m, 16);
+        const int64_t s = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / tiles, nk / 64));
+        part = std::max(part, (size_t)n * p * (size_t)ceil_div(nk, ceil_div(nk, s)) * 4);
+    }
+    return b + align256(part);
 }
 
 bool redomap2_tc_ok(const MmArgs& a) { return a.in_dt == 2 && tc_shape_ok(a.n, a.m, a.p, a.A, a.B); }
@@ -331,35 +370,73 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     constexpr int E = VecE<Tin>::E;
     const bool vec = ((uintptr_t)A % 16 == 0) && ((uintptr_t)Bt % 16 == 0) && (a.m % E == 0);
     const int64_t outs = a.n * a.p;
-    if (version == 2) {
-        const int64_t s = mm_flat_splits(a.n, a.m, a.p);
-        int64_t kchunk = ceil_div(a.m, s);
-        kchunk = ceil_div(kchunk, (int64_t)E) * E;  // keep vector alignment of every chunk
-        const int nsplit = (int)ceil_div(a.m, kchunk);
-        float* part = (float*)(ws + used);
-        const int64_t gy = std::min<int64_t>(outs, 65535), gz = ceil_div(outs, gy);
-        dim3 g((unsigned)nsplit, (unsigned)gy, (unsigned)gz);
-        if (vec) mm_flat_kernel<Tin, true><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
-        else mm_flat_kernel<Tin, false><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
+    float* part = (float*)(ws + used);
+    constexpr bool kBf16 = std::is_same<Tin, __nv_bfloat16>::value;
+    const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, Bt);
+    if (version == 2) {  // ---- V_FLAT: every level parallel (split-K)
+        if (flat_use_dot(a.n, a.p)) {
+            const int64_t s = mm_flat_splits(a.n, a.m, a.p);
+            int64_t kchunk = ceil_div(a.m, s);
+            kchunk = ceil_div(kchunk, (int64_t)E) * E;  // keep vector alignment of every chunk
+            const int nsplit = (int)ceil_div(a.m, kchunk);
+            const int64_t gy = std::min<int64_t>(outs, 65535), gz = ceil_div(outs, gy);
+            dim3 g((unsigned)nsplit, (unsigned)gy, (unsigned)gz);
+            if (vec) mm_flat_kernel<Tin, true><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
+            else mm_flat_kernel<Tin, false><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess || nsplit == 1) return e;
+            mm_flat_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 8), 256, 0, a.stream>>>(
+                part, a.C, outs, nsplit);
+            return cudaGetLastError();
+        }
+        // bf16: 128x256 tensor-core tiles split along k (even a mostly empty
+        // tile beats SIMT here); f32: SIMT 32x32 (16x16 when skinny) tiles
+        if (tc)
+            return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, true), a.stream);
+        const int BM = std::max(a.n, a.p) <= 16 ? 16 : kFlatTileBM;
+        const int64_t s = simt_flat_splits(a.n, a.m, a.p);
+        const int64_t nk = ceil_div(a.m, kFlatTileBK), kps = ceil_div(nk, s), splits = ceil_div(nk, kps);
+        dim3 g((unsigned)ceil_div(a.p, BM), (unsigned)ceil_div(a.n, BM), (unsigned)splits);
+        if (BM == 16) {
+            if (vec)
+                mm_tile_simt_kernel<Tin, 16, 16, kFlatTileBK * 2, true><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m,
+                                                                                          a.p, ceil_div(kps, 2));
+            else
+                mm_tile_simt_kernel<Tin, 16, 16, kFlatTileBK * 2, false><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m,
+                                                                                           a.p, ceil_div(kps, 2));
+        } else if (vec) {
+            mm_tile_simt_kernel<Tin, kFlatTileBM, kFlatTileBM, kFlatTileBK, true>
+                <<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
+        } else {
+            mm_tile_simt_kernel<Tin, kFlatTileBM, kFlatTileBM, kFlatTileBK, false>
+                <<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
+        }
         cudaError_t e = cudaGetLastError();
-        if (e != cudaSuccess || nsplit == 1) return e;
-        mm_flat_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 8), 256, 0, a.stream>>>(part, a.C, outs,
-                                                                                                       nsplit);
+        if (e != cudaSuccess || splits == 1) return e;
+        mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, a.stream>>>(
+            part, a.C, outs, (int)splits);
         return cudaGetLastError();
     }
-    if (version == 1) {
+    if (version == 1) {  // ---- V_MIDDLE: a warp per output
         const int64_t grid = ceil_div(outs, 8);
         if (vec) mm_mid_kernel<Tin, true><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
         else mm_mid_kernel<Tin, false><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
         return cudaGetLastError();
     }
-    // V_TOP
-    if constexpr (std::is_same<Tin, __nv_bfloat16>::value) {
-        if (tc_shape_ok(a.n, a.m, a.p, A, Bt)) return launch_mm_top_tc(A, Bt, a.C, a.n, a.m, a.p, a.stream);
-    }
-    dim3 g((unsigned)ceil_div(a.p, TBN), (unsigned)ceil_div(a.n, TBM));
-    if (vec) mm_top_simt_kernel<Tin, true><<<g, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
-    else mm_top_simt_kernel<Tin, false><<<g, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+    // ---- V_TOP: output tiles, sequential k (tensor cores for bf16)
+    if (tc) return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, false), a.stream);
+    // SIMT TOP: 128x128 tiles; when the tile grid leaves SMs idle, k is split
+    // into >= 64-tile chunks (each CTA still walks its chunk sequentially)
+    const int64_t tiles = ceil_div(a.n, 128) * ceil_div(a.p, 128), nk = ceil_div(a.m, 16);
+    const int64_t s = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / tiles, nk / 64));
+    const int64_t kps = ceil_div(nk, s), splits = ceil_div(nk, kps);
+    dim3 g((unsigned)ceil_div(a.p, 128), (unsigned)ceil_div(a.n, 128), (unsigned)splits);
+    if (vec) mm_tile_simt_kernel<Tin, 128, 128, 16, true><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
+    else mm_tile_simt_kernel<Tin, 128, 128, 16, false><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess || splits == 1) return e;
+    mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, a.stream>>>(part, a.C, outs,
+                                                                                                   (int)splits);
     return cudaGetLastError();
 }
 

@@ -16,6 +16,7 @@
 #include <cuda.h>
 #include <cuda_bf16.h>
 
+#include <algorithm>
 #include <mutex>
 
 #include "common.cuh"
@@ -89,16 +90,21 @@ __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, uint32_t (&r)
 
 // ------------------------------------------------------------------ kernel
 
+// blockIdx.z = k-split: the CTA accumulates k-tiles [z*kps, (z+1)*kps) and
+// writes its fp32 tile to C (one split) or to part[z] (split-K, summed by
+// mm_splitk_finalize in a fixed order).
 __global__ void __launch_bounds__(128, 1) mm_top_tc_kernel(const __grid_constant__ CUtensorMap mapA,
                                                            const __grid_constant__ CUtensorMap mapB, float* C,
-                                                           int64_t n, int64_t m, int64_t p) {
+                                                           float* part, int64_t n, int64_t m, int64_t p, int kps) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
     __shared__ alignas(8) uint64_t full[TC_STAGES], empty[TC_STAGES], done;
     __shared__ uint32_t tmem_base;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int m0 = blockIdx.y * TC_BM, n0 = blockIdx.x * TC_BN;
-    const int nk = (int)ceil_div(m, TC_BK);
+    const int kt0 = blockIdx.z * kps;
+    const int nk = min(kps, (int)ceil_div(m, TC_BK) - kt0);
+    float* out = gridDim.z == 1 ? C : part + (int64_t)blockIdx.z * n * p;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < TC_STAGES; ++s) {
@@ -130,8 +136,8 @@ __global__ void __launch_bounds__(128, 1) mm_top_tc_kernel(const __grid_constant
             uint8_t* sa = smem + s * TC_STAGE_BYTES;
             uint8_t* sb = sa + TC_A_BYTES;
             mbar_arrive_expect_tx(&full[s], TC_STAGE_BYTES);
-            tma_load_2d(sa, &mapA, kt * TC_BK, m0, &full[s]);
-            tma_load_2d(sb, &mapB, kt * TC_BK, n0, &full[s]);
+            tma_load_2d(sa, &mapA, (kt0 + kt) * TC_BK, m0, &full[s]);
+            tma_load_2d(sb, &mapB, (kt0 + kt) * TC_BK, n0, &full[s]);
         }
     } else if (warp == 1 && lane == 0) {
         // ---- MMA issuer
@@ -154,29 +160,26 @@ __global__ void __launch_bounds__(128, 1) mm_top_tc_kernel(const __grid_constant
     }
     __syncwarp();
 
-    // ---- epilogue: TMEM -> registers -> C
+    // ---- epilogue: TMEM -> registers -> padded smem (the drained ring) ->
+    // row-contiguous, coalesced stores (a warp writes 32 consecutive columns
+    // of one row per instruction)
     mbar_wait(&done, 0);
     __syncwarp();
     tc_fence_after();
-    const int64_t row = m0 + warp * 32 + lane;
+    float* stage = reinterpret_cast<float*>(smem) + warp * (32 * 33);
 #pragma unroll 1
     for (int c = 0; c < TC_BN; c += 32) {
         uint32_t r[32];
         tmem_ld_32x32b_x32(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c, r);
-        if (row < n) {
-            float* dst = C + row * p + n0 + c;
-            const int64_t ncol = p - (n0 + c);
-            if (ncol >= 32 && ((uintptr_t)dst % 16 == 0)) {
 #pragma unroll
-                for (int q = 0; q < 8; ++q)
-                    *reinterpret_cast<float4*>(dst + 4 * q) =
-                        make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]),
-                                    __uint_as_float(r[4 * q + 2]), __uint_as_float(r[4 * q + 3]));
-            } else {
-                for (int q = 0; q < 32; ++q)
-                    if (q < ncol) dst[q] = __uint_as_float(r[q]);
-            }
+        for (int q = 0; q < 32; ++q) stage[lane * 33 + q] = __uint_as_float(r[q]);
+        __syncwarp();
+        const int64_t col = (int64_t)n0 + c + lane;
+        for (int rr = 0; rr < 32; ++rr) {
+            const int64_t row = (int64_t)m0 + warp * 32 + rr;
+            if (row < n && col < p) out[row * p + col] = stage[rr * 33 + lane];
         }
+        __syncwarp();
     }
     tc_fence_before();
     __syncthreads();
@@ -222,16 +225,44 @@ bool tc_shape_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* Bt)
            n < (1ll << 31) && p < (1ll << 31) && m < (1ll << 31) && encode_fn() != nullptr;
 }
 
-cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, int64_t n, int64_t m, int64_t p,
-                             cudaStream_t s) {
+__global__ void mm_splitk_finalize(const float* __restrict__ part, float* __restrict__ C, int64_t outs, int splits) {
+    for (int64_t o = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; o < outs; o += (int64_t)gridDim.x * blockDim.x) {
+        float r = 0.f;
+        for (int s = 0; s < splits; ++s) r += part[(int64_t)s * outs + o];
+        C[o] = r;
+    }
+}
+
+// splits: 1 = plain TOP tile; >1 = k split across CTAs (ws holds the partial
+// tiles).  tc_splits() picks them: TOP only fills idle SMs (>= 8 k-tiles per
+// split); FLAT (segred over all three levels) splits as far as 2 CTAs per SM.
+int tc_splits(int64_t n, int64_t m, int64_t p, bool flat) {
+    const int64_t tiles = ceil_div(n, TC_BM) * ceil_div(p, TC_BN);
+    const int64_t nk = ceil_div(m, TC_BK);
+    int64_t s = flat ? ceil_div((int64_t)296, tiles) : (int64_t)148 / tiles;
+    const int64_t cap = flat ? nk : std::max<int64_t>(1, nk / 8);
+    s = std::max<int64_t>(1, std::min(s, cap));
+    const int64_t kps = ceil_div(nk, s);
+    return (int)ceil_div(nk, kps);
+}
+
+cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* part, int64_t n, int64_t m, int64_t p,
+                             int splits, cudaStream_t s) {
     CUtensorMap ma, mb;
     if (!make_map(&ma, A, n, m, TC_BM) || !make_map(&mb, Bt, p, m, TC_BN)) return cudaErrorInvalidValue;
     static std::once_flag once;
     std::call_once(once, [] {
         cudaFuncSetAttribute(mm_top_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM);
     });
-    dim3 g((unsigned)ceil_div(p, TC_BN), (unsigned)ceil_div(n, TC_BM));
-    mm_top_tc_kernel<<<g, 128, TC_SMEM, s>>>(ma, mb, C, n, m, p);
+    const int nk = (int)ceil_div(m, TC_BK);
+    const int kps = (int)ceil_div(nk, splits);
+    splits = (int)ceil_div(nk, kps);
+    dim3 g((unsigned)ceil_div(p, TC_BN), (unsigned)ceil_div(n, TC_BM), (unsigned)splits);
+    mm_top_tc_kernel<<<g, 128, TC_SMEM, s>>>(ma, mb, C, part, n, m, p, kps);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess || splits == 1) return e;
+    const int64_t outs = n * p;
+    mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, s>>>(part, C, outs, splits);
     return cudaGetLastError();
 }
 
