@@ -290,7 +290,7 @@ def tridag(a, b, c, y, version="auto", out=None, ws=None, stream=None, return_ch
             raise TypeError("tridag takes contiguous float32 tensors")
     if out is None:
         out = torch.empty_like(y)
-    wb = lib().ifl_workspace_bytes(b"tridag", S, L, 0, 1, VERSIONS[version])
+    wb = lib().ifl_workspace_bytes(b"tridag", S, L, R, 1, VERSIONS[version])
     if ws is None and wb:
         ws = workspace(wb, y.device, "tridag")
     ch = ifl_choice()

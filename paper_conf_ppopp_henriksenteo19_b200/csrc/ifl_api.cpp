@@ -249,7 +249,7 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
         return 0;
     }
     if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
-    if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(n, m, version);
+    if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
     return 0;
 }
 
@@ -349,7 +349,7 @@ int ifl_tridag(const float* a, const float* b, const float* c, const float* y, f
     if (ch.version == IFL_V_MIDDLE && !fits)
         return fail(IFL_ENOTFIT, "ifl_tridag: V_MIDDLE does not fit L=%lld in shared memory", (long long)L);
     if (S * L == 0) return IFL_OK;
-    const size_t need = ifl::tridag_ws_bytes(S, L, ch.version);
+    const size_t need = ifl::tridag_ws_bytes(coef_rows, L, ch.version);
     if (need && (!ws || ws_bytes < need))
         return fail(IFL_EWORKSPACE, "ifl_tridag: needs %zu workspace bytes, got %zu", need, ws_bytes);
     ifl::TriArgs t{a, b, c, y, x, S, L, coef_rows, ws, ws_bytes, (cudaStream_t)stream};

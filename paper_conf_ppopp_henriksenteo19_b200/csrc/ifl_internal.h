@@ -61,7 +61,7 @@ struct TriArgs {
     size_t ws_bytes;
     cudaStream_t stream;
 };
-size_t tridag_ws_bytes(int64_t S, int64_t L, int version);
+size_t tridag_ws_bytes(int64_t coef_rows, int64_t L, int version);
 bool tridag_mid_fits(int64_t L);
 cudaError_t launch_tridag(int version, const TriArgs& a);
 

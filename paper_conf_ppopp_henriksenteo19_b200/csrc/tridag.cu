@@ -1,8 +1,386 @@
-// tridag.cu -- placeholder, filled in below.
+// tridag.cu -- batched tridiagonal solves as three scans (LocVolCalib,
+// P:400-420; Fig 6b "tridag as = scan (+) . scan (x) . scan (.)"), in the three
+// versions Fig 6c shows:
+//   V_TOP    segmap^1 <xs> (tridag xs): one thread per system, the scans run
+//            sequentially (they are then just the Thomas recurrences);
+//   V_MIDDLE segmap^1 <xs> (segscan^0 ...): a thread group per system, all
+//            three scans in registers / shared memory (needs the system to
+//            fit: the A-fit clause of P:358);
+//   V_FLAT   three segscan^1 over the flattened S*L array in global memory:
+//            y' is written out by the forward scan and read back by the
+//            backward one ("at least two global accesses per element for each
+//            scan").
+// The paper does not give the operators; reading R8:
+//   (+)  2x2 matrix products, M_j = [[b_j, -a_j c_{j-1}], [1, 0]]; with
+//        P_j = M_j...M_0 the eliminated diagonal is beta_j = P_j[0][0] /
+//        P_j[1][0]; every product is renormalised (scale-invariant ratio);
+//   (x)  affine maps y'_j = alpha_j y'_{j-1} + y_j, alpha_j = -a_j / beta_{j-1};
+//   (.)  reversed affine maps x_j = delta_j x_{j+1} + y'_j / beta_j,
+//        delta_j = -c_j / beta_j.
+// Coefficients are [R][L], shared by every system s with s % R == r (R9), so
+// the (+) scan runs once per coefficient row into the workspace (invbeta,
+// alpha, delta), and the per-system work is the two affine scans.  alpha_0 = 0
+// and delta_{L-1} = 0, so the affine scans reset at system boundaries on their
+// own: the flattened scans need no segment flags.
+#include <algorithm>
+
 #include "common.cuh"
 #include "ifl_internal.h"
+
 namespace ifl {
-size_t tridag_ws_bytes(int64_t, int64_t, int) { return 0; }
-bool tridag_mid_fits(int64_t L) { return L <= 4096; }
-cudaError_t launch_tridag(int, const TriArgs&) { return cudaErrorNotSupported; }
+
+// ------------------------------------------------------------ operators
+
+struct Aff {  // x -> a*x + g
+    float a, g;
+};
+// compose: newer o older
+__device__ __forceinline__ Aff aff_after(Aff newer, Aff older) {
+    return {newer.a * older.a, fmaf(newer.a, older.g, newer.g)};
+}
+
+struct Mat2 {
+    float m00, m01, m10, m11;
+};
+__device__ __forceinline__ Mat2 mat_mul(Mat2 y, Mat2 x) {  // y * x (newer on the left)
+    Mat2 r{fmaf(y.m00, x.m00, y.m01 * x.m10), fmaf(y.m00, x.m01, y.m01 * x.m11),
+           fmaf(y.m10, x.m00, y.m11 * x.m10), fmaf(y.m10, x.m01, y.m11 * x.m11)};
+    const float s = fabsf(r.m00) + fabsf(r.m01) + fabsf(r.m10) + fabsf(r.m11);
+    const float inv = s > 0.f ? 1.0f / s : 1.0f;
+    return {r.m00 * inv, r.m01 * inv, r.m10 * inv, r.m11 * inv};
+}
+__device__ __forceinline__ Mat2 mat_id() { return {1.f, 0.f, 0.f, 1.f}; }
+
+// ------------------------------------------------- scan (+): coefficients
+
+// V_TOP: one thread per coefficient row, sequential (the Thomas recurrence).
+__global__ void tridag_coef_seq(const float* __restrict__ a, const float* __restrict__ b, const float* __restrict__ c,
+                                float* __restrict__ invb, float* __restrict__ alpha, float* __restrict__ delta,
+                                int64_t R, int64_t L) {
+    for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < R; r += (int64_t)gridDim.x * blockDim.x) {
+        const float* ar = a + r * L;
+        const float* br = b + r * L;
+        const float* cr = c + r * L;
+        float beta = br[0];
+        alpha[r * L] = 0.f;
+        for (int64_t j = 0; j < L; ++j) {
+            if (j > 0) {
+                const float al = -ar[j] / beta;
+                alpha[r * L + j] = al;
+                beta = fmaf(al, cr[j - 1], br[j]);  // b_j - a_j c_{j-1} / beta_{j-1}
+            }
+            invb[r * L + j] = 1.0f / beta;
+            delta[r * L + j] = j + 1 < L ? -cr[j] / beta : 0.f;
+        }
+    }
+}
+
+// V_MIDDLE / V_FLAT: a CTA per coefficient row, the normalised 2x2 matrix
+// scan of the paper's first scan, in shared memory.  256 threads, each a
+// contiguous run of ceil(L/256) rows.
+__global__ void __launch_bounds__(256) tridag_coef_mat2(const float* __restrict__ a, const float* __restrict__ b,
+                                                        const float* __restrict__ c, float* __restrict__ invb,
+                                                        float* __restrict__ alpha, float* __restrict__ delta,
+                                                        int64_t L) {
+    __shared__ Mat2 wsum[8];
+    __shared__ float sbeta_prev[257];
+    const int64_t r = blockIdx.x;
+    const float* ar = a + r * L;
+    const float* br = b + r * L;
+    const float* cr = c + r * L;
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int64_t per = ceil_div(L, 256);
+    const int64_t j0 = t * per, j1 = std::min(L, j0 + per);
+    auto Mj = [&](int64_t j) -> Mat2 {
+        return j == 0 ? Mat2{br[0], 0.f, 1.f, 0.f} : Mat2{br[j], -ar[j] * cr[j - 1], 1.f, 0.f};
+    };
+    // thread aggregate (product of its run, newer on the left)
+    Mat2 agg = mat_id();
+    for (int64_t j = j0; j < j1; ++j) agg = mat_mul(Mj(j), agg);
+    // inclusive warp scan, then across warps
+    Mat2 inc = agg;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        Mat2 o{__shfl_up_sync(0xffffffffu, inc.m00, off), __shfl_up_sync(0xffffffffu, inc.m01, off),
+               __shfl_up_sync(0xffffffffu, inc.m10, off), __shfl_up_sync(0xffffffffu, inc.m11, off)};
+        if (lane >= off) inc = mat_mul(inc, o);
+    }
+    if (lane == 31) wsum[w] = inc;
+    Mat2 ex{__shfl_up_sync(0xffffffffu, inc.m00, 1), __shfl_up_sync(0xffffffffu, inc.m01, 1),
+            __shfl_up_sync(0xffffffffu, inc.m10, 1), __shfl_up_sync(0xffffffffu, inc.m11, 1)};
+    if (lane == 0) ex = mat_id();
+    __syncthreads();
+    Mat2 pre = mat_id();
+    for (int k = 0; k < w; ++k) pre = mat_mul(wsum[k], pre);
+    ex = mat_mul(ex, pre);
+    // walk the run: P_j = M_j ... M_0, beta_j = P_j[0][0] / P_j[1][0]
+    Mat2 P = ex;
+    float beta_last = 0.f;
+    for (int64_t j = j0; j < j1; ++j) {
+        P = mat_mul(Mj(j), P);
+        const float beta = P.m00 / P.m10;
+        invb[r * L + j] = 1.0f / beta;
+        delta[r * L + j] = j + 1 < L ? -cr[j] / beta : 0.f;
+        beta_last = beta;
+    }
+    sbeta_prev[t + 1] = beta_last;  // beta at the end of this thread's run
+    __syncthreads();
+    // alpha_j = -a_j / beta_{j-1}: the first item of a run needs the previous run's beta
+    for (int64_t j = j0; j < j1; ++j) {
+        float bprev;
+        if (j == 0) {
+            alpha[r * L] = 0.f;
+            continue;
+        }
+        if (j == j0) {
+            int q = t;  // nearest preceding non-empty run
+            while (q > 0 && (int64_t)(q - 1) * per >= L) --q;
+            bprev = sbeta_prev[q];
+        } else {
+            bprev = 1.0f / invb[r * L + j - 1];
+        }
+        alpha[r * L + j] = -ar[j] / bprev;
+    }
+}
+
+// ---------------------------------------------------------------- V_TOP
+
+// One thread per system; the forward scan stores y' into x, the backward
+// scan overwrites it with x.  Coefficient arrays are tiny and L2-resident.
+__global__ void __launch_bounds__(256) tridag_top_kernel(const float* __restrict__ y, float* __restrict__ x,
+                                                         const float* __restrict__ invb, const float* __restrict__ alpha,
+                                                         const float* __restrict__ delta, int64_t S, int64_t L,
+                                                         int64_t R) {
+    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < S; s += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = s % R;
+        const float* ys = y + s * L;
+        float* xs = x + s * L;
+        const float* al = alpha + r * L;
+        const float* ib = invb + r * L;
+        const float* de = delta + r * L;
+        float v = 0.f;
+        for (int64_t j = 0; j < L; ++j) {  // (x): y'_j = alpha_j y'_{j-1} + y_j
+            v = fmaf(__ldg(al + j), v, __ldg(ys + j));
+            xs[j] = v;
+        }
+        float u = 0.f;
+        for (int64_t j = L - 1; j >= 0; --j) {  // (.): x_j = delta_j x_{j+1} + y'_j / beta_j
+            u = fmaf(__ldg(de + j), u, xs[j] * __ldg(ib + j));
+            xs[j] = u;
+        }
+    }
+}
+
+// ------------------------------------------------------------- V_MIDDLE
+
+constexpr int kTriItems = 4;
+
+// Group-wide exclusive scan of affine maps (older lanes first).  G threads
+// per group; G <= 32 uses shuffles only, larger groups go through shared
+// memory (warp totals).  REV scans from the last lane backwards.
+template <bool REV>
+__device__ __forceinline__ Aff group_exscan(Aff v, int G, Aff* wtot, Aff& total) {
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int width = G < 32 ? G : 32;
+    const int gl = threadIdx.x % width;
+    Aff inc = v;
+    for (int off = 1; off < width; off <<= 1) {
+        const float oa = REV ? __shfl_down_sync(0xffffffffu, inc.a, off, width) : __shfl_up_sync(0xffffffffu, inc.a, off, width);
+        const float og = REV ? __shfl_down_sync(0xffffffffu, inc.g, off, width) : __shfl_up_sync(0xffffffffu, inc.g, off, width);
+        const bool ok = REV ? (gl + off < width) : (gl >= off);
+        if (ok) inc = aff_after(inc, Aff{oa, og});
+    }
+    Aff ex;
+    ex.a = REV ? __shfl_down_sync(0xffffffffu, inc.a, 1, width) : __shfl_up_sync(0xffffffffu, inc.a, 1, width);
+    ex.g = REV ? __shfl_down_sync(0xffffffffu, inc.g, 1, width) : __shfl_up_sync(0xffffffffu, inc.g, 1, width);
+    const bool first = REV ? (gl == width - 1) : (gl == 0);
+    if (first) ex = Aff{1.f, 0.f};
+    if (G <= 32) {
+        const int src = REV ? 0 : width - 1;
+        total = Aff{__shfl_sync(0xffffffffu, inc.a, src, width), __shfl_sync(0xffffffffu, inc.g, src, width)};
+        return ex;
+    }
+    const int wpg = G >> 5, w0 = (threadIdx.x / G) * wpg;
+    if (REV ? lane == 0 : lane == 31) wtot[w] = inc;
+    __syncthreads();
+    Aff before{1.f, 0.f};
+    total = Aff{1.f, 0.f};
+    for (int k = 0; k < wpg; ++k) {
+        const int kk = REV ? (wpg - 1 - k) : k;  // oldest first
+        const Aff t = wtot[w0 + kk];
+        if (REV ? (w0 + kk > w) : (w0 + kk < w)) before = aff_after(t, before);
+        total = aff_after(t, total);
+    }
+    __syncthreads();
+    return aff_after(ex, before);
+}
+
+int tridag_group(int64_t L) {
+    int64_t g = 1;
+    while (g < 256 && g * kTriItems < L) g <<= 1;
+    return (int)std::max<int64_t>(g, 1);
+}
+
+template <int IT>
+__global__ void __launch_bounds__(256) tridag_mid_kernel(const float* __restrict__ y, float* __restrict__ x,
+                                                         const float* __restrict__ invb, const float* __restrict__ alpha,
+                                                         const float* __restrict__ delta, int64_t S, int64_t L,
+                                                         int64_t R, int G) {
+    __shared__ Aff wtot[8];
+    const int g = threadIdx.x % G;
+    const int64_t s = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
+    const bool live = s < S;
+    const int64_t r = live ? s % R : 0;
+    const float* ys = y + (live ? s * L : 0);
+    float* xs = x + (live ? s * L : 0);
+    const int64_t j0 = (int64_t)g * IT;
+    float yv[IT], al[IT], ib[IT], de[IT];
+#pragma unroll
+    for (int k = 0; k < IT; ++k) {
+        const int64_t j = j0 + k;
+        const bool ok = live && j < L;
+        yv[k] = ok ? __ldg(ys + j) : 0.f;
+        al[k] = ok ? __ldg(alpha + r * L + j) : 1.f;
+        ib[k] = ok ? __ldg(invb + r * L + j) : 0.f;
+        de[k] = ok ? __ldg(delta + r * L + j) : 1.f;
+    }
+    // (x) forward: thread composite of its items, group exclusive prefix, apply
+    Aff f{1.f, 0.f};
+#pragma unroll
+    for (int k = 0; k < IT; ++k) f = aff_after(Aff{al[k], yv[k]}, f);
+    Aff tot;
+    const Aff pf = group_exscan<false>(f, G, wtot, tot);
+    float v = pf.g;  // y' before this thread's first item (the prefix applied to 0)
+#pragma unroll
+    for (int k = 0; k < IT; ++k) {
+        v = fmaf(al[k], v, yv[k]);
+        yv[k] = v * ib[k];  // epsilon_j = y'_j / beta_j
+    }
+    // (.) backward
+    Aff bk{1.f, 0.f};
+#pragma unroll
+    for (int k = IT - 1; k >= 0; --k) bk = aff_after(Aff{de[k], yv[k]}, bk);
+    const Aff pb = group_exscan<true>(bk, G, wtot, tot);
+    float u = pb.g;
+#pragma unroll
+    for (int k = IT - 1; k >= 0; --k) {
+        u = fmaf(de[k], u, yv[k]);
+        yv[k] = u;
+    }
+#pragma unroll
+    for (int k = 0; k < IT; ++k)
+        if (live && j0 + k < L) xs[j0 + k] = yv[k];
+}
+
+bool tridag_mid_fits(int64_t L) { return L >= 1 && L <= 256 * 16; }
+
+// --------------------------------------------------------------- V_FLAT
+
+// One affine scan over the flattened S*L array.  A CTA takes a tile of whole
+// systems (tile = L * floor(4096 / L), or one system when L > 4096), 256
+// threads each a contiguous run; the CTA scans the thread composites (no
+// segment flags: alpha_0 = 0 / delta_{L-1} = 0 reset the maps).
+// FWD: y'_j = alpha_j y'_{j-1} + y_j   (reads y, writes y' into x)
+// BWD: x_j = delta_j x_{j+1} + y'_j / beta_j   (reads and writes x)
+template <bool FWD>
+__global__ void __launch_bounds__(256) tridag_flat_kernel(const float* __restrict__ y, float* __restrict__ x,
+                                                          const float* __restrict__ invb,
+                                                          const float* __restrict__ alpha,
+                                                          const float* __restrict__ delta, int64_t S, int64_t L,
+                                                          int64_t R, int64_t sys_per_tile) {
+    __shared__ Aff wtot[8];
+    const int64_t s0 = (int64_t)blockIdx.x * sys_per_tile;
+    const int64_t nsys = std::min(sys_per_tile, S - s0);
+    const int64_t base = s0 * L, cnt = nsys * L;
+    const int64_t per = ceil_div(cnt, 256);
+    const int64_t e0 = threadIdx.x * per, e1 = std::min(cnt, e0 + per);
+    auto coef = [&](int64_t e, float& m, float& add) {  // map of flat element base+e
+        const int64_t gi = base + e;
+        const int64_t s = gi / L, j = gi - s * L, r = s % R;
+        if (FWD) {
+            m = __ldg(alpha + r * L + j);
+            add = __ldg(y + gi);
+        } else {
+            m = __ldg(delta + r * L + j);
+            add = x[gi] * __ldg(invb + r * L + j);
+        }
+    };
+    Aff f{1.f, 0.f};
+    if (FWD) {
+        for (int64_t e = e0; e < e1; ++e) {
+            float m, ad;
+            coef(e, m, ad);
+            f = aff_after(Aff{m, ad}, f);
+        }
+    } else {
+        for (int64_t e = e1 - 1; e >= e0; --e) {
+            float m, ad;
+            coef(e, m, ad);
+            f = aff_after(Aff{m, ad}, f);
+        }
+    }
+    Aff tot;
+    const Aff pf = group_exscan<!FWD>(f, 256, wtot, tot);
+    float v = pf.g;
+    if (FWD) {
+        for (int64_t e = e0; e < e1; ++e) {
+            float m, ad;
+            coef(e, m, ad);
+            v = fmaf(m, v, ad);
+            x[base + e] = v;
+        }
+    } else {
+        for (int64_t e = e1 - 1; e >= e0; --e) {
+            float m, ad;
+            coef(e, m, ad);
+            v = fmaf(m, v, ad);
+            x[base + e] = v;
+        }
+    }
+}
+
+// ------------------------------------------------------------------ launch
+
+// invbeta, alpha, delta: one float each per coefficient element ([R][L])
+size_t tridag_ws_bytes(int64_t R, int64_t L, int version) {
+    (void)version;
+    return (size_t)R * L * 3 * sizeof(float);
+}
+
+cudaError_t launch_tridag(int version, const TriArgs& t) {
+    const int64_t R = t.coef_rows, L = t.L, S = t.S;
+    float* invb = (float*)t.ws;
+    float* alpha = invb + R * L;
+    float* delta = alpha + R * L;
+    cudaError_t e;
+    if (version == 0) {
+        const int g = (int)std::min<int64_t>(ceil_div(R, 128), 148 * 8);
+        tridag_coef_seq<<<g, 128, 0, t.stream>>>(t.a, t.b, t.c, invb, alpha, delta, R, L);
+    } else {
+        tridag_coef_mat2<<<(unsigned)R, 256, 0, t.stream>>>(t.a, t.b, t.c, invb, alpha, delta, L);
+    }
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    if (version == 0) {
+        const int g = (int)std::min<int64_t>(ceil_div(S, 256), 148 * 16);
+        tridag_top_kernel<<<g, 256, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R);
+        return cudaGetLastError();
+    }
+    if (version == 1) {
+        const int G = tridag_group(L);
+        const int B = std::max(G, 32) > 256 ? G : 256;
+        const int64_t grid = ceil_div(S, B / G);
+        const int64_t it = ceil_div(L, G);
+        if (it <= 4) tridag_mid_kernel<4><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
+        else if (it <= 8) tridag_mid_kernel<8><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
+        else tridag_mid_kernel<16><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
+        return cudaGetLastError();
+    }
+    const int64_t spt = std::max<int64_t>(1, 4096 / L);
+    const int64_t grid = ceil_div(S, spt);
+    tridag_flat_kernel<true><<<(unsigned)grid, 256, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, spt);
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    tridag_flat_kernel<false><<<(unsigned)grid, 256, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, spt);
+    return cudaGetLastError();
+}
+
 }  // namespace ifl

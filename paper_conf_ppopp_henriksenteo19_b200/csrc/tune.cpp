@@ -111,7 +111,7 @@ size_t ws_bytes_of(Kind k, const int64_t* s) {
     case K_SEGSCAN: return ifl_workspace_bytes("segscan", s[0], s[1], 0, IFL_F32, -1);
     case K_MM_F32: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_F32, -1);
     case K_MM_BF16: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_BF16, -1);
-    case K_TRIDAG: return ifl_workspace_bytes("tridag", s[0], s[1], 0, IFL_F32, -1);
+    case K_TRIDAG: return ifl_workspace_bytes("tridag", s[0], s[1], s[2], IFL_F32, -1);
     default: return 0;
     }
 }
@@ -136,7 +136,7 @@ size_t shape_bytes(Kind k, const int64_t* s) {
     case K_TRIDAG: {
         const int64_t S = s[0], L = s[1], R = s[2];
         return 3 * align256(R * L * 4) + 2 * align256(S * L * 4) +
-               align256(ifl_workspace_bytes("tridag", S, L, 0, IFL_F32, -1));
+               align256(ifl_workspace_bytes("tridag", S, L, R, IFL_F32, -1));
     }
     default: return 0;
     }
@@ -180,7 +180,7 @@ int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_
         char* x = y + align256(S * L * 4);
         char* ws = x + align256(S * L * 4);
         return ifl_tridag((float*)a, (float*)b, (float*)c, (float*)y, (float*)x, S, L, R, version, ws,
-                          ifl_workspace_bytes("tridag", S, L, 0, IFL_F32, -1), st, nullptr);
+                          ifl_workspace_bytes("tridag", S, L, R, IFL_F32, -1), st, nullptr);
     }
     default: return IFL_EINVAL;
     }
