@@ -1,0 +1,123 @@
+"""Multi-GPU layer: rule G3 lifted to a third hardware level,
+l = 2 = devices.  The paper is single-GPU; it notes the rules apply to
+other heterogeneous hardware.
+
+One process per GPU, ``torch.distributed`` for the plumbing (NCCL over
+NVLink on B200, gloo for the CPU tests).  For segred over an [n][m] array
+the device-level guard is ``n >= t_dev`` (Par over devices = n):
+
+  * outer split (n >= t_dev): rank r owns rows [r*ceil(n/G), ...) and runs
+    the single-GPU selector on its block -- independent units, NO collective
+    on the data path (``all_gather`` only if the caller wants the full
+    result replicated);
+  * inner split (n < t_dev): rank r owns columns [r*m/G, (r+1)*m/G) of every
+    row; the local segred runs WITHOUT d (canonical neutral element), one
+    ``all_reduce``/``reduce`` of the n partials combines them -- the one real
+    exchange step -- and d is applied once, after the collective.
+
+Bitwise operators have no NCCL reduction: partials are all-gathered and
+combined with the library's own segred over the [n][G] partial matrix.
+redomap2 splits the rows of A (B replicated) and tridag the systems: both
+are outer splits without a collective.
+
+The local computation is injectable (``local_segred``) so the host logic
+(plans, collectives, d handling) is tested with world size 2 on gloo/CPU.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import torch
+import torch.distributed as td
+
+_REDUCE = {"sum": td.ReduceOp.SUM, "prod": td.ReduceOp.PRODUCT, "min": td.ReduceOp.MIN, "max": td.ReduceOp.MAX,
+           "and": td.ReduceOp.BAND, "or": td.ReduceOp.BOR, "xor": td.ReduceOp.BXOR}
+_BITWISE = ("and", "or", "xor")
+
+
+@dataclass
+class Plan:
+    mode: str        # "outer" or "inner"
+    lo: int          # first owned row (outer) or column (inner)
+    hi: int          # one past the last owned row / column
+
+
+def plan_segred(n: int, m: int, world: int, rank: int, t_dev: int | None = None) -> Plan:
+    """Device-level G3 guard: split rows when there are >= t_dev of them
+    (default: the number of devices), else split every row's columns."""
+    t_dev = world if t_dev is None else t_dev
+    if n >= t_dev:
+        per = -(-n // world)
+        lo = min(n, rank * per)
+        return Plan("outer", lo, min(n, lo + per))
+    lo = (m * rank) // world
+    return Plan("inner", lo, (m * (rank + 1)) // world)
+
+
+def _default_local(x: torch.Tensor, op: str, f: str, ne):
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.segred(x, op, f, ne=ne)
+
+
+def _apply_ne(partial: torch.Tensor, op: str, ne, local_segred):
+    """out[i] = d (+) partial[i]: a segred over [n][1] with neutral element d."""
+    if ne is None:
+        return partial
+    return local_segred(partial.reshape(-1, 1).contiguous(), op, "id", ne)
+
+
+def segred_dist(x_block: torch.Tensor, n: int, m: int, op: str = "sum", f: str = "id", ne=None,
+                plan: Plan | None = None, group=None, gather: bool = False, local_segred=None,
+                gather_partials: bool | None = None) -> torch.Tensor:
+    """Distributed segred.  ``x_block`` is this rank's block: rows
+    [plan.lo, plan.hi) x all m columns (outer) or all n rows x columns
+    [plan.lo, plan.hi) (inner).  Returns this rank's rows of the result
+    (outer; all rows if ``gather``) or the full [n] result on every rank
+    (inner)."""
+    local = local_segred or _default_local
+    world = td.get_world_size(group)
+    rank = td.get_rank(group)
+    plan = plan or plan_segred(n, m, world, rank)
+    if plan.mode == "outer":
+        out = local(x_block, op, f, ne)
+        if not gather:
+            return out
+        per = -(-n // world)
+        buf = torch.empty(per * world, dtype=out.dtype, device=out.device)
+        padded = torch.empty(per, dtype=out.dtype, device=out.device)
+        padded[: out.numel()] = out
+        td.all_gather_into_tensor(buf, padded, group=group)
+        return buf[:n]
+    # inner split: partials without d, one exchange, then d once
+    part = local(x_block, op, f, None)
+    if gather_partials is None:
+        gather_partials = op in _BITWISE and td.get_backend(group) == "nccl"
+    if gather_partials:
+        allp = torch.empty(world * n, dtype=part.dtype, device=part.device)
+        td.all_gather_into_tensor(allp, part.contiguous(), group=group)
+        stacked = allp.view(world, n).t().contiguous()  # [n][G] partials, rank order
+        total = local(stacked, op, "id", None)
+    else:
+        total = part.clone()
+        td.all_reduce(total, op=_REDUCE[op], group=group)
+    return _apply_ne(total, op, ne, local)
+
+
+def rows_of(n: int, world: int, rank: int):
+    per = -(-n // world)
+    lo = min(n, rank * per)
+    return lo, min(n, lo + per)
+
+
+def redomap2_dist(A_rows: torch.Tensor, B: torch.Tensor, **kw) -> torch.Tensor:
+    """Row split of A (B replicated): independent output row blocks."""
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.redomap2(A_rows, B, **kw)
+
+
+def tridag_dist(a, b, c, y_rows: torch.Tensor, **kw) -> torch.Tensor:
+    """System split: independent systems.  The caller passes the systems
+    s in [lo, hi) with lo a multiple of coef_rows (rows_of keeps that when
+    the per-rank count is a multiple of it) so that s % R is preserved."""
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.tridag(a, b, c, y_rows, **kw)

@@ -1,0 +1,101 @@
+"""Multi-process (world size 2, gloo, CPU) tests of the device-level split of
+dist.py: plans, the single exchange step of the inner split, d applied once
+after the collective, and the all-gather path used for bitwise operators.
+The per-rank local segred is the CPU oracle here (tests may use it); on the
+GPU box the same host logic calls the CUDA library."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as td
+import torch.multiprocessing as mp
+
+import ifl_inputs as gen
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _oracle_local(x, op, f, ne):
+    """Stands in for the GPU segred: same dtype in and out (f32 partials)."""
+    import oracle
+    xn = x.numpy()
+    if xn.dtype == np.float64:
+        xn = xn.astype(np.float32)
+    r = oracle.segred(xn, op, f, ne)
+    if r.dtype == np.float64:
+        r = r.astype(np.float32)
+    return torch.from_numpy(np.ascontiguousarray(r))
+
+
+def _worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    td.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    import oracle
+    results = []
+    try:
+        cases = [("I32_FULL", op) for op in ("sum", "prod", "min", "max", "and", "or", "xor")] + \
+                [("F32_EXACT", "sum"), ("F32_SIGNED", "max")]
+        for (n, m) in [(1, 1000), (3, 77), (5, 2), (64, 31)]:
+            for dist_name, op in cases:
+                if op == "prod":
+                    dist_name = "I32_SMALL"
+                X = gen.matrix(dist_name, 5, n, m)
+                d = 3 if X.dtype == torch.int32 else 1.5
+                want = oracle.segred(X.numpy(), op, "id", d)
+                for t_dev in (1, world + 1):  # force outer and inner
+                    plan = dist.plan_segred(n, m, world, rank, t_dev)
+                    blk = X[plan.lo:plan.hi] if plan.mode == "outer" else X[:, plan.lo:plan.hi].contiguous()
+                    for gp in ((None, True) if plan.mode == "inner" else (None,)):
+                        out = dist.segred_dist(blk, n, m, op, "id", d, plan=plan, gather=True,
+                                               local_segred=_oracle_local, gather_partials=gp)
+                        got = out.numpy()
+                        if X.dtype == torch.int32:
+                            ok = np.array_equal(got, want)
+                        else:
+                            ok = np.allclose(got, want, rtol=0, atol=1e-9)
+                        results.append((plan.mode, n, m, dist_name, op, gp, bool(ok)))
+        q.put((rank, results))
+    except Exception as e:  # report instead of hanging the parent
+        q.put((rank, [("error", repr(e), False)]))
+    finally:
+        td.destroy_process_group()
+
+
+def test_segred_dist_world2():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, rows in res:
+        bad = [r for r in rows if not r[-1]]
+        assert not bad, f"rank {rank}: {bad[:5]}"
+        assert any(r[0] == "outer" for r in rows) and any(r[0] == "inner" for r in rows)
+
+
+def test_plans_cover_exactly():
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    for world in (1, 2, 3, 8):
+        for (n, m) in [(1, 10), (7, 3), (100, 1), (8, 8)]:
+            plans = [dist.plan_segred(n, m, world, r) for r in range(world)]
+            assert len({p.mode for p in plans}) == 1
+            if plans[0].mode == "outer":
+                cover = [i for p in plans for i in range(p.lo, p.hi)]
+                assert cover == list(range(n))
+            else:
+                cover = [j for p in plans for j in range(p.lo, p.hi)]
+                assert cover == list(range(m))

@@ -1,0 +1,60 @@
+"""GPU side of the device-level split (dist.py) on one B200: an NCCL
+communicator of world size 1 (plumbing), and G "virtual shards" of one array
+combined with the library's own kernels exactly as the inner split does
+(SURVEY 4(3)(i)).  Checked against the oracle."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+
+import ifl_inputs as gen
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ifl():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_ppopp_henriksenteo19_b200 import build
+    build.build()
+    import paper_conf_ppopp_henriksenteo19_b200 as m
+    return m
+
+
+def test_nccl_world1(ifl, orc):
+    import torch.distributed as td
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    td.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        for op in ("sum", "max", "xor"):
+            X = gen.matrix("I32_FULL", 8, 3, 100003)
+            want = orc.segred(X.numpy(), op, "id", 5)
+            for t_dev in (1, 2):
+                plan = dist.plan_segred(3, 100003, 1, 0, t_dev)
+                out = dist.segred_dist(X.cuda(), 3, 100003, op, "id", 5, plan=plan, gather=True)
+                np.testing.assert_array_equal(out.cpu().numpy(), want)
+    finally:
+        td.destroy_process_group()
+
+
+@pytest.mark.parametrize("G", [2, 4, 8])
+def test_virtual_shards(ifl, orc, G):
+    """Inner split on one GPU: column shards -> partials without d -> the
+    library's segred over the [n][G] partial matrix -> d applied once."""
+    n, m = 4, (1 << 20) + 3
+    X = gen.matrix("I32_FULL", 8, n, m).cuda()
+    for op in ("sum", "min", "xor", "prod"):
+        Xo = X if op != "prod" else gen.matrix("I32_SMALL", 8, n, m).cuda()
+        cuts = [(m * r) // G for r in range(G + 1)]
+        parts = [ifl.segred(Xo[:, cuts[r]:cuts[r + 1]].contiguous(), op) for r in range(G)]
+        stacked = torch.stack(parts, 1).contiguous()
+        total = ifl.segred(stacked, op, ne=7)
+        np.testing.assert_array_equal(total.cpu().numpy(), orc.segred(Xo.cpu().numpy(), op, "id", 7))
