@@ -254,7 +254,10 @@ def run_ours(args, rank, world, device):
 
     auto_ms = {(k, n): time_call(k, n, m, "auto") for k, n, m in calls}
     per_call_ms = [auto_ms[(k, n)] for k, n, m in calls]
-    forced = {(k, n, v): time_call(k, n, m, v) for k, n, m in calls for v in ("top", "middle", "flat")}
+    if args.no_forced:  # launch-list runs: only the contract region
+        forced = {(k, n, v): auto_ms[(k, n)] for k, n, m in calls for v in ("top", "middle", "flat")}
+    else:
+        forced = {(k, n, v): time_call(k, n, m, v) for k, n, m in calls for v in ("top", "middle", "flat")}
     table = []
     ratios = []
     fixed_tot = {v: 0.0 for v in ("top", "middle", "flat")}
@@ -394,8 +397,12 @@ def main():
     ap.add_argument("--no-tune", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-forced", action="store_true",
+                    help="skip the per-shape forced-version timings (for the ncu launch list of the timed region)")
     ap.add_argument("--thresholds", default=None)
     ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"))
+    ap.add_argument("--suite", default="sweep", choices=["sweep", "config0", "redomap2", "tridag", "dist"],
+                    help="sweep = the contract line (configs[1]); the others measure one more SURVEY 8(a) row")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -403,6 +410,15 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
 
+    if args.suite != "sweep" and args.impl == "ours":
+        import bench_suites
+        line = bench_suites.SUITES[args.suite]()
+        os.makedirs(os.path.dirname(args.detail), exist_ok=True)
+        with open(args.detail.replace(".json", f"_{args.suite}.json"), "w") as fp:
+            json.dump(line, fp, indent=1)
+        slim = {k: v for k, v in line.items() if k not in ("shapes", "sites", "rows")}
+        print(json.dumps(slim), flush=True)
+        return
     if args.impl == "reference":
         line = run_reference(args, rank, world)
         if line is not None:

@@ -1,0 +1,252 @@
+"""Per-row measurement suites for bench.py (``python bench.py --suite X``).
+Each prints ONE JSON line for its BASELINE.json config.  All device times
+are CUDA-graph replays timed with CUDA events on the launching stream."""
+from __future__ import annotations
+
+import json
+import os
+import statistics
+import time
+
+import numpy as np
+import torch
+
+import ifl_inputs as gen
+import paper_conf_ppopp_henriksenteo19_b200 as ifl
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+
+
+def gtime(fn, R=4, reps=3):
+    fn()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    fn()
+    e1.record()
+    torch.cuda.synchronize()
+    one = e0.elapsed_time(e1)
+    if one > 50.0:
+        return one
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g):
+        for _ in range(R):
+            fn()
+    g.replay()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        e0.record()
+        g.replay()
+        e1.record()
+        torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1) / R)
+    return statistics.median(ts)
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), float(d["bf16_tflops"]), "measured (MEASURED_PEAKS.json)"
+    return 6650.0, 1590.0, "fallback (B200_PROFILING.md)"
+
+
+def base_line(metric, value, unit, cfg, hib=True, dtype="f32"):
+    return {"metric": metric, "value": value, "unit": unit, "n_gpus": 1, "higher_is_better": hib,
+            "vs_baseline": None, "dtype": dtype, "data": "synthetic", "config": cfg}
+
+
+# ------------------------------------------------------------------ config 0
+
+
+def suite_config0():
+    import oracle
+    n = m = 1024
+    x = gen.matrix("I32_FULL", 1, n, m)
+    xd = x.cuda()
+    out = torch.empty(n, dtype=torch.int32, device="cuda")
+    ws = ifl.workspace(ifl.workspace_bytes("segred", n, m, dt="i32"))
+    res = {}
+    for v in ("top", "middle", "flat", "auto"):
+        res[v] = gtime(lambda: ifl.segred(xd, out=out, ws=ws, version=v)) * 1e3
+        assert np.array_equal(out.cpu().numpy(), oracle.segred(x.numpy(), "sum"))
+    t0 = time.perf_counter()
+    for _ in range(5):
+        oracle.segred(x.numpy(), "sum")
+    cpu_s = (time.perf_counter() - t0) / 5
+    line = base_line("int32 segmented sum latency, 1024x1024 (configs[0])", round(res["auto"], 3), "us",
+                     {"workload": "configs[0] int32 segred sum 1024x1024", "per_version_us": res}, hib=False,
+                     dtype="int32")
+    line["cpu_baseline"] = {"value": round(cpu_s * 1e6, 1), "unit": "us", "cores": 1, "kind": "oracle",
+                            "sample": "full 1024x1024"}
+    line["note"] = "4.2 MB is L2-resident and below launch latency: latency, not a bandwidth roofline"
+    return line
+
+
+# ------------------------------------------------------------------ redomap2
+
+
+def mm_shapes(k):
+    return [(1 << a, 1 << (k - 2 * a), 1 << a) for a in range(0, k // 2 + 1)]
+
+
+def suite_redomap2():
+    hbm, tc_peak, src = peaks()
+    rows = []
+    tuned = {}
+    for dt, tdt, site, ktrain, ks in (("bf16", torch.bfloat16, "redomap2.bf16", 25, (30,)),
+                                      ("f32", torch.float32, "redomap2.f32", 23, (25,))):
+        # P:138 protocol (tune on a smaller constant-work family, test on a
+        # larger one); on B200 k = 20 is launch-bound and L2-resident, so the
+        # training family is k = 25 (bf16) / 23 (f32), testing k = 30 / 25
+        train = mm_shapes(ktrain)
+        need = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data, len(train))
+        scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
+        a, b, tbl = ifl.tune(site, train, reps=3, cost=1, scratch=scratch)
+        tuned[site] = {"t_top": a, "t_intra": b}
+        del scratch
+        for k in ks:
+            for (n, m, p) in mm_shapes(k):
+                A = gen.generate("BF16_SIGNED", 6, n * m, device="cuda").view(n, m).to(tdt)
+                Bt = gen.generate("BF16_SIGNED", 7, p * m, device="cuda").view(p, m).to(tdt)
+                C = torch.empty(n, p, device="cuda")
+                ws = ifl.workspace(ifl.workspace_bytes("redomap2", n, m, p, dt), "cuda", "mm")
+                r = {"dt": dt, "k": k, "n": n, "m": m, "p": p}
+                for v in ("top", "middle", "flat", "auto"):
+                    hopeless = (v == "middle" and (n * p > (1 << 22) or m >= (1 << 24))) or \
+                               (v == "top" and dt == "f32" and n * p < 64 and m >= (1 << 22)) or \
+                               (v == "flat" and n * p > (1 << 24))
+                    r[v] = None if hopeless else gtime(lambda: ifl.redomap2(A, Bt, out=C, ws=ws, version=v)) * 1e3
+                r["chosen"] = ifl.redomap2(A, Bt, out=C, ws=ws, return_choice=True)[1].version
+                best = min(t for t in (r["top"], r["middle"], r["flat"]) if t is not None)
+                r["best_over_auto"] = best / r["auto"]
+                r["flops"] = 2.0 * n * m * p
+                r["bytes"] = (2 if dt == "bf16" else 4) * (n * m + m * p) + 4 * n * p
+                rows.append(r)
+                del A, Bt, C
+    # dense bf16 square (tensor-core roofline)
+    sq = {}
+    for q in (2048, 4096, 8192):
+        A = gen.generate("BF16_SIGNED", 6, q * q, device="cuda").view(q, q).to(torch.bfloat16)
+        Bt = gen.generate("BF16_SIGNED", 7, q * q, device="cuda").view(q, q).to(torch.bfloat16)
+        C = torch.empty(q, q, device="cuda")
+        t = gtime(lambda: ifl.redomap2(A, Bt, out=C, version="top"), R=2)
+        sq[q] = {"us": t * 1e3, "TFLOPs": 2.0 * q ** 3 / (t * 1e-3) / 1e12}
+        del A, Bt, C
+    tot_t = sum(r["auto"] for r in rows if r["dt"] == "bf16" and r["k"] == 30)
+    tot_b = sum(r["bytes"] for r in rows if r["dt"] == "bf16" and r["k"] == 30)
+    line = base_line("map-map-redomap (matmul-shaped) sweep throughput, configs[2] k=30 bf16",
+                     round(tot_b / (tot_t * 1e-6) / 1e9, 1), "GB/s",
+                     {"workload": "configs[2]: A[2^a][2^(k-2a)] x B[2^(k-2a)][2^a], test k=30 (bf16) / 25 (f32), "
+                                  "tuned on k=25 / 23 (P:138 protocol)", "thresholds": tuned}, dtype="bf16")
+    line["min_shape_best_over_auto"] = round(min(r["best_over_auto"] for r in rows), 4)
+    top = sq[8192]
+    line["roofline"] = {"bound": "tensor", "kernel": "mm_top_tc_kernel (8192^3 bf16)",
+                        "achieved": round(top["TFLOPs"], 1), "peak": tc_peak, "unit": "TFLOP/s",
+                        "frac": round(top["TFLOPs"] / tc_peak, 4), "traffic": None, "peak_source": src}
+    line["dense_square"] = sq
+    line["shapes"] = rows
+    return line
+
+
+# -------------------------------------------------------------------- tridag
+
+LVC = {"small": (16, 256, 32, 256), "medium": (128, 64, 256, 32), "large": (256, 64, 256, 256)}
+
+
+def sites(ds):
+    numS, numT, numX, numY = LVC[ds]
+    return [(numS * numX, numY, numX), (numS * numY, numX, numY)], numT
+
+
+def suite_tridag():
+    hbm, _, src = peaks()
+    # tune on other data (seed 9) over the small and large datasets' sites
+    train = [s for ds in ("small", "large") for s in sites(ds)[0]]
+    need = ifl.lib().ifl_tune_scratch_bytes(b"tridag", np.asarray(train, np.int64).ctypes.data, len(train))
+    scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
+    a_, b_, tbl = ifl.tune("tridag", train, reps=3, cost=1, scratch=scratch)
+    del scratch
+    rows = []
+    for ds in ("small", "medium", "large"):
+        shp, numT = sites(ds)
+        for (S, L, R) in shp:
+            a, b, c, y = (t.cuda() for t in gen.tridag_system(7, S, L, R))
+            x = torch.empty_like(y)
+            ws = ifl.workspace(ifl.workspace_bytes("tridag", S, L, R), "cuda", "tri")
+            r = {"dataset": ds, "S": S, "L": L, "R": R, "numT": numT}
+            for v in ("top", "middle", "flat", "auto"):
+                if v == "middle" and L > 4096:
+                    r[v] = None
+                    continue
+                r[v] = gtime(lambda: ifl.tridag(a, b, c, y, out=x, ws=ws, version=v)) * 1e3
+            r["chosen"] = ifl.tridag(a, b, c, y, out=x, ws=ws, return_choice=True)[1].version
+            best = min(t for t in (r["top"], r["middle"], r["flat"]) if t is not None)
+            r["best_over_auto"] = best / r["auto"]
+            r["GBps"] = 8.0 * S * L / (r["auto"] * 1e-6) / 1e9
+            rows.append(r)
+    # whole-run time per dataset: numT steps x both sites (P:400 structure)
+    per_ds = {}
+    for ds in ("small", "medium", "large"):
+        rr = [r for r in rows if r["dataset"] == ds]
+        per_ds[ds] = {"ms_numT_steps": sum(r["auto"] for r in rr) * rr[0]["numT"] / 1e3,
+                      "GBps": sum(8.0 * r["S"] * r["L"] for r in rr) / (sum(r["auto"] for r in rr) * 1e-6) / 1e9}
+    large = [r for r in rows if r["dataset"] == "large"]
+    ach = sum(8.0 * r["S"] * r["L"] for r in large) / (sum(r["auto"] for r in large) * 1e-6) / 1e9
+    line = base_line("batched tridiagonal solves via three scans (LocVolCalib sites), large dataset",
+                     round(ach, 1), "GB/s",
+                     {"workload": "configs[3]: LocVolCalib small/medium/large per-site tridag (P:402), "
+                                  "tuned on small+large with other data", "thresholds": {"t_top": a_, "t_intra": b_}})
+    line["per_dataset"] = per_ds
+    line["min_shape_best_over_auto"] = round(min(r["best_over_auto"] for r in rows), 4)
+    line["roofline"] = {"bound": "hbm", "kernel": "tridag (large, both sites, AUTO)", "achieved": round(ach, 1),
+                        "peak": hbm, "unit": "GB/s", "frac": round(ach / hbm, 4), "traffic": None,
+                        "peak_source": src}
+    line["sites"] = rows
+    return line
+
+
+# ---------------------------------------------------------------------- dist
+
+
+def suite_dist():
+    """configs[4]: 2^30-element f32 segred on this GPU through dist.py with a
+    world-1 NCCL communicator: outer (no collective) and inner (one
+    all_reduce) splits, n in {1, 2^4, 2^10, 2^16, 2^20, 2^24}."""
+    import socket
+
+    import torch.distributed as td
+
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    hbm, _, src = peaks()
+    if not td.is_initialized():
+        s = socket.socket()
+        s.bind(("127.0.0.1", 0))
+        os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(s.getsockname()[1]))
+        s.close()
+        td.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    N = 1 << 30
+    x = gen.generate("F32_UNIT", 8, N, device="cuda")
+    rows = []
+    for lg in (0, 4, 10, 16, 20, 24):
+        n, m = 1 << lg, N >> lg
+        xv = x.view(n, m)
+        r = {"n": n, "m": m}
+        for mode, t_dev in (("outer", 1), ("inner", 2)):
+            plan = dist.plan_segred(n, m, 1, 0, t_dev)
+            t = gtime(lambda: dist.segred_dist(xv, n, m, "sum", plan=plan), R=2)
+            r[mode + "_us"] = t * 1e3
+            r[mode + "_GBps"] = 4.0 * (N + n) / (t * 1e-3) / 1e9
+        rows.append(r)
+    best = max(max(r["outer_GBps"], r["inner_GBps"]) for r in rows)
+    line = base_line("2^30-element segmented reduce, GB/s per GPU (configs[4])", round(best, 1), "GB/s",
+                     {"workload": "configs[4]: 2^30 f32 segred via dist.py, world size 1 on this box"})
+    line["scaling"] = "weak"
+    line["rows"] = rows
+    line["roofline"] = {"bound": "hbm", "kernel": "segred (outer plan)", "achieved": round(best, 1), "peak": hbm,
+                        "unit": "GB/s", "frac": round(best / hbm, 4), "traffic": None, "peak_source": src}
+    return line
+
+
+SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist}

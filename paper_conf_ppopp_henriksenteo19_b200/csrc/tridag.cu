@@ -235,14 +235,31 @@ __global__ void __launch_bounds__(256) tridag_mid_kernel(const float* __restrict
     float* xs = x + (live ? s * L : 0);
     const int64_t j0 = (int64_t)g * IT;
     float yv[IT], al[IT], ib[IT], de[IT];
+    // 128-bit loads when the thread's IT items are whole aligned float4s
+    const bool vec = live && (L % 4 == 0) && (j0 + IT <= L) && (((uintptr_t)ys & 15) == 0) &&
+                     (((uintptr_t)(alpha + r * L) & 15) == 0);
+    if (vec) {
 #pragma unroll
-    for (int k = 0; k < IT; ++k) {
-        const int64_t j = j0 + k;
-        const bool ok = live && j < L;
-        yv[k] = ok ? __ldg(ys + j) : 0.f;
-        al[k] = ok ? __ldg(alpha + r * L + j) : 1.f;
-        ib[k] = ok ? __ldg(invb + r * L + j) : 0.f;
-        de[k] = ok ? __ldg(delta + r * L + j) : 1.f;
+        for (int k = 0; k < IT; k += 4) {
+            const float4 y4 = __ldg(reinterpret_cast<const float4*>(ys + j0 + k));
+            const float4 a4 = __ldg(reinterpret_cast<const float4*>(alpha + r * L + j0 + k));
+            const float4 i4 = __ldg(reinterpret_cast<const float4*>(invb + r * L + j0 + k));
+            const float4 d4 = __ldg(reinterpret_cast<const float4*>(delta + r * L + j0 + k));
+            yv[k] = y4.x; yv[k + 1] = y4.y; yv[k + 2] = y4.z; yv[k + 3] = y4.w;
+            al[k] = a4.x; al[k + 1] = a4.y; al[k + 2] = a4.z; al[k + 3] = a4.w;
+            ib[k] = i4.x; ib[k + 1] = i4.y; ib[k + 2] = i4.z; ib[k + 3] = i4.w;
+            de[k] = d4.x; de[k + 1] = d4.y; de[k + 2] = d4.z; de[k + 3] = d4.w;
+        }
+    } else {
+#pragma unroll
+        for (int k = 0; k < IT; ++k) {
+            const int64_t j = j0 + k;
+            const bool ok = live && j < L;
+            yv[k] = ok ? __ldg(ys + j) : 0.f;
+            al[k] = ok ? __ldg(alpha + r * L + j) : 1.f;
+            ib[k] = ok ? __ldg(invb + r * L + j) : 0.f;
+            de[k] = ok ? __ldg(delta + r * L + j) : 1.f;
+        }
     }
     // (x) forward: thread composite of its items, group exclusive prefix, apply
     Aff f{1.f, 0.f};
@@ -267,9 +284,15 @@ __global__ void __launch_bounds__(256) tridag_mid_kernel(const float* __restrict
         u = fmaf(de[k], u, yv[k]);
         yv[k] = u;
     }
+    if (vec && ((((uintptr_t)xs) & 15) == 0)) {
 #pragma unroll
-    for (int k = 0; k < IT; ++k)
-        if (live && j0 + k < L) xs[j0 + k] = yv[k];
+        for (int k = 0; k < IT; k += 4)
+            *reinterpret_cast<float4*>(xs + j0 + k) = make_float4(yv[k], yv[k + 1], yv[k + 2], yv[k + 3]);
+    } else {
+#pragma unroll
+        for (int k = 0; k < IT; ++k)
+            if (live && j0 + k < L) xs[j0 + k] = yv[k];
+    }
 }
 
 bool tridag_mid_fits(int64_t L) { return L >= 1 && L <= 256 * 16; }

@@ -1,0 +1,29 @@
+#!/bin/bash
+# Profiling pass (run under gpurun): ncu launch list of the bench command and
+# full captures of the dominant kernel of each version family.  Outputs land in
+# gpurun_out/ and are summarised into profiles/ by tools/summarize_ncu.py.
+set -u
+mkdir -p gpurun_out/ncu
+# 1. launch list (cold-cache, serialised: compare SHARES, not absolutes)
+timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
+  --log-file gpurun_out/ncu/launches.csv \
+  python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu --no-forced > gpurun_out/ncu/bench_under_ncu.json 2>&1
+echo "launch list rc=$?"
+# 2. full captures (one launch each)
+cap() {  # name op version n m kernel-regex
+  timeout 300 ncu --set full --import-source on --clock-control none -k regex:"$6" -s 2 -c 1 \
+    -o gpurun_out/ncu/$1 python tools/prof_one.py --op $2 --version $3 --n $4 --m $5 > /dev/null 2>&1
+  echo "$1 rc=$?"
+}
+cap segscan_flat_n1      segscan flat   1        67108864 flat_scan
+cap segscan_flat_n4096   segscan flat   4096     16384    flat_scan
+cap segred_flat_n1       segred  flat   1        67108864 flat_red_kernel
+cap segred_middle_n1024  segred  middle 1024     65536    segred_mid
+cap segscan_middle_n2e18 segscan middle 262144   256      segscan_mid
+cap segred_top_n2e24     segred  top    16777216 4        top_small
+cap segscan_top_n2e23    segscan top    8388608  8        top_warp
+for f in gpurun_out/ncu/*.ncu-rep; do
+  ncu -i $f --page raw --csv > ${f%.ncu-rep}.raw.csv 2>/dev/null
+done
+for f in gpurun_out/ncu/*.ncu-rep; do case $f in *segscan_flat_n1*) ;; *) rm -f $f;; esac; done
+ls -la gpurun_out/ncu
