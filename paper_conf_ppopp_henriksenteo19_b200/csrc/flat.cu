@@ -134,7 +134,11 @@ __device__ __forceinline__ void store_items(T* buf, const T (&v)[FI]) {
 // CTA-wide exclusive scan of the thread aggregates (fl, sv) under the
 // segmented operator.  Returns the thread's exclusive prefix (exf, exv) and
 // the tile aggregate (aggf, aggv).  Contains one __syncthreads.
-template <typename T, int OP>
+// barrier among the FB consumer threads only (named barrier 1): used by the
+// warp-specialised scan kernel, whose producer warp must not take part
+__device__ __forceinline__ void consumer_sync() { asm volatile("bar.sync 1, %0;" ::"n"(FB) : "memory"); }
+
+template <typename T, int OP, bool NAMED = false>
 __device__ __forceinline__ void cta_seg_scan(uint32_t fl, T sv, uint32_t& exf, T& exv, uint32_t& aggf, T& aggv,
                                              T* s_wval, uint32_t* s_wflag) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -157,7 +161,8 @@ __device__ __forceinline__ void cta_seg_scan(uint32_t fl, T sv, uint32_t& exf, T
         exv = identity<OP, T>();
         exf = 0;
     }
-    __syncthreads();
+    if (NAMED) consumer_sync();
+    else __syncthreads();
     T pw = identity<OP, T>();
     uint32_t pf = 0;
     aggv = identity<OP, T>();
@@ -377,37 +382,37 @@ __device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, 
     }
 }
 
-// L2-blocked two-phase segscan.  Persistent CTAs, co-resident by cooperative
-// launch, own chunks of kChunkTiles consecutive tiles statically
-// (chunk c = round * grid + blockIdx).  Per chunk:
+// L2-blocked two-phase segscan, warp-specialised.  Persistent CTAs,
+// co-resident by cooperative launch, own chunks of kChunkTiles consecutive
+// tiles statically (chunk c = round * grid + blockIdx).  Per chunk:
 //   phase 1  (only if the next chunk continues a segment into it) stream the
-//            chunk through the TMA ring with an L2 evict_last policy and fold
-//            the tile aggregates into the chunk aggregate; publish it;
+//            chunk with an L2 evict_last policy and fold the tile aggregates
+//            into the chunk aggregate; publish it;
 //   look-back (only if the chunk does not begin a segment) over the chunk
-//            aggregates, CTA-wide, to the nearest inclusive prefix or chunk
-//            containing a segment start -- that is at most one round back,
-//            and the previous round's prefixes are long final;
+//            aggregates, CTA-wide, bounded arithmetically to the chunk holding
+//            the last segment start -- at most one round back;
 //   phase 3  stream the chunk again (evict_first: the round, ~48 MB, is still
 //            in the 126 MB L2, so DRAM sees one read and one write per
-//            element), scan with the running carry, and store each tile from
-//            its ring slot with the TMA engine (evict_first).
-// The ring runs over the CTA's whole virtual item sequence, so loads for the
-// next phase / chunk are in flight during the look-back and the scans.
-// Status words carry an epoch tag; the last CTA to finish bumps the epoch
-// (one 64-bit {epoch | done} word), so no per-call memset is needed.
+//            element), scan with the running carry, store each tile from its
+//            ring slot with the TMA engine.
+// Warp 8 is the producer: it walks the CTA's item sequence (phase-1 tiles ++
+// phase-3 tiles, chunk after chunk), waits for a ring slot to be released
+// (mbarrier `empty`), writes the slot's metadata and issues the TMA load
+// (completion on `full`).  Warps 0-7 consume; they synchronise among
+// themselves with a named barrier, so the producer never stalls them and the
+// 64-bit tile arithmetic stays off their critical path.  Status words carry
+// an epoch tag; the last CTA to finish bumps the epoch (one 64-bit
+// {epoch | done} word), so no per-call memset is needed.
 constexpr int kChunkTiles = 8;
-
-struct ScanItem {
-    int chunk, j, phase;  // phase 1 = aggregate pass, 3 = scan pass
-};
+constexpr int kScanThreads = FB + 32;
 
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
-                                                          uint8_t* ws, int num_tiles, int num_chunks, bool tma_in,
-                                                          bool tma_out) {
+__global__ void __launch_bounds__(kScanThreads, 2) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
+                                                                    uint8_t* ws, int num_tiles, int num_chunks,
+                                                                    bool tma_in, bool tma_out) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
-    __shared__ alignas(8) uint64_t full[kSlots];
+    __shared__ alignas(8) uint64_t full[kSlots], empty[kSlots];
     __shared__ SlotMeta meta[kSlots];
     __shared__ uint32_t s_tag;
     __shared__ T s_wval[FB / 32];
@@ -419,65 +424,80 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
     const int G = gridDim.x;
     const int64_t chunk_elems = (int64_t)kChunkTiles * FT;
-    // chunk c needs its predecessors' carry / its successor needs c's aggregate
     auto need_carry = [&](int c) { return c > 0 && ((int64_t)c * chunk_elems) % m != 0; };
     auto need_agg = [&](int c) { return need_carry(c + 1) && c + 1 < num_chunks; };
     auto chunk_tiles = [&](int c) { return min(kChunkTiles, num_tiles - c * kChunkTiles); };
 
-    // producer state (thread 0): walks chunk by chunk, phase 1 (if needed) then 3
-    int p_chunk = blockIdx.x, p_phase = 0, p_j = 0;
-    auto p_norm = [&]() {  // settle (p_chunk, p_phase, p_j) on a valid item or past the end
-        while (p_chunk < num_chunks) {
-            if (p_phase == 0) {
-                p_phase = need_agg(p_chunk) ? 1 : 3;
-                p_j = 0;
-            }
-            if (p_j < chunk_tiles(p_chunk)) return;
-            if (p_phase == 1) {
-                p_phase = 3;
-                p_j = 0;
-            } else {
-                p_chunk += G;
-                p_phase = 0;
-            }
-        }
-    };
-    uint32_t free_mask = (1u << kSlots) - 1;
-    int next_slot = 0, pend_slot = -1;
-    uint64_t pol_keep = 0, pol_stream = 0;
-    auto produce_all = [&]() {  // thread 0: fill every free slot, in sequence order
-        p_norm();
-        while (p_chunk < num_chunks && ((free_mask >> next_slot) & 1u)) {
-            free_mask &= ~(1u << next_slot);
-            const int tile = p_chunk * kChunkTiles + p_j;
-            SlotMeta& sm = meta[next_slot];
-            fill_meta(sm, tile, N, m);
-            if (tma_in && sm.cnt == FT) {
-                T* dst = ring + next_slot * FT;
-                mbar_arrive_expect_tx(&full[next_slot], FT * sizeof(T));
-                bulk_g2s_hint(dst, in + (int64_t)tile * FT, FT * sizeof(T), &full[next_slot],
-                              p_phase == 1 ? pol_keep : pol_stream);
-            }
-            next_slot = (next_slot + 1) % kSlots;
-            ++p_j;
-            p_norm();
-        }
-    };
-
     if (t == 0) {
         s_tag = (uint32_t)(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)) >> 32) & 0x1FFFFFFFu;
-        pol_keep = policy_evict_last();
-        pol_stream = policy_evict_first();
-        for (int q = 0; q < kSlots; ++q) mbar_init(&full[q], 1);
+        for (int q = 0; q < kSlots; ++q) {
+            mbar_init(&full[q], 1);
+            mbar_init(&empty[q], 1);
+        }
         fence_mbar_init();
-        produce_all();
     }
     __syncthreads();
+
+    if (w == FB / 32) {
+        // ================= producer warp (one lane)
+        if (lane == 0) {
+            const uint64_t pol_keep = policy_evict_last(), pol_stream = policy_evict_first();
+            int wv = 0;
+            for (int c = blockIdx.x; c < num_chunks; c += G) {
+                const int L = chunk_tiles(c);
+                const int t0 = c * kChunkTiles;
+                // tile metadata advanced incrementally (no 64-bit division per tile)
+                const int64_t cbase = (int64_t)t0 * FT;
+                for (int ph = need_agg(c) ? 1 : 3; ph <= 3; ph += 2) {
+                    int64_t pos = cbase % m, seg = cbase / m;
+                    for (int j = 0; j < L; ++j, ++wv) {
+                        const int sl = wv % kSlots;
+                        if (wv >= kSlots) mbar_wait(&empty[sl], ((wv / kSlots) - 1) & 1);
+                        SlotMeta& sm = meta[sl];
+                        const int tile = t0 + j;
+                        sm.tile = tile;
+                        sm.cnt = (int)std::min((int64_t)FT, N - (int64_t)tile * FT);
+                        sm.pos = pos;
+                        sm.seg = seg;
+                        if (tma_in && sm.cnt == FT) {
+                            mbar_arrive_expect_tx(&full[sl], FT * sizeof(T));
+                            bulk_g2s_hint(ring + sl * FT, in + (int64_t)tile * FT, FT * sizeof(T), &full[sl],
+                                          ph == 1 ? pol_keep : pol_stream);
+                        } else {
+                            mbar_arrive_expect_tx(&full[sl], 0);  // consumers copy it themselves
+                        }
+                        pos += FT;
+                        if (pos >= m) {  // m > FT: at most one wrap; otherwise divide (32-bit range)
+                            if (m > FT) {
+                                pos -= m;
+                                seg += 1;
+                            } else {
+                                seg += pos / m;
+                                pos %= m;
+                            }
+                        }
+                    }
+                }
+            }
+        }
+        return;
+    }
+
+    // ================= consumer warps 0-7
     const uint32_t tag = s_tag;
     uint32_t phase_bits = 0;
-    int vi = 0;  // consumer position in the virtual sequence
-
-    // consume one item: returns with the tile's values scanned in registers
+    int vi = 0;
+    int pend_slot = -1;  // slot whose bulk store may still be reading smem (thread 0)
+    auto release = [&](int sl) { mbar_arrive_expect_tx(&empty[sl], 0); };
+    auto acquire = [&](int sl, T* buf, const SlotMeta& sm) {
+        mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
+        phase_bits ^= 1u << sl;
+        if (!(tma_in && sm.cnt == FT)) {  // partial / misaligned tile: cooperative copy
+            const int64_t base = (int64_t)sm.tile * FT;
+            for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
+            consumer_sync();
+        }
+    };
     for (int c = blockIdx.x; c < num_chunks; c += G) {
         const int L = chunk_tiles(c);
         const bool agg_needed = need_agg(c), carry_needed = need_carry(c);
@@ -487,9 +507,15 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
         if (agg_needed) {
             for (int j = 0; j < L; ++j, ++vi) {
                 const int sl = vi % kSlots;
-                const SlotMeta sm = meta[sl];
                 T* buf = ring + sl * FT;
-                acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
+                mbar_wait(&full[sl], (phase_bits >> sl) & 1u);  // meta is valid once the slot is full
+                const SlotMeta sm = meta[sl];
+                phase_bits ^= 1u << sl;
+                if (!(tma_in && sm.cnt == FT)) {
+                    const int64_t base = (int64_t)sm.tile * FT;
+                    for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
+                    consumer_sync();
+                }
                 const ThreadPos tp = thread_pos(sm, m);
                 T v[FI];
                 load_items(buf, v);
@@ -498,28 +524,25 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
                 local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
                 uint32_t exf, aggf;
                 T exv, aggv;
-                cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
-                run_v = aggf ? aggv : combine<OP>(run_v, aggv);
-                run_f |= aggf;
-                __syncthreads();  // slot consumed, s_wval reusable
+                cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+                // everyone's items are in registers (the barrier inside the scan): free the slot
                 if (t == 0) {
-                    free_mask |= 1u << sl;
-                    if (pend_slot >= 0) {
+                    if (pend_slot >= 0) {  // a phase-3 store before this phase-1 run
                         bulk_wait_read0();
-                        free_mask |= 1u << pend_slot;
+                        release(pend_slot);
                         pend_slot = -1;
                     }
-                    produce_all();
+                    release(sl);
                 }
+                run_v = aggf ? aggv : combine<OP>(run_v, aggv);
+                run_f |= aggf;
+                consumer_sync();  // s_wval reuse
             }
             if (t == 0)
                 st_release_u64(&status[c], pack_status(tag, (run_f || !carry_needed) ? ST_P : ST_A, run_f,
                                                        to_bits(run_v)));
         }
-        // ---- look-back over preceding chunk aggregates.  The carry spans the
-        // chunks from cs (holding the last segment start before this chunk) to
-        // c-1; every one of them publishes (its successor continues a segment),
-        // and nothing older is ever waited on.
+        // ---- look-back over preceding chunk aggregates (chunks cs .. c-1)
         T carry = identity<OP, T>();
         if (carry_needed) {
             const int64_t cstart = (int64_t)c * chunk_elems;
@@ -536,7 +559,7 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
                 const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
                 const uint32_t tb = __ballot_sync(0xffffffffu, term);
                 if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
-                __syncthreads();
+                consumer_sync();
                 int stop = FB;
 #pragma unroll
                 for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
@@ -547,12 +570,12 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
                     if (lane + off < 32) val = combine<OP>(older, val);
                 }
                 if (lane == 0) s_lbval[w] = val;
-                __syncthreads();
+                consumer_sync();
                 T win = identity<OP, T>();
 #pragma unroll
                 for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
                 carry = combine<OP>(win, carry);
-                __syncthreads();
+                consumer_sync();
                 if (stop < FB) break;
                 pred -= FB;
             }
@@ -562,10 +585,16 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
         // ---- phase 3
         for (int j = 0; j < L; ++j, ++vi) {
             const int sl = vi % kSlots;
-            const SlotMeta sm = meta[sl];
             T* buf = ring + sl * FT;
+            mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
+            const SlotMeta sm = meta[sl];
+            phase_bits ^= 1u << sl;
+            if (!(tma_in && sm.cnt == FT)) {
+                const int64_t base = (int64_t)sm.tile * FT;
+                for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
+                consumer_sync();
+            }
             const int64_t base = (int64_t)sm.tile * FT;
-            acquire_tile(buf, in, sm, tma_in, &full[sl], phase_bits, sl);
             const ThreadPos tp = thread_pos(sm, m);
             T v[FI];
             load_items(buf, v);
@@ -574,7 +603,7 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
             local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
             uint32_t exf, aggf;
             T exv, aggv;
-            cta_seg_scan<T, OP>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+            cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
             {
                 const T carry_t = exf ? exv : combine<OP>(carry, exv);
                 const int lim = min(tp.nx0, tp.nvalid);
@@ -586,26 +615,26 @@ __global__ void __launch_bounds__(FB, 2) flat_scan_kernel(const T* in, T* out, i
             store_items(buf, v);
             const bool bulk = tma_out && sm.cnt == FT;
             if (bulk) fence_proxy_async_smem();
-            __syncthreads();
+            consumer_sync();
             if (bulk) {
-                if (t == 0) bulk_s2g_hint(out + base, buf, FT * sizeof(T), pol_stream);
+                if (t == 0) bulk_s2g_hint(out + base, buf, FT * sizeof(T), policy_evict_first());
             } else {
                 for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
-                __syncthreads();
+                consumer_sync();
             }
             if (t == 0) {
                 bulk_commit();  // one group per phase-3 item (empty for cooperative stores)
                 if (pend_slot >= 0) {
-                    bulk_wait_read1();  // all but the newest group have read their slots
-                    free_mask |= 1u << pend_slot;
+                    bulk_wait_read1();  // the previous item's store has read its slot
+                    release(pend_slot);
                 }
                 pend_slot = sl;
-                produce_all();
             }
         }
     }
     if (t == 0) {
         bulk_wait0();
+        if (pend_slot >= 0) release(pend_slot);
         __threadfence();
         const unsigned long long old = atomicAdd(ctr, 1ull);
         if ((uint32_t)old == (uint32_t)G - 1) atomicAdd(ctr, (1ull << 32) - (unsigned long long)G);
@@ -626,13 +655,13 @@ static int sm_count() {
 }
 
 template <typename K>
-static int resident_ctas(K kernel, size_t smem) {
+static int resident_ctas(K kernel, size_t smem, int threads = FB) {
     static thread_local std::unordered_map<const void*, int> cache;
     auto it = cache.find((const void*)kernel);
     if (it != cache.end()) return it->second;
     cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, FB, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem);
     if (per_sm < 1) per_sm = 1;
     const int n = per_sm * sm_count();
     cache[(const void*)kernel] = n;
@@ -654,11 +683,11 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         if (scan) {
             auto k = flat_scan_kernel<T, OP, F>;
             const int chunks = (int)ceil_div(tiles, kChunkTiles);
-            const int grid = (int)std::min<int64_t>(chunks, resident_ctas(k, smem));
+            const int grid = (int)std::min<int64_t>(chunks, resident_ctas(k, smem, kScanThreads));
             // cooperative launch: all CTAs co-resident (static chunk ownership + look-back)
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = dim3((unsigned)grid);
-            cfg.blockDim = dim3(FB);
+            cfg.blockDim = dim3(kScanThreads);
             cfg.dynamicSmemBytes = smem;
             cfg.stream = a.stream;
             cudaLaunchAttribute attr[1];
