@@ -276,6 +276,27 @@ def run_ours(args, rank, world, device):
                       "best_single": min(tv, key=tv.get), "best_over_auto": best / ta,
                       "auto_GBps": b / (ta / 1e3) / 1e9, "frac_of_8TBps": b / (ta / 1e3) / 1e9 / NOMINAL_HBM_GBS})
 
+    # ---- context: the best G3 threshold pair for THIS sweep (exact search over
+    # the measured forced-version table) -- separates the held-out tuner's
+    # generalisation error from the kernels' own gaps
+    g3_best = {}
+    if not args.no_forced:
+        for kind in ("segred", "segscan"):
+            ks = [(n, m) for k2, n, m in calls if k2 == kind]
+            site = kind + ".b4"
+            pt, pm, tbl = [], [], []
+            for (n, m) in ks:
+                c = ifl.select(site, n, m)
+                pt.append(c.par_top)
+                pm.append(c.par_mid)
+                tbl.append([forced[(kind, n, v)] for v in ("top", "middle", "flat")])
+            a, b, _ = ifl.tune_search(pt, pm, tbl, cost=1)
+            ratios_k = []
+            for (n, m), ptop, pmid, row in zip(ks, pt, pm, tbl):
+                v = 0 if ptop >= a else (1 if pmid >= b else 2)
+                ratios_k.append(min(row) / row[v])
+            g3_best[kind] = {"t_top": a, "t_intra": b, "min_shape_best_over_chosen": round(min(ratios_k), 4)}
+
     # ---- dominant kernel roofline (CUDA-event durations on the launch stream)
     groups = {}
     for (kind, n, m), t in zip(calls, per_call_ms):
@@ -328,7 +349,7 @@ def run_ours(args, rank, world, device):
         "value": value, "total_ms": total_ms, "step_ms": step_ms, "step_bytes": step_bytes, "table": table,
         "ratios": ratios, "fixed_tot": fixed_tot, "auto_tot": auto_tot, "tuned": tuned, "clocks": ck,
         "dom": dom, "achieved": achieved, "peak": pk, "traffic": traffic, "e2e": e2e, "groups": groups,
-        "launches": launches_per_step * args.steps,
+        "launches": launches_per_step * args.steps, "g3_best": g3_best,
     }
     return res
 
@@ -465,6 +486,7 @@ def main():
             "frac_of_measured_hbm": round(r["value"] / world / pk["hbm_gbs"], 4),
             "speedup_vs_best_single_version": round(best_fixed / r["auto_tot"], 4),
             "min_shape_best_over_auto": round(min(r["ratios"]), 4),
+            "g3_best_thresholds_on_test_sweep": r["g3_best"] or None,
             "roofline": {"bound": "hbm", "kernel": r["dom"], "achieved": round(r["achieved"], 1),
                          "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": round(r["achieved"] / pk["hbm_gbs"], 4),
                          "traffic": r["traffic"], "peak_source": pk["source"]},

@@ -405,15 +405,16 @@ __device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, 
 // {epoch | done} word), so no per-call memset is needed.
 constexpr int kChunkTiles = 8;
 constexpr int kScanThreads = FB + 32;
+constexpr int kScanSlots = 3;  // 60 KB ring: three CTAs (27 warps) per SM
 
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kScanThreads, 2) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
+__global__ void __launch_bounds__(kScanThreads, 3) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
                                                                     uint8_t* ws, int num_tiles, int num_chunks,
                                                                     bool tma_in, bool tma_out) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
-    __shared__ alignas(8) uint64_t full[kSlots], empty[kSlots];
-    __shared__ SlotMeta meta[kSlots];
+    __shared__ alignas(8) uint64_t full[kScanSlots], empty[kScanSlots];
+    __shared__ SlotMeta meta[kScanSlots];
     __shared__ uint32_t s_tag;
     __shared__ T s_wval[FB / 32];
     __shared__ uint32_t s_wflag[FB / 32];
@@ -430,7 +431,7 @@ __global__ void __launch_bounds__(kScanThreads, 2) flat_scan_kernel(const T* in,
 
     if (t == 0) {
         s_tag = (uint32_t)(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)) >> 32) & 0x1FFFFFFFu;
-        for (int q = 0; q < kSlots; ++q) {
+        for (int q = 0; q < kScanSlots; ++q) {
             mbar_init(&full[q], 1);
             mbar_init(&empty[q], 1);
         }
@@ -451,8 +452,8 @@ __global__ void __launch_bounds__(kScanThreads, 2) flat_scan_kernel(const T* in,
                 for (int ph = need_agg(c) ? 1 : 3; ph <= 3; ph += 2) {
                     int64_t pos = cbase % m, seg = cbase / m;
                     for (int j = 0; j < L; ++j, ++wv) {
-                        const int sl = wv % kSlots;
-                        if (wv >= kSlots) mbar_wait(&empty[sl], ((wv / kSlots) - 1) & 1);
+                        const int sl = wv % kScanSlots;
+                        if (wv >= kScanSlots) mbar_wait(&empty[sl], ((wv / kScanSlots) - 1) & 1);
                         SlotMeta& sm = meta[sl];
                         const int tile = t0 + j;
                         sm.tile = tile;
@@ -506,7 +507,7 @@ __global__ void __launch_bounds__(kScanThreads, 2) flat_scan_kernel(const T* in,
         T run_v = identity<OP, T>();
         if (agg_needed) {
             for (int j = 0; j < L; ++j, ++vi) {
-                const int sl = vi % kSlots;
+                const int sl = vi % kScanSlots;
                 T* buf = ring + sl * FT;
                 mbar_wait(&full[sl], (phase_bits >> sl) & 1u);  // meta is valid once the slot is full
                 const SlotMeta sm = meta[sl];
@@ -584,7 +585,7 @@ __global__ void __launch_bounds__(kScanThreads, 2) flat_scan_kernel(const T* in,
         }
         // ---- phase 3
         for (int j = 0; j < L; ++j, ++vi) {
-            const int sl = vi % kSlots;
+            const int sl = vi % kScanSlots;
             T* buf = ring + sl * FT;
             mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
             const SlotMeta sm = meta[sl];
@@ -682,13 +683,14 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         const T d = bits_to<T>(a.ne_bits);
         if (scan) {
             auto k = flat_scan_kernel<T, OP, F>;
+            const size_t smem_s = (size_t)kScanSlots * FT * sizeof(T);
             const int chunks = (int)ceil_div(tiles, kChunkTiles);
-            const int grid = (int)std::min<int64_t>(chunks, resident_ctas(k, smem, kScanThreads));
+            const int grid = (int)std::min<int64_t>(chunks, resident_ctas(k, smem_s, kScanThreads));
             // cooperative launch: all CTAs co-resident (static chunk ownership + look-back)
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = dim3((unsigned)grid);
             cfg.blockDim = dim3(kScanThreads);
-            cfg.dynamicSmemBytes = smem;
+            cfg.dynamicSmemBytes = smem_s;
             cfg.stream = a.stream;
             cudaLaunchAttribute attr[1];
             attr[0].id = cudaLaunchAttributeCooperative;

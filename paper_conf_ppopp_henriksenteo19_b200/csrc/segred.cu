@@ -330,7 +330,7 @@ cudaError_t launch_segred_top(const SegArgs& a) {
 // --------------------------------------------------------------- V_MIDDLE
 
 int mid_group_size(int64_t m) {
-    int64_t g = 2;
+    int64_t g = 1;  // rows of <= 8 (16) elements: one thread already holds a whole row
     while (g < 1024 && g * 16 < m) g <<= 1;
     return (int)g;
 }

@@ -310,7 +310,7 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
 constexpr int kMidItems = 8;  // consecutive elements per thread per round
 
 int midscan_group_size(int64_t m) {
-    int64_t g = 2;
+    int64_t g = 1;  // rows of <= 8 (16) elements: one thread already holds a whole row
     while (g < 1024 && g * kMidItems < m) g <<= 1;
     return (int)g;
 }
@@ -331,18 +331,19 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
     for (int64_t base = 0; base < m; base += (int64_t)G * kMidItems, par ^= 1) {
         const int64_t k0 = base + (int64_t)g * kMidItems;
         T v[kMidItems];
-        if (live && vec && k0 + kMidItems <= m) {
-            T e[4];
-            unpack4<T>(ldg_stream4(row + k0), e);
 #pragma unroll
-            for (int u = 0; u < 4; ++u) v[u] = apply_map<F>(e[u]);
-            unpack4<T>(ldg_stream4(row + k0 + 4), e);
+        for (int h = 0; h < kMidItems / 4; ++h) {  // two 128-bit halves, each vectorised when whole
+            const int64_t kh = k0 + 4 * h;
+            if (live && vec && kh + 4 <= m) {
+                T e[4];
+                unpack4<T>(ldg_stream4(row + kh), e);
 #pragma unroll
-            for (int u = 0; u < 4; ++u) v[4 + u] = apply_map<F>(e[u]);
-        } else {
+                for (int u = 0; u < 4; ++u) v[4 * h + u] = apply_map<F>(e[u]);
+            } else {
 #pragma unroll
-            for (int u = 0; u < kMidItems; ++u)
-                v[u] = (live && k0 + u < m) ? apply_map<F>(ldg1(row + k0 + u)) : identity<OP, T>();
+                for (int u = 0; u < 4; ++u)
+                    v[4 * h + u] = (live && kh + u < m) ? apply_map<F>(ldg1(row + kh + u)) : identity<OP, T>();
+            }
         }
 #pragma unroll
         for (int u = 1; u < kMidItems; ++u) v[u] = combine<OP>(v[u - 1], v[u]);
@@ -375,16 +376,18 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
 #pragma unroll
         for (int u = 0; u < kMidItems; ++u) v[u] = combine<OP>(pre, v[u]);
         if (live) {
-            if (vec && k0 + kMidItems <= m) {
-                V q0, q1;
-                q0.x = v[0]; q0.y = v[1]; q0.z = v[2]; q0.w = v[3];
-                q1.x = v[4]; q1.y = v[5]; q1.z = v[6]; q1.w = v[7];
-                *reinterpret_cast<V*>(orow + k0) = q0;
-                *reinterpret_cast<V*>(orow + k0 + 4) = q1;
-            } else {
 #pragma unroll
-                for (int u = 0; u < kMidItems; ++u)
-                    if (k0 + u < m) orow[k0 + u] = v[u];
+            for (int h = 0; h < kMidItems / 4; ++h) {
+                const int64_t kh = k0 + 4 * h;
+                if (vec && kh + 4 <= m) {
+                    V q;
+                    q.x = v[4 * h]; q.y = v[4 * h + 1]; q.z = v[4 * h + 2]; q.w = v[4 * h + 3];
+                    *reinterpret_cast<V*>(orow + kh) = q;
+                } else {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        if (kh + u < m) orow[kh + u] = v[4 * h + u];
+                }
             }
         }
         carry = combine<OP>(carry, total);
