@@ -207,51 +207,70 @@ __device__ __forceinline__ void acquire_tile(T* slot, const T* in, const SlotMet
 
 // ------------------------------------------------------------ segred pass 1
 
+// Warp-specialised like the scan: warp 8 is the producer (static round-robin
+// tiles blockIdx + i*grid; waits for a ring slot to be released, writes its
+// metadata, issues the TMA load); warps 0-7 consume.  A slot is released by
+// each consumer warp as soon as its items are in registers (count-8 mbarrier),
+// so the next load into it is issued while the tile is still being reduced.
+constexpr int kRedSlots = 3;
+
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(FB, 2) flat_red_kernel(const T* in, T* out, int64_t N, int64_t m, T d, T* head,
-                                                         T* tail, int num_tiles, bool tma) {
+__global__ void __launch_bounds__(FB + 32, 3) flat_red_kernel(const T* in, T* out, int64_t N, int64_t m, T d, T* head,
+                                                              T* tail, int num_tiles, bool tma) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
-    __shared__ alignas(8) uint64_t full[kSlots];
-    __shared__ SlotMeta meta[kSlots];
-    __shared__ T s_wval[FB / 32];
-    __shared__ uint32_t s_wflag[FB / 32];
-    const int t = threadIdx.x;
+    __shared__ alignas(8) uint64_t full[kRedSlots], empty[kRedSlots];
+    __shared__ SlotMeta meta[kRedSlots];
+    __shared__ T s_wval[2][FB / 32];
+    __shared__ uint32_t s_wflag[2][FB / 32];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
     const int G = gridDim.x;
     if (t == 0) {
-        for (int s = 0; s < kSlots; ++s) mbar_init(&full[s], 1);
-        fence_mbar_init();
-        for (int s = 0; s < kSlots; ++s) {
-            const int tile = blockIdx.x + s * G;
-            if (tile < num_tiles) {
-                fill_meta(meta[s], tile, N, m);
-                if (tma && meta[s].cnt == FT) issue_tile_load(ring + s * FT, in, tile, &full[s]);
-            } else {
-                meta[s].tile = num_tiles;
-            }
+        for (int q = 0; q < kRedSlots; ++q) {
+            mbar_init(&full[q], 1);
+            mbar_init(&empty[q], FB / 32);
         }
+        fence_mbar_init();
     }
     __syncthreads();
+    if (w == FB / 32) {  // ================= producer warp
+        if (lane == 0) {
+            for (int wv = 0;; ++wv) {
+                const int tile = blockIdx.x + wv * G;
+                if (tile >= num_tiles) break;
+                const int sl = wv % kRedSlots;
+                if (wv >= kRedSlots) mbar_wait(&empty[sl], ((wv / kRedSlots) - 1) & 1);
+                fill_meta(meta[sl], tile, N, m);
+                if (tma && meta[sl].cnt == FT) {
+                    mbar_arrive_expect_tx(&full[sl], FT * sizeof(T));
+                    bulk_g2s(ring + sl * FT, in + (int64_t)tile * FT, FT * sizeof(T), &full[sl]);
+                } else {
+                    mbar_arrive_expect_tx(&full[sl], 0);
+                }
+            }
+        }
+        return;
+    }
+    // ================= consumer warps 0-7
     uint32_t phase_bits = 0;
     for (int i = 0;; ++i) {
-        const int s = i % kSlots;
-        const SlotMeta sm = meta[s];
-        if (sm.tile >= num_tiles) break;
-        T* buf = ring + s * FT;
-        acquire_tile(buf, in, sm, tma, &full[s], phase_bits, s);
+        const int tile0 = blockIdx.x + i * G;
+        if (tile0 >= num_tiles) break;
+        const int sl = i % kRedSlots;
+        T* buf = ring + sl * FT;
+        mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
+        phase_bits ^= 1u << sl;
+        const SlotMeta sm = meta[sl];
+        if (!(tma && sm.cnt == FT)) {
+            const int64_t base = (int64_t)sm.tile * FT;
+            for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
+            consumer_sync();
+        }
         const ThreadPos tp = thread_pos(sm, m);
         T v[FI];
         load_items(buf, v);
-        __syncthreads();  // slot s fully read: refill it right away
-        if (t == 0) {
-            const int nt = sm.tile + kSlots * G;
-            if (nt < num_tiles) {
-                fill_meta(meta[s], nt, N, m);
-                if (tma && meta[s].cnt == FT) issue_tile_load(buf, in, nt, &full[s]);
-            } else {
-                meta[s].tile = num_tiles;
-            }
-        }
+        __syncwarp();
+        if (lane == 0) mbar_arrive_expect_tx(&empty[sl], 0);  // this warp is done with the slot
         bool has_start = false, stash = false;
         T acc, stash_v = identity<OP, T>();
         if (tp.nx0 > tp.nvalid) {
@@ -290,14 +309,14 @@ __global__ void __launch_bounds__(FB, 2) flat_red_kernel(const T* in, T* out, in
         }
         uint32_t exf, aggf;
         T exv, aggv;
-        cta_seg_scan<T, OP>(has_start ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+        // double-buffered warp totals: no extra barrier between tiles
+        cta_seg_scan<T, OP, true>(has_start ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[i & 1], s_wflag[i & 1]);
         if (stash) {
             const T val = combine<OP>(exv, stash_v);
             if (exf) out[tp.seg] = val;  // began earlier in this tile: complete
             else head[sm.tile] = val;    // began before this tile: head partial
         }
         if (t == 0) tail[sm.tile] = aggv;
-        __syncthreads();  // s_wval reuse
     }
 }
 
@@ -703,8 +722,9 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
         T* tail = head + tiles;
         auto k = flat_red_kernel<T, OP, F>;
-        const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem));
-        k<<<grid, FB, smem, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, head, tail, (int)tiles, tma_in);
+        const size_t smem_r = (size_t)kRedSlots * FT * sizeof(T);
+        const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem_r, FB + 32));
+        k<<<grid, FB + 32, smem_r, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, head, tail, (int)tiles, tma_in);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
         if (a.m > FT) {

@@ -173,7 +173,7 @@ __global__ void __launch_bounds__(256) tridag_top_kernel(const float* __restrict
 
 // ------------------------------------------------------------- V_MIDDLE
 
-constexpr int kTriItems = 4;
+constexpr int kTriItems = 8;
 
 // Group-wide exclusive scan of affine maps (older lanes first).  G threads
 // per group; G <= 32 uses shuffles only, larger groups go through shared
