@@ -90,35 +90,57 @@ __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, uint32_t (&r)
 
 // ------------------------------------------------------------------ kernel
 
-// blockIdx.z = k-split: the CTA accumulates k-tiles [z*kps, (z+1)*kps) and
-// writes its fp32 tile to C (one split) or to part[z] (split-K, summed by
-// mm_splitk_finalize in a fixed order).
-__global__ void __launch_bounds__(128, 1) mm_top_tc_kernel(const __grid_constant__ CUtensorMap mapA,
-                                                           const __grid_constant__ CUtensorMap mapB, float* C,
-                                                           float* part, int64_t n, int64_t m, int64_t p, int kps) {
+// Persistent, warp-specialised: 6 warps.
+//   warp 0 (lane 0)  TMA producer over every (tile, k-tile) of the CTA's items
+//   warp 1           TMEM allocation (512 columns = two 256-column fp32
+//                    accumulators); lane 0 issues the MMAs
+//   warps 2-5        epilogue; warp w reads TMEM lanes 32*(w % 4) .. +31
+// Item = (k-split z, output tile); items are strided by gridDim.x.  The MMA
+// warp accumulates item i into accumulator i & 1 while the epilogue drains
+// item i-1 from the other one (tmem_full / tmem_empty mbarriers).
+constexpr int TC_THREADS = 192;
+constexpr int TC_EPI_BYTES = 4 * 32 * 33 * 4;
+constexpr int TC_SMEM_P = TC_STAGES * TC_STAGE_BYTES + TC_EPI_BYTES + 1024;
+
+__global__ void __launch_bounds__(TC_THREADS, 1) mm_top_tc_kernel(const __grid_constant__ CUtensorMap mapA,
+                                                                  const __grid_constant__ CUtensorMap mapB, float* C,
+                                                                  float* part, int64_t n, int64_t m, int64_t p,
+                                                                  int kps, int splits) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
-    __shared__ alignas(8) uint64_t full[TC_STAGES], empty[TC_STAGES], done;
+    float* stage_base = reinterpret_cast<float*>(smem + TC_STAGES * TC_STAGE_BYTES);
+    __shared__ alignas(8) uint64_t full[TC_STAGES], empty[TC_STAGES], tfull[2], tempty[2];
     __shared__ uint32_t tmem_base;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const int m0 = blockIdx.y * TC_BM, n0 = blockIdx.x * TC_BN;
-    const int kt0 = blockIdx.z * kps;
-    const int nk = min(kps, (int)ceil_div(m, TC_BK) - kt0);
-    float* out = gridDim.z == 1 ? C : part + (int64_t)blockIdx.z * n * p;
+    const int ntx = (int)ceil_div(p, TC_BN), nty = (int)ceil_div(n, TC_BM);
+    const int ntiles = ntx * nty;
+    const int items = ntiles * splits;
+    const int nk_all = (int)ceil_div(m, TC_BK);
+    auto decode = [&](int it, int& z, int& m0, int& n0, int& kt0, int& nk) {
+        z = it / ntiles;
+        const int rem = it - z * ntiles;
+        m0 = (rem / ntx) * TC_BM;
+        n0 = (rem % ntx) * TC_BN;
+        kt0 = z * kps;
+        nk = min(kps, nk_all - kt0);
+    };
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < TC_STAGES; ++s) {
             mbar_init(&full[s], 1);
             mbar_init(&empty[s], 1);
         }
-        mbar_init(&done, 1);
+        for (int a = 0; a < 2; ++a) {
+            mbar_init(&tfull[a], 1);
+            mbar_init(&tempty[a], 4);
+        }
         fence_mbar_init();
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapA)) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
     }
-    if (warp == 2) {  // TMEM allocation: one warp, 256 fp32 columns x 128 lanes
+    if (warp == 1) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)),
-                     "n"(TC_TMEM_COLS)
+                     "n"(2 * TC_TMEM_COLS)
                      : "memory");
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
     }
@@ -127,64 +149,85 @@ __global__ void __launch_bounds__(128, 1) mm_top_tc_kernel(const __grid_constant
     tc_fence_after();
     const uint32_t tmem = tmem_base;
 
-    if (warp == 0 && lane == 0) {
-        // ---- TMA producer
-        for (int kt = 0; kt < nk; ++kt) {
-            const int s = kt % TC_STAGES;
-            const uint32_t ph = (kt / TC_STAGES) & 1;
-            mbar_wait(&empty[s], ph ^ 1);
-            uint8_t* sa = smem + s * TC_STAGE_BYTES;
-            uint8_t* sb = sa + TC_A_BYTES;
-            mbar_arrive_expect_tx(&full[s], TC_STAGE_BYTES);
-            tma_load_2d(sa, &mapA, (kt0 + kt) * TC_BK, m0, &full[s]);
-            tma_load_2d(sb, &mapB, (kt0 + kt) * TC_BK, n0, &full[s]);
-        }
-    } else if (warp == 1 && lane == 0) {
-        // ---- MMA issuer
-        constexpr uint32_t idesc = umma_idesc_bf16(TC_BM, TC_BN);
-        for (int kt = 0; kt < nk; ++kt) {
-            const int s = kt % TC_STAGES;
-            const uint32_t ph = (kt / TC_STAGES) & 1;
-            mbar_wait(&full[s], ph);
-            tc_fence_after();
-            const uint32_t sa = smem_u32(smem + s * TC_STAGE_BYTES);
-            const uint32_t sb = sa + TC_A_BYTES;
-#pragma unroll
-            for (int kk = 0; kk < TC_BK / 16; ++kk) {  // 16 bf16 = 32 bytes per UMMA K step
-                umma_bf16(tmem, umma_desc_sw128(sa + kk * 32), umma_desc_sw128(sb + kk * 32), idesc,
-                          (kt | kk) != 0 ? 1u : 0u);
+    if (warp == 0) {
+        if (lane == 0) {  // ---- TMA producer
+            int gk = 0;
+            for (int it = blockIdx.x; it < items; it += gridDim.x) {
+                int z, m0, n0, kt0, nk;
+                decode(it, z, m0, n0, kt0, nk);
+                for (int kt = 0; kt < nk; ++kt, ++gk) {
+                    const int s = gk % TC_STAGES;
+                    mbar_wait(&empty[s], ((gk / TC_STAGES) & 1) ^ 1);
+                    uint8_t* sa = smem + s * TC_STAGE_BYTES;
+                    mbar_arrive_expect_tx(&full[s], TC_STAGE_BYTES);
+                    tma_load_2d(sa, &mapA, (kt0 + kt) * TC_BK, m0, &full[s]);
+                    tma_load_2d(sa + TC_A_BYTES, &mapB, (kt0 + kt) * TC_BK, n0, &full[s]);
+                }
             }
-            umma_commit(&empty[s]);  // stage reusable once these MMAs have read it
         }
-        umma_commit(&done);  // accumulator complete
-    }
-    __syncwarp();
-
-    // ---- epilogue: TMEM -> registers -> padded smem (the drained ring) ->
-    // row-contiguous, coalesced stores (a warp writes 32 consecutive columns
-    // of one row per instruction)
-    mbar_wait(&done, 0);
-    __syncwarp();
-    tc_fence_after();
-    float* stage = reinterpret_cast<float*>(smem) + warp * (32 * 33);
-#pragma unroll 1
-    for (int c = 0; c < TC_BN; c += 32) {
-        uint32_t r[32];
-        tmem_ld_32x32b_x32(tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c, r);
+    } else if (warp == 1) {
+        if (lane == 0) {  // ---- MMA issuer
+            constexpr uint32_t idesc = umma_idesc_bf16(TC_BM, TC_BN);
+            int gk = 0, li = 0;
+            for (int it = blockIdx.x; it < items; it += gridDim.x, ++li) {
+                int z, m0, n0, kt0, nk;
+                decode(it, z, m0, n0, kt0, nk);
+                const int acc = li & 1;
+                mbar_wait(&tempty[acc], ((li >> 1) & 1) ^ 1);  // epilogue has drained this accumulator
+                tc_fence_after();
+                const uint32_t d = tmem + (uint32_t)(acc * TC_TMEM_COLS);
+                for (int kt = 0; kt < nk; ++kt, ++gk) {
+                    const int s = gk % TC_STAGES;
+                    mbar_wait(&full[s], (gk / TC_STAGES) & 1);
+                    tc_fence_after();
+                    const uint32_t sa = smem_u32(smem + s * TC_STAGE_BYTES);
+                    const uint32_t sb = sa + TC_A_BYTES;
 #pragma unroll
-        for (int q = 0; q < 32; ++q) stage[lane * 33 + q] = __uint_as_float(r[q]);
-        __syncwarp();
-        const int64_t col = (int64_t)n0 + c + lane;
-        for (int rr = 0; rr < 32; ++rr) {
-            const int64_t row = (int64_t)m0 + warp * 32 + rr;
-            if (row < n && col < p) out[row * p + col] = stage[rr * 33 + lane];
+                    for (int kk = 0; kk < TC_BK / 16; ++kk)
+                        umma_bf16(d, umma_desc_sw128(sa + kk * 32), umma_desc_sw128(sb + kk * 32), idesc,
+                                  (kt | kk) != 0 ? 1u : 0u);
+                    umma_commit(&empty[s]);
+                }
+                umma_commit(&tfull[acc]);
+            }
         }
-        __syncwarp();
+    } else {
+        // ---- epilogue warps 2..5: TMEM -> registers -> padded smem -> coalesced rows
+        const int quad = warp & 3;  // TMEM lane quadrant this warp may access
+        float* stage = stage_base + (warp - 2) * (32 * 33);
+        int li = 0;
+        for (int it = blockIdx.x; it < items; it += gridDim.x, ++li) {
+            int z, m0, n0, kt0, nk;
+            decode(it, z, m0, n0, kt0, nk);
+            float* out = splits == 1 ? C : part + (int64_t)z * n * p;
+            const int acc = li & 1;
+            mbar_wait(&tfull[acc], (li >> 1) & 1);
+            __syncwarp();
+            tc_fence_after();
+#pragma unroll 1
+            for (int c = 0; c < TC_BN; c += 32) {
+                uint32_t r[32];
+                tmem_ld_32x32b_x32(tmem + ((uint32_t)(quad * 32) << 16) + (uint32_t)(acc * TC_TMEM_COLS + c), r);
+#pragma unroll
+                for (int q = 0; q < 32; ++q) stage[lane * 33 + q] = __uint_as_float(r[q]);
+                __syncwarp();
+                const int64_t col = (int64_t)n0 + c + lane;
+                for (int rr = 0; rr < 32; ++rr) {
+                    const int64_t row = (int64_t)m0 + quad * 32 + rr;
+                    if (row < n && col < p) out[row * p + col] = stage[rr * 33 + lane];
+                }
+                __syncwarp();
+            }
+            tc_fence_before();
+            __syncwarp();
+            if (lane == 0) mbar_arrive_expect_tx(&tempty[acc], 0);
+        }
     }
     tc_fence_before();
     __syncthreads();
-    if (warp == 2)
-        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(TC_TMEM_COLS) : "memory");
+    if (warp == 1)
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "n"(2 * TC_TMEM_COLS)
+                     : "memory");
 }
 
 // ------------------------------------------------------------------ host side
@@ -252,13 +295,21 @@ cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* par
     if (!make_map(&ma, A, n, m, TC_BM) || !make_map(&mb, Bt, p, m, TC_BN)) return cudaErrorInvalidValue;
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(mm_top_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM);
+        cudaFuncSetAttribute(mm_top_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
     });
     const int nk = (int)ceil_div(m, TC_BK);
     const int kps = (int)ceil_div(nk, splits);
     splits = (int)ceil_div(nk, kps);
-    dim3 g((unsigned)ceil_div(p, TC_BN), (unsigned)ceil_div(n, TC_BM), (unsigned)splits);
-    mm_top_tc_kernel<<<g, 128, TC_SMEM, s>>>(ma, mb, C, part, n, m, p, kps);
+    const int64_t items = ceil_div(n, TC_BM) * ceil_div(p, TC_BN) * splits;
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        if (sms <= 0) sms = 148;
+    }
+    const int grid = (int)std::min<int64_t>(items, sms);
+    mm_top_tc_kernel<<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, C, part, n, m, p, kps, splits);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess || splits == 1) return e;
     const int64_t outs = n * p;

@@ -317,48 +317,113 @@ __global__ void __launch_bounds__(256) tridag_flat_kernel(const float* __restric
     const int64_t base = s0 * L, cnt = nsys * L;
     const int64_t per = ceil_div(cnt, 256);
     const int64_t e0 = threadIdx.x * per, e1 = std::min(cnt, e0 + per);
-    auto coef = [&](int64_t e, float& m, float& add) {  // map of flat element base+e
-        const int64_t gi = base + e;
-        const int64_t s = gi / L, j = gi - s * L, r = s % R;
+    // walk (system, position) incrementally: one division per thread, not per element
+    auto walk = [&](auto&& body) {
+        if (e0 >= e1) return;
         if (FWD) {
-            m = __ldg(alpha + r * L + j);
+            int64_t s = s0 + e0 / L, j = e0 % L, r = s % R;
+            for (int64_t e = e0; e < e1; ++e) {
+                body(base + e, r * L + j);
+                if (++j == L) {
+                    j = 0;
+                    if (++r == R) r = 0;
+                }
+            }
+        } else {
+            int64_t s = s0 + (e1 - 1) / L, j = (e1 - 1) % L, r = s % R;
+            for (int64_t e = e1 - 1; e >= e0; --e) {
+                body(base + e, r * L + j);
+                if (j-- == 0) {
+                    j = L - 1;
+                    r = (r == 0) ? R - 1 : r - 1;
+                }
+            }
+        }
+    };
+    auto coef = [&](int64_t gi, int64_t ci, float& mm, float& add) {
+        if (FWD) {
+            mm = __ldg(alpha + ci);
             add = __ldg(y + gi);
         } else {
-            m = __ldg(delta + r * L + j);
-            add = x[gi] * __ldg(invb + r * L + j);
+            mm = __ldg(delta + ci);
+            add = x[gi] * __ldg(invb + ci);
         }
     };
     Aff f{1.f, 0.f};
-    if (FWD) {
-        for (int64_t e = e0; e < e1; ++e) {
-            float m, ad;
-            coef(e, m, ad);
-            f = aff_after(Aff{m, ad}, f);
+    walk([&](int64_t gi, int64_t ci) {
+        float mm, ad;
+        coef(gi, ci, mm, ad);
+        f = aff_after(Aff{mm, ad}, f);
+    });
+    Aff tot;
+    const Aff pf = group_exscan<!FWD>(f, 256, wtot, tot);
+    float v = pf.g;
+    walk([&](int64_t gi, int64_t ci) {
+        float mm, ad;
+        coef(gi, ci, mm, ad);
+        v = fmaf(mm, v, ad);
+        x[gi] = v;
+    });
+}
+
+// Fast path of the flattened scans when L is a multiple of 16 dividing the
+// 4096-element tile: every thread's 16 consecutive elements lie in one
+// system, so y / x and the coefficient runs move as 128-bit words.
+template <bool FWD>
+__global__ void __launch_bounds__(256) tridag_flat16_kernel(const float* __restrict__ y, float* __restrict__ x,
+                                                            const float* __restrict__ invb,
+                                                            const float* __restrict__ alpha,
+                                                            const float* __restrict__ delta, int64_t S, int64_t L,
+                                                            int64_t R) {
+    __shared__ Aff wtot[8];
+    constexpr int IT = 16;
+    const int64_t e0 = (int64_t)blockIdx.x * 4096 + threadIdx.x * IT;  // global flat index of the run
+    const bool live = e0 < S * L;
+    const int64_t s = live ? e0 / L : 0, j0 = live ? e0 - s * L : 0, r = s % R;
+    float mm[IT], ad[IT];
+    if (live) {
+#pragma unroll
+        for (int q = 0; q < IT; q += 4) {
+            const float4 c4 = __ldg(reinterpret_cast<const float4*>((FWD ? alpha : delta) + r * L + j0 + q));
+            mm[q] = c4.x; mm[q + 1] = c4.y; mm[q + 2] = c4.z; mm[q + 3] = c4.w;
+            if (FWD) {
+                const float4 y4 = __ldg(reinterpret_cast<const float4*>(y + e0 + q));
+                ad[q] = y4.x; ad[q + 1] = y4.y; ad[q + 2] = y4.z; ad[q + 3] = y4.w;
+            } else {
+                const float4 x4 = *reinterpret_cast<const float4*>(x + e0 + q);
+                const float4 i4 = __ldg(reinterpret_cast<const float4*>(invb + r * L + j0 + q));
+                ad[q] = x4.x * i4.x; ad[q + 1] = x4.y * i4.y; ad[q + 2] = x4.z * i4.z; ad[q + 3] = x4.w * i4.w;
+            }
         }
     } else {
-        for (int64_t e = e1 - 1; e >= e0; --e) {
-            float m, ad;
-            coef(e, m, ad);
-            f = aff_after(Aff{m, ad}, f);
+#pragma unroll
+        for (int q = 0; q < IT; ++q) {
+            mm[q] = 1.f;
+            ad[q] = 0.f;
         }
+    }
+    Aff f{1.f, 0.f};
+    if (FWD) {
+#pragma unroll
+        for (int q = 0; q < IT; ++q) f = aff_after(Aff{mm[q], ad[q]}, f);
+    } else {
+#pragma unroll
+        for (int q = IT - 1; q >= 0; --q) f = aff_after(Aff{mm[q], ad[q]}, f);
     }
     Aff tot;
     const Aff pf = group_exscan<!FWD>(f, 256, wtot, tot);
     float v = pf.g;
     if (FWD) {
-        for (int64_t e = e0; e < e1; ++e) {
-            float m, ad;
-            coef(e, m, ad);
-            v = fmaf(m, v, ad);
-            x[base + e] = v;
-        }
+#pragma unroll
+        for (int q = 0; q < IT; ++q) ad[q] = v = fmaf(mm[q], v, ad[q]);
     } else {
-        for (int64_t e = e1 - 1; e >= e0; --e) {
-            float m, ad;
-            coef(e, m, ad);
-            v = fmaf(m, v, ad);
-            x[base + e] = v;
-        }
+#pragma unroll
+        for (int q = IT - 1; q >= 0; --q) ad[q] = v = fmaf(mm[q], v, ad[q]);
+    }
+    if (live) {
+#pragma unroll
+        for (int q = 0; q < IT; q += 4)
+            *reinterpret_cast<float4*>(x + e0 + q) = make_float4(ad[q], ad[q + 1], ad[q + 2], ad[q + 3]);
     }
 }
 
@@ -396,6 +461,14 @@ cudaError_t launch_tridag(int version, const TriArgs& t) {
         if (it <= 4) tridag_mid_kernel<4><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
         else if (it <= 8) tridag_mid_kernel<8><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
         else tridag_mid_kernel<16><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
+        return cudaGetLastError();
+    }
+    const bool aligned = ((uintptr_t)t.y % 16 == 0) && ((uintptr_t)t.x % 16 == 0) && ((uintptr_t)t.ws % 16 == 0);
+    if (aligned && L % 16 == 0 && 4096 % L == 0) {
+        const int64_t grid16 = ceil_div(S * L, 4096);
+        tridag_flat16_kernel<true><<<(unsigned)grid16, 256, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        tridag_flat16_kernel<false><<<(unsigned)grid16, 256, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R);
         return cudaGetLastError();
     }
     const int64_t spt = std::max<int64_t>(1, 4096 / L);
