@@ -151,8 +151,14 @@ def run_ours(args, rank, world, device):
             tuned[site] = {"t_top": a, "t_intra": b}
             del scratch
         log(f"[bench] tuned in {time.time() - t0:.1f}s: {tuned}")
+        if rank == 0:  # reused by the ncu launch-list pass (--no-tune --thresholds)
+            os.makedirs(os.path.dirname(args.detail), exist_ok=True)
+            ifl.save_thresholds(os.path.join(os.path.dirname(args.detail), "thresholds.txt"))
     if args.thresholds:
         ifl.load_thresholds(args.thresholds)
+        for site in ("segred.b4", "segscan.b4"):
+            a, b = ifl.get_thresholds(site)
+            tuned[site] = {"t_top": a, "t_intra": b, "from": os.path.basename(args.thresholds)}
 
     # ---- resident inputs: two copies > L2, alternate per step
     xs = [gen.generate("F32_UNIT", 2 + rank * 101, N, device=device),
@@ -410,6 +416,7 @@ def run_reference(args, rank, world):
 
 
 def main():
+    os.environ.setdefault("NCCL_DEBUG", "WARN")  # keep NCCL's banner off the JSON stdout
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)

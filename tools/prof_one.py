@@ -14,10 +14,31 @@ ap.add_argument("--op", default="segred")
 ap.add_argument("--version", default="flat")
 ap.add_argument("--n", type=int, default=1)
 ap.add_argument("--m", type=int, default=1 << 26)
+ap.add_argument("--p", type=int, default=1, help="redomap2: columns of C; tridag: coefficient rows R")
+ap.add_argument("--dt", default="bf16", help="redomap2 input dtype")
 ap.add_argument("--reps", type=int, default=3)
 a = ap.parse_args()
-x = gen.generate("F32_UNIT", 2, a.n * a.m, device="cuda").view(a.n, a.m)
-fn = ifl.segred if a.op == "segred" else ifl.segscan
+if a.op == "redomap2":
+    tdt = torch.bfloat16 if a.dt == "bf16" else torch.float32
+    A = gen.generate("BF16_SIGNED", 6, a.n * a.m, device="cuda").view(a.n, a.m).to(tdt)
+    Bt = gen.generate("BF16_SIGNED", 7, a.p * a.m, device="cuda").view(a.p, a.m).to(tdt)
+    C = torch.empty(a.n, a.p, device="cuda")
+    ws = ifl.workspace(ifl.workspace_bytes("redomap2", a.n, a.m, a.p, a.dt), "cuda", "mm")
+    x = None
+
+    def fn(_x, version):
+        return ifl.redomap2(A, Bt, out=C, ws=ws, version=version)
+elif a.op == "tridag":
+    ta, tb, tc, ty = (t.cuda() for t in gen.tridag_system(7, a.n, a.m, a.p))
+    tx = torch.empty_like(ty)
+    ws = ifl.workspace(ifl.workspace_bytes("tridag", a.n, a.m, a.p), "cuda", "tri")
+    x = None
+
+    def fn(_x, version):
+        return ifl.tridag(ta, tb, tc, ty, out=tx, ws=ws, version=version)
+else:
+    x = gen.generate("F32_UNIT", 2, a.n * a.m, device="cuda").view(a.n, a.m)
+    fn = ifl.segred if a.op == "segred" else ifl.segscan
 for _ in range(a.reps):
     fn(x, version=a.version)
 torch.cuda.synchronize()

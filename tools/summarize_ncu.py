@@ -38,9 +38,13 @@ ALG = {  # algorithmic bytes of the captured launch
     "segscan_flat_n1": 8 * 2**26, "segscan_flat_n4096": 8 * 2**26, "segred_flat_n1": 4 * (2**26 + 1),
     "segred_middle_n1024": 4 * (2**26 + 1024), "segscan_middle_n2e18": 8 * 2**26,
     "segred_top_n2e24": 4 * (2**26 + 2**24), "segscan_top_n2e23": 8 * 2**26,
+    "redomap2_tc_8192": 2 * (2 * 8192 * 8192) + 4 * 8192 * 8192, "redomap2_flat_n1": 2 * (2 * 2**30) + 4,
+    "tridag_middle_large": 8 * 65536 * 256, "tridag_flat_large": 8 * 65536 * 256,
 }
 GROUP = {"segscan_flat_n1": "segscan_flat", "segred_flat_n1": "segred_flat", "segred_middle_n1024": "segred_middle",
-         "segscan_middle_n2e18": "segscan_middle", "segred_top_n2e24": "segred_top", "segscan_top_n2e23": "segscan_top"}
+         "segscan_middle_n2e18": "segscan_middle", "segred_top_n2e24": "segred_top", "segscan_top_n2e23": "segscan_top",
+         "redomap2_tc_8192": "redomap2_tc", "redomap2_flat_n1": "redomap2_flat", "tridag_middle_large": "tridag_middle",
+         "tridag_flat_large": "tridag_flat"}
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_sector_hit_rate.pct",
         "sm__warps_active.avg.pct_of_peak_sustained_active", "smsp__issue_active.avg.pct_of_peak_sustained_active",
@@ -84,7 +88,7 @@ for f in sorted(glob.glob(os.path.join(src, "*.raw.csv"))):
         traffic[GROUP[name]] = {"capture": name, "dram_bytes_per_launch": rdb + wrb, "algorithmic_bytes": alg,
                                 "ratio": round(ratio, 4), "ncu_time_us": round(t_us, 2)}
 md.append("\nLaunch-list shares (`--metrics gpu__time_duration.sum`, bench command with "
-          "`--steps 2 --warmup 3 --no-tune`): `profiles/%s_ncu_launches_summary.csv`." % tag)
+          "`--steps 2 --warmup 3 --no-e2e --no-cpu --no-forced`): `profiles/%s_ncu_launches_summary.csv`." % tag)
 open(f"profiles/{tag}_ncu_summary.md", "w").write("\n".join(md) + "\n")
 json.dump(traffic, open("profiles/ncu_traffic.json", "w"), indent=1)
 print("\n".join(md))
