@@ -98,14 +98,26 @@ __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, uint32_t (&r)
 // Item = (k-split z, output tile); items are strided by gridDim.x.  The MMA
 // warp accumulates item i into accumulator i & 1 while the epilogue drains
 // item i-1 from the other one (tmem_full / tmem_empty mbarriers).
+// Epilogue: with TST (C 16-byte aligned, p % 4 == 0) each warp writes its
+// 32 x 32 fp32 chunk into a 128-byte-swizzled, double-buffered staging tile
+// and one lane stores it with a 3-D TMA bulk-tensor store ({col,row,split});
+// otherwise a padded smem transpose feeds coalesced row stores.
 constexpr int TC_THREADS = 192;
-constexpr int TC_EPI_BYTES = 4 * 32 * 33 * 4;
+constexpr int TC_EPI_BYTES = 4 * 2 * 32 * 32 * 4;  // 4 warps x 2 buffers x 4 KB (>= 4 x 32 x 33 x 4)
 constexpr int TC_SMEM_P = TC_STAGES * TC_STAGE_BYTES + TC_EPI_BYTES + 1024;
 
-__global__ void __launch_bounds__(TC_THREADS, 1) mm_top_tc_kernel(const __grid_constant__ CUtensorMap mapA,
-                                                                  const __grid_constant__ CUtensorMap mapB, float* C,
-                                                                  float* part, int64_t n, int64_t m, int64_t p,
-                                                                  int kps, int splits) {
+__device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void* src, int c0, int c1, int c2) {
+    asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+                     reinterpret_cast<uint64_t>(map)),
+                 "r"(smem_u32(src)), "r"(c0), "r"(c1), "r"(c2)
+                 : "memory");
+}
+
+template <bool TST>
+__global__ void __launch_bounds__(TC_THREADS, 1)
+    mm_top_tc_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
+                     const __grid_constant__ CUtensorMap mapC, float* C, float* part, int64_t n, int64_t m,
+                     int64_t p, int kps, int splits) {
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
     float* stage_base = reinterpret_cast<float*>(smem + TC_STAGES * TC_STAGE_BYTES);
@@ -137,6 +149,7 @@ __global__ void __launch_bounds__(TC_THREADS, 1) mm_top_tc_kernel(const __grid_c
         fence_mbar_init();
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapA)) : "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapB)) : "memory");
+        if (TST) asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&mapC)) : "memory");
     }
     if (warp == 1) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tmem_base)),
@@ -194,8 +207,8 @@ __global__ void __launch_bounds__(TC_THREADS, 1) mm_top_tc_kernel(const __grid_c
     } else {
         // ---- epilogue warps 2..5: TMEM -> registers -> padded smem -> coalesced rows
         const int quad = warp & 3;  // TMEM lane quadrant this warp may access
-        float* stage = stage_base + (warp - 2) * (32 * 33);
-        int li = 0;
+        float* stage = stage_base + (warp - 2) * (2 * 32 * 32);
+        int li = 0, nst = 0;
         for (int it = blockIdx.x; it < items; it += gridDim.x, ++li) {
             int z, m0, n0, kt0, nk;
             decode(it, z, m0, n0, kt0, nk);
@@ -208,20 +221,42 @@ __global__ void __launch_bounds__(TC_THREADS, 1) mm_top_tc_kernel(const __grid_c
             for (int c = 0; c < TC_BN; c += 32) {
                 uint32_t r[32];
                 tmem_ld_32x32b_x32(tmem + ((uint32_t)(quad * 32) << 16) + (uint32_t)(acc * TC_TMEM_COLS + c), r);
-#pragma unroll
-                for (int q = 0; q < 32; ++q) stage[lane * 33 + q] = __uint_as_float(r[q]);
-                __syncwarp();
-                const int64_t col = (int64_t)n0 + c + lane;
-                for (int rr = 0; rr < 32; ++rr) {
-                    const int64_t row = (int64_t)m0 + quad * 32 + rr;
-                    if (row < n && col < p) out[row * p + col] = stage[rr * 33 + lane];
+                if (c + 32 == TC_BN) {  // accumulator drained: let the MMA warp reuse it
+                    tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) mbar_arrive_expect_tx(&tempty[acc], 0);
                 }
-                __syncwarp();
+                if constexpr (TST) {
+                    if (n0 + c >= p) continue;
+                    float* buf = stage + (nst & 1) * (32 * 32);
+                    if (lane == 0) bulk_wait_read1();  // the store that last read buf has finished
+                    __syncwarp();
+                    float4* row = reinterpret_cast<float4*>(buf + lane * 32);
+#pragma unroll
+                    for (int q = 0; q < 8; ++q)
+                        row[q ^ (lane & 7)] = make_float4(__uint_as_float(r[4 * q]), __uint_as_float(r[4 * q + 1]),
+                                                          __uint_as_float(r[4 * q + 2]), __uint_as_float(r[4 * q + 3]));
+                    fence_proxy_async_smem();
+                    __syncwarp();
+                    if (lane == 0) {
+                        tma_store_3d(&mapC, buf, n0 + c, m0 + quad * 32, splits == 1 ? 0 : z);
+                        bulk_commit();
+                    }
+                    ++nst;
+                } else {
+#pragma unroll
+                    for (int q = 0; q < 32; ++q) stage[lane * 33 + q] = __uint_as_float(r[q]);
+                    __syncwarp();
+                    const int64_t col = (int64_t)n0 + c + lane;
+                    for (int rr = 0; rr < 32; ++rr) {
+                        const int64_t row = (int64_t)m0 + quad * 32 + rr;
+                        if (row < n && col < p) out[row * p + col] = stage[rr * 33 + lane];
+                    }
+                    __syncwarp();
+                }
             }
-            tc_fence_before();
-            __syncwarp();
-            if (lane == 0) mbar_arrive_expect_tx(&tempty[acc], 0);
         }
+        if (TST && lane == 0) bulk_wait0();
     }
     tc_fence_before();
     __syncthreads();
@@ -261,6 +296,19 @@ static bool make_map(CUtensorMap* map, const void* base, int64_t rows, int64_t k
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// fp32 output [splits][n][p] as a 3-D map, 32 x 32 boxes, 128-byte swizzle
+static bool make_out_map(CUtensorMap* map, float* base, int64_t n, int64_t p, int splits) {
+    EncodeTiledFn fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[3] = {(cuuint64_t)p, (cuuint64_t)n, (cuuint64_t)splits};
+    const cuuint64_t strides[2] = {(cuuint64_t)p * 4, (cuuint64_t)(n * p * 4)};
+    const cuuint32_t box[3] = {32, 32, 1};
+    const cuuint32_t estr[3] = {1, 1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, base, dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+              CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 // TMA needs 16-byte-aligned bases and row pitches (m % 8 == 0 for bf16);
 // everything else (ragged n, p, m) is covered by TMA zero-fill and masking.
 bool tc_shape_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* Bt) {
@@ -295,11 +343,15 @@ cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* par
     if (!make_map(&ma, A, n, m, TC_BM) || !make_map(&mb, Bt, p, m, TC_BN)) return cudaErrorInvalidValue;
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(mm_top_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
+        cudaFuncSetAttribute(mm_top_tc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
+        cudaFuncSetAttribute(mm_top_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
     });
     const int nk = (int)ceil_div(m, TC_BK);
     const int kps = (int)ceil_div(nk, splits);
     splits = (int)ceil_div(nk, kps);
+    float* out = splits == 1 ? C : part;
+    CUtensorMap mc;
+    const bool tst = p % 4 == 0 && (uintptr_t)out % 16 == 0 && make_out_map(&mc, out, n, p, splits);
     const int64_t items = ceil_div(n, TC_BM) * ceil_div(p, TC_BN) * splits;
     static int sms = 0;
     if (!sms) {
@@ -309,7 +361,10 @@ cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* par
         if (sms <= 0) sms = 148;
     }
     const int grid = (int)std::min<int64_t>(items, sms);
-    mm_top_tc_kernel<<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, C, part, n, m, p, kps, splits);
+    if (tst)
+        mm_top_tc_kernel<true><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, mc, C, part, n, m, p, kps, splits);
+    else
+        mm_top_tc_kernel<false><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, ma, C, part, n, m, p, kps, splits);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess || splits == 1) return e;
     const int64_t outs = n * p;
