@@ -178,12 +178,13 @@ constexpr int kTriItems = 8;
 // Group-wide exclusive scan of affine maps (older lanes first).  G threads
 // per group; G <= 32 uses shuffles only, larger groups go through shared
 // memory (warp totals).  REV scans from the last lane backwards.
-template <bool REV>
-__device__ __forceinline__ Aff group_exscan(Aff v, int G, Aff* wtot, Aff& total) {
+template <bool REV, int G>
+__device__ __forceinline__ Aff group_exscan(Aff v, Aff* wtot, Aff& total) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    const int width = G < 32 ? G : 32;
+    constexpr int width = G < 32 ? G : 32;
     const int gl = threadIdx.x % width;
     Aff inc = v;
+#pragma unroll
     for (int off = 1; off < width; off <<= 1) {
         const float oa = REV ? __shfl_down_sync(0xffffffffu, inc.a, off, width) : __shfl_up_sync(0xffffffffu, inc.a, off, width);
         const float og = REV ? __shfl_down_sync(0xffffffffu, inc.g, off, width) : __shfl_up_sync(0xffffffffu, inc.g, off, width);
@@ -195,16 +196,18 @@ __device__ __forceinline__ Aff group_exscan(Aff v, int G, Aff* wtot, Aff& total)
     ex.g = REV ? __shfl_down_sync(0xffffffffu, inc.g, 1, width) : __shfl_up_sync(0xffffffffu, inc.g, 1, width);
     const bool first = REV ? (gl == width - 1) : (gl == 0);
     if (first) ex = Aff{1.f, 0.f};
-    if (G <= 32) {
+    if constexpr (G <= 32) {
         const int src = REV ? 0 : width - 1;
         total = Aff{__shfl_sync(0xffffffffu, inc.a, src, width), __shfl_sync(0xffffffffu, inc.g, src, width)};
         return ex;
     }
-    const int wpg = G >> 5, w0 = (threadIdx.x / G) * wpg;
+    constexpr int wpg = G >> 5;
+    const int w0 = (threadIdx.x / G) * wpg;
     if (REV ? lane == 0 : lane == 31) wtot[w] = inc;
     __syncthreads();
     Aff before{1.f, 0.f};
     total = Aff{1.f, 0.f};
+#pragma unroll
     for (int k = 0; k < wpg; ++k) {
         const int kk = REV ? (wpg - 1 - k) : k;  // oldest first
         const Aff t = wtot[w0 + kk];
@@ -221,31 +224,33 @@ int tridag_group(int64_t L) {
     return (int)std::max<int64_t>(g, 1);
 }
 
-template <int IT>
+// A group of G threads (IT items each) solves `spg` systems that share one
+// coefficient row r (s = r + R*q, R9): the row's alpha / invbeta / delta are
+// loaded once into registers, and the next system's y is prefetched while
+// the current one is scanned.  Consecutive groups take consecutive r, so a
+// warp-wide load still covers adjacent systems.
+template <int IT, int G>
 __global__ void __launch_bounds__(256) tridag_mid_kernel(const float* __restrict__ y, float* __restrict__ x,
                                                          const float* __restrict__ invb, const float* __restrict__ alpha,
                                                          const float* __restrict__ delta, int64_t S, int64_t L,
-                                                         int64_t R, int G) {
+                                                         int64_t R, int spg) {
     __shared__ Aff wtot[8];
     const int g = threadIdx.x % G;
-    const int64_t s = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
-    const bool live = s < S;
-    const int64_t r = live ? s % R : 0;
-    const float* ys = y + (live ? s * L : 0);
-    float* xs = x + (live ? s * L : 0);
+    const int64_t gid = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
+    const int64_t qc = gid / R, r = gid - qc * R, q0 = qc * spg;
+    // systems of this group: s = r + R*(q0 + i), i < nq
+    const int nq = r + R * q0 < S ? (int)std::min<int64_t>(spg, (S - 1 - r) / R + 1 - q0) : 0;
+    const bool live = nq > 0;  // (a dead group still joins the group scans)
     const int64_t j0 = (int64_t)g * IT;
-    float yv[IT], al[IT], ib[IT], de[IT];
-    // 128-bit loads when the thread's IT items are whole aligned float4s
-    const bool vec = live && (L % 4 == 0) && (j0 + IT <= L) && (((uintptr_t)ys & 15) == 0) &&
+    float yv[IT], yn[IT], al[IT], ib[IT], de[IT];
+    const bool vec = (L % 4 == 0) && (j0 + IT <= L) && (((uintptr_t)y & 15) == 0) && (((uintptr_t)x & 15) == 0) &&
                      (((uintptr_t)(alpha + r * L) & 15) == 0);
-    if (vec) {
+    if (vec && live) {
 #pragma unroll
         for (int k = 0; k < IT; k += 4) {
-            const float4 y4 = __ldg(reinterpret_cast<const float4*>(ys + j0 + k));
             const float4 a4 = __ldg(reinterpret_cast<const float4*>(alpha + r * L + j0 + k));
             const float4 i4 = __ldg(reinterpret_cast<const float4*>(invb + r * L + j0 + k));
             const float4 d4 = __ldg(reinterpret_cast<const float4*>(delta + r * L + j0 + k));
-            yv[k] = y4.x; yv[k + 1] = y4.y; yv[k + 2] = y4.z; yv[k + 3] = y4.w;
             al[k] = a4.x; al[k + 1] = a4.y; al[k + 2] = a4.z; al[k + 3] = a4.w;
             ib[k] = i4.x; ib[k + 1] = i4.y; ib[k + 2] = i4.z; ib[k + 3] = i4.w;
             de[k] = d4.x; de[k + 1] = d4.y; de[k + 2] = d4.z; de[k + 3] = d4.w;
@@ -253,45 +258,71 @@ __global__ void __launch_bounds__(256) tridag_mid_kernel(const float* __restrict
     } else {
 #pragma unroll
         for (int k = 0; k < IT; ++k) {
-            const int64_t j = j0 + k;
-            const bool ok = live && j < L;
-            yv[k] = ok ? __ldg(ys + j) : 0.f;
-            al[k] = ok ? __ldg(alpha + r * L + j) : 1.f;
-            ib[k] = ok ? __ldg(invb + r * L + j) : 0.f;
-            de[k] = ok ? __ldg(delta + r * L + j) : 1.f;
+            const bool ok = live && j0 + k < L;
+            al[k] = ok ? __ldg(alpha + r * L + j0 + k) : 1.f;
+            ib[k] = ok ? __ldg(invb + r * L + j0 + k) : 0.f;
+            de[k] = ok ? __ldg(delta + r * L + j0 + k) : 1.f;
         }
     }
-    // (x) forward: thread composite of its items, group exclusive prefix, apply
-    Aff f{1.f, 0.f};
+    const int64_t stride = R * L;
+    const float* yp = y + (live ? (r + R * q0) * L : 0) + j0;
+    float* xp = x + (live ? (r + R * q0) * L : 0) + j0;
+    auto load_y = [&](int i, float (&dst)[IT]) {
+        const bool ok = i < nq;
+        const float* ys = yp + (ok ? i * stride : 0);
+        if (vec && ok) {
 #pragma unroll
-    for (int k = 0; k < IT; ++k) f = aff_after(Aff{al[k], yv[k]}, f);
-    Aff tot;
-    const Aff pf = group_exscan<false>(f, G, wtot, tot);
-    float v = pf.g;  // y' before this thread's first item (the prefix applied to 0)
+            for (int k = 0; k < IT; k += 4) {
+                const float4 y4 = ldg_stream4<float>(ys + k);
+                dst[k] = y4.x; dst[k + 1] = y4.y; dst[k + 2] = y4.z; dst[k + 3] = y4.w;
+            }
+        } else {
 #pragma unroll
-    for (int k = 0; k < IT; ++k) {
-        v = fmaf(al[k], v, yv[k]);
-        yv[k] = v * ib[k];  // epsilon_j = y'_j / beta_j
-    }
-    // (.) backward
-    Aff bk{1.f, 0.f};
+            for (int k = 0; k < IT; ++k) dst[k] = (ok && j0 + k < L) ? __ldg(ys + k) : 0.f;
+        }
+    };
+    load_y(0, yv);
+    // every group runs the same trip count so that group scans over shared
+    // memory (G > 32) stay block-uniform
+    for (int i = 0; i < spg; ++i) {
+        if (spg > 1) load_y(i + 1, yn);  // prefetch the next system of this row
+        // (x) forward: thread composite of its items, group exclusive prefix, apply
+        Aff f{1.f, 0.f};
 #pragma unroll
-    for (int k = IT - 1; k >= 0; --k) bk = aff_after(Aff{de[k], yv[k]}, bk);
-    const Aff pb = group_exscan<true>(bk, G, wtot, tot);
-    float u = pb.g;
+        for (int k = 0; k < IT; ++k) f = aff_after(Aff{al[k], yv[k]}, f);
+        Aff tot;
+        const Aff pf = group_exscan<false, G>(f, wtot, tot);
+        float v = pf.g;  // y' before this thread's first item (the prefix applied to 0)
 #pragma unroll
-    for (int k = IT - 1; k >= 0; --k) {
-        u = fmaf(de[k], u, yv[k]);
-        yv[k] = u;
-    }
-    if (vec && ((((uintptr_t)xs) & 15) == 0)) {
+        for (int k = 0; k < IT; ++k) {
+            v = fmaf(al[k], v, yv[k]);
+            yv[k] = v * ib[k];  // epsilon_j = y'_j / beta_j
+        }
+        // (.) backward
+        Aff bk{1.f, 0.f};
 #pragma unroll
-        for (int k = 0; k < IT; k += 4)
-            *reinterpret_cast<float4*>(xs + j0 + k) = make_float4(yv[k], yv[k + 1], yv[k + 2], yv[k + 3]);
-    } else {
+        for (int k = IT - 1; k >= 0; --k) bk = aff_after(Aff{de[k], yv[k]}, bk);
+        const Aff pb = group_exscan<true, G>(bk, wtot, tot);
+        float u = pb.g;
 #pragma unroll
-        for (int k = 0; k < IT; ++k)
-            if (live && j0 + k < L) xs[j0 + k] = yv[k];
+        for (int k = IT - 1; k >= 0; --k) {
+            u = fmaf(de[k], u, yv[k]);
+            yv[k] = u;
+        }
+        if (i < nq) {
+            float* xs = xp + i * stride;
+            if (vec) {
+#pragma unroll
+                for (int k = 0; k < IT; k += 4)
+                    __stcs(reinterpret_cast<float4*>(xs + k), make_float4(yv[k], yv[k + 1], yv[k + 2], yv[k + 3]));
+            } else {
+#pragma unroll
+                for (int k = 0; k < IT; ++k)
+                    if (j0 + k < L) xs[k] = yv[k];
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < IT; ++k) yv[k] = yn[k];
     }
 }
 
@@ -356,7 +387,7 @@ __global__ void __launch_bounds__(256) tridag_flat_kernel(const float* __restric
         f = aff_after(Aff{mm, ad}, f);
     });
     Aff tot;
-    const Aff pf = group_exscan<!FWD>(f, 256, wtot, tot);
+    const Aff pf = group_exscan<!FWD, 256>(f, wtot, tot);
     float v = pf.g;
     walk([&](int64_t gi, int64_t ci) {
         float mm, ad;
@@ -411,7 +442,7 @@ __global__ void __launch_bounds__(256) tridag_flat16_kernel(const float* __restr
         for (int q = IT - 1; q >= 0; --q) f = aff_after(Aff{mm[q], ad[q]}, f);
     }
     Aff tot;
-    const Aff pf = group_exscan<!FWD>(f, 256, wtot, tot);
+    const Aff pf = group_exscan<!FWD, 256>(f, wtot, tot);
     float v = pf.g;
     if (FWD) {
 #pragma unroll
@@ -456,11 +487,29 @@ cudaError_t launch_tridag(int version, const TriArgs& t) {
     if (version == 1) {
         const int G = tridag_group(L);
         const int B = std::max(G, 32) > 256 ? G : 256;
-        const int64_t grid = ceil_div(S, B / G);
+        // systems per group: as many as keep ~8 CTAs' worth of groups on
+        // every SM (one coefficient load then serves them all)
+        const int64_t Rr = std::min(R, S), Q = ceil_div(S, Rr);
+        const int64_t want_groups = (int64_t)148 * 8 * (B / G);
+        const int spg = (int)std::max<int64_t>(1, std::min<int64_t>({(int64_t)8, Q, (Rr * Q) / want_groups}));
+        const int64_t groups = Rr * ceil_div(Q, spg);
+        const int64_t grid = ceil_div(groups, B / G);
         const int64_t it = ceil_div(L, G);
-        if (it <= 4) tridag_mid_kernel<4><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
-        else if (it <= 8) tridag_mid_kernel<8><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
-        else tridag_mid_kernel<16><<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R, G);
+        auto go = [&](auto kern) {
+            kern<<<(unsigned)grid, B, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, Rr, spg);
+        };
+        switch (G) {
+            case 1: go(it <= 4 ? tridag_mid_kernel<4, 1> : tridag_mid_kernel<8, 1>); break;
+            case 2: go(it <= 4 ? tridag_mid_kernel<4, 2> : tridag_mid_kernel<8, 2>); break;
+            case 4: go(it <= 4 ? tridag_mid_kernel<4, 4> : tridag_mid_kernel<8, 4>); break;
+            case 8: go(it <= 4 ? tridag_mid_kernel<4, 8> : tridag_mid_kernel<8, 8>); break;
+            case 16: go(it <= 4 ? tridag_mid_kernel<4, 16> : tridag_mid_kernel<8, 16>); break;
+            case 32: go(it <= 4 ? tridag_mid_kernel<4, 32> : tridag_mid_kernel<8, 32>); break;
+            case 64: go(it <= 4 ? tridag_mid_kernel<4, 64> : tridag_mid_kernel<8, 64>); break;
+            case 128: go(it <= 4 ? tridag_mid_kernel<4, 128> : tridag_mid_kernel<8, 128>); break;
+            default:
+                go(it <= 4 ? tridag_mid_kernel<4, 256> : it <= 8 ? tridag_mid_kernel<8, 256> : tridag_mid_kernel<16, 256>);
+        }
         return cudaGetLastError();
     }
     const bool aligned = ((uintptr_t)t.y % 16 == 0) && ((uintptr_t)t.x % 16 == 0) && ((uintptr_t)t.ws % 16 == 0);
