@@ -127,6 +127,24 @@ def segscan(x: np.ndarray, op: str = "sum", f: str = "id", d=None, reverse=False
     raise TypeError(x.dtype)
 
 
+def segscan_seeded(x: np.ndarray, seed: np.ndarray, op: str = "sum", f: str = "id", with_absum=False):
+    """P:79's scan with d replaced row by row (ifl_segscan_seeded):
+    out[i,j] = seed[i] (+) f(x[i,0]) (+) ... (+) f(x[i,j]).  Row i is exactly
+    segscan(x[i:i+1], d=seed[i]); for f32 the tolerance base adds |seed[i]|."""
+    x = np.ascontiguousarray(x)
+    n, m = x.shape
+    outs, abs_ = [], []
+    for i in range(n):
+        o, ab = segscan(x[i:i + 1], op, f, d=seed[i], with_absum=True)
+        outs.append(o)
+        if ab is not None:
+            abs_.append(ab + abs(float(seed[i])))
+    out = np.concatenate(outs) if n else (np.empty((0, m), np.int32 if x.dtype == np.int32 else np.float64))
+    if not with_absum:
+        return out
+    return out, (np.concatenate(abs_) if abs_ else None)
+
+
 def colred(x: np.ndarray, op: str = "sum", f: str = "id", d=None):
     """P:156 (G4 left-hand side): column reduction of an [n][m] matrix."""
     x = np.ascontiguousarray(x)

@@ -60,6 +60,7 @@ _i64, _int, _vp, _sz = ctypes.c_int64, ctypes.c_int, ctypes.c_void_p, ctypes.c_s
 _SIGS = {
     "ifl_segred": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segscan": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_segscan_seeded": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_redomap2": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_tridag": ([_vp, _vp, _vp, _vp, _vp, _i64, _i64, _i64, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_workspace_bytes": ([ctypes.c_char_p, _i64, _i64, _i64, _int, _int], _sz),
@@ -204,11 +205,13 @@ def _choice_out(c: ifl_choice) -> Choice:
 # ---------------------------------------------------------- segred / segscan
 
 
-def _seg(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws, stream, return_choice):
+def _seg(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws, stream, return_choice,
+         seed=None):
     host = not x.is_cuda
     if host:  # end-to-end path: pinned host -> device -> host
         xd = x.to("cuda", non_blocking=True)
-        r = _seg(scan, xd, op, f, ne, version, None, ws, stream, return_choice)
+        sd = None if seed is None else seed.to("cuda", non_blocking=True)
+        r = _seg(scan, xd, op, f, ne, version, None, ws, stream, return_choice, sd)
         if return_choice:
             r, c = r
         o = torch.empty(r.shape, dtype=r.dtype, pin_memory=True) if out is None else out
@@ -233,7 +236,12 @@ def _seg(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws
     args = (x.data_ptr(), out.data_ptr(), n, m, DTYPES[dt], OPS[op], MAPS[f], _ne_buf(ne, dt))
     tail = (VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel() * ws.element_size(),
             _stream(stream), ctypes.byref(c))
-    if scan:
+    if seed is not None:
+        if seed.dtype != x.dtype or seed.numel() != n or not seed.is_contiguous() or seed.device != x.device:
+            raise ValueError("seed must be a contiguous [n] tensor of x's dtype on x's device")
+        rc = lib().ifl_segscan_seeded(*args[:7], seed.data_ptr(), *tail)
+        entry = "segscan_seeded"
+    elif scan:
         rc = lib().ifl_segscan(*args, 0, *tail)
     else:
         rc = lib().ifl_segred(*args, *tail)
@@ -246,9 +254,14 @@ def segred(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stre
     return _seg(False, x, op, f, ne, version, out, ws, stream, return_choice)
 
 
-def segscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False):
-    """Inclusive per-row scanomap (example P:116)."""
-    return _seg(True, x, op, f, ne, version, out, ws, stream, return_choice)
+def segscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False,
+            seed=None):
+    """Inclusive per-row scanomap (example P:116).  ``seed``
+    (an [n] tensor) replaces ne row by row: out[i,j] = seed[i] (+) f(x[i,0])
+    (+) ... (+) f(x[i,j]) -- the carry-in of a column block (ifl_segscan_seeded)."""
+    if seed is not None and ne is not None:
+        raise ValueError("pass either ne or seed")
+    return _seg(True, x, op, f, ne, version, out, ws, stream, return_choice, seed)
 
 
 # ------------------------------------------------------------------ redomap2

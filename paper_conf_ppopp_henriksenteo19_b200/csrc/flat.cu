@@ -373,7 +373,8 @@ __global__ void __launch_bounds__(512) flat_red_fix_long(T* out, int64_t n, int6
 
 // Thread-local segmented inclusive scan of the thread's items (in registers).
 template <typename T, int OP, int F>
-__device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, T d, bool& has_start, T& acc) {
+__device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, T d, bool& has_start, T& acc,
+                                               const T* __restrict__ seed) {
     has_start = false;
     acc = identity<OP, T>();
     if (tp.nx0 > tp.nvalid) {  // no boundary: plain inclusive scan
@@ -384,12 +385,14 @@ __device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, 
         }
     } else {
         int nx = tp.nx0;
+        int64_t ss = tp.seg + (tp.nx0 > 0 ? 1 : 0);  // segment the next start begins
 #pragma unroll
         for (int k = 0; k < FI; ++k) {
             if (k < tp.nvalid) {
                 const T x = apply_map<F>(v[k]);
                 if (k == nx) {
-                    acc = combine<OP>(d, x);
+                    acc = combine<OP>(seed ? seed[ss] : d, x);
+                    ++ss;
                     has_start = true;
                     nx += tp.mi;
                 } else {
@@ -429,7 +432,7 @@ constexpr int kScanSlots = 3;  // 60 KB ring: three CTAs (27 warps) per SM
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(kScanThreads, 3) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
                                                                     uint8_t* ws, int num_tiles, int num_chunks,
-                                                                    bool tma_in, bool tma_out) {
+                                                                    bool tma_in, bool tma_out, const T* __restrict__ seed) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
     __shared__ alignas(8) uint64_t full[kScanSlots], empty[kScanSlots];
@@ -541,7 +544,7 @@ __global__ void __launch_bounds__(kScanThreads, 3) flat_scan_kernel(const T* in,
                 load_items(buf, v);
                 bool hs;
                 T acc;
-                local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
+                local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
                 uint32_t exf, aggf;
                 T exv, aggv;
                 cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
@@ -620,7 +623,7 @@ __global__ void __launch_bounds__(kScanThreads, 3) flat_scan_kernel(const T* in,
             load_items(buf, v);
             bool hs;
             T acc;
-            local_seg_scan<T, OP, F>(v, tp, d, hs, acc);
+            local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
             uint32_t exf, aggf;
             T exv, aggv;
             cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
@@ -717,7 +720,8 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
             cfg.attrs = attr;
             cfg.numAttrs = 1;
             int nt = (int)tiles;
-            return cudaLaunchKernelEx(&cfg, k, (const T*)a.in, (T*)a.out, N, a.m, d, ws, nt, chunks, tma_in, tma_out);
+            return cudaLaunchKernelEx(&cfg, k, (const T*)a.in, (T*)a.out, N, a.m, d, ws, nt, chunks, tma_in, tma_out,
+                                      (const T*)a.seed);
         }
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
         T* tail = head + tiles;

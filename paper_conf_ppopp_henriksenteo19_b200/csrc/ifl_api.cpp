@@ -260,8 +260,9 @@ int ifl_workspace_init(void* ws, size_t ws_bytes, void* stream) {
 }
 
 static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f,
-                   const void* ne, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
-    const char* what = scan ? "ifl_segscan" : "ifl_segred";
+                   const void* ne, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice,
+                   const void* seed = nullptr) {
+    const char* what = seed ? "ifl_segscan_seeded" : scan ? "ifl_segscan" : "ifl_segred";
     int rc = validate_seg(scan, in, out, n, m, dt, op, f, version, what);
     if (rc) return rc;
     const size_t ob = (size_t)(scan ? n * m : n) * 4, ib = (size_t)(n * m) * 4;
@@ -270,6 +271,8 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
     } else if (overlap(in, ib, out, ob)) {
         return fail(IFL_EINVAL, "%s: out overlaps in", what);
     }
+    if (seed && (overlap(seed, (size_t)n * 4, out, ob) || overlap(seed, (size_t)n * 4, in, ib)))
+        return fail(IFL_EINVAL, "%s: seed overlaps in/out", what);
     uint32_t bits = canonical_bits(dt, op);
     if (ne) memcpy(&bits, ne, 4);
     const char* site = scan ? "segscan.b4" : "segred.b4";
@@ -283,7 +286,7 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
         return cuda_status(ifl::launch_fill(out, n, bits, (cudaStream_t)stream), what);
     }
     (void)v;
-    ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream};
+    ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream, seed};
     cudaError_t e;
     switch (c.version) {
     case IFL_V_TOP: e = scan ? ifl::launch_segscan_top(a) : ifl::launch_segred_top(a); break;
@@ -307,6 +310,12 @@ int ifl_segscan(const void* in, void* out, int64_t n, int64_t m, int dt, int op,
                 int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
     if (reverse) return fail(IFL_EUNSUPPORTED, "ifl_segscan: reverse scans are not exposed");
     return run_seg(true, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+}
+
+int ifl_segscan_seeded(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* seed,
+                       int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    if (n > 0 && m > 0 && !seed) return fail(IFL_EINVAL, "ifl_segscan_seeded: seed is NULL");
+    return run_seg(true, in, out, n, m, dt, op, f, nullptr, version, ws, ws_bytes, stream, choice, seed);
 }
 
 int ifl_redomap2(const void* A, const void* B, float* C, int64_t n, int64_t m, int64_t p, int in_dt, int b_kmajor,

@@ -17,6 +17,7 @@ struct SegArgs {
     void* ws;
     size_t ws_bytes;
     cudaStream_t stream;
+    const void* seed = nullptr;  // segscan: per-row d (device [n]) or NULL = ne_bits for every row
 };
 
 // Flat engine tile geometry (flat.cu).  ws layout: 256-byte header then one

@@ -92,7 +92,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
 
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T* out, int64_t n, int64_t m, T d,
-                                                                  bool vec) {
+                                                                  bool vec, const T* __restrict__ seed) {
     __shared__ T tile[kTopWords];
     const int t = threadIdx.x;
     const int rpt = stop_rpt(m);
@@ -108,7 +108,7 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
             for (int j = 0; j < rpt; ++j) {
                 const int r = t + j * kTopThreads;
                 if (r < rows) {
-                    Acc<OP, T> a(d);  // d (+) f(x0) (+) ...: d applied once, at the row start
+                    Acc<OP, T> a(seed ? seed[r0 + r] : d);  // d (+) f(x0) (+) ...: d applied once, at the row start
                     for (int k = 0; k < mm; ++k) {
                         a.add(apply_map<F>(tile[spadq(r * mm + k)]));
                         tile[spadq(r * mm + k)] = a.get();
@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
             top_xfer<false>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
             __syncthreads();
         } else {
-            Acc<OP, T> a(d);
+            Acc<OP, T> a((seed && t < rows) ? seed[r0 + t] : d);
             for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
                 const int kt = (int)min((int64_t)kTopKT, m - k0);
                 top_xfer<true>(tile, in, out, r0, rows, m, k0, kt, false, vec);
@@ -149,7 +149,8 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
 // V_TOP for m in {1, 2, 4} with 16-byte-aligned in/out: each 128-bit word
 // holds 4/m whole rows, scanned in registers and stored back as one word.
 template <typename T, int OP, int F, int M>
-__global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* out, int64_t n, T d) {
+__global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* out, int64_t n, T d,
+                                                                const T* __restrict__ seed) {
     using V = typename Vec4<T>::type;
     const int64_t N = n * M, nv = N >> 2;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -167,7 +168,8 @@ __global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* 
 #pragma unroll
             for (int k = 0; k < 4; ++k) {
                 const T x = apply_map<F>(e[k]);
-                e[k] = (k % M == 0) ? combine<OP>(d, x) : combine<OP>(e[k - 1 < 0 ? 0 : k - 1], x);
+                e[k] = (k % M == 0) ? combine<OP>(seed ? seed[(4 * v + k) / M] : d, x)
+                                    : combine<OP>(e[k - 1 < 0 ? 0 : k - 1], x);
             }
             V r;
             r.x = e[0]; r.y = e[1]; r.z = e[2]; r.w = e[3];
@@ -176,7 +178,7 @@ __global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* 
     }
     const int64_t r0 = (nv * 4) / M;
     for (int64_t r = r0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += stride) {
-        T a = d;
+        T a = seed ? seed[r] : d;
         for (int k = 0; k < M; ++k) {
             a = combine<OP>(a, apply_map<F>(in[r * M + k]));
             out[r * M + k] = a;
@@ -189,7 +191,7 @@ __global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* 
 // coalesced 128-bit accesses through a padded per-warp tile, and every lane
 // walks its own row sequentially (conflict-free: one pad word per 32).
 template <typename T, int OP, int F, int M, bool SCAN>
-__global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int64_t n, T d) {
+__global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int64_t n, T d, const T* __restrict__ seed) {
     using V = typename Vec4<T>::type;
     constexpr int W4 = M / 4;
     __shared__ T sm[8][32 * M + M];
@@ -216,7 +218,7 @@ __global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int6
         __syncwarp();
         if (lane < rows) {  // rows of <= 32 elements: plain chains (no compensation needed)
             if constexpr (SCAN) {
-                T a = d;
+                T a = seed ? seed[r0 + lane] : d;
 #pragma unroll
                 for (int k = 0; k < M; ++k) {
                     const int q = lane * M + k;
@@ -273,6 +275,7 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        const T* seed = (const T*)a.seed;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) &&
                          (a.m <= kTopKT || a.m % 4 == 0);
         if (vec && (a.m == 1 || a.m == 2 || a.m == 4)) {
@@ -280,27 +283,27 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
             const int grid = stop_grid(ceil_div(nv, 256 * 4)) * 2;
             const T d = bits_to<T>(a.ne_bits);
             if (a.m == 1)
-                segscan_top_small_kernel<T, OP, F, 1><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+                segscan_top_small_kernel<T, OP, F, 1><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             else if (a.m == 2)
-                segscan_top_small_kernel<T, OP, F, 2><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+                segscan_top_small_kernel<T, OP, F, 2><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             else
-                segscan_top_small_kernel<T, OP, F, 4><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+                segscan_top_small_kernel<T, OP, F, 4><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             return cudaGetLastError();
         }
         if (vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
             const int grid = stop_grid(ceil_div(a.n, 256));
             const T d = bits_to<T>(a.ne_bits);
             if (a.m == 8)
-                top_warp_kernel<T, OP, F, 8, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+                top_warp_kernel<T, OP, F, 8, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             else if (a.m == 16)
-                top_warp_kernel<T, OP, F, 16, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+                top_warp_kernel<T, OP, F, 16, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             else
-                top_warp_kernel<T, OP, F, 32, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+                top_warp_kernel<T, OP, F, 32, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             return cudaGetLastError();
         }
         const int64_t nblk = ceil_div(a.n, (int64_t)kTopThreads * stop_rpt(a.m));
         segscan_top_kernel<T, OP, F><<<stop_grid(nblk), kTopThreads, 0, a.stream>>>(
-            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec);
+            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec, seed);
         return cudaGetLastError();
     });
 }
@@ -317,7 +320,7 @@ int midscan_group_size(int64_t m) {
 
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, int64_t n, int64_t m, T d, int G,
-                                                           bool vec) {
+                                                           bool vec, const T* __restrict__ seed) {
     __shared__ T wtot[2][32];
     using V = typename Vec4<T>::type;
     const int g = threadIdx.x % G;
@@ -326,7 +329,7 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
     const bool live = i < n;
     const T* row = in + (live ? i * m : 0);
     T* orow = out + (live ? i * m : 0);
-    T carry = d;
+    T carry = (seed && live) ? seed[i] : d;
     int par = 0;
     for (int64_t base = 0; base < m; base += (int64_t)G * kMidItems, par ^= 1) {
         const int64_t k0 = base + (int64_t)g * kMidItems;
@@ -403,7 +406,8 @@ cudaError_t launch_segscan_mid(const SegArgs& a) {
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) && (a.m % 4 == 0);
         const int64_t grid = ceil_div(a.n, B / G);
         segscan_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, a.m,
-                                                                         bits_to<T>(a.ne_bits), G, vec);
+                                                                         bits_to<T>(a.ne_bits), G, vec,
+                                                                         (const T*)a.seed);
         return cudaGetLastError();
     });
 }

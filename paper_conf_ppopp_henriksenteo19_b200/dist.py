@@ -17,6 +17,14 @@ the device-level guard is ``n >= t_dev`` (Par over devices = n):
 
 Bitwise operators have no NCCL reduction: partials are all-gathered and
 combined with the library's own segred over the [n][G] partial matrix.
+
+segscan uses the same guard.  Outer split: independent rows, no collective.
+Inner split: (1) local segred of the rank's column block without d -> n
+totals; (2) one ``all_gather`` of the [G][n] totals -- the exchange step;
+(3) carry-in of rank r = d (+) tot_0 (+) ... (+) tot_{r-1}, an ordered
+segred over the [n][r] matrix of lower ranks' totals; (4) the local scan
+seeded row by row with that carry (ifl_segscan_seeded).  Three global
+accesses per element (read, read + write), as SURVEY 8(e) plans.
 redomap2 splits the rows of A (B replicated) and tridag the systems: both
 are outer splits without a collective.
 
@@ -101,6 +109,42 @@ def segred_dist(x_block: torch.Tensor, n: int, m: int, op: str = "sum", f: str =
         total = part.clone()
         td.all_reduce(total, op=_REDUCE[op], group=group)
     return _apply_ne(total, op, ne, local)
+
+
+def _default_local_scan(x: torch.Tensor, op: str, f: str, ne, seed):
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.segscan(x, op, f, ne=ne, seed=seed)
+
+
+def segscan_dist(x_block: torch.Tensor, n: int, m: int, op: str = "sum", f: str = "id", ne=None,
+                 plan: Plan | None = None, group=None, local_segred=None, local_segscan=None) -> torch.Tensor:
+    """Distributed segscan.  ``x_block`` as for segred_dist; returns this
+    rank's block of the [n][m] result (its rows for the outer split, its
+    columns of every row for the inner split)."""
+    red = local_segred or _default_local
+    scan = local_segscan or _default_local_scan
+    world = td.get_world_size(group)
+    rank = td.get_rank(group)
+    plan = plan or plan_segred(n, m, world, rank)
+    if plan.mode == "outer" or world == 1:
+        return scan(x_block, op, f, ne, None)
+    # (1) block totals without d (canonical neutral element)
+    if x_block.shape[1] > 0:
+        tot = red(x_block, op, f, None).contiguous()
+    else:
+        tot = red(x_block.new_empty((n, 0)), op, f, None).contiguous()
+    # (2) the exchange step: every rank's totals
+    allt = torch.empty(world * n, dtype=tot.dtype, device=tot.device)
+    td.all_gather_into_tensor(allt, tot, group=group)
+    if x_block.shape[1] == 0:
+        return x_block.new_empty((n, 0))
+    # (3) carry-in = d (+) totals of ranks 0..r-1, in rank order
+    if rank == 0:
+        return scan(x_block, op, f, ne, None)
+    lower = allt.view(world, n)[:rank].t().contiguous()  # [n][rank]
+    seed = red(lower, op, "id", ne).contiguous()
+    # (4) local scan continued from the carry
+    return scan(x_block, op, f, None, seed)
 
 
 def rows_of(n: int, world: int, rank: int):

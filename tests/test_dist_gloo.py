@@ -87,6 +87,69 @@ def test_segred_dist_world2():
         assert any(r[0] == "outer" for r in rows) and any(r[0] == "inner" for r in rows)
 
 
+def _oracle_local_scan(x, op, f, ne, seed):
+    """Stands in for the GPU segscan (seeded when seed is given)."""
+    import oracle
+    xn = x.numpy()
+    if seed is None:
+        r = oracle.segscan(xn, op, f, ne)
+    else:
+        r = oracle.segscan_seeded(xn, seed.numpy(), op, f)
+    if r.dtype == np.float64:
+        r = r.astype(np.float32)
+    return torch.from_numpy(np.ascontiguousarray(r))
+
+
+def _scan_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    td.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    import oracle
+    results = []
+    try:
+        cases = [("I32_FULL", op) for op in ("sum", "min", "max", "and", "or", "xor")] + \
+                [("I32_SMALL", "prod"), ("F32_EXACT", "sum")]
+        for (n, m) in [(1, 1000), (3, 77), (5, 2), (2, 1), (64, 31)]:
+            for dist_name, op in cases:
+                X = gen.matrix(dist_name, 6, n, m)
+                d = 3 if X.dtype == torch.int32 else 1.5
+                want = oracle.segscan(X.numpy(), op, "id", d)
+                for t_dev in (1, world + 1):  # force outer and inner
+                    plan = dist.plan_segred(n, m, world, rank, t_dev)
+                    blk = X[plan.lo:plan.hi] if plan.mode == "outer" else X[:, plan.lo:plan.hi].contiguous()
+                    out = dist.segscan_dist(blk, n, m, op, "id", d, plan=plan, local_segred=_oracle_local,
+                                            local_segscan=_oracle_local_scan).numpy()
+                    ref = want[plan.lo:plan.hi] if plan.mode == "outer" else want[:, plan.lo:plan.hi]
+                    if X.dtype == torch.int32:
+                        ok = np.array_equal(out, ref)
+                    else:
+                        ok = np.allclose(out, ref, rtol=0, atol=1e-9)
+                    results.append((plan.mode, n, m, dist_name, op, bool(ok)))
+        q.put((rank, results))
+    except Exception as e:  # report instead of hanging the parent
+        import traceback
+        q.put((rank, [("error", traceback.format_exc(), False)]))
+    finally:
+        td.destroy_process_group()
+
+
+def test_segscan_dist_world2():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_scan_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, rows in res:
+        bad = [r for r in rows if not r[-1]]
+        assert not bad, f"rank {rank}: {bad[:5]}"
+        assert any(r[0] == "outer" for r in rows) and any(r[0] == "inner" for r in rows)
+
+
 def test_plans_cover_exactly():
     from paper_conf_ppopp_henriksenteo19_b200 import dist
     for world in (1, 2, 3, 8):

@@ -58,3 +58,44 @@ def test_virtual_shards(ifl, orc, G):
         stacked = torch.stack(parts, 1).contiguous()
         total = ifl.segred(stacked, op, ne=7)
         np.testing.assert_array_equal(total.cpu().numpy(), orc.segred(Xo.cpu().numpy(), op, "id", 7))
+
+
+@pytest.mark.parametrize("G", [2, 8])
+def test_virtual_shards_segscan(ifl, orc, G):
+    """segscan inner split on one GPU, step by step as dist.segscan_dist runs
+    it per rank: block totals without d -> carry-in d (+) lower totals ->
+    seeded local scan; the concatenated blocks equal the full scan."""
+    n, m = 3, (1 << 20) + 5
+    for op in ("sum", "max", "xor"):
+        X = gen.matrix("I32_FULL", 9, n, m).cuda()
+        cuts = [(m * r) // G for r in range(G + 1)]
+        blocks = [X[:, cuts[r]:cuts[r + 1]].contiguous() for r in range(G)]
+        tots = torch.stack([ifl.segred(b, op) for b in blocks], 0)  # [G][n], what all_gather delivers
+        outs = []
+        for r in range(G):
+            if r == 0:
+                outs.append(ifl.segscan(blocks[0], op, ne=11))
+            else:
+                seed = ifl.segred(tots[:r].t().contiguous(), op, ne=11)
+                outs.append(ifl.segscan(blocks[r], op, seed=seed))
+        got = torch.cat(outs, 1).cpu().numpy()
+        np.testing.assert_array_equal(got, orc.segscan(X.cpu().numpy(), op, "id", 11))
+
+
+def test_nccl_world1_segscan(ifl, orc):
+    import torch.distributed as td
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    td.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        X = gen.matrix("I32_FULL", 10, 2, 70001)
+        for t_dev in (1, 2):
+            plan = dist.plan_segred(2, 70001, 1, 0, t_dev)
+            out = dist.segscan_dist(X.cuda(), 2, 70001, "sum", "id", 5, plan=plan)
+            np.testing.assert_array_equal(out.cpu().numpy(), orc.segscan(X.numpy(), "sum", "id", 5))
+    finally:
+        td.destroy_process_group()

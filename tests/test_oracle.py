@@ -326,3 +326,39 @@ def test_tridag_against_scipy_and_residual(orc):
         Ax[1:] += a[r, 1:] * x[s, :-1]
         Ax[:-1] += c[r, :-1] * x[s, 1:]
         assert np.abs(Ax - y[s]).max() < 1e-12
+
+
+# ---- segscan_seeded (ifl_segscan_seeded): per-row d
+def test_seeded_closed_form(orc):
+    # ones with seed s_i: out[i, j] = s_i + j + 1
+    n, m = 4, 9
+    seed = np.array([0, 5, -3, 100], np.int32)
+    got = orc.segscan_seeded(np.ones((n, m), np.int32), seed, "sum")
+    np.testing.assert_array_equal(got, seed[:, None] + np.arange(1, m + 1)[None, :])
+    # max with seed above every element: the row is constant seed
+    x = np.arange(n * m, dtype=np.int32).reshape(n, m)
+    np.testing.assert_array_equal(orc.segscan_seeded(x, np.full(n, 10**6, np.int32), "max"),
+                                  np.full((n, m), 10**6, np.int32))
+
+
+def test_seeded_continues_a_split_row(orc):
+    # P:79 associativity: scanning columns [k, m) seeded with the inclusive
+    # scan of [0, k) gives the tail of the full-row scan (the carry step of
+    # the multi-GPU inner split)
+    rng = np.random.default_rng(5)
+    for op in ("sum", "min", "max", "xor"):
+        x = rng.integers(-1000, 1000, size=(3, 40), dtype=np.int32)
+        full = orc.segscan(x, op)
+        for k in (1, 17, 39):
+            tail = orc.segscan_seeded(np.ascontiguousarray(x[:, k:]), full[:, k - 1].copy(), op)
+            np.testing.assert_array_equal(tail, full[:, k:])
+    xf = rng.standard_normal((2, 50)).astype(np.float32)
+    full = orc.segscan(xf, "sum")
+    tail, ab = orc.segscan_seeded(np.ascontiguousarray(xf[:, 20:]), full[:, 19].astype(np.float32), "sum",
+                                  with_absum=True)
+    assert (np.abs(tail - full[:, 20:]) <= 1e-6 * (ab + 1)).all()
+
+
+def test_seeded_equal_seeds_is_plain_scan(orc):
+    x = np.arange(24, dtype=np.int32).reshape(3, 8)
+    np.testing.assert_array_equal(orc.segscan_seeded(x, np.full(3, 7, np.int32), "sum"), orc.segscan(x, "sum", "id", 7))
