@@ -153,15 +153,63 @@ def rows_of(n: int, world: int, rank: int):
     return lo, min(n, lo + per)
 
 
-def redomap2_dist(A_rows: torch.Tensor, B: torch.Tensor, **kw) -> torch.Tensor:
-    """Row split of A (B replicated): independent output row blocks."""
+def plan_redomap2(n: int, m: int, p: int, world: int, rank: int, t_dev: int | None = None) -> Plan:
+    """Device-level guard for redomap2 (Par_dev = n, rows of C): split the
+    rows of A when n >= t_dev (B replicated, no collective), else split k
+    (columns of A / rows of yss) and sum the [n][p] partials with one
+    all_reduce ("split-K, then ncclReduce")."""
+    t_dev = world if t_dev is None else t_dev
+    if n >= t_dev:
+        lo, hi = rows_of(n, world, rank)
+        return Plan("outer", lo, hi)
+    return Plan("inner", (m * rank) // world, (m * (rank + 1)) // world)
+
+
+def _default_local_mm(A, B, b_kmajor):
     import paper_conf_ppopp_henriksenteo19_b200 as ifl
-    return ifl.redomap2(A_rows, B, **kw)
+    return ifl.redomap2(A, B, b_kmajor=b_kmajor)
 
 
-def tridag_dist(a, b, c, y_rows: torch.Tensor, **kw) -> torch.Tensor:
-    """System split: independent systems.  The caller passes the systems
-    s in [lo, hi) with lo a multiple of coef_rows (rows_of keeps that when
-    the per-rank count is a multiple of it) so that s % R is preserved."""
+def redomap2_dist(A_block: torch.Tensor, B_block: torch.Tensor, n: int, m: int, p: int, plan: Plan | None = None,
+                  group=None, b_kmajor: bool = True, gather: bool = False, local_redomap2=None) -> torch.Tensor:
+    """Distributed C = xss x yss.  Outer plan: A_block = rows
+    [lo, hi) of A, B_block = all of B; returns those rows of C (all rows if
+    ``gather``).  Inner plan: A_block = A[:, lo:hi], B_block = the matching
+    k-block of B (Bt[:, lo:hi] when b_kmajor, else B[lo:hi]); returns the
+    full C on every rank after one all_reduce of the fp32 partials."""
+    local = local_redomap2 or _default_local_mm
+    world = td.get_world_size(group)
+    rank = td.get_rank(group)
+    plan = plan or plan_redomap2(n, m, p, world, rank)
+    if plan.mode == "outer":
+        C = local(A_block, B_block, b_kmajor)
+        if not gather:
+            return C
+        per = -(-n // world)
+        buf = torch.empty(per * world * p, dtype=C.dtype, device=C.device)
+        padded = torch.zeros(per * p, dtype=C.dtype, device=C.device)
+        padded[: C.numel()] = C.reshape(-1)
+        td.all_gather_into_tensor(buf, padded, group=group)
+        return buf.view(per * world, p)[:n]
+    if A_block.shape[1] == 0:
+        C = torch.zeros(n, p, dtype=torch.float32, device=A_block.device)
+    else:
+        C = local(A_block, B_block, b_kmajor).contiguous()
+    td.all_reduce(C, op=td.ReduceOp.SUM, group=group)
+    return C
+
+
+def tridag_dist(a: torch.Tensor, b: torch.Tensor, c: torch.Tensor, y_rows: torch.Tensor, lo: int,
+                local_tridag=None, **kw) -> torch.Tensor:
+    """System split (independent units, no collective).  y_rows holds the
+    systems s in [lo, lo + len); coefficients are the full [R][L] arrays and
+    system s uses row s % R (R9), so when lo % R != 0 the rows are rotated
+    to keep that mapping for the local call (R * L elements, tiny)."""
+    R = a.shape[0]
+    sh = lo % R
+    if sh:
+        a, b, c = (torch.roll(t, -sh, dims=0).contiguous() for t in (a, b, c))
+    if local_tridag is not None:
+        return local_tridag(a, b, c, y_rows)
     import paper_conf_ppopp_henriksenteo19_b200 as ifl
     return ifl.tridag(a, b, c, y_rows, **kw)

@@ -150,6 +150,69 @@ def test_segscan_dist_world2():
         assert any(r[0] == "outer" for r in rows) and any(r[0] == "inner" for r in rows)
 
 
+def _mm_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    td.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    import oracle
+    results = []
+
+    def local_mm(A, B, b_kmajor):  # the oracle stands in for the GPU (fp64 -> fp32 partials)
+        return torch.from_numpy(oracle.redomap2(A.numpy(), B.numpy(), b_kmajor=b_kmajor).astype(np.float32))
+
+    def local_tri(a, b, c, y):
+        return torch.from_numpy(oracle.tridag(a.numpy(), b.numpy(), c.numpy(), y.numpy(), a.shape[0])
+                                .astype(np.float32))
+    try:
+        for (n, m, p) in [(1, 64, 1), (3, 50, 5), (8, 16, 3), (2, 1, 7)]:
+            # small integers in f32: every partial and sum is exact
+            A = (gen.matrix("I32_SMALL", 11, n, m) % 5).float()
+            Bt = (gen.matrix("I32_SMALL", 12, p, m) % 5).float()
+            want = oracle.redomap2(A.numpy(), Bt.numpy(), b_kmajor=True)
+            for t_dev in (1, world + 1):
+                for kmaj in (True, False):
+                    plan = dist.plan_redomap2(n, m, p, world, rank, t_dev)
+                    Bfull = Bt if kmaj else Bt.t().contiguous()
+                    if plan.mode == "outer":
+                        Ab, Bb = A[plan.lo:plan.hi].contiguous(), Bfull
+                    else:
+                        Ab = A[:, plan.lo:plan.hi].contiguous()
+                        Bb = Bt[:, plan.lo:plan.hi].contiguous() if kmaj else Bfull[plan.lo:plan.hi].contiguous()
+                    C = dist.redomap2_dist(Ab, Bb, n, m, p, plan=plan, b_kmajor=kmaj, gather=True,
+                                           local_redomap2=local_mm).numpy()
+                    results.append(("mm", plan.mode, n, m, p, kmaj, bool(np.array_equal(C, want))))
+        # tridag: system split with a block start that is not a multiple of R
+        S, L, R = 10, 16, 4
+        a, b, c, y = gen.tridag_system(3, S, L, R)
+        want = oracle.tridag(a.numpy(), b.numpy(), c.numpy(), y.numpy(), R)
+        lo, hi = [(0, 5), (5, 10)][rank]
+        x = dist.tridag_dist(a, b, c, y[lo:hi].contiguous(), lo, local_tridag=local_tri).numpy()
+        results.append(("tridag", lo, hi, bool(np.allclose(x, want[lo:hi], rtol=1e-5, atol=1e-5))))
+        q.put((rank, results))
+    except Exception:
+        import traceback
+        q.put((rank, [("error", traceback.format_exc(), False)]))
+    finally:
+        td.destroy_process_group()
+
+
+def test_redomap2_tridag_dist_world2():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_mm_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, rows in res:
+        bad = [r for r in rows if not r[-1]]
+        assert not bad, f"rank {rank}: {bad[:5]}"
+        assert any(r[:2] == ("mm", "outer") for r in rows) and any(r[:2] == ("mm", "inner") for r in rows)
+
+
 def test_plans_cover_exactly():
     from paper_conf_ppopp_henriksenteo19_b200 import dist
     for world in (1, 2, 3, 8):

@@ -99,3 +99,33 @@ def test_nccl_world1_segscan(ifl, orc):
             np.testing.assert_array_equal(out.cpu().numpy(), orc.segscan(X.numpy(), "sum", "id", 5))
     finally:
         td.destroy_process_group()
+
+
+def test_redomap2_tridag_dist_gpu(ifl, orc):
+    """redomap2_dist (outer and split-K plans, NCCL world 1) and tridag_dist
+    with a block start that is not a multiple of R, on the GPU kernels."""
+    import torch.distributed as td
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    td.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        n, m, p = 3, 4096, 40
+        A = (gen.matrix("I32_SMALL", 11, n, m) % 5).float()
+        Bt = (gen.matrix("I32_SMALL", 12, p, m) % 5).float()
+        want = orc.redomap2(A.numpy(), Bt.numpy(), b_kmajor=True)
+        for t_dev in (1, 4):
+            plan = dist.plan_redomap2(n, m, p, 1, 0, t_dev)
+            C = dist.redomap2_dist(A.cuda(), Bt.cuda(), n, m, p, plan=plan, gather=True)
+            np.testing.assert_array_equal(C.cpu().numpy(), want)
+    finally:
+        td.destroy_process_group()
+    S, L, R = 64, 256, 8
+    a, b, c, y = gen.tridag_system(4, S, L, R)
+    want = orc.tridag(a.numpy(), b.numpy(), c.numpy(), y.numpy(), R)
+    lo = 11
+    x = dist.tridag_dist(a.cuda(), b.cuda(), c.cuda(), y[lo:].contiguous().cuda(), lo).cpu().numpy()
+    assert (np.abs(x - want[lo:]) <= 1e-5 * np.maximum(1.0, np.abs(want[lo:]).max(1, keepdims=True))).all()
