@@ -22,7 +22,7 @@ from dataclasses import dataclass
 import torch
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libifl.so")
+LIB_PATH = os.environ.get("IFL_LIB_PATH") or os.path.join(_PKG, "libifl.so")  # override: experiment builds
 
 IFL_OK, IFL_EINVAL, IFL_EUNSUPPORTED, IFL_EWORKSPACE, IFL_ENOTFIT, IFL_ECUDA = 0, -1, -2, -3, -4, -5
 DTYPES = {"i32": 0, "f32": 1, "bf16": 2}

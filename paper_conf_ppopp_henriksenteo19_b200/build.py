@@ -20,8 +20,11 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-OBJ = os.path.join(PKG, "build_obj")
-LIB = os.path.join(PKG, "libifl.so")
+# IFL_BUILD_TAG builds an experiment variant side by side (build_obj_<tag>,
+# libifl_<tag>.so; load it with IFL_LIB_PATH) -- tools only, never the product
+_TAG = os.environ.get("IFL_BUILD_TAG", "")
+OBJ = os.path.join(PKG, "build_obj" + (f"_{_TAG}" if _TAG else ""))
+LIB = os.path.join(PKG, "libifl" + (f"_{_TAG}" if _TAG else "") + ".so")
 NVCC = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + CSRC, "-I" + os.path.join(ROOT, "include")]

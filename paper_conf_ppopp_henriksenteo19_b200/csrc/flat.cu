@@ -212,10 +212,16 @@ __device__ __forceinline__ void acquire_tile(T* slot, const T* in, const SlotMet
 // metadata, issues the TMA load); warps 0-7 consume.  A slot is released by
 // each consumer warp as soon as its items are in registers (count-8 mbarrier),
 // so the next load into it is issued while the tile is still being reduced.
-constexpr int kRedSlots = 3;
+#ifndef IFL_RED_SLOTS  // experiment overrides (tools/flat_probe.py with IFL_BUILD_TAG builds)
+#define IFL_RED_SLOTS 3
+#endif
+#ifndef IFL_RED_MINB
+#define IFL_RED_MINB 3
+#endif
+constexpr int kRedSlots = IFL_RED_SLOTS;
 
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(FB + 32, 3) flat_red_kernel(const T* in, T* out, int64_t N, int64_t m, T d, T* head,
+__global__ void __launch_bounds__(FB + 32, IFL_RED_MINB) flat_red_kernel(const T* in, T* out, int64_t N, int64_t m, T d, T* head,
                                                               T* tail, int num_tiles, bool tma) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
@@ -425,12 +431,21 @@ __device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, 
 // 64-bit tile arithmetic stays off their critical path.  Status words carry
 // an epoch tag; the last CTA to finish bumps the epoch (one 64-bit
 // {epoch | done} word), so no per-call memset is needed.
-constexpr int kChunkTiles = 8;
+#ifndef IFL_CHUNK_TILES
+#define IFL_CHUNK_TILES 8
+#endif
+constexpr int kChunkTiles = IFL_CHUNK_TILES;
 constexpr int kScanThreads = FB + 32;
-constexpr int kScanSlots = 3;  // 60 KB ring: three CTAs (27 warps) per SM
+#ifndef IFL_SCAN_SLOTS
+#define IFL_SCAN_SLOTS 3  // 60 KB ring: three CTAs (27 warps) per SM
+#endif
+#ifndef IFL_SCAN_MINB
+#define IFL_SCAN_MINB 3
+#endif
+constexpr int kScanSlots = IFL_SCAN_SLOTS;
 
 template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kScanThreads, 3) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
+__global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
                                                                     uint8_t* ws, int num_tiles, int num_chunks,
                                                                     bool tma_in, bool tma_out, const T* __restrict__ seed) {
     extern __shared__ __align__(128) uint8_t smem_raw[];

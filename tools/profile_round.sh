@@ -11,6 +11,7 @@ mkdir -p gpurun_out/ncu
 timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv \
   --log-file gpurun_out/ncu/launches.csv \
   python bench.py --steps 2 --warmup 3 --no-tune --thresholds gpurun_out/thresholds.txt --no-e2e --no-cpu --no-forced \
+  --detail gpurun_out/ncu/bench_detail_under_ncu.json \
   > gpurun_out/ncu/bench_under_ncu.json 2>&1
 echo "launch list rc=$?"
 # 2. full captures (one launch each)
