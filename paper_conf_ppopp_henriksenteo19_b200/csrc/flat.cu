@@ -20,13 +20,14 @@
 //           (the open segment at its end, or the whole tile) in the workspace;
 //   pass 2  every segment that crosses tiles ta < tb is
 //           out = tail[ta] (+) tail[ta+1..tb-1] (+) head[tb]   (a tree reduce).
-// segscan (single pass, decoupled look-back):
-//   tiles are claimed dynamically; each publishes a 64-bit status word
-//   (aggregate / inclusive prefix, segment flag, epoch tag) and looks back for
-//   its carry only if it does not begin with a segment start; results return to
-//   the slot and the TMA engine stores the tile (cp.async.bulk shared->global).
-//   The workspace is re-armed by the last CTA (counter reset, epoch bump), so no
-//   per-call memset is needed.
+// segscan (L2-blocked two-phase, see flat_scan_kernel): chunks of kChunkTiles
+//   tiles; a chunk's aggregate is computed in a first pass whose data stays in
+//   L2, a CTA-wide look-back over chunk status words (aggregate / inclusive
+//   prefix, segment flag, epoch tag; relaxed loads -- the word is
+//   self-contained) gives its carry, and the scan pass re-reads it from L2 and
+//   stores each tile from its ring slot with the TMA engine (cp.async.bulk
+//   shared->global).  The workspace is re-armed by the last CTA (counter
+//   reset, epoch bump), so no per-call memset is needed.
 // Workspace: [header 256 B][status: 8 B/tile][head: 4 B/tile][tail: 4 B/tile].
 #include <string.h>
 
@@ -577,7 +578,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
                 consumer_sync();  // s_wval reuse
             }
             if (t == 0)
-                st_release_u64(&status[c], pack_status(tag, (run_f || !carry_needed) ? ST_P : ST_A, run_f,
+                st_relaxed_u64(&status[c], pack_status(tag, (run_f || !carry_needed) ? ST_P : ST_A, run_f,
                                                        to_bits(run_v)));
         }
         // ---- look-back over preceding chunk aggregates (chunks cs .. c-1)
@@ -591,7 +592,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
                 uint64_t word = 0;
                 if (idx >= cs) {
                     do {
-                        word = ld_acquire_u64(&status[idx]);
+                        word = ld_relaxed_u64(&status[idx]);  // self-contained word: no acquire needed
                     } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
                 }
                 const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
@@ -618,7 +619,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
                 pred -= FB;
             }
             if (agg_needed && !run_f && t == 0)
-                st_release_u64(&status[c], pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, run_v))));
+                st_relaxed_u64(&status[c], pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, run_v))));
         }
         // ---- phase 3
         for (int j = 0; j < L; ++j, ++vi) {
