@@ -264,4 +264,80 @@ __device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
 
 __host__ __device__ constexpr int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
+// ------------------------------------------------ V_TOP warp-tile kernel
+// V_TOP (thread per segment) for m = M in {16, 32, 64}, 16-byte-aligned in/out:
+// each warp owns 32 consecutive rows (one contiguous 32*M-element block).  The
+// block is loaded with coalesced 128-bit loads (all in flight at once), staged
+// in shared memory with a row stride of M+4 words (16-byte aligned; the
+// 128-bit stores and the lanes' row walks are bank-conflict-free), and each
+// lane then walks its own row sequentially -- the inner level of P:233's e_top.
+// For SCAN the results go back through the same tile and leave with coalesced
+// 128-bit stores.  Non-persistent: one warp-tile per warp, top_tile_warps(M)
+// warps per CTA (the tile is 32 * (M + 4) words per warp).
+__host__ __device__ constexpr int top_tile_warps(int M) { return M <= 32 ? 8 : 4; }
+template <typename T, int OP, int F, int M, bool SCAN>
+__global__ void __launch_bounds__(32 * top_tile_warps(M)) top_tile_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                                          int64_t n, T d, const T* __restrict__ seed) {
+    using V = typename Vec4<T>::type;
+    constexpr int S = M + 4, W4 = M / 4, WPC = top_tile_warps(M);  // row stride (words), words per row
+    __shared__ __align__(16) T sm[WPC][32 * S];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    T* s = sm[warp];
+    const int64_t r0 = ((int64_t)blockIdx.x * WPC + warp) * 32;
+    if (r0 >= n) return;
+    const int rows = (int)min((int64_t)32, n - r0);
+    const T* src = in + r0 * M;
+    V q[W4];
+#pragma unroll
+    for (int u = 0; u < W4; ++u) {
+        const int q4 = lane + 32 * u;  // 16-byte word of the block
+        if (q4 < rows * W4) q[u] = ldg_stream4(src + 4 * q4);
+    }
+#pragma unroll
+    for (int u = 0; u < W4; ++u) {
+        const int q4 = lane + 32 * u;
+        if (q4 < rows * W4) *reinterpret_cast<V*>(&s[(q4 / W4) * S + 4 * (q4 % W4)]) = q[u];
+    }
+    __syncwarp();
+    if (lane < rows) {
+        T* row = s + lane * S;
+        if constexpr (SCAN) {
+            T a = seed ? seed[r0 + lane] : d;
+#pragma unroll
+            for (int j = 0; j < W4; ++j) {
+                V v = *reinterpret_cast<const V*>(row + 4 * j);
+                a = combine<OP>(a, apply_map<F>(v.x));
+                v.x = a;
+                a = combine<OP>(a, apply_map<F>(v.y));
+                v.y = a;
+                a = combine<OP>(a, apply_map<F>(v.z));
+                v.z = a;
+                a = combine<OP>(a, apply_map<F>(v.w));
+                v.w = a;
+                *reinterpret_cast<V*>(row + 4 * j) = v;
+            }
+        } else {
+            T a[4] = {d, identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+#pragma unroll
+            for (int j = 0; j < W4; ++j) {
+                const V v = *reinterpret_cast<const V*>(row + 4 * j);
+                a[0] = combine<OP>(a[0], apply_map<F>(v.x));
+                a[1] = combine<OP>(a[1], apply_map<F>(v.y));
+                a[2] = combine<OP>(a[2], apply_map<F>(v.z));
+                a[3] = combine<OP>(a[3], apply_map<F>(v.w));
+            }
+            out[r0 + lane] = combine<OP>(combine<OP>(a[0], a[1]), combine<OP>(a[2], a[3]));
+        }
+    }
+    if constexpr (SCAN) {
+        __syncwarp();
+        T* dst = out + r0 * M;
+#pragma unroll
+        for (int u = 0; u < W4; ++u) {
+            const int q4 = lane + 32 * u;
+            if (q4 < rows * W4) *reinterpret_cast<V*>(dst + 4 * q4) = *reinterpret_cast<const V*>(&s[(q4 / W4) * S + 4 * (q4 % W4)]);
+        }
+    }
+}
+
 }  // namespace ifl

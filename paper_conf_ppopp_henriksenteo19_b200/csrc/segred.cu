@@ -17,6 +17,16 @@
 #include "dispatch.cuh"
 #include "ifl_internal.h"
 
+#ifndef IFL_MID_GMAX
+#define IFL_MID_GMAX 512  // largest V_MIDDLE group (threads per segment; 1024 measured slower)
+#endif
+#ifndef IFL_ROW_L1
+#define IFL_ROW_L1 0  // row kernels: L1-allocating loads (a row's 16-byte words share sectors)
+#endif
+#ifndef IFL_TOP_ROW
+#define IFL_TOP_ROW 1  // m in {8,16,32}: thread-per-row register kernel (0: smem-staged warp tiles)
+#endif
+
 namespace ifl {
 
 // ------------------------------------------------------------------ V_TOP
@@ -277,6 +287,30 @@ __global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int6
     }
 }
 
+// V_TOP for m in {8, 16, 32}, 16-byte-aligned: one thread per row, its m/4
+// 128-bit words loaded straight into registers (all in flight at once); a
+// warp's 32 rows are one contiguous block, so every word of it is used.
+template <typename T, int OP, int F, int M>
+__global__ void __launch_bounds__(256) segred_top_row_kernel(const T* __restrict__ in, T* __restrict__ out, int64_t n,
+                                                             T d) {
+    using V = typename Vec4<T>::type;
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= n) return;
+    const T* p = in + r * M;
+    V q[M / 4];
+#pragma unroll
+    for (int u = 0; u < M / 4; ++u) q[u] = IFL_ROW_L1 ? __ldg(reinterpret_cast<const V*>(p + 4 * u)) : ldg_stream4(p + 4 * u);
+    T a[4] = {d, identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+#pragma unroll
+    for (int u = 0; u < M / 4; ++u) {
+        T e[4];
+        unpack4<T>(q[u], e);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) a[k] = combine<OP>(a[k], apply_map<F>(e[k]));
+    }
+    out[r] = combine<OP>(combine<OP>(a[0], a[1]), combine<OP>(a[2], a[3]));
+}
+
 static int top_grid(int64_t nblk) {
     static int sms = 0;
     if (!sms) {
@@ -305,6 +339,24 @@ cudaError_t launch_segred_top(const SegArgs& a) {
                 segred_top_small_kernel<T, OP, F, 4><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
             return cudaGetLastError();
         }
+        if (vec && a.m == 64) {
+            top_tile_kernel<T, OP, F, 64, false><<<(unsigned)ceil_div(a.n, 32 * top_tile_warps(64)),
+                                                   32 * top_tile_warps(64), 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, bits_to<T>(a.ne_bits), nullptr);
+            return cudaGetLastError();
+        }
+        if (IFL_TOP_ROW && vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
+            const unsigned grid = (unsigned)ceil_div(a.n, 256);
+            const T d = bits_to<T>(a.ne_bits);
+            if (a.m == 8)
+                segred_top_row_kernel<T, OP, F, 8><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else if (a.m == 16)
+                segred_top_row_kernel<T, OP, F, 16><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d);
+            else
+                top_tile_kernel<T, OP, F, 32, false><<<(unsigned)ceil_div(a.n, 256), 256, 0, a.stream>>>(
+                    (const T*)a.in, (T*)a.out, a.n, d, nullptr);
+            return cudaGetLastError();
+        }
         if (vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
             const int grid = top_grid(ceil_div(a.n, 256));
             const T d = bits_to<T>(a.ne_bits);
@@ -331,7 +383,7 @@ cudaError_t launch_segred_top(const SegArgs& a) {
 
 int mid_group_size(int64_t m) {
     int64_t g = 1;  // rows of <= 8 (16) elements: one thread already holds a whole row
-    while (g < 1024 && g * 16 < m) g <<= 1;
+    while (g < IFL_MID_GMAX && g * 16 < m) g <<= 1;
     return (int)g;
 }
 

@@ -16,6 +16,17 @@
 #include "dispatch.cuh"
 #include "ifl_internal.h"
 
+#ifndef IFL_MIDSCAN_GMAX
+#define IFL_MIDSCAN_GMAX 256  // largest V_MIDDLE scan group (threads per segment; longer rows take
+                              // several pipelined rounds -- 512 / 1024 measured slower)
+#endif
+#ifndef IFL_ROW_L1
+#define IFL_ROW_L1 0  // row kernels: L1-allocating loads (a row's 16-byte words share sectors)
+#endif
+#ifndef IFL_TOP_ROW
+#define IFL_TOP_ROW 1  // m in {8,16,32}: thread-per-row register kernel (0: smem-staged warp tiles)
+#endif
+
 namespace ifl {
 
 constexpr int kTopThreads = 256;
@@ -260,6 +271,35 @@ __global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int6
     }
 }
 
+// V_TOP for m in {8, 16, 32}, 16-byte-aligned: one thread per row, its m/4
+// 128-bit words loaded straight into registers, scanned, stored back.
+template <typename T, int OP, int F, int M>
+__global__ void __launch_bounds__(256) segscan_top_row_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                              int64_t n, T d, const T* __restrict__ seed) {
+    using V = typename Vec4<T>::type;
+    const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (r >= n) return;
+    const T* p = in + r * M;
+    V q[M / 4];
+#pragma unroll
+    for (int u = 0; u < M / 4; ++u) q[u] = IFL_ROW_L1 ? __ldg(reinterpret_cast<const V*>(p + 4 * u)) : ldg_stream4(p + 4 * u);
+    T a = seed ? seed[r] : d;
+    T* o = out + r * M;
+#pragma unroll
+    for (int u = 0; u < M / 4; ++u) {
+        T e[4];
+        unpack4<T>(q[u], e);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+            a = combine<OP>(a, apply_map<F>(e[k]));
+            e[k] = a;
+        }
+        V w;
+        w.x = e[0]; w.y = e[1]; w.z = e[2]; w.w = e[3];
+        *reinterpret_cast<V*>(o + 4 * u) = w;
+    }
+}
+
 static int stop_grid(int64_t nblk) {
     static int sms = 0;
     if (!sms) {
@@ -290,6 +330,23 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
                 segscan_top_small_kernel<T, OP, F, 4><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
             return cudaGetLastError();
         }
+        if (vec && a.m == 64) {
+            top_tile_kernel<T, OP, F, 64, true><<<(unsigned)ceil_div(a.n, 32 * top_tile_warps(64)),
+                                                  32 * top_tile_warps(64), 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, bits_to<T>(a.ne_bits), seed);
+            return cudaGetLastError();
+        }
+        if (IFL_TOP_ROW && vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
+            const unsigned grid = (unsigned)ceil_div(a.n, 256);
+            const T d = bits_to<T>(a.ne_bits);
+            if (a.m == 8)
+                segscan_top_row_kernel<T, OP, F, 8><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
+            else if (a.m == 16)
+                top_tile_kernel<T, OP, F, 16, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
+            else
+                top_tile_kernel<T, OP, F, 32, true><<<grid, 256, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, d, seed);
+            return cudaGetLastError();
+        }
         if (vec && (a.m == 8 || a.m == 16 || a.m == 32)) {
             const int grid = stop_grid(ceil_div(a.n, 256));
             const T d = bits_to<T>(a.ne_bits);
@@ -314,7 +371,7 @@ constexpr int kMidItems = 8;  // consecutive elements per thread per round
 
 int midscan_group_size(int64_t m) {
     int64_t g = 1;  // rows of <= 8 (16) elements: one thread already holds a whole row
-    while (g < 1024 && g * kMidItems < m) g <<= 1;
+    while (g < IFL_MIDSCAN_GMAX && g * kMidItems < m) g <<= 1;
     return (int)g;
 }
 
@@ -397,6 +454,105 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
     }
 }
 
+#ifndef IFL_MULTI_MINB
+#define IFL_MULTI_MINB 6
+#endif
+// V_MIDDLE for rows of several rounds: the next round's items are loaded before
+// this round is scanned (register double buffer), so every round's loads overlap
+// the previous round's group scan and barriers.
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
+    segscan_mid_multi_kernel(const T* in, T* out, int64_t n, int64_t m, T d, int G, bool vec,
+                             const T* __restrict__ seed) {
+    __shared__ T wtot[2][32];
+    using V = typename Vec4<T>::type;
+    const int g = threadIdx.x % G;
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int64_t i = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
+    const bool live = i < n;
+    const T* row = in + (live ? i * m : 0);
+    T* orow = out + (live ? i * m : 0);
+    T carry = (seed && live) ? seed[i] : d;
+    int par = 0;
+    const int64_t step = (int64_t)G * kMidItems;
+    // raw items of one round (two 128-bit halves, each vectorised when whole; f applied at use,
+    // so the next round's loads stay in flight while this round is scanned)
+    auto load_round = [&](int64_t base, T (&r)[kMidItems]) {
+        const int64_t k0 = base + (int64_t)g * kMidItems;
+#pragma unroll
+        for (int h = 0; h < kMidItems / 4; ++h) {
+            const int64_t kh = k0 + 4 * h;
+            if (live && vec && kh + 4 <= m) {
+                T e[4];
+                unpack4<T>(ldg_stream4(row + kh), e);
+#pragma unroll
+                for (int u = 0; u < 4; ++u) r[4 * h + u] = e[u];
+            } else {
+#pragma unroll
+                for (int u = 0; u < 4; ++u) r[4 * h + u] = (live && kh + u < m) ? ldg1(row + kh + u) : T();
+            }
+        }
+    };
+    T nxt[kMidItems];
+    load_round(0, nxt);
+    for (int64_t base = 0; base < m; base += step, par ^= 1) {
+        const int64_t k0 = base + (int64_t)g * kMidItems;
+        T v[kMidItems];
+#pragma unroll
+        for (int u = 0; u < kMidItems; ++u) v[u] = nxt[u];
+        if (base + step < m) load_round(base + step, nxt);  // prefetch the next round
+#pragma unroll
+        for (int u = 0; u < kMidItems; ++u)
+            v[u] = (live && k0 + u < m) ? apply_map<F>(v[u]) : identity<OP, T>();
+#pragma unroll
+        for (int u = 1; u < kMidItems; ++u) v[u] = combine<OP>(v[u - 1], v[u]);
+        // inclusive scan of thread totals across the group
+        T s = v[kMidItems - 1];
+        const int width = G < 32 ? G : 32;
+        const int gl = threadIdx.x % width;  // lane within the (sub)warp group
+        for (int off = 1; off < width; off <<= 1) {
+            T o = __shfl_up_sync(0xffffffffu, s, off, width);
+            if (gl >= off) s = combine<OP>(o, s);
+        }
+        T ex = __shfl_up_sync(0xffffffffu, s, 1, width);
+        if (gl == 0) ex = identity<OP, T>();
+        T total;
+        if (G <= 32) {
+            total = __shfl_sync(0xffffffffu, s, width - 1, width);
+        } else {
+            if (lane == 31) wtot[par][w] = s;
+            __syncthreads();
+            const int wpg = G >> 5, w0 = (threadIdx.x / G) * wpg;
+            T before = identity<OP, T>();
+            total = identity<OP, T>();
+            for (int k = 0; k < wpg; ++k) {
+                if (w0 + k < w) before = combine<OP>(before, wtot[par][w0 + k]);
+                total = combine<OP>(total, wtot[par][w0 + k]);
+            }
+            ex = combine<OP>(before, ex);
+        }
+        const T pre = combine<OP>(carry, ex);
+#pragma unroll
+        for (int u = 0; u < kMidItems; ++u) v[u] = combine<OP>(pre, v[u]);
+        if (live) {
+#pragma unroll
+            for (int h = 0; h < kMidItems / 4; ++h) {
+                const int64_t kh = k0 + 4 * h;
+                if (vec && kh + 4 <= m) {
+                    V q;
+                    q.x = v[4 * h]; q.y = v[4 * h + 1]; q.z = v[4 * h + 2]; q.w = v[4 * h + 3];
+                    *reinterpret_cast<V*>(orow + kh) = q;
+                } else {
+#pragma unroll
+                    for (int u = 0; u < 4; ++u)
+                        if (kh + u < m) orow[kh + u] = v[4 * h + u];
+                }
+            }
+        }
+        carry = combine<OP>(carry, total);
+    }
+}
+
 cudaError_t launch_segscan_mid(const SegArgs& a) {
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
@@ -405,9 +561,12 @@ cudaError_t launch_segscan_mid(const SegArgs& a) {
         const int B = G > 256 ? G : 256;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) && (a.m % 4 == 0);
         const int64_t grid = ceil_div(a.n, B / G);
-        segscan_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, a.m,
-                                                                         bits_to<T>(a.ne_bits), G, vec,
-                                                                         (const T*)a.seed);
+        if (a.m > (int64_t)G * kMidItems)  // several rounds per row: pipelined loads
+            segscan_mid_multi_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), G, vec, (const T*)a.seed);
+        else
+            segscan_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), G, vec, (const T*)a.seed);
         return cudaGetLastError();
     });
 }

@@ -203,3 +203,19 @@ def test_config1_sweep_full_size_sampled(ifl, orc, scan):
                 got = fn(xv, "sum", f, version=v)
                 assert_parity(orc, xs, got[rows], scan, "sum", f, None, "f32")
         del xv
+
+
+@pytest.mark.parametrize("version", VERS)
+@pytest.mark.parametrize("scan", [False, True])
+def test_small_m_kernels(ifl, orc, version, scan):
+    """Row lengths with dedicated TOP kernels (m in {1,2,4}: packed words;
+    {8,16}: thread-per-row registers; {16,32,64}: warp tiles via shared memory),
+    ragged row counts (partial warps / CTAs), every op, int32 and f32."""
+    fn = ifl.segscan if scan else ifl.segred
+    for m in (1, 2, 4, 8, 16, 32, 64):
+        for n in (1, 31, 33, 257, 4099):
+            for dt, ops in (("i32", OPS_I), ("f32", OPS_F)):
+                for op in ops:
+                    x, xd = gen_for(op, dt, 5, n, m)
+                    got = fn(xd, op, "sq" if op == "sum" else "id", version=version)
+                    assert_parity(orc, x, got, scan, op, "sq" if op == "sum" else "id", None, dt)
