@@ -207,6 +207,67 @@ def suite_tridag():
     return line
 
 
+# ----------------------------------------------------------------------- lvc
+
+# FP32 lanes x SMs: the ALU roof for V_OUTER, which keeps every system in
+# registers for all numT steps (no HBM traffic inside the loop).  Algorithmic
+# work per element and step = the Thomas recurrences with the loop-invariant
+# elimination hoisted: 1 FMA (forward), 1 MUL (1/beta), 1 FMA (backward).
+LVC_OPS_PER_ELEM_STEP = 3
+
+
+def alu_peak_ops(sm_mhz=1965.0):
+    return 148 * 128 * sm_mhz * 1e6
+
+
+def suite_lvc():
+    """NEXT-1: the whole LocVolCalib loop of Fig 6a
+    dataset, every version of Fig 6c plus the outermost branch (V_OUTER), the
+    per-site G3 tuned as in the tridag suite and the outermost t0 tuned on
+    reduced-numT copies of the datasets (the tuner sees other data)."""
+    hbm, _, src = peaks()
+    ifl.reset_thresholds()
+    train = [s for ds in ("small", "large") for s in sites(ds)[0]]
+    need = ifl.lib().ifl_tune_scratch_bytes(b"tridag", np.asarray(train, np.int64).ctypes.data, len(train))
+    scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
+    ifl.tune("tridag", train, reps=3, cost=1, scratch=scratch)
+    del scratch
+    ltrain = [(S, 8, X, Y) for (S, T, X, Y) in gen.LVC_DATASETS.values()]
+    t0, _, ltbl = ifl.tune("lvc", ltrain, reps=3, cost=1)
+    rows = []
+    for ds, (S, T, X, Y) in gen.LVC_DATASETS.items():
+        (ax, bx, cx), (ay, by, cy), xs, ys = gen.lvc_problem(17, S, X, Y, "cuda")
+        xc, yc = (ax, bx, cx), (ay, by, cy)
+        E = S * X * Y
+        r = {"dataset": ds, "numS": S, "numT": T, "numX": X, "numY": Y}
+        for v in ("outer", "top", "middle", "flat", "auto"):
+            r[v + "_ms"] = gtime(lambda: ifl.lvc(xs, ys, xc, yc, T, version=v), R=2)
+        r["chosen"] = ifl.lvc(xs, ys, xc, yc, T, return_choice=True).version
+        best = min(r[v + "_ms"] for v in ("outer", "top", "middle", "flat"))
+        best_step = min(r[v + "_ms"] for v in ("top", "middle", "flat"))
+        r["best_over_auto"] = round(best / r["auto_ms"], 4)
+        r["speedup_outer_vs_best_per_step"] = round(best_step / r["outer_ms"], 3)
+        # per-step traffic the stepwise versions must move (read y + write x per
+        # element, both sites); V_OUTER moves it once for the whole loop
+        r["per_step_equiv_GBps"] = round(8.0 * 2 * E * T / (r["auto_ms"] * 1e-3) / 1e9, 1)
+        r["alu_Gops"] = round(LVC_OPS_PER_ELEM_STEP * 2 * E * T / (r["outer_ms"] * 1e-3) / 1e9, 1)
+        rows.append(r)
+    peak = alu_peak_ops()
+    large = [r for r in rows if r["dataset"] == "large"][0]
+    ach = LVC_OPS_PER_ELEM_STEP * 2 * (256 * 256 * 256) * 64 / (large["outer_ms"] * 1e-3)
+    line = base_line("LocVolCalib loop (Fig 6a): numT steps of tridag on both sites, large dataset",
+                     round(large["auto_ms"], 4), "ms", {"workload": "SURVEY 8(f) NEXT-1: whole LocVolCalib-shaped "
+                     "program, P:402 datasets, coefficients loop-invariant", "t0": t0}, hib=False)
+    line["per_dataset"] = rows
+    line["lvc_tune_table_ms"] = ltbl.tolist()
+    line["min_shape_best_over_auto"] = min(r["best_over_auto"] for r in rows)
+    line["roofline"] = {"bound": "alu", "kernel": "lvc_outer_kernel (large)", "achieved": round(ach / 1e12, 3),
+                        "peak": round(peak / 1e12, 2), "unit": "Tops/s (FP32 lanes x SMs x 1965 MHz)",
+                        "frac": round(ach / peak, 4), "traffic": None,
+                        "note": f"{LVC_OPS_PER_ELEM_STEP} Thomas ops per element and step; HBM peak {hbm} GB/s ({src})"}
+    return line
+
+
 # ---------------------------------------------------------------------- dist
 
 
@@ -249,4 +310,5 @@ def suite_dist():
     return line
 
 
-SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist}
+SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist,
+          "lvc": suite_lvc}

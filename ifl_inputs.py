@@ -99,3 +99,32 @@ def tridag_system(seed: int, S: int, L: int, coef_rows: int, device="cpu"):
     b = (1.0 + a.abs() + c.abs() + u(2, coef_rows * L).view(coef_rows, L))
     y = generate("F32_SIGNED", seed * 16 + 3, S * L, device).view(S, L)
     return a.contiguous(), b.contiguous(), c.contiguous(), y
+
+
+LVC_DATASETS = {  # (numS, numT, numX, numY)
+    "small": (16, 256, 32, 256),
+    "medium": (128, 64, 256, 32),
+    "large": (256, 64, 256, 256),
+}
+
+
+def lvc_problem(seed: int, numS: int, numX: int, numY: int, device="cpu"):
+    """Inputs of the LocVolCalib loop (Fig 6a), DESIGN.md recipe:
+    per site, coefficient rows a, c ~ -U(0, 0.5), b = 1 + |a| + |c| (the
+    implicit diffusion step I - dt*D: interior rows sum to 1, so repeated
+    solves neither blow up nor underflow over numT steps); x-site
+    coefficients [numX][numY], y-site [numY][numX]; xsss [numS][numX][numY]
+    and ysss [numS][numY][numX] ~ U(-1, 1)."""
+    u = lambda k, cnt: generate("F32_UNIT", seed * 16 + k, cnt, device)
+
+    def site(k0, R, L):
+        a = (-0.5 * u(k0, R * L)).view(R, L)
+        c = (-0.5 * u(k0 + 1, R * L)).view(R, L)
+        b = 1.0 + a.abs() + c.abs()
+        return a.contiguous(), b.contiguous(), c.contiguous()
+
+    ax, bx, cx = site(0, numX, numY)
+    ay, by, cy = site(2, numY, numX)
+    xsss = generate("F32_SIGNED", seed * 16 + 4, numS * numX * numY, device).view(numS, numX, numY)
+    ysss = generate("F32_SIGNED", seed * 16 + 5, numS * numY * numX, device).view(numS, numY, numX)
+    return (ax, bx, cx), (ay, by, cy), xsss, ysss

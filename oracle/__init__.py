@@ -56,6 +56,7 @@ def lib() -> ctypes.CDLL:
             "oracle_segred_f32_literal": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_float],
             "oracle_redomap2": [_vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int],
             "oracle_tridag": [_vp, _vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _vp],
+            "oracle_lvc": [_vp] * 10 + [_c_i64] * 4 + [_vp],
         }.items():
             fn = getattr(L, name)
             fn.argtypes = argt
@@ -197,3 +198,22 @@ def tridag(a, b, c, y, coef_rows: int):
     rc = lib().oracle_tridag(_ptr(a), _ptr(b), _ptr(c), _ptr(y), _ptr(x), S, L, coef_rows, _ptr(work))
     _check(rc)
     return x
+
+
+def lvc(ax, bx, cx, ay, by, cy, xsss, ysss, numT: int):
+    """The LocVolCalib loop of Fig 6a: numT steps of
+    ``map tridag`` over xsss [numS][numX][numY] (coefficients [numX][numY])
+    and ysss [numS][numY][numX] (coefficients [numY][numX]); Thomas solves in
+    double, state kept in double.  Returns (xsss', ysss') as float64."""
+    ax, bx, cx, ay, by, cy, xsss, ysss = (np.ascontiguousarray(v, dtype=np.float32)
+                                          for v in (ax, bx, cx, ay, by, cy, xsss, ysss))
+    numS, numX, numY = xsss.shape
+    assert ysss.shape == (numS, numY, numX)
+    assert ax.shape == bx.shape == cx.shape == (numX, numY)
+    assert ay.shape == by.shape == cy.shape == (numY, numX)
+    xo = np.empty(xsss.shape, np.float64)
+    yo = np.empty(ysss.shape, np.float64)
+    work = np.empty(max(numX, numY, 1), np.float64)
+    _check(lib().oracle_lvc(_ptr(ax), _ptr(bx), _ptr(cx), _ptr(ay), _ptr(by), _ptr(cy), _ptr(xsss), _ptr(ysss),
+                            _ptr(xo), _ptr(yo), numS, int(numT), numX, numY, _ptr(work)))
+    return xo, yo

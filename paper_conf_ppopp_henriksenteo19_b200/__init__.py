@@ -28,9 +28,9 @@ IFL_OK, IFL_EINVAL, IFL_EUNSUPPORTED, IFL_EWORKSPACE, IFL_ENOTFIT, IFL_ECUDA = 0
 DTYPES = {"i32": 0, "f32": 1, "bf16": 2}
 OPS = {"sum": 0, "prod": 1, "min": 2, "max": 3, "and": 4, "or": 5, "xor": 6}
 MAPS = {"id": 0, "sq": 1, "abs": 2}
-VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2}
-VERSION_NAMES = {0: "top", 1: "middle", 2: "flat"}
-SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag")
+VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3}
+VERSION_NAMES = {-1: "auto", 0: "top", 1: "middle", 2: "flat", 3: "outer"}
+SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -63,6 +63,7 @@ _SIGS = {
     "ifl_segscan_seeded": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_redomap2": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_tridag": ([_vp, _vp, _vp, _vp, _vp, _i64, _i64, _i64, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_lvc": ([_vp] * 8 + [_i64] * 4 + [_int, _vp, _sz, _vp, _vp], _int),
     "ifl_workspace_bytes": ([ctypes.c_char_p, _i64, _i64, _i64, _int, _int], _sz),
     "ifl_workspace_init": ([_vp, _sz, _vp], _int),
     "ifl_select": ([ctypes.c_char_p, _i64, _i64, _i64, _vp], _int),
@@ -314,6 +315,30 @@ def tridag(a, b, c, y, version="auto", out=None, ws=None, stream=None, return_ch
     return (out, _choice_out(ch)) if return_choice else out
 
 
+# ----------------------------------------------------------------------- lvc
+
+
+def lvc(xsss, ysss, xcoef, ycoef, numT: int, version="auto", ws=None, stream=None, return_choice=False):
+    """The LocVolCalib loop of Fig 6a, in place on xsss
+    [numS][numX][numY] and ysss [numS][numY][numX]; xcoef = (a, b, c) each
+    [numX][numY], ycoef = (a, b, c) each [numY][numX]."""
+    numS, numX, numY = xsss.shape
+    ts = (xsss, ysss) + tuple(xcoef) + tuple(ycoef)
+    for t in ts:
+        if t.dtype != torch.float32 or not t.is_contiguous() or not t.is_cuda:
+            raise TypeError("lvc takes contiguous float32 CUDA tensors")
+    if tuple(ysss.shape) != (numS, numY, numX):
+        raise ValueError("ysss must be [numS][numY][numX]")
+    wb = lib().ifl_workspace_bytes(b"lvc", numX, numY, 0, 1, -1)
+    if ws is None and wb:
+        ws = workspace(wb, xsss.device, "lvc")
+    ch = ifl_choice()
+    rc = lib().ifl_lvc(*(t.data_ptr() for t in ts), numS, int(numT), numX, numY, VERSIONS[version], _ptr(ws),
+                       0 if ws is None else ws.numel(), _stream(stream), ctypes.byref(ch))
+    _check(rc, "ifl_lvc")
+    return _choice_out(ch) if return_choice else None
+
+
 # ---------------------------------------------------------------------- tuner
 
 
@@ -327,6 +352,8 @@ def tune(site: str, shapes, reps: int = 5, cost: int = 0, scratch: torch.Tensor 
     need = lib().ifl_tune_scratch_bytes(_b(site), sh.ctypes.data, ns)
     if scratch is None or scratch.numel() < need:
         scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
+    if sh.ndim != 2 or sh.shape[1] != (2 if site.startswith("seg") else 4 if site == "lvc" else 3):
+        raise ValueError(f"{site}: shapes must be tuples of the site's arity")
     tbl = np.zeros(ns * 3, np.float64)
     a, b = ctypes.c_int64(), ctypes.c_int64()
     _check(lib().ifl_tune(_b(site), sh.ctypes.data, ns, reps, cost, scratch.data_ptr(), scratch.numel(),

@@ -38,7 +38,7 @@ int cuda_status(cudaError_t e, const char* what) {
 constexpr int64_t kDefaultThreshold = 1 << 15;
 constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE kernel (reading R3)
 
-const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag"};
+const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc"};
 
 struct Table {
     std::mutex mu;
@@ -162,6 +162,14 @@ int ifl_select(const char* site, int64_t n, int64_t m, int64_t p, ifl_choice* ch
     if (!known_site(site)) return fail(IFL_EINVAL, "ifl_select: unknown site '%s'", site ? site : "(null)");
     if (n < 0 || m < 0 || p < 0) return fail(IFL_EINVAL, "ifl_select: negative size");
     bool fits = true;
+    if (strcmp(site, "lvc") == 0) {  // outermost guard of Fig 6c: numS >= t0 (and V_OUTER fits)
+        int64_t t0, tu;
+        ifl_get_thresholds("lvc", &t0, &tu);
+        ifl_choice c{(n >= t0 && m <= ifl::kLvcMaxL && p <= ifl::kLvcMaxL) ? IFL_V_OUTER : IFL_AUTO,
+                     n, sat_mul(n, sat_mul(m, p)), t0, tu};
+        if (choice) *choice = c;
+        return IFL_OK;
+    }
     if (strcmp(site, "tridag") == 0) fits = ifl::tridag_mid_fits(m);
     return select_version(site, n, m, p, fits, choice) >= 0 ? IFL_OK : IFL_EINVAL;
 }
@@ -250,6 +258,8 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
     }
     if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
     if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
+    if (strcmp(entry, "lvc") == 0)  // (numX, numY): the coefficient scans of both sites
+        return ifl::tridag_ws_bytes(n, m, version) + ifl::tridag_ws_bytes(m, n, version);
     return 0;
 }
 
@@ -365,4 +375,71 @@ int ifl_tridag(const float* a, const float* b, const float* c, const float* y, f
     return cuda_status(ifl::launch_tridag(ch.version, t), "ifl_tridag");
 }
 
+int ifl_lvc(float* xsss, float* ysss, const float* ax, const float* bx, const float* cx, const float* ay,
+            const float* by, const float* cy, int64_t numS, int64_t numT, int64_t numX, int64_t numY, int version,
+            void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    return ifl::lvc_run(xsss, ysss, ax, bx, cx, ay, by, cy, numS, numT, numX, numY, version, ws, ws_bytes, stream,
+                        choice, true);
+}
+
 }  // extern "C"
+
+// allow_outer = false: the else-branch of the outermost guard (per-step,
+// per-site G3) even when numS >= t0 -- what the tuner times as the alternative.
+int ifl::lvc_run(float* xsss, float* ysss, const float* ax, const float* bx, const float* cx, const float* ay,
+                 const float* by, const float* cy, int64_t numS, int64_t numT, int64_t numX, int64_t numY,
+                 int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice, bool allow_outer) {
+    if (numS < 0 || numT < 0 || numX < 0 || numY < 0) return fail(IFL_EINVAL, "ifl_lvc: negative size");
+    if (mul_overflows(numX, numY) || mul_overflows(numS, numX * numY) || mul_overflows(numS * numX * numY, 4))
+        return fail(IFL_EINVAL, "ifl_lvc: size overflow");
+    if (version < IFL_AUTO || version > IFL_V_OUTER) return fail(IFL_EINVAL, "ifl_lvc: bad version %d", version);
+    const int64_t E = numS * numX * numY;
+    if (E > 0 && (!xsss || !ysss || !ax || !bx || !cx || !ay || !by || !cy))
+        return fail(IFL_EINVAL, "ifl_lvc: NULL pointer");
+    if (E > 0 && overlap(xsss, (size_t)E * 4, ysss, (size_t)E * 4)) return fail(IFL_EINVAL, "ifl_lvc: xsss overlaps ysss");
+    const bool outer_fits = numX <= ifl::kLvcMaxL && numY <= ifl::kLvcMaxL;
+    // outermost guard of Fig 6c: if numS >= t0 then V_OUTER (reading R1: >=)
+    int64_t t0, t_unused;
+    ifl_get_thresholds("lvc", &t0, &t_unused);
+    ifl_choice ch{IFL_AUTO, numS, numS * numX * numY, t0, t_unused};
+    if (allow_outer && numS >= t0 && outer_fits) ch.version = IFL_V_OUTER;
+    if (version != IFL_AUTO) ch.version = version;
+    if (choice) *choice = ch;
+    if (ch.version == IFL_V_OUTER && !outer_fits)
+        return fail(IFL_ENOTFIT, "ifl_lvc: V_OUTER keeps systems in registers; needs numX, numY <= %lld",
+                    (long long)ifl::kLvcMaxL);
+    if (ch.version == IFL_V_MIDDLE && !(ifl::tridag_mid_fits(numX) && ifl::tridag_mid_fits(numY)))
+        return fail(IFL_ENOTFIT, "ifl_lvc: V_MIDDLE does not fit");
+    if (E == 0 || numT == 0) return IFL_OK;
+    const size_t need = ifl_workspace_bytes("lvc", numX, numY, 0, IFL_F32, IFL_AUTO);
+    if (!ws || ws_bytes < need) return fail(IFL_EWORKSPACE, "ifl_lvc: needs %zu workspace bytes, got %zu", need, ws_bytes);
+    cudaStream_t st = (cudaStream_t)stream;
+    float* wx = (float*)ws;
+    float* wy = wx + 3 * numX * numY;
+    // site x: numS*numX systems of length numY, coefficient rows [numX][numY]; site y mirrored
+    ifl::TriArgs tx{ax, bx, cx, xsss, xsss, numS * numX, numY, numX, wx, (size_t)numX * numY * 12, st};
+    ifl::TriArgs ty{ay, by, cy, ysss, ysss, numS * numY, numX, numY, wy, (size_t)numX * numY * 12, st};
+    int vx = ch.version, vy = ch.version;
+    if (ch.version == IFL_AUTO) {  // recurse: G3 of the per-site tridag (Fig 6c versions 1-3)
+        vx = select_version("tridag", tx.S, tx.L, 0, ifl::tridag_mid_fits(tx.L), nullptr);
+        vy = select_version("tridag", ty.S, ty.L, 0, ifl::tridag_mid_fits(ty.L), nullptr);
+    }
+    // the (+) scan of the coefficients is loop-invariant: once per site
+    cudaError_t e = ifl::launch_tridag_coef(vx == IFL_V_TOP ? 0 : 1, tx);
+    if (e == cudaSuccess) e = ifl::launch_tridag_coef(vy == IFL_V_TOP ? 0 : 1, ty);
+    if (e != cudaSuccess) return cuda_status(e, "ifl_lvc");
+    if (ch.version == IFL_V_OUTER) {
+        const int64_t RLx = numX * numY;
+        ifl::LvcSite sx{xsss, tx.S, tx.L, tx.coef_rows, wx, wx + RLx, wx + 2 * RLx};
+        ifl::LvcSite sy{ysss, ty.S, ty.L, ty.coef_rows, wy, wy + RLx, wy + 2 * RLx};
+        return cuda_status(ifl::launch_lvc_outer(sx, sy, numT, st), "ifl_lvc");
+    }
+    for (int64_t t = 0; t < numT; ++t) {  // one step: both sites, in place
+        e = ifl::launch_tridag_solve(vx, tx);
+        if (e == cudaSuccess) e = ifl::launch_tridag_solve(vy, ty);
+        if (e != cudaSuccess) return cuda_status(e, "ifl_lvc");
+    }
+    return IFL_OK;
+}
+
+

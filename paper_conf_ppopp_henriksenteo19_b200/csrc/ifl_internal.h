@@ -5,6 +5,8 @@
 #include <stddef.h>
 #include <stdint.h>
 
+#include "../../include/ifl.h"
+
 namespace ifl {
 
 // Arguments of one segred/segscan call after validation and version choice.
@@ -64,6 +66,22 @@ struct TriArgs {
 };
 size_t tridag_ws_bytes(int64_t coef_rows, int64_t L, int version);
 bool tridag_mid_fits(int64_t L);
-cudaError_t launch_tridag(int version, const TriArgs& a);
+cudaError_t launch_tridag(int version, const TriArgs& a);       // coef + solve
+cudaError_t launch_tridag_coef(int version, const TriArgs& a);  // (+) scan of the coefficient rows -> ws
+cudaError_t launch_tridag_solve(int version, const TriArgs& a); // (x) and (.) scans per system (ws from _coef)
+
+// Whole LocVolCalib-shaped program (lvc.cu): V_OUTER keeps every system in
+// registers across all numT steps.  fits: both lengths <= kLvcMaxL.
+constexpr int64_t kLvcMaxL = 512;
+struct LvcSite {
+    float* xs;       // [S][L] in place
+    int64_t S, L, R; // systems, length, coefficient rows
+    const float *invb, *alpha, *delta;  // [R][L] each, from launch_tridag_coef
+};
+cudaError_t launch_lvc_outer(const LvcSite& x, const LvcSite& y, int64_t numT, cudaStream_t s);
+// ifl_lvc with the outermost branch optionally disabled (the tuner's alternative)
+int lvc_run(float* xsss, float* ysss, const float* ax, const float* bx, const float* cx, const float* ay,
+            const float* by, const float* cy, int64_t numS, int64_t numT, int64_t numX, int64_t numY, int version,
+            void* ws, size_t ws_bytes, void* stream, ifl_choice* choice, bool allow_outer);
 
 }  // namespace ifl

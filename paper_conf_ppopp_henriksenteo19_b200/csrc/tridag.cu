@@ -466,19 +466,35 @@ size_t tridag_ws_bytes(int64_t R, int64_t L, int version) {
     return (size_t)R * L * 3 * sizeof(float);
 }
 
-cudaError_t launch_tridag(int version, const TriArgs& t) {
-    const int64_t R = t.coef_rows, L = t.L, S = t.S;
+// The (+) scan of every coefficient row into the workspace (invbeta, alpha,
+// delta): sequential per row for V_TOP, the CTA-wide 2x2 matrix scan otherwise.
+cudaError_t launch_tridag_coef(int version, const TriArgs& t) {
+    const int64_t R = t.coef_rows, L = t.L;
     float* invb = (float*)t.ws;
     float* alpha = invb + R * L;
     float* delta = alpha + R * L;
-    cudaError_t e;
     if (version == 0) {
         const int g = (int)std::min<int64_t>(ceil_div(R, 128), 148 * 8);
         tridag_coef_seq<<<g, 128, 0, t.stream>>>(t.a, t.b, t.c, invb, alpha, delta, R, L);
     } else {
         tridag_coef_mat2<<<(unsigned)R, 256, 0, t.stream>>>(t.a, t.b, t.c, invb, alpha, delta, L);
     }
-    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+    return cudaGetLastError();
+}
+
+cudaError_t launch_tridag(int version, const TriArgs& t) {
+    cudaError_t e = launch_tridag_coef(version, t);
+    if (e != cudaSuccess) return e;
+    return launch_tridag_solve(version, t);
+}
+
+// The per-system (x) / (.) scans, given the coefficient scans in the workspace.
+cudaError_t launch_tridag_solve(int version, const TriArgs& t) {
+    const int64_t R = t.coef_rows, L = t.L, S = t.S;
+    float* invb = (float*)t.ws;
+    float* alpha = invb + R * L;
+    float* delta = alpha + R * L;
+    cudaError_t e;
     if (version == 0) {
         const int g = (int)std::min<int64_t>(ceil_div(S, 256), 148 * 16);
         tridag_top_kernel<<<g, 256, 0, t.stream>>>(t.y, t.x, invb, alpha, delta, S, L, R);

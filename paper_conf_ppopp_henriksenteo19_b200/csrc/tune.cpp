@@ -89,7 +89,7 @@ extern "C" int ifl_tune_search(const int64_t* par_top, const int64_t* par_mid, c
 
 namespace {
 
-enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_BAD };
+enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_BAD };
 
 Kind kind_of(const char* site) {
     if (!site) return K_BAD;
@@ -98,10 +98,11 @@ Kind kind_of(const char* site) {
     if (!strcmp(site, "redomap2.f32")) return K_MM_F32;
     if (!strcmp(site, "redomap2.bf16")) return K_MM_BF16;
     if (!strcmp(site, "tridag")) return K_TRIDAG;
+    if (!strcmp(site, "lvc")) return K_LVC;
     return K_BAD;
 }
 
-int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN) ? 2 : 3; }
+int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN) ? 2 : k == K_LVC ? 4 : 3; }
 
 size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 
@@ -112,6 +113,7 @@ size_t ws_bytes_of(Kind k, const int64_t* s) {
     case K_MM_F32: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_F32, -1);
     case K_MM_BF16: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_BF16, -1);
     case K_TRIDAG: return ifl_workspace_bytes("tridag", s[0], s[1], s[2], IFL_F32, -1);
+    case K_LVC: return ifl_workspace_bytes("lvc", s[2], s[3], 0, IFL_F32, -1);
     default: return 0;
     }
 }
@@ -137,6 +139,10 @@ size_t shape_bytes(Kind k, const int64_t* s) {
         const int64_t S = s[0], L = s[1], R = s[2];
         return 3 * align256(R * L * 4) + 2 * align256(S * L * 4) +
                align256(ifl_workspace_bytes("tridag", S, L, R, IFL_F32, -1));
+    }
+    case K_LVC: {  // (numS, numT, numX, numY): xsss, ysss, 6 coefficient arrays, ws
+        const int64_t E = s[0] * s[2] * s[3], RL = s[2] * s[3];
+        return 2 * align256(E * 4) + 6 * align256(RL * 4) + align256(ws_bytes_of(k, s));
     }
     default: return 0;
     }
@@ -182,6 +188,20 @@ int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_
         return ifl_tridag((float*)a, (float*)b, (float*)c, (float*)y, (float*)x, S, L, R, version, ws,
                           ifl_workspace_bytes("tridag", S, L, R, IFL_F32, -1), st, nullptr);
     }
+    case K_LVC: {
+        // table slot 0 (TOP) = the outermost version V_OUTER, slot 2 (FLAT) =
+        // its else-branch (per-step, per-site G3); slot 1 is unavailable
+        if (version == IFL_V_MIDDLE) return IFL_ENOTFIT;
+        const int64_t E = s[0] * s[2] * s[3], RL = s[2] * s[3];
+        float* xs = (float*)scratch;
+        float* ys = (float*)(scratch + align256(E * 4));
+        char* co = scratch + 2 * align256(E * 4);
+        const float* cf[6];
+        for (int q = 0; q < 6; ++q) cf[q] = (const float*)(co + q * align256(RL * 4));
+        char* ws = co + 6 * align256(RL * 4);
+        return ifl::lvc_run(xs, ys, cf[0], cf[1], cf[2], cf[3], cf[4], cf[5], s[0], s[1], s[2], s[3],
+                            version == IFL_V_TOP ? IFL_V_OUTER : IFL_AUTO, ws, ws_bytes_of(k, s), st, nullptr, false);
+    }
     default: return IFL_EINVAL;
     }
 }
@@ -223,6 +243,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         const int64_t* s = shapes + i * ar;
         ifl_choice c;
         ifl_select(site, s[0], s[1], ar == 3 && k != K_TRIDAG ? s[2] : 0, &c);
+        if (k == K_LVC) c.par_mid = 0;  // one guard: Par = numS
         ptop[i] = c.par_top;
         pmid[i] = c.par_mid;
         // zero this shape's workspace (the tail of its scratch layout); the

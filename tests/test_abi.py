@@ -241,3 +241,31 @@ def test_tune_search_minimax_cost(L):
     a0, b0, _ = ifl.tune_search(pt, pm, table, cost=0)
     a1, b1, _ = ifl.tune_search(pt, pm, table, cost=1)
     assert _path_cost(pt, pm, table, a0, b0) <= _path_cost(pt, pm, table, a1, b1)
+
+
+def test_lvc_validation_and_guard(L):
+    P = [256] * 8
+    # negative size / bad version / NULL pointers / overlapping arrays (no launch)
+    assert L.ifl_lvc(*P, -1, 2, 4, 4, -1, None, 0, None, None) == ifl.IFL_EINVAL
+    assert L.ifl_lvc(*P[:7], 256, 2, 2, 4, 4, 7, None, 0, None, None) == ifl.IFL_EINVAL
+    assert L.ifl_lvc(0, *P[1:], 2, 2, 4, 4, -1, None, 0, None, None) == ifl.IFL_EINVAL
+    assert L.ifl_lvc(*P, 2, 2, 4, 4, -1, None, 0, None, None) == ifl.IFL_EINVAL  # xsss == ysss
+    # V_OUTER keeps systems in registers: lengths > 512 do not fit (P:358 fit clause)
+    xs, ys = 1 << 20, 1 << 24
+    assert L.ifl_lvc(xs, ys, *P[2:], 2, 2, 4, 600, 3, None, 0, None, None) == ifl.IFL_ENOTFIT
+    # no workspace
+    assert L.ifl_lvc(xs, ys, *P[2:], 2, 2, 4, 8, 3, None, 0, None, None) == ifl.IFL_EWORKSPACE
+    # empty problem and zero steps are no-ops
+    assert L.ifl_lvc(xs, ys, *P[2:], 0, 2, 4, 8, -1, None, 0, None, None) == 0
+    assert L.ifl_lvc(xs, ys, *P[2:], 2, 0, 4, 8, -1, None, 0, None, None) == 0
+    assert ifl.workspace_bytes("lvc", 32, 256) == 6 * 32 * 256 * 4
+    # outermost guard of Fig 6c: numS >= t0 (R1) and fit
+    try:
+        ifl.set_thresholds("lvc", 100, 0)
+        assert ifl.select("lvc", 100, 32, 256).version == "outer"
+        assert ifl.select("lvc", 99, 32, 256).version == "auto"
+        assert ifl.select("lvc", 100, 32, 513).version == "auto"
+        c = ifl.select("lvc", 128, 256, 32)
+        assert (c.par_top, c.t_top) == (128, 100)
+    finally:
+        ifl.reset_thresholds()

@@ -362,3 +362,88 @@ def test_seeded_continues_a_split_row(orc):
 def test_seeded_equal_seeds_is_plain_scan(orc):
     x = np.arange(24, dtype=np.int32).reshape(3, 8)
     np.testing.assert_array_equal(orc.segscan_seeded(x, np.full(3, 7, np.int32), "sum"), orc.segscan(x, "sum", "id", 7))
+
+
+# ------------------------------------------------------- lvc (Fig 6a loop)
+
+
+def _spectral_powers(lam, L, T, y):
+    """tridiag(-lam, 1+2 lam, -lam)^{-T} y by the sine eigenbasis of the
+    Dirichlet second difference: v_k(j) = sin(pi k (j+1) / (L+1)),
+    mu_k = 1 + 4 lam sin^2(pi k / (2 (L+1))) -- a closed form that shares
+    nothing with the Thomas recurrence."""
+    j = np.arange(L)
+    k = np.arange(1, L + 1)
+    V = np.sin(np.pi * np.outer(k, j + 1) / (L + 1))  # [k][j], V V^T = (L+1)/2 I
+    mu = 1 + 4 * lam * np.sin(np.pi * k / (2 * (L + 1))) ** 2
+    coef = (V @ y.T) * (2.0 / (L + 1)) * mu[:, None] ** (-T)
+    return (V.T @ coef).T
+
+
+def test_lvc_spectral_closed_form(orc):
+    lam = 0.375  # exact in f32
+    numS, numX, numY = 2, 5, 7
+    for T in (0, 1, 3, 8):
+        ax = np.full((numX, numY), -lam, np.float32)
+        bx = np.full((numX, numY), 1 + 2 * lam, np.float32)
+        ay = np.full((numY, numX), -lam, np.float32)
+        by = np.full((numY, numX), 1 + 2 * lam, np.float32)
+        (_, _, _), (_, _, _), xs, ys = gen.lvc_problem(3, numS, numX, numY)
+        xs, ys = xs.numpy(), ys.numpy()
+        xo, yo = orc.lvc(ax, bx, ax, ay, by, ay, xs, ys, T)
+        want_x = _spectral_powers(lam, numY, T, xs.reshape(-1, numY).astype(np.float64)).reshape(xs.shape)
+        want_y = _spectral_powers(lam, numX, T, ys.reshape(-1, numX).astype(np.float64)).reshape(ys.shape)
+        np.testing.assert_allclose(xo, want_x, rtol=1e-11, atol=1e-12)
+        np.testing.assert_allclose(yo, want_y, rtol=1e-11, atol=1e-12)
+
+
+def _banded_matvec(a, b, c, x):
+    """A x for A = tridiag(a[1:], b, c[:-1]) row by row (a[0], c[L-1] unused)."""
+    Ax = b * x
+    Ax[..., 1:] += a[..., 1:] * x[..., :-1]
+    Ax[..., :-1] += c[..., :-1] * x[..., 1:]
+    return Ax
+
+
+def test_lvc_step_residuals_and_scipy(orc):
+    # each step solves A x_t = x_{t-1} (residual by a plain matvec), and the
+    # loop equals scipy's banded solver applied numT times
+    from scipy.linalg import solve_banded
+    numS, numX, numY, T = 3, 6, 9, 4
+    (ax, bx, cx), (ay, by, cy), xs, ys = (v if isinstance(v, torch.Tensor) else tuple(t.numpy() for t in v)
+                                          for v in gen.lvc_problem(5, numS, numX, numY))
+    xs, ys = xs.numpy(), ys.numpy()
+    prev_x, prev_y = xs.astype(np.float64), ys.astype(np.float64)
+    for t in range(1, T + 1):
+        xo, yo = orc.lvc(ax, bx, cx, ay, by, cy, xs, ys, t)
+        rx = _banded_matvec(ax.astype(np.float64)[None], bx.astype(np.float64)[None], cx.astype(np.float64)[None], xo) - prev_x
+        ry = _banded_matvec(ay.astype(np.float64)[None], by.astype(np.float64)[None], cy.astype(np.float64)[None], yo) - prev_y
+        assert np.abs(rx).max() < 1e-12 and np.abs(ry).max() < 1e-12
+        prev_x, prev_y = xo, yo
+    # scipy, applied T times per system
+    want = xs.astype(np.float64).copy()
+    for s in range(numS):
+        for x in range(numX):
+            ab = np.zeros((3, numY))
+            ab[0, 1:] = cx[x, :-1]
+            ab[1] = bx[x]
+            ab[2, :-1] = ax[x, 1:]
+            for _ in range(T):
+                want[s, x] = solve_banded((1, 1), ab, want[s, x])
+    np.testing.assert_allclose(prev_x, want, rtol=1e-10, atol=1e-12)
+
+
+def test_lvc_sites_independent_and_tridag_consistent(orc):
+    numS, numX, numY = 2, 4, 8
+    (ax, bx, cx), (ay, by, cy), xs, ys = gen.lvc_problem(11, numS, numX, numY)
+    ax, bx, cx, ay, by, cy, xs, ys = (t.numpy() for t in (ax, bx, cx, ay, by, cy, xs, ys))
+    xo, yo = orc.lvc(ax, bx, cx, ay, by, cy, xs, ys, 2)
+    xo2, _ = orc.lvc(ax, bx, cx, ay, by, cy, xs, np.zeros_like(ys), 2)
+    np.testing.assert_array_equal(xo, xo2)  # the y-site never touches xsss
+    # one step = one tridag call per site with coefficient rows shared (R9)
+    x1, y1 = orc.lvc(ax, bx, cx, ay, by, cy, xs, ys, 1)
+    np.testing.assert_allclose(x1.reshape(-1, numY), orc.tridag(ax, bx, cx, xs.reshape(-1, numY), numX), rtol=1e-14)
+    np.testing.assert_allclose(y1.reshape(-1, numX), orc.tridag(ay, by, cy, ys.reshape(-1, numX), numY), rtol=1e-14)
+    # the diffusion-like recipe keeps the state O(1) over many steps (no underflow)
+    xT, _ = orc.lvc(ax, bx, cx, ay, by, cy, np.ones_like(xs), ys, 256)
+    assert 0.05 < np.abs(xT).max() <= 1.0 + 1e-12
