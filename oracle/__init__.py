@@ -53,6 +53,8 @@ def lib() -> ctypes.CDLL:
             "oracle_segred_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double],
             "oracle_segscan_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double, _c_int],
             "oracle_colred_f32": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double],
+            "oracle_colscan_i32": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_int32],
+            "oracle_colscan_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_double],
             "oracle_segred_f32_literal": [_vp, _vp, _c_i64, _c_i64, _c_int, _c_int, ctypes.c_float],
             "oracle_redomap2": [_vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int],
             "oracle_tridag": [_vp, _vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _vp],
@@ -160,6 +162,22 @@ def colred(x: np.ndarray, op: str = "sum", f: str = "id", d=None):
     out = np.empty(m, np.float64)
     _check(lib().oracle_colred_f32(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f], d))
     return out
+
+
+def colscan(x: np.ndarray, op: str = "sum", f: str = "id", d=None, with_absum=False):
+    """G4 (P:156) with scan: out[i][j] = d (+) f(x[0][j]) (+) ... (+) f(x[i][j])."""
+    x = np.ascontiguousarray(x)
+    n, m = x.shape
+    if x.dtype == np.int32:
+        d = canonical_ne(op, "i32") if d is None else int(d)
+        out = np.empty((n, m), np.int32)
+        _check(lib().oracle_colscan_i32(_ptr(x), _ptr(out), n, m, OPS[op], MAPS[f], _i32(d)))
+        return out
+    d = canonical_ne(op, "f32") if d is None else float(np.float32(d))
+    out = np.empty((n, m), np.float64)
+    ab = np.empty((n, m), np.float64)
+    _check(lib().oracle_colscan_f32(_ptr(x), _ptr(out), _ptr(ab), n, m, OPS[op], MAPS[f], d))
+    return (out, ab) if with_absum else out
 
 
 def segred_f32_literal(x: np.ndarray, op: str = "sum", f: str = "id", d=None):

@@ -447,3 +447,39 @@ def test_lvc_sites_independent_and_tridag_consistent(orc):
     # the diffusion-like recipe keeps the state O(1) over many steps (no underflow)
     xT, _ = orc.lvc(ax, bx, cx, ay, by, cy, np.ones_like(xs), ys, 256)
     assert 0.05 < np.abs(xT).max() <= 1.0 + 1e-12
+
+
+# ------------------------------------------- colscan (G4 with scan, NEXT-3)
+
+
+def test_colscan_closed_forms(orc):
+    n, m = 9, 5
+    np.testing.assert_array_equal(orc.colscan(np.ones((n, m), np.int32)), np.tile(np.arange(1, n + 1)[:, None], (1, m)))
+    x = np.tile(np.arange(n, dtype=np.int32)[:, None], (1, m))
+    i = np.arange(n)
+    np.testing.assert_array_equal(orc.colscan(x), np.tile((i * (i + 1) // 2)[:, None], (1, m)))
+    # max-scan down a column that increases: the column itself
+    np.testing.assert_array_equal(orc.colscan(x, "max"), x)
+    assert orc.colscan(np.zeros((0, 3), np.int32)).shape == (0, 3)
+
+
+@pytest.mark.parametrize("op", INT_OPS)
+def test_colscan_g4_identity_and_numpy(orc, op):
+    # G4: the column scan is the row scan of the transpose; its last row is colred
+    M = gen.matrix("I32_FULL", 21, 13, 29).numpy()
+    cs = orc.colscan(M, op, "sq")
+    np.testing.assert_array_equal(cs, orc.segscan(np.ascontiguousarray(M.T), op, "sq").T)
+    np.testing.assert_array_equal(cs[-1], orc.colred(M, op, "sq"))
+    if op == "sum":  # numpy: square mod 2^32 in int64, cumsum, then wrap
+        sq = (M.astype(np.int64) * M.astype(np.int64)) % 2**32
+        np.testing.assert_array_equal(cs, ((sq.cumsum(0) + 2**31) % 2**32 - 2**31).astype(np.int32))
+
+
+def test_colscan_f32_numpy_and_exact(orc):
+    Mf = gen.matrix("F32_EXACT", 23, 40, 17).numpy()
+    np.testing.assert_array_equal(orc.colscan(Mf), Mf.astype(np.float64).cumsum(0))
+    Mu = gen.matrix("F32_SIGNED", 24, 50, 7).numpy()
+    out, ab = orc.colscan(Mu, "sum", "abs", with_absum=True)
+    np.testing.assert_allclose(out, np.abs(Mu).astype(np.float64).cumsum(0), rtol=1e-13)
+    np.testing.assert_allclose(ab, out, rtol=1e-13)  # f = abs: the bound scale equals the result
+    np.testing.assert_array_equal(orc.colscan(Mu, "min")[-1], orc.colred(Mu, "min"))
