@@ -268,6 +268,65 @@ def suite_lvc():
     return line
 
 
+# ----------------------------------------------------------------------- col
+
+
+def suite_col():
+    """NEXT-3: column (axis-0) segred / segscan, G4,
+    over the same constant-work sweep as configs[1]: [n][m] f32 with
+    n*m = 2^26, n = 2^k.  Thresholds tuned on the 2^25 and 2^27 sweeps
+    (bracketing, other data); every forced version timed where it can occupy the GPU
+    (TOP needs >= 4096 column threads, MIDDLE >= 64 column tiles -- the
+    others run a few threads for seconds and are reported as null)."""
+    hbm, _, src = peaks()
+    ifl.reset_thresholds()
+    L2N = 26
+    sh = [(1 << k, 1 << (L2N - k)) for k in range(L2N + 1)]
+    tuned = {}
+    for site in ("colred.b4", "colscan.b4"):
+        train = [(1 << k, 1 << (lg - k)) for lg in (25, 27) for k in range(lg + 1)]
+        need = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data, len(train))
+        scratch = torch.empty(need, dtype=torch.uint8, device="cuda")
+        scratch.view(-1)[: (need // 4) * 4].view(torch.float32).copy_(gen.generate("F32_UNIT", 4, need // 4, "cuda"))
+        a, b, _ = ifl.tune(site, train, reps=3, cost=1, scratch=scratch)
+        del scratch
+        tuned[site] = {"t_top": a, "t_intra": b}
+    N = 1 << L2N
+    xs = gen.generate("F32_UNIT", 2, N, device="cuda")
+    out = torch.empty(N, dtype=torch.float32, device="cuda")
+    ws = ifl.workspace(max(ifl.workspace_bytes("colscan", n, m) for n, m in sh), "cuda", "colsuite")
+    rows = []
+    for kind in ("colred", "colscan"):
+        fn = ifl.colscan if kind == "colscan" else ifl.colred
+        for (n, m) in sh:
+            x = xs.view(n, m)
+            o = out.view(n, m) if kind == "colscan" else out[:m]
+            r = {"op": kind, "n": n, "m": m}
+            for v in ("top", "middle", "flat", "auto"):
+                if (v == "top" and m < 4096 * (4 if m % 4 == 0 else 1)) or (v == "middle" and (m + 127) // 128 < 64):
+                    r[v] = None
+                    continue
+                r[v] = gtime(lambda: fn(x, out=o, ws=ws, version=v)) * 1e3
+            r["chosen"] = fn(x, out=o, ws=ws, return_choice=True)[1].version
+            best = min(t for t in (r["top"], r["middle"], r["flat"]) if t is not None)
+            r["best_over_auto"] = round(best / r["auto"], 4)
+            byt = (8 * n * m) if kind == "colscan" else 4 * (n * m + m)
+            r["GBps"] = round(byt / (r["auto"] * 1e-6) / 1e9, 1)
+            rows.append(r)
+    tot_b = sum((8 * r["n"] * r["m"]) if r["op"] == "colscan" else 4 * (r["n"] * r["m"] + r["m"]) for r in rows)
+    tot_t = sum(r["auto"] for r in rows)
+    agg = tot_b / (tot_t * 1e-6) / 1e9
+    line = base_line("colred/colscan GB/s over the n x m sweep (G4 axis-0 reductions)", round(agg, 1), "GB/s",
+                     {"workload": "SURVEY 8(f) NEXT-3: column segred + segscan, f32 sum, n*m = 2^26, n = 2^0..2^26, "
+                                  "AUTO with tuned thresholds", "thresholds": tuned})
+    line["min_shape_best_over_auto"] = min(r["best_over_auto"] for r in rows)
+    line["roofline"] = {"bound": "hbm", "kernel": "colred+colscan sweep (AUTO)", "achieved": round(agg, 1),
+                        "peak": hbm, "unit": "GB/s", "frac": round(agg / hbm, 4), "traffic": None,
+                        "peak_source": src}
+    line["shapes"] = rows
+    return line
+
+
 # ---------------------------------------------------------------------- dist
 
 
@@ -311,4 +370,4 @@ def suite_dist():
 
 
 SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist,
-          "lvc": suite_lvc}
+          "lvc": suite_lvc, "col": suite_col}

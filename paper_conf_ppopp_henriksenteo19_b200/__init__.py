@@ -30,7 +30,7 @@ OPS = {"sum": 0, "prod": 1, "min": 2, "max": 3, "and": 4, "or": 5, "xor": 6}
 MAPS = {"id": 0, "sq": 1, "abs": 2}
 VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3}
 VERSION_NAMES = {-1: "auto", 0: "top", 1: "middle", 2: "flat", 3: "outer"}
-SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc")
+SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -61,6 +61,8 @@ _SIGS = {
     "ifl_segred": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segscan": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segscan_seeded": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_colred": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_colscan": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_redomap2": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_tridag": ([_vp, _vp, _vp, _vp, _vp, _i64, _i64, _i64, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_lvc": ([_vp] * 8 + [_i64] * 4 + [_int, _vp, _sz, _vp, _vp], _int),
@@ -265,6 +267,40 @@ def segscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, str
     return _seg(True, x, op, f, ne, version, out, ws, stream, return_choice, seed)
 
 
+# ----------------------------------------------------------- colred / colscan
+
+
+def _col(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws, stream, return_choice):
+    if x.dim() != 2 or not x.is_contiguous() or not x.is_cuda:
+        raise ValueError("expected a contiguous [n][m] CUDA tensor")
+    dt = _TORCH_DT.get(x.dtype)
+    if dt not in ("i32", "f32"):
+        raise TypeError(f"unsupported dtype {x.dtype}")
+    n, m = x.shape
+    if out is None:
+        out = torch.empty((n, m) if scan else (m,), dtype=x.dtype, device=x.device)
+    entry = "colscan" if scan else "colred"
+    wb = lib().ifl_workspace_bytes(_b(entry), n, m, 0, DTYPES[dt], VERSIONS[version])
+    if ws is None and wb:
+        ws = workspace(wb, x.device, "col")
+    c = ifl_choice()
+    fn = lib().ifl_colscan if scan else lib().ifl_colred
+    rc = fn(x.data_ptr(), out.data_ptr(), n, m, DTYPES[dt], OPS[op], MAPS[f], _ne_buf(ne, dt), VERSIONS[version],
+            _ptr(ws), 0 if ws is None else ws.numel() * ws.element_size(), _stream(stream), ctypes.byref(c))
+    _check(rc, "ifl_" + entry)
+    return (out, _choice_out(c)) if return_choice else out
+
+
+def colred(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False):
+    """out[j] = ne (+) f(x[0,j]) (+) ... (+) f(x[n-1,j]) -- G4's column reduction."""
+    return _col(False, x, op, f, ne, version, out, ws, stream, return_choice)
+
+
+def colscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False):
+    """out[i,j] = ne (+) f(x[0,j]) (+) ... (+) f(x[i,j]) -- column-wise inclusive scan (G4 with scan)."""
+    return _col(True, x, op, f, ne, version, out, ws, stream, return_choice)
+
+
 # ------------------------------------------------------------------ redomap2
 
 
@@ -352,7 +388,7 @@ def tune(site: str, shapes, reps: int = 5, cost: int = 0, scratch: torch.Tensor 
     need = lib().ifl_tune_scratch_bytes(_b(site), sh.ctypes.data, ns)
     if scratch is None or scratch.numel() < need:
         scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
-    if sh.ndim != 2 or sh.shape[1] != (2 if site.startswith("seg") else 4 if site == "lvc" else 3):
+    if sh.ndim != 2 or sh.shape[1] != (2 if site.startswith(("seg", "col")) else 4 if site == "lvc" else 3):
         raise ValueError(f"{site}: shapes must be tuples of the site's arity")
     tbl = np.zeros(ns * 3, np.float64)
     a, b = ctypes.c_int64(), ctypes.c_int64()

@@ -116,6 +116,7 @@ __device__ __forceinline__ T ldg1(const T* p) { return __ldg(p); }
 template <int OP, typename T>
 struct Acc {
     T s;
+    __device__ __forceinline__ Acc() {}
     __device__ __forceinline__ explicit Acc(T init) : s(init) {}
     __device__ __forceinline__ void add(T x) { s = combine<OP>(s, x); }
     __device__ __forceinline__ T get() const { return s; }
@@ -123,6 +124,7 @@ struct Acc {
 template <>
 struct Acc<OP_SUM, float> {
     float s, c;
+    __device__ __forceinline__ Acc() {}
     __device__ __forceinline__ explicit Acc(float init) : s(init), c(0.0f) {}
     __device__ __forceinline__ void add(float x) {
         const float y = __fsub_rn(x, c);

@@ -38,7 +38,8 @@ int cuda_status(cudaError_t e, const char* what) {
 constexpr int64_t kDefaultThreshold = 1 << 15;
 constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE kernel (reading R3)
 
-const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc"};
+const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
+                              "colred.b4", "colscan.b4"};
 
 struct Table {
     std::mutex mu;
@@ -75,6 +76,11 @@ bool mul_overflows(int64_t a, int64_t b) { return a > 0 && b > 0 && a > INT64_MA
 void par_values(const char* site, int64_t n, int64_t m, int64_t p, int mode, int64_t* ptop, int64_t* pmid) {
     int64_t outer = n;
     if (strncmp(site, "redomap2", 8) == 0) outer = sat_mul(n, p);
+    if (strncmp(site, "col", 3) == 0) {  // G4: the segments are the m columns, each of n rows
+        *ptop = m;
+        *pmid = mode == 1 ? sat_mul(m, std::min(n, ifl::kColGroup)) : sat_mul(m, n);
+        return;
+    }
     *ptop = outer;
     *pmid = mode == 1 ? sat_mul(outer, std::min(m, kBmax)) : sat_mul(outer, m);
 }
@@ -155,7 +161,8 @@ extern "C" {
 const char* ifl_last_error(void) { return g_err.c_str(); }
 
 const char* ifl_build_info(void) {
-    return "ifl " __DATE__ " sm_100a; versions: top/middle/flat; segred segscan redomap2 tridag tune";
+    return "ifl " __DATE__ " sm_100a; versions: top/middle/flat(/outer); segred segscan colred colscan redomap2 tridag "
+           "lvc tune";
 }
 
 int ifl_select(const char* site, int64_t n, int64_t m, int64_t p, ifl_choice* choice) {
@@ -257,6 +264,7 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
         return 0;
     }
     if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
+    if (strcmp(entry, "colred") == 0 || strcmp(entry, "colscan") == 0) return ifl::col_ws_bytes(n, m, version);
     if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
     if (strcmp(entry, "lvc") == 0)  // (numX, numY): the coefficient scans of both sites
         return ifl::tridag_ws_bytes(n, m, version) + ifl::tridag_ws_bytes(m, n, version);
@@ -309,6 +317,44 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
     }
     }
     return cuda_status(e, what);
+}
+
+// Column (axis-0) reduce / scan (G4).  out: [m] (reduce) or [n][m] (scan).
+static int run_col(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne,
+                   int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    const char* what = scan ? "ifl_colscan" : "ifl_colred";
+    // validate_seg checks the [n][m] input; the output of a column reduce has m elements
+    int rc = validate_seg(true, in, scan ? out : (n * m > 0 ? out : const_cast<void*>(in)), n, m, dt, op, f, version, what);
+    if (rc) return rc;
+    if (!scan && m > 0 && !out) return fail(IFL_EINVAL, "%s: out is NULL", what);
+    const size_t ob = (size_t)(scan ? n * m : m) * 4, ib = (size_t)(n * m) * 4;
+    if (scan ? (in != out && overlap(in, ib, out, ob)) : overlap(in, ib, out, ob))
+        return fail(IFL_EINVAL, "%s: in/out overlap", what);
+    uint32_t bits = canonical_bits(dt, op);
+    if (ne) memcpy(&bits, ne, 4);
+    ifl_choice c;
+    select_version(scan ? "colscan.b4" : "colred.b4", n, m, 0, true, &c);
+    if (version != IFL_AUTO) c.version = version;
+    if (choice) *choice = c;
+    if (m == 0) return IFL_OK;
+    if (n == 0) return scan ? IFL_OK : cuda_status(ifl::launch_fill(out, m, bits, (cudaStream_t)stream), what);
+    if (c.version == IFL_V_FLAT) {
+        const size_t need = ifl::col_ws_bytes(n, m, IFL_V_FLAT);
+        if (!ws || ws_bytes < need)
+            return fail(IFL_EWORKSPACE, "%s: V_FLAT needs %zu workspace bytes, got %zu", what, need, ws_bytes);
+    }
+    ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream, nullptr};
+    return cuda_status(ifl::launch_col(a, scan, c.version), what);
+}
+
+int ifl_colred(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int version,
+               void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    return run_col(false, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+}
+
+int ifl_colscan(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int version,
+                void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    return run_col(true, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
 }
 
 int ifl_segred(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int version,

@@ -41,6 +41,17 @@ cudaError_t launch_fill(void* out, int64_t count, uint32_t bits, cudaStream_t s)
 int mid_group_size(int64_t m);
 int midscan_group_size(int64_t m);
 
+// Column (axis-0) segred / segscan, G4 (colred.cu).  version 0/1/2 = TOP /
+// MIDDLE / FLAT; FLAT needs col_ws_bytes of workspace (per-chunk partials).
+struct ColGeom {
+    int64_t nv, mv;  // the (possibly virtual, narrow mode) [nv][mv] view the kernels walk
+    int64_t ntiles, P, rows_per_chunk;
+};
+ColGeom col_geom(int64_t n, int64_t m, int version, bool vec4, int narrow_width);
+size_t col_ws_bytes(int64_t n, int64_t m, int version);
+cudaError_t launch_col(const SegArgs& a, bool scan, int version);
+constexpr int64_t kColGroup = 8;  // threads per column in V_MIDDLE (reading R3's group size)
+
 // redomap2 (redomap2.cu) and tridag (tridag.cu)
 struct MmArgs {
     const void* A;

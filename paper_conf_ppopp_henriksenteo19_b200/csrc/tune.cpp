@@ -89,7 +89,7 @@ extern "C" int ifl_tune_search(const int64_t* par_top, const int64_t* par_mid, c
 
 namespace {
 
-enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_BAD };
+enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_COLRED, K_COLSCAN, K_BAD };
 
 Kind kind_of(const char* site) {
     if (!site) return K_BAD;
@@ -99,12 +99,15 @@ Kind kind_of(const char* site) {
     if (!strcmp(site, "redomap2.bf16")) return K_MM_BF16;
     if (!strcmp(site, "tridag")) return K_TRIDAG;
     if (!strcmp(site, "lvc")) return K_LVC;
+    if (!strcmp(site, "colred.b4")) return K_COLRED;
+    if (!strcmp(site, "colscan.b4")) return K_COLSCAN;
     return K_BAD;
 }
 
-int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN) ? 2 : k == K_LVC ? 4 : 3; }
+int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN) ? 2 : k == K_LVC ? 4 : 3; }
 
 size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
+int64_t ceil_div_i64(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 size_t ws_bytes_of(Kind k, const int64_t* s) {
     switch (k) {
@@ -114,6 +117,8 @@ size_t ws_bytes_of(Kind k, const int64_t* s) {
     case K_MM_BF16: return ifl_workspace_bytes("redomap2", s[0], s[1], s[2], IFL_BF16, -1);
     case K_TRIDAG: return ifl_workspace_bytes("tridag", s[0], s[1], s[2], IFL_F32, -1);
     case K_LVC: return ifl_workspace_bytes("lvc", s[2], s[3], 0, IFL_F32, -1);
+    case K_COLRED: return ifl_workspace_bytes("colred", s[0], s[1], 0, IFL_F32, -1);
+    case K_COLSCAN: return ifl_workspace_bytes("colscan", s[0], s[1], 0, IFL_F32, -1);
     default: return 0;
     }
 }
@@ -139,6 +144,14 @@ size_t shape_bytes(Kind k, const int64_t* s) {
         const int64_t S = s[0], L = s[1], R = s[2];
         return 3 * align256(R * L * 4) + 2 * align256(S * L * 4) +
                align256(ifl_workspace_bytes("tridag", S, L, R, IFL_F32, -1));
+    }
+    case K_COLRED: {
+        const int64_t n = s[0], m = s[1];
+        return align256(n * m * 4) + align256(m * 4) + align256(ws_bytes_of(k, s));
+    }
+    case K_COLSCAN: {
+        const int64_t n = s[0], m = s[1];
+        return 2 * align256(n * m * 4) + align256(ws_bytes_of(k, s));
     }
     case K_LVC: {  // (numS, numT, numX, numY): xsss, ysss, 6 coefficient arrays, ws
         const int64_t E = s[0] * s[2] * s[3], RL = s[2] * s[3];
@@ -188,6 +201,16 @@ int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_
         return ifl_tridag((float*)a, (float*)b, (float*)c, (float*)y, (float*)x, S, L, R, version, ws,
                           ifl_workspace_bytes("tridag", S, L, R, IFL_F32, -1), st, nullptr);
     }
+    case K_COLRED:
+    case K_COLSCAN: {
+        const int64_t n = s[0], m = s[1];
+        const bool scan = k == K_COLSCAN;
+        char* in = scratch;
+        char* out = in + align256(n * m * 4);
+        char* ws = out + align256((scan ? n * m : m) * 4);
+        return (scan ? ifl_colscan : ifl_colred)(in, out, n, m, IFL_F32, IFL_SUM, IFL_F_ID, nullptr, version, ws,
+                                                 ws_bytes_of(k, s), st, nullptr);
+    }
     case K_LVC: {
         // table slot 0 (TOP) = the outermost version V_OUTER, slot 2 (FLAT) =
         // its else-branch (per-step, per-site G3); slot 1 is unavailable
@@ -216,6 +239,18 @@ size_t max_shape_bytes(Kind k, const int64_t* shapes, int nshapes) {
     size_t mx = 0;
     for (int i = 0; i < nshapes; ++i) mx = std::max(mx, shape_bytes(k, shapes + i * arity(k)));
     return align256(mx);
+}
+
+// Column sites: a forced TOP / MIDDLE on a narrow array runs a handful of
+// threads down millions of rows (seconds per run).  Such a version cannot win
+// (do not spend the budget on settings that cannot), so it is not run:
+// TOP needs >= 4096 column threads, MIDDLE >= 64 column-tile CTAs.
+bool hopeless(Kind k, const int64_t* s, int v) {
+    if (k != K_COLRED && k != K_COLSCAN) return false;
+    const int64_t m = s[1];
+    if (v == IFL_V_TOP) return (m % 4 == 0 ? m / 4 : m) < 4096;
+    if (v == IFL_V_MIDDLE) return ceil_div_i64(m, (m >= 128 && m % 4 == 0) ? 128 : 32) < 64;
+    return false;
 }
 
 }  // namespace
@@ -259,6 +294,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         double best_ms = std::numeric_limits<double>::infinity();
         for (int vv = 0; vv < 3; ++vv) {
             const int v = 2 - vv;
+            if (hopeless(k, s, v)) continue;  // stays +inf: unavailable to the search
             cudaMemsetAsync(flush, 0, kFlushBytes, st);
             cudaEventRecord(e0, st);
             int r = run_forced(k, s, v, (char*)scratch, st);  // warm-up; also feasibility (ENOTFIT)

@@ -269,3 +269,14 @@ def test_lvc_validation_and_guard(L):
         assert (c.par_top, c.t_top) == (128, 100)
     finally:
         ifl.reset_thresholds()
+
+
+def test_col_selector_g4(L):
+    ifl.set_thresholds("colred.b4", 4096, 1024)
+    try:
+        assert ifl.select("colred.b4", 10, 4096).version == "top"      # Par_top = m
+        c = ifl.select("colred.b4", 100, 200)
+        assert c.version == "middle" and c.par_mid == 200 * 8           # m * min(n, 8)
+        assert ifl.select("colred.b4", 100000, 100).version == "flat"
+    finally:
+        ifl.reset_thresholds()
