@@ -128,3 +128,20 @@ def lvc_problem(seed: int, numS: int, numX: int, numY: int, device="cpu"):
     xsss = generate("F32_SIGNED", seed * 16 + 4, numS * numX * numY, device).view(numS, numX, numY)
     ysss = generate("F32_SIGNED", seed * 16 + 5, numS * numY * numX, device).view(numS, numY, numX)
     return (ax, bx, cx), (ay, by, cy), xsss, ysss
+
+
+def irregular_offsets(seed: int, n: int, mean: float, alpha: float = 1.5, max_len: int | None = None):
+    """Segment descriptor for irregular nested parallelism (DESIGN.md
+    recipe): n segment lengths from a Pareto-like heavy tail with the given
+    mean (power-law degree distributions of sparse / graph workloads):
+    len_i = floor(mean * (alpha - 1) / alpha * u_i^(-1/alpha)), u_i ~ U(0, 1],
+    capped at max_len; about (1 - (alpha-1)/alpha * mean)-fraction of short
+    and some empty segments at small means.  Returns int64 offsets [n + 1]."""
+    import numpy as np
+    u = 1.0 - generate("F32_UNIT", seed, n).double().numpy()  # (0, 1]
+    lens = np.floor(mean * (alpha - 1) / alpha * u ** (-1.0 / alpha)).astype(np.int64)
+    if max_len is not None:
+        lens = np.minimum(lens, max_len)
+    off = np.zeros(n + 1, np.int64)
+    np.cumsum(lens, out=off[1:])
+    return off

@@ -59,6 +59,10 @@ def lib() -> ctypes.CDLL:
             "oracle_redomap2": [_vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int],
             "oracle_tridag": [_vp, _vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _vp],
             "oracle_lvc": [_vp] * 10 + [_c_i64] * 4 + [_vp],
+            "oracle_segred_irr_i32": [_vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_int32],
+            "oracle_segscan_irr_i32": [_vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_int32],
+            "oracle_segred_irr_f32": [_vp, _vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_double],
+            "oracle_segscan_irr_f32": [_vp, _vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_double],
         }.items():
             fn = getattr(L, name)
             fn.argtypes = argt
@@ -235,3 +239,26 @@ def lvc(ax, bx, cx, ay, by, cy, xsss, ysss, numT: int):
     _check(lib().oracle_lvc(_ptr(ax), _ptr(bx), _ptr(cx), _ptr(ay), _ptr(by), _ptr(cy), _ptr(xsss), _ptr(ysss),
                             _ptr(xo), _ptr(yo), numS, int(numT), numX, numY, _ptr(work)))
     return xo, yo
+
+
+def seg_irr(x: np.ndarray, offsets: np.ndarray, scan: bool, op: str = "sum", f: str = "id", d=None,
+            with_absum=False):
+    """Irregular segments (P:532 future work): segment i is
+    x[offsets[i]:offsets[i+1]]; reduce (out [n]) or inclusive scan (out like x)
+    of every segment as P:79 defines them; an empty segment reduces to d."""
+    x = np.ascontiguousarray(x).reshape(-1)
+    off = np.ascontiguousarray(offsets, dtype=np.int64)
+    n = off.shape[0] - 1
+    assert off[-1] == x.shape[0]
+    if x.dtype == np.int32:
+        d = canonical_ne(op, "i32") if d is None else int(d)
+        out = np.empty(x.shape[0] if scan else n, np.int32)
+        fn = lib().oracle_segscan_irr_i32 if scan else lib().oracle_segred_irr_i32
+        _check(fn(_ptr(x), _ptr(out), _ptr(off), n, OPS[op], MAPS[f], _i32(d)))
+        return (out, None) if with_absum else out
+    d = canonical_ne(op, "f32") if d is None else float(np.float32(d))
+    out = np.empty(x.shape[0] if scan else n, np.float64)
+    ab = np.empty_like(out)
+    fn = lib().oracle_segscan_irr_f32 if scan else lib().oracle_segred_irr_f32
+    _check(fn(_ptr(x), _ptr(out), _ptr(ab), _ptr(off), n, OPS[op], MAPS[f], d))
+    return (out, ab) if with_absum else out

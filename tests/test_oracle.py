@@ -483,3 +483,57 @@ def test_colscan_f32_numpy_and_exact(orc):
     np.testing.assert_allclose(out, np.abs(Mu).astype(np.float64).cumsum(0), rtol=1e-13)
     np.testing.assert_allclose(ab, out, rtol=1e-13)  # f = abs: the bound scale equals the result
     np.testing.assert_array_equal(orc.colscan(Mu, "min")[-1], orc.colred(Mu, "min"))
+
+
+# ------------------------------------------- irregular segments (NEXT-4)
+
+
+def _wrap(v):
+    return ((np.asarray(v, dtype=np.int64) + 2**31) % 2**32 - 2**31).astype(np.int32)
+
+
+def test_irr_regular_descriptor_equals_rows(orc):
+    # offsets i*m describe the regular [n][m] nest: same results as the row oracle
+    for op in INT_OPS:
+        x = gen.matrix("I32_FULL", 41, 9, 13).numpy()
+        off = np.arange(10, dtype=np.int64) * 13
+        np.testing.assert_array_equal(orc.seg_irr(x, off, False, op, "sq"), orc.segred(x, op, "sq"))
+        np.testing.assert_array_equal(orc.seg_irr(x, off, True, op, "abs"), orc.segscan(x, op, "abs").reshape(-1))
+
+
+def test_irr_closed_forms_and_empty(orc):
+    lens = np.array([0, 3, 0, 0, 1, 7, 0], np.int64)
+    off = np.r_[0, np.cumsum(lens)]
+    ones = np.ones(off[-1], np.int32)
+    np.testing.assert_array_equal(orc.seg_irr(ones, off, False), lens)        # sum of ones = length
+    pos = np.concatenate([np.arange(1, L + 1) for L in lens])
+    np.testing.assert_array_equal(orc.seg_irr(ones, off, True), pos)          # scan of ones = j + 1
+    for op in INT_OPS:                                                        # empty reduce = d
+        out = orc.seg_irr(ones, off, False, op, d=-5)
+        assert (out[lens == 0] == -5).all()
+    with pytest.raises(ValueError):
+        orc.seg_irr(ones, np.array([0, 5, 3, 11], np.int64), False)           # decreasing descriptor
+
+
+def test_irr_numpy_cumsum_and_brute_force(orc):
+    rng = np.random.default_rng(3)
+    for trial in range(5):
+        lens = rng.integers(0, 9, size=rng.integers(1, 40)).astype(np.int64)
+        off = np.r_[0, np.cumsum(lens)]
+        x = gen.generate("I32_FULL", 50 + trial, int(off[-1])).numpy()
+        cs = np.r_[0, np.cumsum(x.astype(np.int64))]
+        np.testing.assert_array_equal(orc.seg_irr(x, off, False), _wrap(cs[off[1:]] - cs[off[:-1]]))
+        seg_of = np.repeat(np.arange(len(lens)), lens)
+        np.testing.assert_array_equal(orc.seg_irr(x, off, True), _wrap(cs[1:] - cs[off[:-1]][seg_of]))
+        for op, fn in (("max", max), ("min", min), ("xor", lambda a, b: a ^ b)):
+            want = []
+            for i in range(len(lens)):  # brute force in Python ints
+                acc = orc.canonical_ne(op, "i32")
+                for k in range(off[i], off[i + 1]):
+                    acc = fn(acc, int(x[k]))
+                want.append(acc)
+            np.testing.assert_array_equal(orc.seg_irr(x, off, False, op), np.array(want, np.int32))
+        xf = gen.generate("F32_SIGNED", 60 + trial, int(off[-1])).numpy()
+        got, ab = orc.seg_irr(xf, off, False, with_absum=True)
+        want = np.array([math.fsum(xf[off[i]:off[i + 1]].astype(np.float64)) for i in range(len(lens))])
+        assert (np.abs(got - want) <= 1e-12 * (ab + 1)).all()
