@@ -327,6 +327,91 @@ def suite_col():
     return line
 
 
+# ----------------------------------------------------------------------- irr
+
+
+def _irr_case(seed, total_log2, mean):
+    n = max(1, (1 << total_log2) // int(mean))
+    off = gen.irregular_offsets(seed, n, float(mean))
+    return off
+
+
+def suite_irr():
+    """NEXT-4: irregular segments -- segred + segscan
+    over Pareto(1.5)-distributed segment lengths (the heavy-tailed degree
+    distributions of graph / sparse workloads), ~2^26 f32 elements, mean
+    length 2^0..2^16.  The inspector (ifl_irr_inspect, timed separately)
+    supplies max_len for the guard's imbalance measure; thresholds come from
+    the exact search (ifl_tune_search) over forced-version timings of the same
+    sweep at 2^24 and 2^27 elements with other seeds."""
+    hbm, _, src = peaks()
+    ifl.reset_thresholds()
+    means = [1 << k for k in range(0, 17, 2)]
+
+    def run_case(off, seed, versions, R=4):
+        offd = torch.from_numpy(off).cuda()
+        total = int(off[-1])
+        x = gen.generate("F32_UNIT", seed, total, "cuda")
+        ob = torch.empty(max(total, off.size - 1), device="cuda")
+        t0 = time.perf_counter()
+        mx = ifl.irr_inspect(offd, total)
+        t_insp = (time.perf_counter() - t0) * 1e3
+        ws = ifl.workspace(ifl.workspace_bytes("segscan_irr", off.size - 1, total), "cuda", "irrsuite")
+        r = {}
+        for kind in ("segred", "segscan"):
+            fn = ifl.segscan_irr if kind == "segscan" else ifl.segred_irr
+            o = ob[:total] if kind == "segscan" else ob[: off.size - 1]
+            for v in versions:
+                r[(kind, v)] = gtime(lambda: fn(x, offd, out=o, ws=ws, version=v, max_len=mx), R=R) * 1e3
+            r[(kind, "choice")] = fn(x, offd, out=o, ws=ws, max_len=mx, return_choice=True)[1]
+        return r, mx, total, t_insp
+
+    # ---- tune (other seeds, bracketing sizes)
+    thr = {}
+    tabs = {"segred": ([], [], []), "segscan": ([], [], [])}
+    for lg in (24, 27):
+        for k, mean in enumerate(means):
+            off = _irr_case(200 + k + lg, lg, mean)
+            r, mx, total, _ = run_case(off, 300 + k, ("top", "middle", "flat"), R=2)
+            for kind in ("segred", "segscan"):
+                c = ifl.select(kind + ".irr", off.size - 1, total, mx)
+                tabs[kind][0].append(c.par_top)
+                tabs[kind][1].append(c.par_mid)
+                tabs[kind][2].append([r[(kind, "top")], r[(kind, "middle")], r[(kind, "flat")]])
+    for kind in ("segred", "segscan"):
+        a, b, npaths = ifl.tune_search(tabs[kind][0], tabs[kind][1], tabs[kind][2], cost=1)
+        ifl.set_thresholds(kind + ".irr", a, b)
+        thr[kind + ".irr"] = {"t_top": a, "t_intra": b, "paths": npaths}
+    # ---- test sweep (2^26)
+    rows = []
+    for k, mean in enumerate(means):
+        off = _irr_case(100 + k, 26, mean)
+        r, mx, total, t_insp = run_case(off, 2, ("top", "middle", "flat", "auto"))
+        n = off.size - 1
+        for kind in ("segred", "segscan"):
+            byt = (8 * total + 8 * (n + 1)) if kind == "segscan" else (4 * total + 4 * n + 8 * (n + 1))
+            row = {"op": kind, "mean": mean, "n": n, "total": total, "max_len": mx, "inspect_ms": round(t_insp, 3),
+                   "chosen": r[(kind, "choice")].version}
+            for v in ("top", "middle", "flat", "auto"):
+                row[v] = round(r[(kind, v)], 2)
+            best = min(row["top"], row["middle"], row["flat"])
+            row["best_over_auto"] = round(best / row["auto"], 4)
+            row["GBps"] = round(byt / (row["auto"] * 1e-6) / 1e9, 1)
+            row["bytes"] = byt
+            rows.append(row)
+    agg = sum(r["bytes"] for r in rows) / (sum(r["auto"] for r in rows) * 1e-6) / 1e9
+    line = base_line("irregular segred/segscan GB/s over a Pareto segment-length sweep (P:532)", round(agg, 1),
+                     "GB/s", {"workload": "SURVEY 8(f) NEXT-4: f32 sum, ~2^26 elements, Pareto(1.5) lengths, mean "
+                                          "2^0..2^16, AUTO with the inspector's max_len and tuned thresholds",
+                              "thresholds": thr})
+    line["min_shape_best_over_auto"] = min(r["best_over_auto"] for r in rows)
+    line["roofline"] = {"bound": "hbm", "kernel": "irregular sweep (AUTO, data + offsets bytes)",
+                        "achieved": round(agg, 1), "peak": hbm, "unit": "GB/s", "frac": round(agg / hbm, 4),
+                        "traffic": None, "peak_source": src}
+    line["shapes"] = rows
+    return line
+
+
 # ---------------------------------------------------------------------- dist
 
 
@@ -370,4 +455,4 @@ def suite_dist():
 
 
 SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist,
-          "lvc": suite_lvc, "col": suite_col}
+          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr}

@@ -30,7 +30,8 @@ OPS = {"sum": 0, "prod": 1, "min": 2, "max": 3, "and": 4, "or": 5, "xor": 6}
 MAPS = {"id": 0, "sq": 1, "abs": 2}
 VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3}
 VERSION_NAMES = {-1: "auto", 0: "top", 1: "middle", 2: "flat", 3: "outer"}
-SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4")
+SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4",
+         "segred.irr", "segscan.irr")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -63,6 +64,9 @@ _SIGS = {
     "ifl_segscan_seeded": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_colred": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_colscan": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_segred_irr": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_segscan_irr": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_irr_inspect": ([_vp, _i64, _i64, _vp, _vp, _vp], _int),
     "ifl_redomap2": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_tridag": ([_vp, _vp, _vp, _vp, _vp, _i64, _i64, _i64, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_lvc": ([_vp] * 8 + [_i64] * 4 + [_int, _vp, _sz, _vp, _vp], _int),
@@ -299,6 +303,55 @@ def colred(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stre
 def colscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False):
     """out[i,j] = ne (+) f(x[0,j]) (+) ... (+) f(x[i,j]) -- column-wise inclusive scan (G4 with scan)."""
     return _col(True, x, op, f, ne, version, out, ws, stream, return_choice)
+
+
+# -------------------------------------------------------- irregular segments
+
+
+def irr_inspect(offsets: torch.Tensor, total: int, stream=None) -> int:
+    """Inspector: validate the descriptor and return the longest
+    segment (synchronises the stream)."""
+    ws = workspace(16, offsets.device, "irr_inspect")
+    mx = ctypes.c_int64()
+    _check(lib().ifl_irr_inspect(offsets.data_ptr(), offsets.numel() - 1, int(total), ws.data_ptr(), _stream(stream),
+                                 ctypes.byref(mx)), "ifl_irr_inspect")
+    return mx.value
+
+
+def _irr(scan, x, offsets, op, f, ne, version, max_len, out, ws, stream, return_choice):
+    if x.dim() != 1 or not x.is_contiguous() or not x.is_cuda:
+        raise ValueError("expected a contiguous 1-D CUDA tensor of segment data")
+    if offsets.dtype != torch.int64 or not offsets.is_contiguous() or offsets.device != x.device:
+        raise ValueError("offsets must be a contiguous int64 tensor on x's device")
+    dt = _TORCH_DT.get(x.dtype)
+    if dt not in ("i32", "f32"):
+        raise TypeError(f"unsupported dtype {x.dtype}")
+    n, total = offsets.numel() - 1, x.numel()
+    if out is None:
+        out = torch.empty(total if scan else n, dtype=x.dtype, device=x.device)
+    entry = "segscan_irr" if scan else "segred_irr"
+    wb = lib().ifl_workspace_bytes(_b(entry), n, total, 0, DTYPES[dt], VERSIONS[version])
+    if ws is None and wb:
+        ws = workspace(wb, x.device, "irr")
+    c = ifl_choice()
+    fn = lib().ifl_segscan_irr if scan else lib().ifl_segred_irr
+    rc = fn(x.data_ptr(), out.data_ptr(), offsets.data_ptr(), n, total, int(max_len), DTYPES[dt], OPS[op], MAPS[f],
+            _ne_buf(ne, dt), VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel() * ws.element_size(),
+            _stream(stream), ctypes.byref(c))
+    _check(rc, "ifl_" + entry)
+    return (out, _choice_out(c)) if return_choice else out
+
+
+def segred_irr(x, offsets, op="sum", f="id", ne=None, version="auto", max_len=0, out=None, ws=None, stream=None,
+               return_choice=False):
+    """out[i] = ne (+) f(x[offsets[i]]) (+) ... (+) f(x[offsets[i+1]-1]) (irregular segments)."""
+    return _irr(False, x, offsets, op, f, ne, version, max_len, out, ws, stream, return_choice)
+
+
+def segscan_irr(x, offsets, op="sum", f="id", ne=None, version="auto", max_len=0, out=None, ws=None, stream=None,
+                return_choice=False):
+    """Inclusive scan of every irregular segment."""
+    return _irr(True, x, offsets, op, f, ne, version, max_len, out, ws, stream, return_choice)
 
 
 # ------------------------------------------------------------------ redomap2

@@ -39,7 +39,7 @@ constexpr int64_t kDefaultThreshold = 1 << 15;
 constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE kernel (reading R3)
 
 const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
-                              "colred.b4", "colscan.b4"};
+                              "colred.b4", "colscan.b4", "segred.irr", "segscan.irr"};
 
 struct Table {
     std::mutex mu;
@@ -112,6 +112,16 @@ int select_version(const char* site, int64_t n, int64_t m, int64_t p, bool mid_f
     return v;
 }
 
+// Irregular segments: G3 with the inspector's imbalance measure.
+// Par_top = total / max_len (longest-segment equivalents: what a thread per
+// segment really runs in parallel), or n when max_len is unknown (0);
+// Par_mid = n * min(mean length, 32) (a warp per segment, reading R3).
+void irr_par(int64_t n, int64_t total, int64_t max_len, int64_t* ptop, int64_t* pmid) {
+    *ptop = max_len > 0 ? std::min(n, total / max_len) : n;
+    const int64_t mean = n > 0 ? (total + n - 1) / n : 0;
+    *pmid = sat_mul(n, std::min<int64_t>(mean, 32));
+}
+
 uint32_t canonical_bits(int dt, int op) {
     if (dt == IFL_I32) {
         switch (op) {
@@ -174,6 +184,16 @@ int ifl_select(const char* site, int64_t n, int64_t m, int64_t p, ifl_choice* ch
         ifl_get_thresholds("lvc", &t0, &tu);
         ifl_choice c{(n >= t0 && m <= ifl::kLvcMaxL && p <= ifl::kLvcMaxL) ? IFL_V_OUTER : IFL_AUTO,
                      n, sat_mul(n, sat_mul(m, p)), t0, tu};
+        if (choice) *choice = c;
+        return IFL_OK;
+    }
+    if (strstr(site, ".irr")) {  // (n, total, max_len)
+        int64_t tt, ti;
+        ifl_get_thresholds(site, &tt, &ti);
+        ifl_choice c{IFL_V_FLAT, 0, 0, tt, ti};
+        irr_par(n, m, p, &c.par_top, &c.par_mid);
+        if (c.par_top >= tt) c.version = IFL_V_TOP;
+        else if (c.par_mid >= ti) c.version = IFL_V_MIDDLE;
         if (choice) *choice = c;
         return IFL_OK;
     }
@@ -265,6 +285,7 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
     }
     if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
     if (strcmp(entry, "colred") == 0 || strcmp(entry, "colscan") == 0) return ifl::col_ws_bytes(n, m, version);
+    if (strcmp(entry, "segred_irr") == 0 || strcmp(entry, "segscan_irr") == 0) return ifl::irr_ws_bytes(m, version);
     if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
     if (strcmp(entry, "lvc") == 0)  // (numX, numY): the coefficient scans of both sites
         return ifl::tridag_ws_bytes(n, m, version) + ifl::tridag_ws_bytes(m, n, version);
@@ -345,6 +366,73 @@ static int run_col(bool scan, const void* in, void* out, int64_t n, int64_t m, i
     }
     ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream, nullptr};
     return cuda_status(ifl::launch_col(a, scan, c.version), what);
+}
+
+static int run_irr(bool scan, const void* in, void* out, const int64_t* off, int64_t n, int64_t total,
+                   int64_t max_len, int dt, int op, int f, const void* ne, int version, void* ws, size_t ws_bytes,
+                   void* stream, ifl_choice* choice) {
+    const char* what = scan ? "ifl_segscan_irr" : "ifl_segred_irr";
+    if (n < 0 || total < 0 || max_len < 0) return fail(IFL_EINVAL, "%s: negative size", what);
+    if (mul_overflows(total, 4)) return fail(IFL_EINVAL, "%s: size overflow", what);
+    int rc = validate_seg(true, in, out, 1, total, dt, op, f, version, what);  // element checks on [total]
+    if (rc && !(total == 0 && rc == IFL_EINVAL)) return rc;
+    if (n > 0 && !off) return fail(IFL_EINVAL, "%s: offsets is NULL", what);
+    if (!scan && n > 0 && !out) return fail(IFL_EINVAL, "%s: out is NULL", what);
+    if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "%s: bad version", what);
+    const size_t ob = (size_t)(scan ? total : n) * 4, ib = (size_t)total * 4;
+    if (scan ? (in != out && overlap(in, ib, out, ob)) : overlap(in, ib, out, ob))
+        return fail(IFL_EINVAL, "%s: in/out overlap", what);
+    uint32_t bits = canonical_bits(dt, op);
+    if (ne) memcpy(&bits, ne, 4);
+    const char* site = scan ? "segscan.irr" : "segred.irr";
+    int64_t tt, ti;
+    ifl_get_thresholds(site, &tt, &ti);
+    ifl_choice c{IFL_V_FLAT, 0, 0, tt, ti};
+    irr_par(n, total, max_len, &c.par_top, &c.par_mid);
+    if (c.par_top >= tt) c.version = IFL_V_TOP;
+    else if (c.par_mid >= ti) c.version = IFL_V_MIDDLE;
+    if (version != IFL_AUTO) c.version = version;
+    if (choice) *choice = c;
+    if (n == 0) return IFL_OK;
+    if (total == 0) return scan ? IFL_OK : cuda_status(ifl::launch_fill(out, n, bits, (cudaStream_t)stream), what);
+    if (c.version == IFL_V_FLAT) {
+        const size_t need = ifl::irr_ws_bytes(total, IFL_V_FLAT);
+        if (!ws || ws_bytes < need)
+            return fail(IFL_EWORKSPACE, "%s: V_FLAT needs %zu workspace bytes, got %zu", what, need, ws_bytes);
+    }
+    ifl::IrrArgs a{in, out, off, n, total, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream};
+    return cuda_status(ifl::launch_irr(a, scan, c.version), what);
+}
+
+int ifl_segred_irr(const void* in, void* out, const int64_t* offsets, int64_t n, int64_t total, int64_t max_len,
+                   int dt, int op, int f, const void* ne, int version, void* ws, size_t ws_bytes, void* stream,
+                   ifl_choice* choice) {
+    return run_irr(false, in, out, offsets, n, total, max_len, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+}
+
+int ifl_segscan_irr(const void* in, void* out, const int64_t* offsets, int64_t n, int64_t total, int64_t max_len,
+                    int dt, int op, int f, const void* ne, int version, void* ws, size_t ws_bytes, void* stream,
+                    ifl_choice* choice) {
+    return run_irr(true, in, out, offsets, n, total, max_len, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+}
+
+int ifl_irr_inspect(const int64_t* offsets, int64_t n, int64_t total, void* ws16, void* stream, int64_t* max_len) {
+    if (n < 0 || total < 0 || (n > 0 && (!offsets || !ws16))) return fail(IFL_EINVAL, "ifl_irr_inspect: bad argument");
+    if (max_len) *max_len = 0;
+    if (n == 0) return total == 0 ? IFL_OK : fail(IFL_EINVAL, "ifl_irr_inspect: no segments but total > 0");
+    cudaStream_t st = (cudaStream_t)stream;
+    cudaError_t e = ifl::launch_irr_inspect(offsets, n, ws16, st);
+    unsigned long long res[2] = {0, 0};
+    int64_t last = 0;
+    if (e == cudaSuccess) e = cudaMemcpyAsync(res, ws16, 16, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&last, offsets + n, 8, cudaMemcpyDeviceToHost, st);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(st);
+    if (e != cudaSuccess) return cuda_status(e, "ifl_irr_inspect");
+    if (res[1] || last != total)
+        return fail(IFL_EINVAL, "ifl_irr_inspect: offsets are not a segment descriptor (off[0] = 0, nondecreasing, "
+                                "off[n] = total = %lld; got off[n] = %lld)", (long long)total, (long long)last);
+    if (max_len) *max_len = (int64_t)res[0];
+    return IFL_OK;
 }
 
 int ifl_colred(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int version,

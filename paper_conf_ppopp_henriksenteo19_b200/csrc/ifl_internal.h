@@ -52,6 +52,23 @@ size_t col_ws_bytes(int64_t n, int64_t m, int version);
 cudaError_t launch_col(const SegArgs& a, bool scan, int version);
 constexpr int64_t kColGroup = 8;  // threads per column in V_MIDDLE (reading R3's group size)
 
+// Irregular segments (irr.cu): segment i = in[off[i] .. off[i+1]-1].
+struct IrrArgs {
+    const void* in;
+    void* out;
+    const int64_t* off;  // device [n + 1]
+    int64_t n, total;
+    int dt, op, f;
+    uint32_t ne_bits;
+    void* ws;
+    size_t ws_bytes;
+    cudaStream_t stream;
+};
+int64_t irr_tiles(int64_t total);
+size_t irr_ws_bytes(int64_t total, int version);
+cudaError_t launch_irr(const IrrArgs& a, bool scan, int version);
+cudaError_t launch_irr_inspect(const int64_t* off, int64_t n, void* res16, cudaStream_t s);
+
 // redomap2 (redomap2.cu) and tridag (tridag.cu)
 struct MmArgs {
     const void* A;

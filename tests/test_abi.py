@@ -280,3 +280,23 @@ def test_col_selector_g4(L):
         assert ifl.select("colred.b4", 100000, 100).version == "flat"
     finally:
         ifl.reset_thresholds()
+
+
+def test_irr_guard_and_validation(L):
+    # the inspector's imbalance measure in G3 -- Par_top = total / max_len
+    ifl.set_thresholds("segscan.irr", 1000, 5000)
+    try:
+        assert ifl.select("segscan.irr", 4000, 64000, 16).version == "top"
+        c = ifl.select("segscan.irr", 4000, 64000, 6400)
+        assert (c.version, c.par_top, c.par_mid) == ("middle", 10, 4000 * 16)
+        assert ifl.select("segscan.irr", 100, 64000, 6400).version == "flat"   # 100 * min(640, 32) < 5000
+        assert ifl.select("segscan.irr", 4000, 64000, 0).par_top == 4000      # max_len unknown: n
+    finally:
+        ifl.reset_thresholds()
+    sig = (256, 512, 1024)
+    assert L.ifl_segred_irr(*sig, -1, 0, 0, 1, 0, 0, None, -1, None, 0, None, None) == ifl.IFL_EINVAL
+    assert L.ifl_segred_irr(256, 512, None, 4, 8, 0, 1, 0, 0, None, -1, None, 0, None, None) == ifl.IFL_EINVAL
+    # forced V_FLAT without workspace
+    assert L.ifl_segred_irr(*sig, 4, 8, 0, 1, 0, 0, None, 2, None, 0, None, None) == ifl.IFL_EWORKSPACE
+    assert ifl.workspace_bytes("segred_irr", 4, 1 << 20, version="flat") > 0
+    assert ifl.workspace_bytes("segred_irr", 4, 1 << 20, version="top") == 0
