@@ -213,3 +213,102 @@ def tridag_dist(a: torch.Tensor, b: torch.Tensor, c: torch.Tensor, y_rows: torch
         return local_tridag(a, b, c, y_rows)
     import paper_conf_ppopp_henriksenteo19_b200 as ifl
     return ifl.tridag(a, b, c, y_rows, **kw)
+
+
+# ------------------------------------------------------------- colred (G4)
+
+
+def plan_colred(n: int, m: int, world: int, rank: int, t_dev: int | None = None) -> Plan:
+    """Device-level guard of the column reduction (the segments are the m
+    columns, Par over devices = m): split the columns when m >= t_dev (outer,
+    no collective), else split the rows (inner: one all_reduce of the m
+    partials)."""
+    t_dev = world if t_dev is None else t_dev
+    if m >= t_dev:
+        lo = (m * rank) // world
+        return Plan("outer", lo, (m * (rank + 1)) // world)
+    per = -(-n // world)
+    lo = min(n, rank * per)
+    return Plan("inner", lo, min(n, lo + per))
+
+
+def _default_local_col(x: torch.Tensor, op: str, f: str, ne):
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.colred(x, op, f, ne=ne)
+
+
+def colred_dist(x_block: torch.Tensor, n: int, m: int, op: str = "sum", f: str = "id", ne=None,
+                plan: Plan | None = None, group=None, gather: bool = False, local_colred=None) -> torch.Tensor:
+    """Distributed column reduction (G4).  ``x_block``: all n rows x
+    columns [plan.lo, plan.hi) (outer; contiguous copy of the column block)
+    or rows [plan.lo, plan.hi) x all m columns (inner).  Returns this rank's
+    columns (outer; all m if ``gather``) or the full [m] result (inner)."""
+    local = local_colred or _default_local_col
+    world = td.get_world_size(group)
+    rank = td.get_rank(group)
+    plan = plan or plan_colred(n, m, world, rank)
+    if plan.mode == "outer":
+        out = local(x_block, op, f, ne)
+        if not gather:
+            return out
+        parts = [None] * world
+        td.all_gather_object(parts, out.cpu(), group=group)
+        return torch.cat(parts).to(out.device)
+    part = local(x_block, op, f, None)  # partials without d
+    if op in _BITWISE and td.get_backend(group) == "nccl":
+        allp = torch.empty(world * m, dtype=part.dtype, device=part.device)
+        td.all_gather_into_tensor(allp, part.contiguous(), group=group)
+        total = local(allp.view(world, m).contiguous(), op, "id", None)
+    else:
+        total = part.clone()
+        td.all_reduce(total, op=_REDUCE[op], group=group)
+    if ne is None:
+        return total
+    return local(total.view(1, m).contiguous(), op, "id", ne)  # d (+) total, once
+
+
+# ------------------------------------------------------- LocVolCalib loop
+
+
+def lvc_dist(xsss_block: torch.Tensor, ysss_block: torch.Tensor, xcoef, ycoef, numT: int, local_lvc=None,
+             **kw):
+    """The LocVolCalib loop split over numS (its outermost map, Fig 6a):
+    every s is an independent unit and the coefficients do not depend on s,
+    so each rank runs its block [numS_r][numX][numY] / [numS_r][numY][numX]
+    with no collective (weak scaling).  In place, like ifl_lvc."""
+    if local_lvc is not None:
+        return local_lvc(xsss_block, ysss_block, xcoef, ycoef, numT)
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.lvc(xsss_block, ysss_block, xcoef, ycoef, numT, **kw)
+
+
+# ------------------------------------------------------ irregular segments
+
+
+def plan_irr(offsets, world: int, rank: int):
+    """Split n irregular segments (host int64 offsets [n+1]) into contiguous
+    segment ranges of about total/G elements each, cut at segment boundaries
+    (independent units, no collective).  Returns (seg_lo, seg_hi)."""
+    import numpy as np
+    off = np.asarray(offsets, dtype=np.int64)
+    n, total = off.size - 1, int(off[-1])
+    cuts = [0] + [int(np.searchsorted(off, (total * r) // world, side="left")) for r in range(1, world)] + [n]
+    cuts = [min(max(c, 0), n) for c in cuts]
+    for r in range(1, len(cuts)):  # monotone
+        cuts[r] = max(cuts[r], cuts[r - 1])
+    return cuts[rank], cuts[rank + 1]
+
+
+def segred_irr_dist(x: torch.Tensor, offsets, seg_lo: int, seg_hi: int, op: str = "sum", f: str = "id", ne=None,
+                    local=None, **kw) -> torch.Tensor:
+    """This rank's segments [seg_lo, seg_hi): the element range
+    x[off[seg_lo]:off[seg_hi]] with rebased offsets; no collective."""
+    import numpy as np
+    off = np.asarray(offsets, dtype=np.int64)
+    e0, e1 = int(off[seg_lo]), int(off[seg_hi])
+    loc_off = torch.from_numpy(off[seg_lo:seg_hi + 1] - e0)
+    xb = x[e0:e1]
+    if local is not None:
+        return local(xb, loc_off, op, f, ne)
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    return ifl.segred_irr(xb.contiguous(), loc_off.to(x.device), op, f, ne=ne, **kw)

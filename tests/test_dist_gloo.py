@@ -225,3 +225,76 @@ def test_plans_cover_exactly():
             else:
                 cover = [j for p in plans for j in range(p.lo, p.hi)]
                 assert cover == list(range(m))
+
+
+# ------------------------------------------- colred / lvc / irregular splits
+
+
+def _worker_ext(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    td.init_process_group("gloo", rank=rank, world_size=world)
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    import oracle
+    res = []
+    try:
+        def loc_col(x, op, f, ne):
+            r = oracle.colred(x.numpy(), op, f, ne)
+            return torch.from_numpy(np.ascontiguousarray(r.astype(x.numpy().dtype)))
+        for (n, m) in [(7, 1), (5, 13), (64, 3), (2, 40)]:
+            for op in ("sum", "min", "xor"):
+                X = gen.matrix("I32_FULL", 9, n, m)
+                want = oracle.colred(X.numpy(), op, "id", 5)
+                for t_dev in (1, 10**9):  # force column split / row split
+                    plan = dist.plan_colred(n, m, world, rank, t_dev)
+                    blk = X[:, plan.lo:plan.hi].contiguous() if plan.mode == "outer" else X[plan.lo:plan.hi]
+                    out = dist.colred_dist(blk, n, m, op, "id", 5, plan=plan, gather=True, local_colred=loc_col)
+                    res.append(("colred", plan.mode, n, m, op, bool(np.array_equal(out.numpy(), want))))
+        # lvc: numS split, each rank's block equals the oracle's rows of the full run
+        xc, yc, xs, ys = gen.lvc_problem(3, 5, 4, 6)
+        wx, wy = oracle.lvc(*(t.numpy() for t in xc + yc), xs.numpy(), ys.numpy(), 3)
+        lo, hi = dist.rows_of(5, world, rank)
+
+        def loc_lvc(xb, yb, xcf, ycf, T):
+            gx, gy = oracle.lvc(*(t.numpy() for t in xcf + ycf), xb.numpy(), yb.numpy(), T)
+            xb.copy_(torch.from_numpy(gx.astype(np.float32)))
+            yb.copy_(torch.from_numpy(gy.astype(np.float32)))
+        xb, yb = xs[lo:hi].clone(), ys[lo:hi].clone()
+        dist.lvc_dist(xb, yb, xc, yc, 3, local_lvc=loc_lvc)
+        res.append(("lvc", lo, hi, bool(np.allclose(xb.numpy(), wx[lo:hi], atol=1e-6) and
+                                         np.allclose(yb.numpy(), wy[lo:hi], atol=1e-6))))
+        # irregular: element-balanced segment ranges; concatenated per-rank results = the whole
+        off = gen.irregular_offsets(4, 300, 10.0)
+        x = gen.generate("I32_FULL", 8, int(off[-1]))
+        want = oracle.seg_irr(x.numpy(), off, False, "sum")
+        s0, s1 = dist.plan_irr(off, world, rank)
+
+        def loc_irr(xb, o, op, f, ne):
+            return torch.from_numpy(oracle.seg_irr(xb.numpy(), o.numpy(), False, op, f, ne))
+        got = dist.segred_irr_dist(x, off, s0, s1, local=loc_irr)
+        parts = [None] * world
+        td.all_gather_object(parts, (s0, s1, got))
+        whole = torch.cat([p[2] for p in sorted(parts, key=lambda p: p[0])]).numpy()
+        cover = sorted((p[0], p[1]) for p in parts)
+        res.append(("irr", s0, s1, bool(np.array_equal(whole, want) and cover[0][0] == 0 and cover[-1][1] == 300)))
+        q.put((rank, res))
+    except Exception as e:
+        q.put((rank, [("error", repr(e), False)]))
+    finally:
+        td.destroy_process_group()
+
+
+def test_colred_lvc_irr_dist_world2():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_ext, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, res in out:
+        bad = [r for r in res if not r[-1]]
+        assert not bad, (rank, bad[:5])
+        assert len(res) > 20

@@ -36,6 +36,25 @@ elif a.op == "tridag":
 
     def fn(_x, version):
         return ifl.tridag(ta, tb, tc, ty, out=tx, ws=ws, version=version)
+elif a.op == "lvc":  # --n numS --m numX --p numY, numT = 64
+    xc, yc, xs, ys = gen.lvc_problem(17, a.n, a.m, a.p, "cuda")
+    x = None
+
+    def fn(_x, version):
+        return ifl.lvc(xs, ys, xc, yc, 64, version=version)
+elif a.op in ("colred", "colscan"):
+    x = gen.generate("F32_UNIT", 2, a.n * a.m, device="cuda").view(a.n, a.m)
+    fn = ifl.colred if a.op == "colred" else ifl.colscan
+elif a.op in ("segred_irr", "segscan_irr"):  # --m = mean segment length, ~2^26 elements
+    off = gen.irregular_offsets(5, max(1, (1 << 26) // a.m), float(a.m))
+    offd = torch.from_numpy(off).cuda()
+    xi = gen.generate("F32_UNIT", 2, int(off[-1]), device="cuda")
+    mx = ifl.irr_inspect(offd, int(off[-1]))
+    x = None
+    g = ifl.segred_irr if a.op == "segred_irr" else ifl.segscan_irr
+
+    def fn(_x, version):
+        return g(xi, offd, version=version, max_len=mx)
 else:
     x = gen.generate("F32_UNIT", 2, a.n * a.m, device="cuda").view(a.n, a.m)
     fn = ifl.segred if a.op == "segred" else ifl.segscan
