@@ -376,6 +376,75 @@ __global__ void __launch_bounds__(512) flat_red_fix_long(T* out, int64_t n, int6
     }
 }
 
+// Long rows (m >= kSplitMinM): the flattened reduction as uniform chunks.
+// Row i is cut into P equal pieces (P*n ~ 2 CTAs per SM); a 512-thread CTA
+// reduces one piece with 4 independent 128-bit loads per thread in flight
+// (no ring, no staging: every element is read once, straight into
+// registers), leaving one partial per piece; a second pass combines the P
+// partials of each row and applies d.  Same two-pass structure as the tiled
+// engine, without its per-tile segment bookkeeping.
+constexpr int64_t kSplitMinM = 1 << 16;
+constexpr int kSplitThreads = 512;
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(kSplitThreads) flat_red_split_kernel(const T* __restrict__ in, int64_t m, int P,
+                                                                       T* __restrict__ part) {
+    using V = typename Vec4<T>::type;
+    __shared__ T red[kSplitThreads / 32];
+    const int64_t row = blockIdx.x / P;
+    const int piece = blockIdx.x % P;
+    const int64_t len = ceil_div(ceil_div(m, P), 4) * 4;  // piece length, a multiple of 4 elements
+    const int64_t a = std::min(m, (int64_t)piece * len), b = std::min(m, a + len);
+    const T* src = in + row * m;
+    T acc4[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+    // scalar head up to 16-byte alignment, vector body, scalar tail
+    int64_t h = (int64_t)(((16u - ((uint32_t)(uintptr_t)(src + a) & 15u)) & 15u) / sizeof(T));
+    if (h > b - a) h = b - a;
+    for (int64_t k = a + threadIdx.x; k < a + h; k += kSplitThreads)
+        acc4[0] = combine<OP>(acc4[0], apply_map<F>(__ldg(src + k)));
+    const T* body = src + a + h;
+    const int64_t nv = (b - a - h) >> 2;
+    int64_t v = threadIdx.x;
+    for (; v + 3 * kSplitThreads < nv; v += 4 * kSplitThreads) {
+        V q[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) q[u] = ldg_stream4(body + 4 * (v + u * kSplitThreads));
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            T e[4];
+            unpack4<T>(q[u], e);
+#pragma unroll
+            for (int c = 0; c < 4; ++c) acc4[c] = combine<OP>(acc4[c], apply_map<F>(e[c]));
+        }
+    }
+    for (; v < nv; v += kSplitThreads) {
+        T e[4];
+        unpack4<T>(ldg_stream4(body + 4 * v), e);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) acc4[c] = combine<OP>(acc4[c], apply_map<F>(e[c]));
+    }
+    for (int64_t k = a + h + 4 * nv + threadIdx.x; k < b; k += kSplitThreads)
+        acc4[1] = combine<OP>(acc4[1], apply_map<F>(__ldg(src + k)));
+    T acc = warp_reduce<OP>(combine<OP>(combine<OP>(acc4[0], acc4[1]), combine<OP>(acc4[2], acc4[3])));
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = acc;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        T r = threadIdx.x < kSplitThreads / 32 ? red[threadIdx.x] : identity<OP, T>();
+        r = warp_reduce<OP>(r);
+        if (threadIdx.x == 0) part[blockIdx.x] = r;
+    }
+}
+
+template <typename T, int OP>
+__global__ void __launch_bounds__(256) flat_red_split_fix(const T* __restrict__ part, T* __restrict__ out, int64_t n,
+                                                          int P, T d) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        T r = d;
+        for (int p = 0; p < P; ++p) r = combine<OP>(r, part[i * P + p]);
+        out[i] = r;
+    }
+}
+
 // ------------------------------------------------------------------ segscan
 
 // Thread-local segmented inclusive scan of the thread's items (in registers).
@@ -741,6 +810,19 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         }
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
         T* tail = head + tiles;
+        if (a.m >= kSplitMinM) {
+            // P pieces per row: ~4 resident 512-thread CTAs per SM over the grid, and
+            // n*P partials fit the head array (P*n <= tiles since pieces >= 8192 > kFlatTile)
+            const int P = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)sm_count() * 4, a.n),
+                                                                      a.m / 8192));
+            flat_red_split_kernel<T, OP, F><<<(unsigned)(a.n * P), kSplitThreads, 0, a.stream>>>(
+                (const T*)a.in, a.m, P, head);
+            cudaError_t e = cudaGetLastError();
+            if (e != cudaSuccess) return e;
+            const int g2 = (int)std::min<int64_t>(ceil_div(a.n, 256), (int64_t)sm_count() * 4);
+            flat_red_split_fix<T, OP><<<g2, 256, 0, a.stream>>>(head, (T*)a.out, a.n, P, d);
+            return cudaGetLastError();
+        }
         auto k = flat_red_kernel<T, OP, F>;
         const size_t smem_r = (size_t)kRedSlots * FT * sizeof(T);
         const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem_r, FB + 32));

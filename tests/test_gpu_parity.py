@@ -219,3 +219,13 @@ def test_small_m_kernels(ifl, orc, version, scan):
                     x, xd = gen_for(op, dt, 5, n, m)
                     got = fn(xd, op, "sq" if op == "sum" else "id", version=version)
                     assert_parity(orc, x, got, scan, op, "sq" if op == "sum" else "id", None, dt)
+
+
+@pytest.mark.parametrize("dt", ["i32", "f32"])
+def test_flat_segred_long_rows_split(ifl, orc, dt):
+    # V_FLAT segred on rows >= 2^16 elements: uniform row pieces + per-row combine
+    for (n, m, mis) in [(1, (1 << 20) + 5, True), (3, (1 << 16) + 13, False), (7, 1 << 17, True), (130, 1 << 16, False)]:
+        for op in (["sum", "min", "xor", "prod"] if dt == "i32" else ["sum", "max"]):
+            x, xd = gen_for(op, dt, 17, n, m, misalign=mis)
+            got = ifl.segred(xd, op, "sq" if op != "prod" else "id", ne=(2 if dt == "i32" else 0.5), version="flat")
+            assert_parity(orc, x, got, False, op, "sq" if op != "prod" else "id", 2 if dt == "i32" else 0.5, dt)
