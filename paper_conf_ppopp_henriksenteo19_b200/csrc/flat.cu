@@ -376,39 +376,33 @@ __global__ void __launch_bounds__(512) flat_red_fix_long(T* out, int64_t n, int6
     }
 }
 
-// Long rows (m >= kSplitMinM): the flattened reduction as uniform chunks.
+// Long rows (m >= kSplitMinM = 8192): the flattened reduction as uniform chunks.
 // Row i is cut into P equal pieces (P*n ~ 2 CTAs per SM); a 512-thread CTA
 // reduces one piece with 4 independent 128-bit loads per thread in flight
 // (no ring, no staging: every element is read once, straight into
 // registers), leaving one partial per piece; a second pass combines the P
 // partials of each row and applies d.  Same two-pass structure as the tiled
 // engine, without its per-tile segment bookkeeping.
-constexpr int64_t kSplitMinM = 1 << 16;
+constexpr int64_t kSplitMinM = 1 << 13;
 constexpr int kSplitThreads = 512;
 
-template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kSplitThreads) flat_red_split_kernel(const T* __restrict__ in, int64_t m, int P,
-                                                                       T* __restrict__ part) {
+// CTA-wide reduction of f over src[a, b) (NT threads, 4 independent 128-bit
+// loads per thread in flight); the total is valid in thread 0.
+template <typename T, int OP, int F, int NT>
+__device__ __forceinline__ T cta_piece_reduce(const T* __restrict__ src, int64_t a, int64_t b, T* red) {
     using V = typename Vec4<T>::type;
-    __shared__ T red[kSplitThreads / 32];
-    const int64_t row = blockIdx.x / P;
-    const int piece = blockIdx.x % P;
-    const int64_t len = ceil_div(ceil_div(m, P), 4) * 4;  // piece length, a multiple of 4 elements
-    const int64_t a = std::min(m, (int64_t)piece * len), b = std::min(m, a + len);
-    const T* src = in + row * m;
     T acc4[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
     // scalar head up to 16-byte alignment, vector body, scalar tail
     int64_t h = (int64_t)(((16u - ((uint32_t)(uintptr_t)(src + a) & 15u)) & 15u) / sizeof(T));
     if (h > b - a) h = b - a;
-    for (int64_t k = a + threadIdx.x; k < a + h; k += kSplitThreads)
-        acc4[0] = combine<OP>(acc4[0], apply_map<F>(__ldg(src + k)));
+    for (int64_t k = a + threadIdx.x; k < a + h; k += NT) acc4[0] = combine<OP>(acc4[0], apply_map<F>(__ldg(src + k)));
     const T* body = src + a + h;
     const int64_t nv = (b - a - h) >> 2;
     int64_t v = threadIdx.x;
-    for (; v + 3 * kSplitThreads < nv; v += 4 * kSplitThreads) {
+    for (; v + 3 * NT < nv; v += 4 * NT) {
         V q[4];
 #pragma unroll
-        for (int u = 0; u < 4; ++u) q[u] = ldg_stream4(body + 4 * (v + u * kSplitThreads));
+        for (int u = 0; u < 4; ++u) q[u] = ldg_stream4(body + 4 * (v + u * NT));
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             T e[4];
@@ -417,22 +411,123 @@ __global__ void __launch_bounds__(kSplitThreads) flat_red_split_kernel(const T* 
             for (int c = 0; c < 4; ++c) acc4[c] = combine<OP>(acc4[c], apply_map<F>(e[c]));
         }
     }
-    for (; v < nv; v += kSplitThreads) {
+    for (; v < nv; v += NT) {
         T e[4];
         unpack4<T>(ldg_stream4(body + 4 * v), e);
 #pragma unroll
         for (int c = 0; c < 4; ++c) acc4[c] = combine<OP>(acc4[c], apply_map<F>(e[c]));
     }
-    for (int64_t k = a + h + 4 * nv + threadIdx.x; k < b; k += kSplitThreads)
-        acc4[1] = combine<OP>(acc4[1], apply_map<F>(__ldg(src + k)));
+    for (int64_t k = a + h + 4 * nv + threadIdx.x; k < b; k += NT) acc4[1] = combine<OP>(acc4[1], apply_map<F>(__ldg(src + k)));
     T acc = warp_reduce<OP>(combine<OP>(combine<OP>(acc4[0], acc4[1]), combine<OP>(acc4[2], acc4[3])));
     if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = acc;
     __syncthreads();
+    T r = identity<OP, T>();
     if (threadIdx.x < 32) {
-        T r = threadIdx.x < kSplitThreads / 32 ? red[threadIdx.x] : identity<OP, T>();
+        r = threadIdx.x < NT / 32 ? red[threadIdx.x] : identity<OP, T>();
         r = warp_reduce<OP>(r);
-        if (threadIdx.x == 0) part[blockIdx.x] = r;
     }
+    return r;
+}
+
+// DIRECT (P = 1, V_MIDDLE's one-CTA-per-row use of the same kernel): the
+// CTA's result is final, part[row] = d (+) row total.
+template <typename T, int OP, int F, bool DIRECT = false, int NT = kSplitThreads>
+__global__ void __launch_bounds__(NT) flat_red_split_kernel(const T* __restrict__ in, int64_t m, int P,
+                                                            T* __restrict__ part, T d) {
+    __shared__ T red[NT / 32];
+    const int64_t row = blockIdx.x / P;
+    const int piece = blockIdx.x % P;
+    const int64_t len = ceil_div(ceil_div(m, P), 4) * 4;  // piece length, a multiple of 4 elements
+    const int64_t a = std::min(m, (int64_t)piece * len), b = std::min(m, a + len);
+    const T r = cta_piece_reduce<T, OP, F, NT>(in + row * m, a, b, red);
+    if (threadIdx.x == 0) part[blockIdx.x] = DIRECT ? combine<OP>(d, r) : r;
+}
+
+// V_MIDDLE on the thread-block-cluster level (P:346's hierarchy one level up,
+// SURVEY 8(f) NEXT-4): when there are fewer rows than SMs, one CLUSTER of C
+// CTAs is the group of a row -- each CTA reduces a piece, the C partials are
+// combined through distributed shared memory by the cluster's rank-0 CTA,
+// which writes d (+) row total.  Still one group per segment, no second pass.
+template <typename T, int OP, int F, int NT>
+__global__ void __launch_bounds__(NT) segred_cluster_kernel(const T* __restrict__ in, T* __restrict__ out, int64_t m,
+                                                            T d) {
+    __shared__ T red[NT / 32];
+    __shared__ T cta_total;
+    unsigned rank, csize;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(csize));
+    const int64_t row = blockIdx.x / csize;
+    const int64_t len = ceil_div(ceil_div(m, (int64_t)csize), 4) * 4;
+    const int64_t a = std::min(m, (int64_t)rank * len), b = std::min(m, a + len);
+    const T r = cta_piece_reduce<T, OP, F, NT>(in + row * m, a, b, red);
+    if (threadIdx.x == 0) cta_total = r;
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (rank == 0 && threadIdx.x == 0) {
+        T t = d;
+        const uint32_t local = (uint32_t)__cvta_generic_to_shared(&cta_total);
+        for (unsigned q = 0; q < csize; ++q) {
+            uint32_t remote;
+            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(local), "r"(q));
+            uint32_t bits;
+            asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(bits) : "r"(remote) : "memory");
+            t = combine<OP>(t, from_bits<T>(bits));
+        }
+        out[row] = t;
+    }
+    // keep every CTA's shared memory alive until rank 0 has read it
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+static int sm_count();
+
+// V_MIDDLE for rows of >= 8192 elements: a 512-thread CTA per row (the group
+// size V_MIDDLE already uses there), 4 independent 128-bit loads per thread.
+cudaError_t launch_segred_rows512(const SegArgs& a) {
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        if (a.n > 0x7fffffffLL) return cudaErrorInvalidValue;
+        // few rows (< 2 per SM): a cluster of C CTAs (512 threads) per row, C a
+        // power of two <= 16 chosen so n*C CTAs fill the GPU (B200: n = 2^5..2^8
+        // rows of 2^18..2^21 elements at 6.4-6.6 TB/s; non-power-of-two C and
+        // 1024-thread CTAs measured slower)
+        const int64_t target = (int64_t)sm_count() * 4;
+        int64_t C = 1;
+        while (C * 2 <= 8 && C * 2 * a.n <= target && C * 2 * 8192 <= a.m) C *= 2;
+        // 16-CTA clusters only while 8-CTA ones leave over half the SMs idle
+        // (measured: 16 rows x 16 CTAs 40.9 us vs x 8 48.1; 32 rows x 16 46.7 vs x 8 40.4)
+        if (C == 8 && 16 * a.n <= (int64_t)sm_count() * 2 && 16 * 8192 <= a.m) C = 16;
+        if (a.n < 2 * sm_count() && C >= 2) {
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3((unsigned)(a.n * C));
+            cfg.blockDim = dim3(kSplitThreads);
+            cfg.stream = a.stream;
+            cudaLaunchAttribute attr[1];
+            attr[0].id = cudaLaunchAttributeClusterDimension;
+            attr[0].val.clusterDim.x = (unsigned)C;
+            attr[0].val.clusterDim.y = 1;
+            attr[0].val.clusterDim.z = 1;
+            cfg.attrs = attr;
+            cfg.numAttrs = 1;
+            auto kc = segred_cluster_kernel<T, OP, F, kSplitThreads>;
+            if (C > 8) cudaFuncSetAttribute(kc, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);  // opt-in
+            cudaError_t e = cudaLaunchKernelEx(&cfg, kc, (const T*)a.in, (T*)a.out, a.m, bits_to<T>(a.ne_bits));
+            if (e != cudaSuccess && C > 8) {  // 16-CTA clusters refused: the portable size
+                (void)cudaGetLastError();
+                attr[0].val.clusterDim.x = 8;
+                cfg.gridDim = dim3((unsigned)(a.n * 8));
+                e = cudaLaunchKernelEx(&cfg, kc, (const T*)a.in, (T*)a.out, a.m, bits_to<T>(a.ne_bits));
+            }
+            return e;
+        }
+        if (a.n < 2 * sm_count())
+            flat_red_split_kernel<T, OP, F, true, 1024><<<(unsigned)a.n, 1024, 0, a.stream>>>(
+                (const T*)a.in, a.m, 1, (T*)a.out, bits_to<T>(a.ne_bits));
+        else
+            flat_red_split_kernel<T, OP, F, true><<<(unsigned)a.n, kSplitThreads, 0, a.stream>>>(
+                (const T*)a.in, a.m, 1, (T*)a.out, bits_to<T>(a.ne_bits));
+        return cudaGetLastError();
+    });
 }
 
 template <typename T, int OP>
@@ -811,12 +906,12 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
         T* tail = head + tiles;
         if (a.m >= kSplitMinM) {
-            // P pieces per row: ~4 resident 512-thread CTAs per SM over the grid, and
-            // n*P partials fit the head array (P*n <= tiles since pieces >= 8192 > kFlatTile)
-            const int P = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div((int64_t)sm_count() * 4, a.n),
-                                                                      a.m / 8192));
-            flat_red_split_kernel<T, OP, F><<<(unsigned)(a.n * P), kSplitThreads, 0, a.stream>>>(
-                (const T*)a.in, a.m, P, head);
+            // P pieces per row: n*P <= the resident CTAs of the GPU (a single wave, no
+            // tail), pieces >= 8192 elements, so n*P <= tiles fits the head array
+            auto ks = flat_red_split_kernel<T, OP, F>;
+            const int64_t R = resident_ctas(ks, 0, kSplitThreads);
+            const int P = (int)std::max<int64_t>(1, std::min<int64_t>(R / a.n, a.m / 8192));
+            ks<<<(unsigned)(a.n * P), kSplitThreads, 0, a.stream>>>((const T*)a.in, a.m, P, head, d);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
             const int g2 = (int)std::min<int64_t>(ceil_div(a.n, 256), (int64_t)sm_count() * 4);

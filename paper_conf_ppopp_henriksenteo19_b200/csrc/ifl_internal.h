@@ -35,6 +35,7 @@ cudaError_t launch_segred_mid(const SegArgs& a);
 cudaError_t launch_segscan_top(const SegArgs& a);
 cudaError_t launch_segscan_mid(const SegArgs& a);
 cudaError_t launch_flat(const SegArgs& a, bool scan);
+cudaError_t launch_segred_rows512(const SegArgs& a);  // V_MIDDLE segred, m >= 8192 (flat.cu)
 cudaError_t launch_fill(void* out, int64_t count, uint32_t bits, cudaStream_t s);
 
 // Group size (threads per segment) used by the V_MIDDLE kernels.

@@ -449,6 +449,7 @@ __global__ void __launch_bounds__(1024) segred_mid_kernel(const T* __restrict__ 
 }
 
 cudaError_t launch_segred_mid(const SegArgs& a) {
+    if (a.m >= 8192) return launch_segred_rows512(a);  // one 512-thread group per row (flat.cu)
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;

@@ -221,11 +221,15 @@ def test_small_m_kernels(ifl, orc, version, scan):
                     assert_parity(orc, x, got, scan, op, "sq" if op == "sum" else "id", None, dt)
 
 
+@pytest.mark.parametrize("version", ["flat", "middle"])
 @pytest.mark.parametrize("dt", ["i32", "f32"])
-def test_flat_segred_long_rows_split(ifl, orc, dt):
-    # V_FLAT segred on rows >= 2^16 elements: uniform row pieces + per-row combine
-    for (n, m, mis) in [(1, (1 << 20) + 5, True), (3, (1 << 16) + 13, False), (7, 1 << 17, True), (130, 1 << 16, False)]:
+def test_segred_long_rows_split_and_cluster(ifl, orc, dt, version):
+    # rows >= 8192 elements: V_FLAT uniform row pieces + per-row combine; V_MIDDLE
+    # one 512/1024-thread CTA per row, or a thread-block cluster per row with a
+    # DSMEM combine when there are fewer rows than SMs
+    for (n, m, mis) in [(1, (1 << 20) + 5, True), (3, (1 << 16) + 13, False), (7, 1 << 17, True),
+                        (130, 1 << 16, False), (300, 8200, True), (64, 1 << 15, False)]:
         for op in (["sum", "min", "xor", "prod"] if dt == "i32" else ["sum", "max"]):
             x, xd = gen_for(op, dt, 17, n, m, misalign=mis)
-            got = ifl.segred(xd, op, "sq" if op != "prod" else "id", ne=(2 if dt == "i32" else 0.5), version="flat")
+            got = ifl.segred(xd, op, "sq" if op != "prod" else "id", ne=(2 if dt == "i32" else 0.5), version=version)
             assert_parity(orc, x, got, False, op, "sq" if op != "prod" else "id", 2 if dt == "i32" else 0.5, dt)
