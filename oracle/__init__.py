@@ -59,6 +59,8 @@ def lib() -> ctypes.CDLL:
             "oracle_redomap2": [_vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int],
             "oracle_tridag": [_vp, _vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _vp],
             "oracle_lvc": [_vp] * 10 + [_c_i64] * 4 + [_vp],
+            "oracle_segarg_i32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int],
+            "oracle_segarg_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int],
             "oracle_segred_irr_i32": [_vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_int32],
             "oracle_segscan_irr_i32": [_vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_int32],
             "oracle_segred_irr_f32": [_vp, _vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_double],
@@ -262,3 +264,15 @@ def seg_irr(x: np.ndarray, offsets: np.ndarray, scan: bool, op: str = "sum", f: 
     fn = lib().oracle_segscan_irr_f32 if scan else lib().oracle_segred_irr_f32
     _check(fn(_ptr(x), _ptr(out), _ptr(ab), _ptr(off), n, OPS[op], MAPS[f], d))
     return (out, ab) if with_absum else out
+
+
+def segarg(x: np.ndarray, which: str = "min"):
+    """Tuple-valued reduction (argmin of NN): per row the
+    (value, index) of the first minimum / maximum; m == 0 -> (d, -1)."""
+    x = np.ascontiguousarray(x)
+    n, m = x.shape
+    val = np.empty(n, x.dtype)
+    idx = np.empty(n, np.int32)
+    fn = lib().oracle_segarg_i32 if x.dtype == np.int32 else lib().oracle_segarg_f32
+    _check(fn(_ptr(x), _ptr(val), _ptr(idx), n, m, 1 if which == "max" else 0))
+    return val, idx

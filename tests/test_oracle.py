@@ -537,3 +537,26 @@ def test_irr_numpy_cumsum_and_brute_force(orc):
         got, ab = orc.seg_irr(xf, off, False, with_absum=True)
         want = np.array([math.fsum(xf[off[i]:off[i + 1]].astype(np.float64)) for i in range(len(lens))])
         assert (np.abs(got - want) <= 1e-12 * (ab + 1)).all()
+
+
+# ------------------------------------------- segarg: tuple-valued (+) (NEXT-3)
+
+
+def test_segarg_numpy_and_closed_forms(orc):
+    x = gen.matrix("I32_SMALL", 51, 37, 53).numpy()  # many ties: values in [-1000, 1000]
+    for which, npf in (("min", np.argmin), ("max", np.argmax)):
+        val, idx = orc.segarg(x, which)
+        np.testing.assert_array_equal(idx, npf(x, axis=1))                 # numpy: first occurrence
+        np.testing.assert_array_equal(val, x[np.arange(37), idx])
+        np.testing.assert_array_equal(val, orc.segred(x, which))           # the value half is segred
+    xf = gen.matrix("F32_SIGNED", 52, 20, 31).numpy()
+    v, i = orc.segarg(xf, "min")
+    np.testing.assert_array_equal(i, np.argmin(xf, axis=1))
+    # closed forms: decreasing rows -> last index; constant rows -> index 0; empty rows -> (d, -1)
+    dec = np.tile(np.arange(9, 0, -1, dtype=np.int32), (3, 1))
+    assert (orc.segarg(dec, "min")[1] == 8).all() and (orc.segarg(dec, "max")[1] == 0).all()
+    assert (orc.segarg(np.full((2, 5), 7, np.int32), "min")[1] == 0).all()
+    big = np.full((2, 4), 2**31 - 1, np.int32)                             # equal to d: still index 0
+    assert (orc.segarg(big, "min")[1] == 0).all()
+    v, i = orc.segarg(np.zeros((3, 0), np.float32), "max")
+    assert (i == -1).all() and np.isneginf(v).all()
