@@ -327,6 +327,64 @@ def suite_col():
     return line
 
 
+# -------------------------------------------------------------------- segarg
+
+
+def suite_arg():
+    """NEXT-3: the tuple-valued per-row argmin (NN's
+    argmin P:474) over the configs[1] constant-work sweep, f32, n*m = 2^26.
+    Thresholds from ifl_tune_search over forced-version timings of the 2^24
+    and 2^25 sweeps (other data); a thread-per-row TOP on fewer than 4096 rows
+    runs for seconds and is reported as null (cannot win)."""
+    hbm, _, src = peaks()
+    ifl.reset_thresholds()
+
+    def sweep(lg, seed, versions):
+        x = gen.generate("F32_SIGNED", seed, 1 << lg, "cuda")
+        out = (torch.empty(1 << lg, device="cuda"), torch.empty(1 << lg, dtype=torch.int32, device="cuda"))
+        ws = ifl.workspace(max(ifl.workspace_bytes("segarg", 1 << k, 1 << (lg - k)) for k in range(lg + 1)) + 16,
+                           "cuda", "argsuite")
+        res = []
+        for k in range(lg + 1):
+            n, m = 1 << k, 1 << (lg - k)
+            xv = x.view(n, m)
+            o = (out[0][:n], out[1][:n])
+            r = {"n": n, "m": m}
+            for v in versions:
+                if v == "top" and n < 4096:
+                    r[v] = None
+                    continue
+                r[v] = gtime(lambda: ifl.segarg(xv, "min", version=v, out=o, ws=ws)) * 1e3
+            if "auto" in versions:
+                r["chosen"] = ifl.segarg(xv, "min", out=o, ws=ws, return_choice=True)[1].version
+            res.append(r)
+        return res
+
+    pt, pm, tbl = [], [], []
+    for lg in (24, 25):
+        for r in sweep(lg, 5 + lg, ("top", "middle", "flat")):
+            c = ifl.select("segarg.b4", r["n"], r["m"])
+            pt.append(c.par_top)
+            pm.append(c.par_mid)
+            tbl.append([float("inf") if r[v] is None else r[v] for v in ("top", "middle", "flat")])
+    a, b, npaths = ifl.tune_search(pt, pm, tbl, cost=1)
+    ifl.set_thresholds("segarg.b4", a, b)
+    rows = sweep(26, 2, ("top", "middle", "flat", "auto"))
+    for r in rows:
+        best = min(r[v] for v in ("top", "middle", "flat") if r[v] is not None)
+        r["best_over_auto"] = round(best / r["auto"], 4)
+        r["GBps"] = round((4 * r["n"] * r["m"] + 8 * r["n"]) / (r["auto"] * 1e-6) / 1e9, 1)
+    tot = sum(4 * r["n"] * r["m"] + 8 * r["n"] for r in rows) / (sum(r["auto"] for r in rows) * 1e-6) / 1e9
+    line = base_line("per-row argmin (tuple-valued reduce) GB/s over the n x m sweep", round(tot, 1), "GB/s",
+                     {"workload": "SURVEY 8(f) NEXT-3: f32 argmin, n*m = 2^26, n = 2^0..2^26, AUTO tuned on the "
+                                  "2^24 / 2^25 sweeps", "thresholds": {"t_top": a, "t_intra": b, "paths": npaths}})
+    line["min_shape_best_over_auto"] = min(r["best_over_auto"] for r in rows)
+    line["roofline"] = {"bound": "hbm", "kernel": "segarg sweep (AUTO)", "achieved": round(tot, 1), "peak": hbm,
+                        "unit": "GB/s", "frac": round(tot / hbm, 4), "traffic": None, "peak_source": src}
+    line["shapes"] = rows
+    return line
+
+
 # ----------------------------------------------------------------------- irr
 
 
@@ -455,4 +513,4 @@ def suite_dist():
 
 
 SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist,
-          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr}
+          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr, "arg": suite_arg}

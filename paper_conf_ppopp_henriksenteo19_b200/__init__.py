@@ -31,7 +31,7 @@ MAPS = {"id": 0, "sq": 1, "abs": 2}
 VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3}
 VERSION_NAMES = {-1: "auto", 0: "top", 1: "middle", 2: "flat", 3: "outer"}
 SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4",
-         "segred.irr", "segscan.irr")
+         "segred.irr", "segscan.irr", "segarg.b4")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -64,6 +64,7 @@ _SIGS = {
     "ifl_segscan_seeded": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_colred": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_colscan": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_segarg": ([_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segred_irr": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segscan_irr": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_irr_inspect": ([_vp, _i64, _i64, _vp, _vp, _vp], _int),
@@ -303,6 +304,31 @@ def colred(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stre
 def colscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False):
     """out[i,j] = ne (+) f(x[0,j]) (+) ... (+) f(x[i,j]) -- column-wise inclusive scan (G4 with scan)."""
     return _col(True, x, op, f, ne, version, out, ws, stream, return_choice)
+
+
+# -------------------------------------------------------------- segarg
+
+
+def segarg(x, which="min", version="auto", out=None, ws=None, stream=None, return_choice=False):
+    """Per-row (value, index) of the first minimum / maximum -- the
+    tuple-valued reduction (argmin of NN).  Returns (val, idx)."""
+    if x.dim() != 2 or not x.is_contiguous() or not x.is_cuda:
+        raise ValueError("expected a contiguous [n][m] CUDA tensor")
+    dt = _TORCH_DT.get(x.dtype)
+    if dt not in ("i32", "f32"):
+        raise TypeError(f"unsupported dtype {x.dtype}")
+    n, m = x.shape
+    val, idx = out if out is not None else (torch.empty(n, dtype=x.dtype, device=x.device),
+                                            torch.empty(n, dtype=torch.int32, device=x.device))
+    wb = lib().ifl_workspace_bytes(b"segarg", n, m, 0, DTYPES[dt], VERSIONS[version])
+    if ws is None and wb:
+        ws = workspace(wb, x.device, "arg")
+    c = ifl_choice()
+    rc = lib().ifl_segarg(x.data_ptr(), val.data_ptr(), idx.data_ptr(), n, m, DTYPES[dt], 1 if which == "max" else 0,
+                          VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel() * ws.element_size(),
+                          _stream(stream), ctypes.byref(c))
+    _check(rc, "ifl_segarg")
+    return ((val, idx), _choice_out(c)) if return_choice else (val, idx)
 
 
 # -------------------------------------------------------- irregular segments

@@ -39,7 +39,7 @@ constexpr int64_t kDefaultThreshold = 1 << 15;
 constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE kernel (reading R3)
 
 const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
-                              "colred.b4", "colscan.b4", "segred.irr", "segscan.irr"};
+                              "colred.b4", "colscan.b4", "segred.irr", "segscan.irr", "segarg.b4"};
 
 struct Table {
     std::mutex mu;
@@ -285,6 +285,7 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
     }
     if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
     if (strcmp(entry, "colred") == 0 || strcmp(entry, "colscan") == 0) return ifl::col_ws_bytes(n, m, version);
+    if (strcmp(entry, "segarg") == 0) return ifl::arg_ws_bytes(n, m, version);
     if (strcmp(entry, "segred_irr") == 0 || strcmp(entry, "segscan_irr") == 0) return ifl::irr_ws_bytes(m, version);
     if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
     if (strcmp(entry, "lvc") == 0)  // (numX, numY): the coefficient scans of both sites
@@ -433,6 +434,37 @@ int ifl_irr_inspect(const int64_t* offsets, int64_t n, int64_t total, void* ws16
                                 "off[n] = total = %lld; got off[n] = %lld)", (long long)total, (long long)last);
     if (max_len) *max_len = (int64_t)res[0];
     return IFL_OK;
+}
+
+int ifl_segarg(const void* in, void* val, int32_t* idx, int64_t n, int64_t m, int dt, int which, int version,
+               void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
+    const char* what = "ifl_segarg";
+    int rc = validate_seg(false, in, val, n, m, dt, IFL_MIN, IFL_F_ID, version, what);
+    if (rc) return rc;
+    if (which != 0 && which != 1) return fail(IFL_EINVAL, "%s: which must be 0 (argmin) or 1 (argmax)", what);
+    if (n > 0 && !idx) return fail(IFL_EINVAL, "%s: idx is NULL", what);
+    if (m > 0x7fffffffLL) return fail(IFL_EINVAL, "%s: rows longer than 2^31 - 1 (int32 indices)", what);
+    if (overlap(in, (size_t)(n * m) * 4, val, (size_t)n * 4) || overlap(in, (size_t)(n * m) * 4, idx, (size_t)n * 4) ||
+        overlap(val, (size_t)n * 4, idx, (size_t)n * 4))
+        return fail(IFL_EINVAL, "%s: overlapping arrays", what);
+    ifl_choice c;
+    select_version("segarg.b4", n, m, 0, true, &c);
+    if (version != IFL_AUTO) c.version = version;
+    if (choice) *choice = c;
+    if (n == 0) return IFL_OK;
+    if (m == 0) {  // (d, -1) per row
+        const uint32_t dbits = canonical_bits(dt, which ? IFL_MAX : IFL_MIN);
+        cudaError_t e = ifl::launch_fill(val, n, dbits, (cudaStream_t)stream);
+        if (e == cudaSuccess) e = ifl::launch_fill(idx, n, 0xffffffffu, (cudaStream_t)stream);
+        return cuda_status(e, what);
+    }
+    if (c.version == IFL_V_FLAT) {
+        const size_t need = ifl::arg_ws_bytes(n, m, IFL_V_FLAT);
+        if (!ws || ws_bytes < need)
+            return fail(IFL_EWORKSPACE, "%s: V_FLAT needs %zu workspace bytes, got %zu", what, need, ws_bytes);
+    }
+    ifl::ArgArgs a{in, val, idx, n, m, dt, which, ws, ws_bytes, (cudaStream_t)stream};
+    return cuda_status(ifl::launch_arg(a, c.version), what);
 }
 
 int ifl_colred(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int version,

@@ -53,6 +53,20 @@ size_t col_ws_bytes(int64_t n, int64_t m, int version);
 cudaError_t launch_col(const SegArgs& a, bool scan, int version);
 constexpr int64_t kColGroup = 8;  // threads per column in V_MIDDLE (reading R3's group size)
 
+// Tuple-valued per-row argmin / argmax (arg.cu).
+struct ArgArgs {
+    const void* in;
+    void* val;
+    int* idx;
+    int64_t n, m;
+    int dt, which;  // which: 0 argmin, 1 argmax
+    void* ws;
+    size_t ws_bytes;
+    cudaStream_t stream;
+};
+size_t arg_ws_bytes(int64_t n, int64_t m, int version);
+cudaError_t launch_arg(const ArgArgs& a, int version);
+
 // Irregular segments (irr.cu): segment i = in[off[i] .. off[i+1]-1].
 struct IrrArgs {
     const void* in;

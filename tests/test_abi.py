@@ -300,3 +300,12 @@ def test_irr_guard_and_validation(L):
     assert L.ifl_segred_irr(*sig, 4, 8, 0, 1, 0, 0, None, 2, None, 0, None, None) == ifl.IFL_EWORKSPACE
     assert ifl.workspace_bytes("segred_irr", 4, 1 << 20, version="flat") > 0
     assert ifl.workspace_bytes("segred_irr", 4, 1 << 20, version="top") == 0
+
+
+def test_segarg_validation(L):
+    assert L.ifl_segarg(256, 512, 1024, -1, 4, 1, 0, -1, None, 0, None, None) == ifl.IFL_EINVAL
+    assert L.ifl_segarg(256, 512, 1024, 4, 4, 1, 2, -1, None, 0, None, None) == ifl.IFL_EINVAL   # which
+    assert L.ifl_segarg(256, 512, None, 4, 4, 1, 0, -1, None, 0, None, None) == ifl.IFL_EINVAL   # idx NULL
+    assert L.ifl_segarg(1 << 20, 512, 1024, 4, 1 << 16, 1, 0, 2, None, 0, None, None) == ifl.IFL_EWORKSPACE
+    assert L.ifl_segarg(256, 512, 1024, 0, 4, 1, 0, -1, None, 0, None, None) == 0                # n == 0
+    assert ifl.workspace_bytes("segarg", 4, 1 << 16, version="flat") > 0
