@@ -327,6 +327,61 @@ def suite_col():
     return line
 
 
+# -------------------------------------------------------------------- mmtree
+
+
+def suite_mmtree():
+    """NEXT-2: the 5-leaf branching tree of matrix
+    multiplication (row-level G3 leaves ROW_TOP / ROW_MIDDLE, then TOP /
+    MIDDLE / FLAT over the two-map context), f32, on the paper's Fig 2 family
+    A[2^a][2^(k-2a)] x B[2^(k-2a)][2^a]: thresholds tuned on k = 20
+    and applied to k = 25 (the paper's protocol), by the chain search over
+    every distinct tree path (Fig 5); the 3-leaf tuning of the same
+    training set is timed beside it."""
+    ifl.reset_thresholds()
+    train, test = mm_shapes(20), mm_shapes(25)
+    # 3-leaf tuning (the row level off), then the 5-leaf tree
+    a3, b3, _ = ifl.tune("redomap2.f32", train, reps=3, cost=1)
+    t_top, t_intra, tbl = ifl.tune("redomap2.f32.tree", train, reps=3, cost=1)
+    rt, ri = ifl.get_thresholds("redomap2.f32.row")
+    rows = []
+    for (n, m, p) in test:
+        A = gen.generate("F32_SIGNED", 6, n * m, "cuda").view(n, m)
+        Bt = gen.generate("F32_SIGNED", 7, p * m, "cuda").view(p, m)
+        C = torch.empty(n, p, device="cuda")
+        ws = ifl.workspace(ifl.workspace_bytes("redomap2", n, m, p, "f32"), "cuda", "mmtree")
+        r = {"n": n, "m": m, "p": p}
+        for v in ("row_top", "row_middle", "top", "middle", "flat"):
+            if v == "row_middle" and m > 8192:
+                r[v] = None
+                continue
+            r[v] = gtime(lambda: ifl.redomap2(A, Bt, out=C, ws=ws, version=v)) * 1e3
+        r["auto5"] = gtime(lambda: ifl.redomap2(A, Bt, out=C, ws=ws)) * 1e3
+        r["chosen5"] = ifl.redomap2(A, Bt, out=C, ws=ws, return_choice=True)[1].version
+        ifl.set_thresholds("redomap2.f32.row", 2**63 - 1, 2**63 - 1)
+        ifl.set_thresholds("redomap2.f32", a3, b3)
+        r["auto3"] = gtime(lambda: ifl.redomap2(A, Bt, out=C, ws=ws)) * 1e3
+        r["chosen3"] = ifl.redomap2(A, Bt, out=C, ws=ws, return_choice=True)[1].version
+        ifl.set_thresholds("redomap2.f32.row", rt, ri)
+        ifl.set_thresholds("redomap2.f32", t_top, t_intra)
+        best = min(r[v] for v in ("row_top", "row_middle", "top", "middle", "flat") if r[v] is not None)
+        r["best_over_auto5"] = round(best / r["auto5"], 4)
+        r["best_over_auto3"] = round(best / r["auto3"], 4)
+        rows.append(r)
+    t5, t3 = sum(r["auto5"] for r in rows), sum(r["auto3"] for r in rows)
+    line = base_line("matmul branching tree (5 leaves) on the Fig 2 family, k = 25, f32: total us", round(t5, 2),
+                     "us", {"workload": "SURVEY 8(f) NEXT-2: A[2^a][2^(25-2a)] x B, a = 0..12, tuned on k = 20",
+                            "thresholds": {"row": [rt, ri], "two_map": [t_top, t_intra], "three_leaf_only": [a3, b3]}},
+                     hib=False)
+    line["total_us_3leaf"] = round(t3, 2)
+    line["speedup_5leaf_vs_3leaf"] = round(t3 / t5, 4)
+    line["min_shape_best_over_auto5"] = min(r["best_over_auto5"] for r in rows)
+    line["min_shape_best_over_auto3"] = min(r["best_over_auto3"] for r in rows)
+    line["train_cost_table_ms"] = tbl.tolist()
+    line["shapes"] = rows
+    return line
+
+
 # -------------------------------------------------------------------- segarg
 
 
@@ -513,4 +568,4 @@ def suite_dist():
 
 
 SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist,
-          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr, "arg": suite_arg}
+          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr, "arg": suite_arg, "mmtree": suite_mmtree}

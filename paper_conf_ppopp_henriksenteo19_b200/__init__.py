@@ -28,10 +28,10 @@ IFL_OK, IFL_EINVAL, IFL_EUNSUPPORTED, IFL_EWORKSPACE, IFL_ENOTFIT, IFL_ECUDA = 0
 DTYPES = {"i32": 0, "f32": 1, "bf16": 2}
 OPS = {"sum": 0, "prod": 1, "min": 2, "max": 3, "and": 4, "or": 5, "xor": 6}
 MAPS = {"id": 0, "sq": 1, "abs": 2}
-VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3}
-VERSION_NAMES = {-1: "auto", 0: "top", 1: "middle", 2: "flat", 3: "outer"}
+VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3, "row_top": 4, "row_middle": 5}
+VERSION_NAMES = {v: k for k, v in VERSIONS.items()}
 SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4",
-         "segred.irr", "segscan.irr", "segarg.b4")
+         "segred.irr", "segscan.irr", "segarg.b4", "redomap2.f32.row", "redomap2.bf16.row")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -84,6 +84,7 @@ _SIGS = {
     "ifl_tune": ([ctypes.c_char_p, _vp, _int, _int, _int, _vp, _sz, _vp, _vp, _vp, _vp], _int),
     "ifl_tune_scratch_bytes": ([ctypes.c_char_p, _vp, _int], _sz),
     "ifl_tune_search": ([_vp, _vp, _vp, _int, _int, _vp, _vp, _vp], _int),
+    "ifl_tune_search_chain": ([_vp, _vp, _int, _int, _int, _vp, _vp], _int),
     "ifl_last_error": ([], ctypes.c_char_p),
     "ifl_build_info": ([], ctypes.c_char_p),
 }
@@ -173,6 +174,20 @@ def tune_search(par_top, par_mid, cost_table, cost: int = 0):
     _check(lib().ifl_tune_search(pt.ctypes.data, pm.ctypes.data, ct.ctypes.data, len(pt), cost,
                                  ctypes.byref(a), ctypes.byref(b), ctypes.byref(npaths)), "ifl_tune_search")
     return a.value, b.value, npaths.value
+
+
+def tune_search_chain(par, cost_table, cost: int = 0):
+    """Chain (Fig 5) search: par [nshapes][G], cost_table [nshapes][G+1] ->
+    (thresholds [G], distinct paths evaluated)."""
+    import numpy as np
+    pa = np.ascontiguousarray(par, dtype=np.int64)
+    ct = np.ascontiguousarray(cost_table, dtype=np.float64)
+    ns, G = pa.shape
+    th = np.zeros(G, np.int64)
+    npaths = ctypes.c_int()
+    _check(lib().ifl_tune_search_chain(pa.ctypes.data, ct.ctypes.data, ns, G, cost, th.ctypes.data,
+                                       ctypes.byref(npaths)), "ifl_tune_search_chain")
+    return [int(t) for t in th], npaths.value
 
 
 # ------------------------------------------------------------- workspaces
@@ -469,11 +484,12 @@ def tune(site: str, shapes, reps: int = 5, cost: int = 0, scratch: torch.Tensor 
         scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
     if sh.ndim != 2 or sh.shape[1] != (2 if site.startswith(("seg", "col")) else 4 if site == "lvc" else 3):
         raise ValueError(f"{site}: shapes must be tuples of the site's arity")
-    tbl = np.zeros(ns * 3, np.float64)
+    nv = 5 if site.endswith(".tree") else 3
+    tbl = np.zeros(ns * nv, np.float64)
     a, b = ctypes.c_int64(), ctypes.c_int64()
     _check(lib().ifl_tune(_b(site), sh.ctypes.data, ns, reps, cost, scratch.data_ptr(), scratch.numel(),
                           _stream(stream), ctypes.byref(a), ctypes.byref(b), tbl.ctypes.data), "ifl_tune")
-    return a.value, b.value, tbl.reshape(ns, 3)
+    return a.value, b.value, tbl.reshape(ns, nv)
 
 
 def build_info() -> str:

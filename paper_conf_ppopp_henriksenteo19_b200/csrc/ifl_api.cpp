@@ -39,7 +39,8 @@ constexpr int64_t kDefaultThreshold = 1 << 15;
 constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE kernel (reading R3)
 
 const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
-                              "colred.b4", "colscan.b4", "segred.irr", "segscan.irr", "segarg.b4"};
+                              "colred.b4", "colscan.b4", "segred.irr", "segscan.irr", "segarg.b4",
+                              "redomap2.f32.row", "redomap2.bf16.row"};
 
 struct Table {
     std::mutex mu;
@@ -48,7 +49,9 @@ struct Table {
     Table() { reset(); }
     void reset() {
         thr.clear();
-        for (const char* s : kSites) thr[s] = {kDefaultThreshold, kDefaultThreshold};
+        for (const char* s : kSites)  // the matmul row level is off until tuned (reading R17)
+            thr[s] = strstr(s, ".row") ? std::make_pair(INT64_MAX, INT64_MAX)
+                                       : std::make_pair(kDefaultThreshold, kDefaultThreshold);
         par_mode = 1;
     }
 };
@@ -120,6 +123,18 @@ void irr_par(int64_t n, int64_t total, int64_t max_len, int64_t* ptop, int64_t* 
     *ptop = max_len > 0 ? std::min(n, total / max_len) : n;
     const int64_t mean = n > 0 ? (total + n - 1) / n : 0;
     *pmid = sat_mul(n, std::min<int64_t>(mean, 32));
+}
+
+// The matmul branching tree (5 leaves): the row-level guards
+// of G3 on the outer map, then the existing G3 over the two-map context.
+void mm_tree_select(int in_dt, int64_t n, int64_t m, int64_t p, ifl_choice* c) {
+    const char* site = in_dt == IFL_BF16 ? "redomap2.bf16" : "redomap2.f32";
+    const char* rsite = in_dt == IFL_BF16 ? "redomap2.bf16.row" : "redomap2.f32.row";
+    select_version(site, n, m, p, true, c);
+    int64_t trt, tri;
+    ifl_get_thresholds(rsite, &trt, &tri);
+    if (n >= trt) c->version = IFL_V_ROW_TOP;
+    else if (sat_mul(n, std::min<int64_t>(p, 8) * 32) >= tri && ifl::mm_row_mid_fits(m)) c->version = IFL_V_ROW_MIDDLE;
 }
 
 uint32_t canonical_bits(int dt, int op) {
@@ -500,15 +515,20 @@ int ifl_redomap2(const void* A, const void* B, float* C, int64_t n, int64_t m, i
     if (mul_overflows(n, m) || mul_overflows(m, p) || mul_overflows(n, p) || mul_overflows(sat_mul(n, p), m))
         return fail(IFL_EINVAL, "ifl_redomap2: size overflow");
     if (in_dt != IFL_F32 && in_dt != IFL_BF16) return fail(IFL_EUNSUPPORTED, "ifl_redomap2: dtype %d", in_dt);
-    if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "ifl_redomap2: bad version");
+    if (version < IFL_AUTO || version > IFL_V_ROW_MIDDLE || version == IFL_V_OUTER)
+        return fail(IFL_EINVAL, "ifl_redomap2: bad version");
     if (n * p > 0 && !C) return fail(IFL_EINVAL, "ifl_redomap2: C is NULL");
     if (n * m > 0 && !A) return fail(IFL_EINVAL, "ifl_redomap2: A is NULL");
     if (m * p > 0 && !B) return fail(IFL_EINVAL, "ifl_redomap2: B is NULL");
     const char* site = in_dt == IFL_BF16 ? "redomap2.bf16" : "redomap2.f32";
     ifl_choice c;
-    select_version(site, n, m, p, true, &c);
+    mm_tree_select(in_dt, n, m, p, &c);
     if (version != IFL_AUTO) c.version = version;
     if (choice) *choice = c;
+    (void)site;
+    if (c.version == IFL_V_ROW_MIDDLE && !ifl::mm_row_mid_fits(m))
+        return fail(IFL_ENOTFIT, "ifl_redomap2: V_ROW_MIDDLE keeps a row of A in shared memory (m <= %lld)",
+                    (long long)ifl::kMmRowMaxM);
     if (n * p == 0) return IFL_OK;
     ifl::MmArgs a{A, B, C, n, m, p, in_dt, b_kmajor ? 1 : 0, ws, ws_bytes, (cudaStream_t)stream};
     // actual need: B transposition (b_kmajor = 0) + split-K partials (V_FLAT)

@@ -98,6 +98,11 @@ struct MmArgs {
 size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version);
 cudaError_t launch_redomap2(int version, const MmArgs& a);
 bool redomap2_tc_ok(const MmArgs& a);
+// row-level leaves of the matmul tree (mm_row.cu); Bt is [p][m]
+constexpr int64_t kMmRowMaxM = 8192;  // V_ROW_MIDDLE keeps a row of A in shared memory
+bool mm_row_mid_fits(int64_t m);
+cudaError_t launch_mm_row(int version, const void* A, const void* Bt, float* C, int64_t n, int64_t m, int64_t p,
+                          int in_dt, cudaStream_t s);
 
 struct TriArgs {
     const float *a, *b, *c, *y;

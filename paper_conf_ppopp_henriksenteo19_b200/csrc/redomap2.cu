@@ -367,6 +367,8 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
         Bt = t;
     }
     if (a.m == 0) return cudaMemsetAsync(a.C, 0, (size_t)a.n * a.p * sizeof(float), a.stream);
+    if (version == IFL_V_ROW_TOP || version == IFL_V_ROW_MIDDLE)  // row-level leaves (mm_row.cu)
+        return launch_mm_row(version, A, Bt, a.C, a.n, a.m, a.p, a.in_dt, a.stream);
     constexpr int E = VecE<Tin>::E;
     const bool vec = ((uintptr_t)A % 16 == 0) && ((uintptr_t)Bt % 16 == 0) && (a.m % E == 0);
     const int64_t outs = a.n * a.p;

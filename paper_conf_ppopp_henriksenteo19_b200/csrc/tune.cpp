@@ -87,9 +87,102 @@ extern "C" int ifl_tune_search(const int64_t* par_top, const int64_t* par_mid, c
     return std::isfinite(bp) ? IFL_OK : IFL_ENOTFIT;
 }
 
+// Generalised search for a CHAIN of G guards -- the branching trees of Fig 5
+// (P:374): leaf k < G is taken when par[s][k] >= t_k and every earlier guard
+// failed, leaf G otherwise.  Every combination of candidate thresholds (the
+// geometric midpoints between adjacent training Par values, per guard) maps to
+// a path (one leaf per shape); each DISTINCT path is costed once (P:374-378
+// memoisation), and once every shape is placed, the later guards are not
+// enumerated at all.  Cost as in ifl_tune_search; ties broken by the sum.
+namespace {
+struct ChainSearch {
+    const int64_t* par;
+    const double* cost;
+    int ns, G, kind;
+    std::vector<std::vector<int64_t>> cand;
+    std::vector<double> best;
+    std::map<std::vector<int>, std::pair<double, double>> memo;
+    std::vector<int> path;
+    std::vector<int64_t> cur, bt;
+    double bp = std::numeric_limits<double>::infinity(), bs = std::numeric_limits<double>::infinity();
+
+    void eval() {
+        auto it = memo.find(path);
+        if (it == memo.end()) {
+            double sum = 0, worst = 0;
+            for (int s = 0; s < ns; ++s) {
+                const double c = cost[s * (G + 1) + path[s]];
+                sum += c;
+                worst = std::max(worst, c / best[s]);
+            }
+            it = memo.emplace(path, std::make_pair(kind == 0 ? sum : worst, sum)).first;
+        }
+        const double p = it->second.first, q = it->second.second;
+        if (p < bp || (p == bp && q < bs)) {
+            bp = p;
+            bs = q;
+            bt = cur;
+        }
+    }
+    void rec(int k, int left) {
+        if (k == G || left == 0) {
+            for (int j = k; j < G; ++j) cur[j] = INT64_MAX;  // later guards are irrelevant
+            std::vector<int> rest;
+            for (int s = 0; s < ns; ++s)
+                if (path[s] < 0) {
+                    path[s] = G;  // the else-leaf
+                    rest.push_back(s);
+                }
+            eval();
+            for (int s : rest) path[s] = -1;
+            return;
+        }
+        for (int64_t t : cand[k]) {
+            cur[k] = t;
+            std::vector<int> took;
+            for (int s = 0; s < ns; ++s)
+                if (path[s] < 0 && par[s * G + k] >= t) {
+                    path[s] = k;
+                    took.push_back(s);
+                }
+            rec(k + 1, left - (int)took.size());
+            for (int s : took) path[s] = -1;
+        }
+    }
+};
+}  // namespace
+
+extern "C" int ifl_tune_search_chain(const int64_t* par, const double* cost_table, int nshapes, int G, int cost,
+                                     int64_t* thresholds, int* n_paths) {
+    if (nshapes <= 0 || G <= 0 || G > 8 || !par || !cost_table || (cost != 0 && cost != 1)) return IFL_EINVAL;
+    ChainSearch cs;
+    cs.par = par;
+    cs.cost = cost_table;
+    cs.ns = nshapes;
+    cs.G = G;
+    cs.kind = cost;
+    cs.cand.resize(G);
+    for (int k = 0; k < G; ++k) {
+        std::vector<int64_t> v(nshapes);
+        for (int s = 0; s < nshapes; ++s) v[s] = par[s * G + k];
+        cs.cand[k] = candidates(v);
+    }
+    cs.best.assign(nshapes, std::numeric_limits<double>::infinity());
+    for (int s = 0; s < nshapes; ++s)
+        for (int v = 0; v <= G; ++v) cs.best[s] = std::min(cs.best[s], cost_table[s * (G + 1) + v]);
+    cs.path.assign(nshapes, -1);
+    cs.cur.assign(G, INT64_MAX);
+    cs.bt.assign(G, INT64_MAX);
+    cs.rec(0, nshapes);
+    if (thresholds)
+        for (int k = 0; k < G; ++k) thresholds[k] = cs.bt[k];
+    if (n_paths) *n_paths = (int)cs.memo.size();
+    return std::isfinite(cs.bp) ? IFL_OK : IFL_ENOTFIT;
+}
+
 namespace {
 
-enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_COLRED, K_COLSCAN, K_BAD };
+enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_COLRED, K_COLSCAN, K_TREE_F32, K_TREE_BF16, K_BAD };
 
 Kind kind_of(const char* site) {
     if (!site) return K_BAD;
@@ -101,8 +194,13 @@ Kind kind_of(const char* site) {
     if (!strcmp(site, "lvc")) return K_LVC;
     if (!strcmp(site, "colred.b4")) return K_COLRED;
     if (!strcmp(site, "colscan.b4")) return K_COLSCAN;
+    if (!strcmp(site, "redomap2.f32.tree")) return K_TREE_F32;
+    if (!strcmp(site, "redomap2.bf16.tree")) return K_TREE_BF16;
     return K_BAD;
 }
+
+Kind mm_of(Kind k) { return k == K_TREE_F32 ? K_MM_F32 : k == K_TREE_BF16 ? K_MM_BF16 : k; }
+bool is_tree(Kind k) { return k == K_TREE_F32 || k == K_TREE_BF16; }
 
 int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN) ? 2 : k == K_LVC ? 4 : 3; }
 
@@ -110,6 +208,7 @@ size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 int64_t ceil_div_i64(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
 size_t ws_bytes_of(Kind k, const int64_t* s) {
+    k = mm_of(k);
     switch (k) {
     case K_SEGRED: return ifl_workspace_bytes("segred", s[0], s[1], 0, IFL_F32, -1);
     case K_SEGSCAN: return ifl_workspace_bytes("segscan", s[0], s[1], 0, IFL_F32, -1);
@@ -125,6 +224,7 @@ size_t ws_bytes_of(Kind k, const int64_t* s) {
 
 // Scratch layout per shape: [in/A/...][out][ws], each 256-byte aligned.
 size_t base_shape_bytes(Kind k, const int64_t* s) {
+    k = mm_of(k);
     switch (k) {
     case K_SEGRED: {
         const int64_t n = s[0], m = s[1];
@@ -169,6 +269,7 @@ size_t shape_bytes(Kind k, const int64_t* s) { return base_shape_bytes(k, s); }
 int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_t st, int copy = 0) {
     // `in` of the seg/col layouts: the first region, or the second copy
     char* const in2 = (two_inputs(k) && copy) ? scratch + base_shape_bytes(k, s) : nullptr;
+    k = mm_of(k);
     switch (k) {
     case K_SEGRED: {
         const int64_t n = s[0], m = s[1];
@@ -282,18 +383,30 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     cudaStream_t st = (cudaStream_t)stream;
     char* flush = (char*)scratch + max_shape_bytes(k, shapes, nshapes);
     if (cudaMemsetAsync(flush, 0, kFlushBytes, st) != cudaSuccess) return IFL_ECUDA;  // valid floats, once
-    std::vector<double> table(nshapes * 3, std::numeric_limits<double>::infinity());
-    std::vector<int64_t> ptop(nshapes), pmid(nshapes);
+    // the matmul tree sites time five leaves (ROW_TOP, ROW_MIDDLE, TOP, MIDDLE,
+    // FLAT) and search a chain of four guards; every other site three versions
+    const bool tree = is_tree(k);
+    const int NV = tree ? 5 : 3;
+    static const int kTreeVersion[5] = {IFL_V_ROW_TOP, IFL_V_ROW_MIDDLE, IFL_V_TOP, IFL_V_MIDDLE, IFL_V_FLAT};
+    std::vector<double> table(nshapes * NV, std::numeric_limits<double>::infinity());
+    std::vector<int64_t> ptop(nshapes), pmid(nshapes), pchain(tree ? nshapes * 4 : 0);
     cudaEvent_t e0, e1;
     if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess) return IFL_ECUDA;
     int rc = IFL_OK;
     for (int i = 0; i < nshapes && rc == IFL_OK; ++i) {
         const int64_t* s = shapes + i * ar;
         ifl_choice c;
-        ifl_select(site, s[0], s[1], ar == 3 && k != K_TRIDAG ? s[2] : 0, &c);
+        const char* psite = tree ? (k == K_TREE_F32 ? "redomap2.f32" : "redomap2.bf16") : site;
+        ifl_select(psite, s[0], s[1], ar == 3 && k != K_TRIDAG ? s[2] : 0, &c);
         if (k == K_LVC) c.par_mid = 0;  // one guard: Par = numS
         ptop[i] = c.par_top;
         pmid[i] = c.par_mid;
+        if (tree) {  // Par of the four guards: n, n*min(p,8)*32, n*p, n*p*min(m,1024)
+            pchain[i * 4 + 0] = s[0];
+            pchain[i * 4 + 1] = s[0] * std::min<int64_t>(s[2], 8) * 32;
+            pchain[i * 4 + 2] = c.par_top;
+            pchain[i * 4 + 3] = c.par_mid;
+        }
         // zero this shape's workspace (the tail of its scratch layout); the
         // input region keeps the caller's data
         const size_t tot = base_shape_bytes(k, s), wsb = ws_bytes_of(k, s);
@@ -305,8 +418,9 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         // is > 50x slower than the best timed so far is recorded from that one
         // run (avoid spending the budget on settings that cannot win)
         double best_ms = std::numeric_limits<double>::infinity();
-        for (int vv = 0; vv < 3; ++vv) {
-            const int v = 2 - vv;
+        for (int vv = 0; vv < NV; ++vv) {
+            const int slot = NV - 1 - vv;                     // table column
+            const int v = tree ? kTreeVersion[slot] : slot;  // version run
             if (hopeless(k, s, v)) continue;  // stays +inf: unavailable to the search
             flush_l2(flush, st);
             cudaEventRecord(e0, st);
@@ -321,7 +435,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
             float warm = 0;
             cudaEventElapsedTime(&warm, e0, e1);
             if (warm > 50.0 * best_ms) {
-                table[i * 3 + v] = warm;
+                table[i * NV + slot] = warm;
                 continue;
             }
             // each rep: L2 evicted (read-flush), then one call.  (Measured on B200:
@@ -341,7 +455,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
                 ms[q] /= back;
             }
             std::sort(ms.begin(), ms.end());
-            table[i * 3 + v] = ms[reps / 2];
+            table[i * NV + slot] = ms[reps / 2];
             best_ms = std::min(best_ms, (double)ms[reps / 2]);
         }
     }
@@ -349,6 +463,18 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     cudaEventDestroy(e1);
     if (rc != IFL_OK) return rc;
     if (cost_table) std::copy(table.begin(), table.end(), cost_table);
+    if (tree) {
+        int64_t th[4];
+        int np;
+        rc = ifl_tune_search_chain(pchain.data(), table.data(), nshapes, 4, cost, th, &np);
+        if (rc != IFL_OK) return rc;
+        if (t_top) *t_top = th[2];
+        if (t_intra) *t_intra = th[3];
+        const bool bf = k == K_TREE_BF16;
+        rc = ifl_set_thresholds(bf ? "redomap2.bf16.row" : "redomap2.f32.row", th[0], th[1]);
+        if (rc != IFL_OK) return rc;
+        return ifl_set_thresholds(bf ? "redomap2.bf16" : "redomap2.f32", th[2], th[3]);
+    }
     int64_t a, b;
     int np;
     rc = ifl_tune_search(ptop.data(), pmid.data(), table.data(), nshapes, cost, &a, &b, &np);

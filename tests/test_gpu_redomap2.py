@@ -104,3 +104,42 @@ def test_tc_dense_square(ifl, orc):
     C = ifl.redomap2(A.cuda(), Bt.cuda(), version="top")
     rows = [0, 1, 127, 128, 511, 1023]
     check(orc, A[rows], Bt, C[rows])
+
+
+# ------------------------------------------ row-level leaves of the matmul tree (NEXT-2)
+
+ROW_SHAPES = [(1, 1, 1), (3, 5, 7), (1000, 64, 3), (130, 77, 260), (7, 8192, 5), (64, 1000, 1), (4096, 16, 16)]
+
+
+@pytest.mark.parametrize("version", ["row_top", "row_middle"])
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+@pytest.mark.parametrize("kmajor", [True, False])
+def test_redomap2_row_versions(ifl, orc, version, dt, kmajor):
+    tdt = torch.float32 if dt == "f32" else torch.bfloat16
+    for (n, m, p) in ROW_SHAPES:
+        A, Bt = operands(dt, n, m, p, seed=21)
+        A, Bt = A.to(tdt), Bt.to(tdt)
+        B = Bt if kmajor else Bt.t().contiguous()
+        C = ifl.redomap2(A.cuda(), B.cuda(), b_kmajor=kmajor, version=version)
+        check(orc, A, Bt, C)
+
+
+def test_redomap2_row_middle_notfit_and_tree(ifl, orc):
+    A, Bt = operands("f32", 3, 9000, 2)
+    with pytest.raises(ifl.IflError) as e:
+        ifl.redomap2(A.cuda(), Bt.cuda(), version="row_middle")
+    assert e.value.code == ifl.IFL_ENOTFIT
+    # the 5-leaf tree tuner: times every leaf, installs the row and the two-map thresholds
+    try:
+        train = [(1 << a, 1 << (18 - 2 * a), 1 << a) for a in range(0, 10)]
+        t_top, t_intra, tbl = ifl.tune("redomap2.f32.tree", train, reps=2, cost=1)
+        assert tbl.shape == (len(train), 5) and np.isfinite(tbl[:, 2:]).all()
+        assert ifl.get_thresholds("redomap2.f32") == (t_top, t_intra)
+        rt, ri = ifl.get_thresholds("redomap2.f32.row")
+        for (n, m, p) in train[:4]:
+            A, Bt = operands("f32", n, m, p, seed=22)
+            C, ch = ifl.redomap2(A.cuda(), Bt.cuda(), return_choice=True)
+            check(orc, A, Bt, C)
+            assert ch.version in ("row_top", "row_middle", "top", "middle", "flat")
+    finally:
+        ifl.reset_thresholds()
