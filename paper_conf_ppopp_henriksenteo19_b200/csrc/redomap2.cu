@@ -340,6 +340,11 @@ size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
     }
     if (version == 0 || version == -1) {
         part = std::max(part, (size_t)n * p * tc_splits(n, m, p, false) * 4);
+        {  // SIMT TOP with 32x32 tiles (small output grids)
+            const int64_t t32 = ceil_div(n, 32) * ceil_div(p, 32), nk32 = ceil_div(m, 32);
+            const int64_t s32 = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / std::max<int64_t>(t32, 1), nk32 / 8));
+            part = std::max(part, (size_t)n * p * s32 * 4);
+        }
         const int64_t tiles = ceil_div(n, 128) * ceil_div(p, 128), nk = ceil_div(m, 16);
         const int64_t s = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / tiles, nk / 64));
         part = std::max(part, (size_t)n * p * (size_t)ceil_div(nk, ceil_div(nk, s)) * 4);
@@ -427,8 +432,22 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     }
     // ---- V_TOP: output tiles, sequential k (tensor cores for bf16)
     if (tc) return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, false), a.stream);
-    // SIMT TOP: 128x128 tiles; when the tile grid leaves SMs idle, k is split
-    // into >= 64-tile chunks (each CTA still walks its chunk sequentially)
+    // SIMT TOP: 128x128 tiles; when fewer than half the SMs would get one, the
+    // 32x32 tiles (k in chunks of >= 8 x 32, each walked sequentially) -- B200:
+    // n = p = 64..512 outputs from 105-60 us down to the 32x32 engine's 11-18 us
+    if (ceil_div(a.n, 128) * ceil_div(a.p, 128) < 74) {
+        const int64_t t32 = ceil_div(a.n, 32) * ceil_div(a.p, 32), nk32 = ceil_div(a.m, 32);
+        const int64_t s32 = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / t32, nk32 / 8));
+        const int64_t kps32 = ceil_div(nk32, s32), sp32 = ceil_div(nk32, kps32);
+        dim3 g32((unsigned)ceil_div(a.p, 32), (unsigned)ceil_div(a.n, 32), (unsigned)sp32);
+        if (vec) mm_tile_simt_kernel<Tin, 32, 32, 32, true><<<g32, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps32);
+        else mm_tile_simt_kernel<Tin, 32, 32, 32, false><<<g32, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps32);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess || sp32 == 1) return e;
+        mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, a.stream>>>(
+            part, a.C, outs, (int)sp32);
+        return cudaGetLastError();
+    }
     const int64_t tiles = ceil_div(a.n, 128) * ceil_div(a.p, 128), nk = ceil_div(a.m, 16);
     const int64_t s = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / tiles, nk / 64));
     const int64_t kps = ceil_div(nk, s), splits = ceil_div(nk, kps);
