@@ -388,8 +388,8 @@ def suite_mmtree():
 def suite_arg():
     """NEXT-3: the tuple-valued per-row argmin (NN's
     argmin P:474) over the configs[1] constant-work sweep, f32, n*m = 2^26.
-    Thresholds from ifl_tune_search over forced-version timings of the 2^24
-    and 2^25 sweeps (other data); a thread-per-row TOP on fewer than 4096 rows
+    Thresholds from ifl_tune_search over forced-version timings of the 2^25
+    and 2^27 sweeps (other data, bracketing the test size as in bench.py); a thread-per-row TOP on fewer than 4096 rows
     runs for seconds and is reported as null (cannot win)."""
     hbm, _, src = peaks()
     ifl.reset_thresholds()
@@ -416,7 +416,7 @@ def suite_arg():
         return res
 
     pt, pm, tbl = [], [], []
-    for lg in (24, 25):
+    for lg in (25, 27):
         for r in sweep(lg, 5 + lg, ("top", "middle", "flat")):
             c = ifl.select("segarg.b4", r["n"], r["m"])
             pt.append(c.par_top)
@@ -432,7 +432,7 @@ def suite_arg():
     tot = sum(4 * r["n"] * r["m"] + 8 * r["n"] for r in rows) / (sum(r["auto"] for r in rows) * 1e-6) / 1e9
     line = base_line("per-row argmin (tuple-valued reduce) GB/s over the n x m sweep", round(tot, 1), "GB/s",
                      {"workload": "SURVEY 8(f) NEXT-3: f32 argmin, n*m = 2^26, n = 2^0..2^26, AUTO tuned on the "
-                                  "2^24 / 2^25 sweeps", "thresholds": {"t_top": a, "t_intra": b, "paths": npaths}})
+                                  "2^25 / 2^27 sweeps", "thresholds": {"t_top": a, "t_intra": b, "paths": npaths}})
     line["min_shape_best_over_auto"] = min(r["best_over_auto"] for r in rows)
     line["roofline"] = {"bound": "hbm", "kernel": "segarg sweep (AUTO)", "achieved": round(tot, 1), "peak": hbm,
                         "unit": "GB/s", "frac": round(tot / hbm, 4), "traffic": None, "peak_source": src}
