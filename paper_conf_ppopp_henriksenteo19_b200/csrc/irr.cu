@@ -12,8 +12,9 @@
 //             16 items) with per-tile segment ranges, a CTA-wide segmented
 //             scan of the thread pieces, and tile aggregates combined by a
 //             single-CTA segmented scan over tiles:
-//               pass 0  tile -> first segment (scatter at segment starts,
-//                       max-scan over tiles); empty segments reduce to d;
+//               pass 0  tile -> the segment holding its first element
+//                       (each segment writes its tile starts; long ones with
+//                       the whole warp); empty segments reduce to d;
 //               pass 1  per tile: complete segments written, head / tail
 //                       pieces and flags recorded;
 //               pass 2  exclusive segmented scan of the tile tails (carry in);
@@ -105,60 +106,41 @@ __global__ void __launch_bounds__(256) irr_mid_kernel(const T* __restrict__ in, 
 
 // ------------------------------------------------------------ V_FLAT
 
-// pass 0a: tile_seg[t] = -1; empty segments reduce to d
-// pass 0b: a non-empty segment holding the first element of tile t claims it
+// pass 0: every tile t learns the (non-empty) segment holding its first
+// element: segment i writes tile_seg[t] for each tile start inside
+// [off[i], off[i+1]) -- each tile exactly once, so no initialisation and no
+// scan are needed.  A lane whose segment covers more than two tile starts
+// hands it to its whole warp (ballot), so a long segment costs ~1/32 of its
+// tiles per lane.  Empty segments reduce to d.
 template <typename T, bool RED>
 __global__ void __launch_bounds__(256) irr_claim_kernel(const int64_t* __restrict__ off, int64_t n,
                                                         int64_t* __restrict__ tile_seg, T* __restrict__ out, T d) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t a = off[i], b = off[i + 1];
-        if (a == b) {
-            if constexpr (RED) out[i] = d;
-            continue;
+    const int lane = threadIdx.x & 31;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    // uniform trip count per warp so the ballots see every lane
+    const int64_t base0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) - lane;
+    for (int64_t b0 = base0; b0 < n; b0 += stride) {
+        const int64_t i = b0 + lane;
+        int64_t t0 = 0, t1 = 0;  // tile starts [t0, t1) inside segment i
+        if (i < n) {
+            const int64_t a = off[i], b = off[i + 1];
+            if (a == b) {
+                if constexpr (RED) out[i] = d;
+            } else {
+                t0 = (a + kIrrTile - 1) / kIrrTile;
+                t1 = (b + kIrrTile - 1) / kIrrTile;
+            }
         }
-        const int64_t t = (a + kIrrTile - 1) / kIrrTile;
-        if (t * kIrrTile < b) tile_seg[t] = i;
-    }
-}
-
-// pass 0c: inclusive max-scan over tiles (segment ids grow with position);
-// a tile no segment start claimed continues the previous tile's segment.
-// One CTA; chunks of 1024 x 16 tiles, each thread's 16 loads in flight.
-__global__ void __launch_bounds__(1024) irr_tileseg_scan_kernel(int64_t* __restrict__ tile_seg, int64_t T) {
-    __shared__ int64_t wmax[32];
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    int64_t carry = -1;
-    for (int64_t c0 = 0; c0 < T; c0 += 1024 * 16) {
-        const int64_t k0 = c0 + (int64_t)t * 16;
-        int64_t v[16];
-#pragma unroll
-        for (int q = 0; q < 16; ++q) v[q] = k0 + q < T ? tile_seg[k0 + q] : -1;
-        int64_t mx = -1;
-#pragma unroll
-        for (int q = 0; q < 16; ++q) mx = max(mx, v[q]);
-        int64_t inc = mx;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int64_t y = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc = max(inc, y);
+        const bool longseg = t1 - t0 > 2;
+        if (!longseg)
+            for (int64_t t = t0; t < t1; ++t) tile_seg[t] = i;
+        unsigned ball = __ballot_sync(0xffffffffu, longseg);
+        while (ball) {  // the warp writes each long segment's tiles together
+            const int src = __ffs(ball) - 1;
+            ball &= ball - 1;
+            const int64_t s0 = __shfl_sync(0xffffffffu, t0, src), s1 = __shfl_sync(0xffffffffu, t1, src);
+            for (int64_t t = s0 + lane; t < s1; t += 32) tile_seg[t] = b0 + src;
         }
-        if (lane == 31) wmax[w] = inc;
-        __syncthreads();
-        int64_t pre = __shfl_up_sync(0xffffffffu, inc, 1);
-        if (lane == 0) pre = -1;
-        int64_t all = -1;
-        for (int k = 0; k < 32; ++k) {
-            if (k < w) pre = max(pre, wmax[k]);
-            all = max(all, wmax[k]);
-        }
-        pre = max(pre, carry);
-#pragma unroll
-        for (int q = 0; q < 16; ++q) {
-            pre = max(pre, v[q]);
-            if (k0 + q < T) tile_seg[k0 + q] = pre;
-        }
-        carry = max(carry, all);
-        __syncthreads();
     }
 }
 
@@ -524,12 +506,10 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         T* tail = head + Tn;
         T* cin = tail + Tn;
         uint32_t* tflag = (uint32_t*)(cin + Tn);
-        cudaError_t e = cudaMemsetAsync(tile_seg, 0xff, (size_t)Tn * 8, a.stream);  // -1
-        if (e != cudaSuccess) return e;
+        cudaError_t e;
         const unsigned gs = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.n, 256), 148 * 16));
         if (scan) irr_claim_kernel<T, false><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
         else irr_claim_kernel<T, true><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
-        irr_tileseg_scan_kernel<<<1, 1024, 0, a.stream>>>(tile_seg, Tn);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
         if (Tn > 0x7fffffffLL) return cudaErrorInvalidValue;
