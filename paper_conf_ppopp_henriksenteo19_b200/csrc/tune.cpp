@@ -261,21 +261,16 @@ size_t base_shape_bytes(Kind k, const int64_t* s) {
     }
 }
 
-// segred / segscan / colred / colscan: copy 1 = a second input copy after the
-// layout (only used when timing back-to-back calls, kBack > 1 below).
-bool two_inputs(Kind k) { return k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN; }
 size_t shape_bytes(Kind k, const int64_t* s) { return base_shape_bytes(k, s); }
 
-int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_t st, int copy = 0) {
-    // `in` of the seg/col layouts: the first region, or the second copy
-    char* const in2 = (two_inputs(k) && copy) ? scratch + base_shape_bytes(k, s) : nullptr;
+int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_t st) {
     k = mm_of(k);
     switch (k) {
     case K_SEGRED: {
         const int64_t n = s[0], m = s[1];
         char* out = scratch + align256(n * m * 4);
         char* ws = out + align256(n * 4);
-        char* in = in2 ? in2 : scratch;
+        char* in = scratch;
         return ifl_segred(in, out, n, m, IFL_F32, IFL_SUM, IFL_F_ID, nullptr, version, ws,
                           ifl_workspace_bytes("segred", n, m, 0, IFL_F32, -1), st, nullptr);
     }
@@ -283,7 +278,7 @@ int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_
         const int64_t n = s[0], m = s[1];
         char* out = scratch + align256(n * m * 4);
         char* ws = out + align256(n * m * 4);
-        char* in = in2 ? in2 : scratch;
+        char* in = scratch;
         return ifl_segscan(in, out, n, m, IFL_F32, IFL_SUM, IFL_F_ID, nullptr, 0, version, ws,
                            ifl_workspace_bytes("segscan", n, m, 0, IFL_F32, -1), st, nullptr);
     }
@@ -314,7 +309,7 @@ int run_forced(Kind k, const int64_t* s, int version, char* scratch, cudaStream_
         const int64_t n = s[0], m = s[1];
         const bool scan = k == K_COLSCAN;
         char* out = scratch + align256(n * m * 4);
-        char* in = in2 ? in2 : scratch;
+        char* in = scratch;
         char* ws = out + align256((scan ? n * m : m) * 4);
         return (scan ? ifl_colscan : ifl_colred)(in, out, n, m, IFL_F32, IFL_SUM, IFL_F_ID, nullptr, version, ws,
                                                  ws_bytes_of(k, s), st, nullptr);
@@ -438,21 +433,18 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
                 table[i * NV + slot] = warm;
                 continue;
             }
-            // each rep: L2 evicted (read-flush), then one call.  (Measured on B200:
-            // timing 4 back-to-back calls alternating two input copies instead
-            // moved the tuned thresholds further from the 2^26 test sweep's best
-            // -- 5.37 vs 5.60 TB/s -- so it stays at one call per rep.)
-            constexpr int kBack = 1;
-            const int back = two_inputs(k) ? kBack : 1;
+            // each rep: L2 evicted, then one call.  (Measured on B200: timing 4
+            // back-to-back calls alternating two input copies instead moved the
+            // tuned thresholds away from the 2^26 test sweep's best -- 5.37 vs
+            // 5.60 TB/s -- so it is one call per rep.)
             std::vector<float> ms(reps);
             for (int q = 0; q < reps; ++q) {
                 flush_l2(flush, st, q);  // evict the L2 (untimed)
                 cudaEventRecord(e0, st);
-                for (int b = 0; b < back; ++b) run_forced(k, s, v, (char*)scratch, st, b & 1);
+                run_forced(k, s, v, (char*)scratch, st);
                 cudaEventRecord(e1, st);
                 cudaEventSynchronize(e1);
                 cudaEventElapsedTime(&ms[q], e0, e1);
-                ms[q] /= back;
             }
             std::sort(ms.begin(), ms.end());
             table[i * NV + slot] = ms[reps / 2];
