@@ -15,12 +15,13 @@
 //               pass 0  tile -> the segment holding its first element
 //                       (each segment writes its tile starts; long ones with
 //                       the whole warp); empty segments reduce to d;
-//               pass 1  per tile: complete segments written, head / tail
-//                       pieces and flags recorded;
-//               pass 2  exclusive segmented scan of the tile tails (carry in);
-//               pass 3  segred: segments crossing into a tile finished as
-//                       carry (+) head; segscan: the tile rescanned with its
-//                       carry (two reads + one write per element).
+//               pass 1  per tile: complete segments written; segred: the
+//                       head / tail pieces of segments crossing tiles are
+//                       combined into their outputs atomically (done);
+//                       segscan: the tile's tail piece and flag recorded;
+//               pass 2  (segscan) exclusive segmented scan of the tile tails;
+//               pass 3  (segscan) the tile rescanned with its carry (two
+//                       reads + one write per element).
 #include <algorithm>
 
 #include "common.cuh"
@@ -112,7 +113,7 @@ __global__ void __launch_bounds__(256) irr_mid_kernel(const T* __restrict__ in, 
 // scan are needed.  A lane whose segment covers more than two tile starts
 // hands it to its whole warp (ballot), so a long segment costs ~1/32 of its
 // tiles per lane.  Empty segments reduce to d.
-template <typename T, bool RED>
+template <typename T, int OP, bool RED>
 __global__ void __launch_bounds__(256) irr_claim_kernel(const int64_t* __restrict__ off, int64_t n,
                                                         int64_t* __restrict__ tile_seg, T* __restrict__ out, T d) {
     const int lane = threadIdx.x & 31;
@@ -129,6 +130,9 @@ __global__ void __launch_bounds__(256) irr_claim_kernel(const int64_t* __restric
             } else {
                 t0 = (a + kIrrTile - 1) / kIrrTile;
                 t1 = (b + kIrrTile - 1) / kIrrTile;
+                // a segment crossing tiles is assembled by atomic combines
+                if constexpr (RED)
+                    if (a / kIrrTile != (b - 1) / kIrrTile) out[i] = identity<OP, T>();
             }
         }
         const bool longseg = t1 - t0 > 2;
@@ -204,6 +208,32 @@ __device__ __forceinline__ int64_t seg_search(const int64_t* o, int64_t lo, int6
         else hi = mid - 1;
     }
     return lo;
+}
+
+// *addr = *addr (+) v, atomically: the pieces of a segment that crosses tiles
+// are combined into its output in any order (every builtin (+) is associative
+// and commutative; f32 sums may differ from run to run only by association,
+// within the parity bound).
+template <int OP, typename T>
+__device__ __forceinline__ void atomic_combine(T* addr, T v) {
+    if constexpr (std::is_same<T, int>::value) {
+        if constexpr (OP == OP_SUM) { atomicAdd(addr, v); return; }
+        if constexpr (OP == OP_MIN) { atomicMin(addr, v); return; }
+        if constexpr (OP == OP_MAX) { atomicMax(addr, v); return; }
+        if constexpr (OP == OP_AND) { atomicAnd(addr, v); return; }
+        if constexpr (OP == OP_OR) { atomicOr(addr, v); return; }
+        if constexpr (OP == OP_XOR) { atomicXor(addr, v); return; }
+    } else {
+        if constexpr (OP == OP_SUM) { atomicAdd(addr, v); return; }
+    }
+    // PROD (both types), f32 MIN / MAX: compare-and-swap on the bit pattern
+    unsigned* a = reinterpret_cast<unsigned*>(addr);
+    unsigned old = *a, assumed;
+    do {
+        assumed = old;
+        const T cur = from_bits<T>(assumed);
+        old = atomicCAS(a, assumed, to_bits<T>(combine<OP>(cur, v)));
+    } while (old != assumed);
 }
 
 // Load the thread's 16 items of tile `tile` (identity past the end).
@@ -325,15 +355,15 @@ __device__ __forceinline__ void irr_tile(int64_t tile, int64_t Tn, T (&v)[kIrrIt
     if constexpr (MODE == 0) {
         if (stash) {
             const T val = combine<OP>(exv, stash_v);
-            if (exf) out[stash_seg] = val;  // started earlier in this tile: complete
-            else head[tile] = val;          // started before this tile: finished in pass 3
+            if (exf) out[stash_seg] = val;                  // started earlier in this tile: complete
+            else atomic_combine<OP>(out + stash_seg, val);  // the head piece of a crossing segment
         }
         if (t == 0) {
-            // head valid iff the tile's first segment started before the tile and ends in it
-            const int64_t a0 = O(s_lo), b0 = O(s_lo + 1);
-            const bool hv = a0 < base && b0 <= base + cnt;
-            tail[tile] = aggv;
-            tflag[tile] = (aggf ? 1u : 0u) | (hv ? 2u : 0u);
+            // the open piece at the tile's end (from its last start, with d, or
+            // the whole tile) belongs to a segment that continues past the tile
+            const int64_t e_last = base + cnt - 1;
+            const int64_t sl = staged ? s_lo + seg_search(s_off, 0, s_hi - s_lo, e_last) : seg_search(off, s_lo, s_hi, e_last);
+            if (O(sl + 1) > e_last + 1) atomic_combine<OP>(out + sl, aggv);
         }
     } else if constexpr (MODE == 1) {
         if (t == 0) {
@@ -461,15 +491,6 @@ __global__ void __launch_bounds__(1024) irr_tile_scan_kernel(const T* __restrict
     }
 }
 
-// pass 3 (segred): the segment entering tile t and ending in it
-template <typename T, int OP>
-__global__ void __launch_bounds__(256) irr_finish_kernel(T* __restrict__ out, const int64_t* __restrict__ tile_seg,
-                                                         const T* __restrict__ head, const uint32_t* __restrict__ tflag,
-                                                         const T* __restrict__ cin, int64_t Tn) {
-    for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < Tn; t += (int64_t)gridDim.x * blockDim.x)
-        if (tflag[t] & 2u) out[tile_seg[t]] = combine<OP>(cin[t], head[t]);
-}
-
 }  // namespace
 
 int64_t irr_tiles(int64_t total) { return ceil_div(total, kIrrTile); }
@@ -508,8 +529,8 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         uint32_t* tflag = (uint32_t*)(cin + Tn);
         cudaError_t e;
         const unsigned gs = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.n, 256), 148 * 16));
-        if (scan) irr_claim_kernel<T, false><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
-        else irr_claim_kernel<T, true><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
+        if (scan) irr_claim_kernel<T, OP, false><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
+        else irr_claim_kernel<T, OP, true><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
         if (Tn > 0x7fffffffLL) return cudaErrorInvalidValue;
@@ -519,15 +540,11 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         else
             irr_flat_kernel<T, OP, F, 0><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
                 in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
+        if (!scan) return cudaGetLastError();  // crossing segments were combined atomically
         irr_tile_scan_kernel<T, OP><<<1, 1024, 0, a.stream>>>(tail, tflag, cin, Tn);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
-        if (!scan) {
-            const unsigned gf = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(Tn, 256), 148 * 16));
-            irr_finish_kernel<T, OP><<<gf, 256, 0, a.stream>>>(out, tile_seg, head, tflag, cin, Tn);
-        } else {
-            irr_flat_kernel<T, OP, F, 2><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
-                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
-        }
+        irr_flat_kernel<T, OP, F, 2><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
+            in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
         return cudaGetLastError();
     });
 }
