@@ -5,7 +5,7 @@
 // elements.  Segment starts are arithmetic (multiples of m): no flag array is
 // read, and d is combined into every segment's first element.  Both kernels
 // are persistent (grid = resident CTAs) and stream tiles through a ring of
-// kSlots shared-memory slots filled by the TMA engine (cp.async.bulk +
+// shared-memory slots (kRedSlots / kScanSlots) filled by the TMA engine (cp.async.bulk +
 // mbarrier), so loads for the next tiles are in flight while a tile is
 // processed.  Per tile:
 //   * thread t takes its 20 consecutive elements (5 conflict-free LDS.128: the
@@ -43,7 +43,6 @@ namespace ifl {
 constexpr int FB = kFlatThreads;
 constexpr int FI = kFlatItems;
 constexpr int FT = (int)kFlatTile;
-constexpr int kSlots = 4;
 static_assert(FI % 4 == 0 && (FI / 4) % 2 == 1, "odd number of 16-byte chunks per thread");
 
 struct FlatHdr {
@@ -877,7 +876,6 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
     if (tiles > 0x3fffffffLL) return cudaErrorInvalidValue;
     const bool tma_in = ((uintptr_t)a.in % 16) == 0;
     const bool tma_out = ((uintptr_t)a.out % 16) == 0;
-    const size_t smem = (size_t)kSlots * FT * 4;
     uint8_t* ws = (uint8_t*)a.ws;
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
