@@ -341,8 +341,9 @@ def suite_mmtree():
     ifl.reset_thresholds()
     train, test = mm_shapes(20), mm_shapes(25)
     # 3-leaf tuning (the row level off), then the 5-leaf tree
-    a3, b3, _ = ifl.tune("redomap2.f32", train, reps=3, cost=1)
-    t_top, t_intra, tbl = ifl.tune("redomap2.f32.tree", train, reps=3, cost=1)
+    # the k = 20 shapes run for microseconds: 9 repetitions (median) per leaf
+    a3, b3, _ = ifl.tune("redomap2.f32", train, reps=9, cost=1)
+    t_top, t_intra, tbl = ifl.tune("redomap2.f32.tree", train, reps=9, cost=1)
     rt, ri = ifl.get_thresholds("redomap2.f32.row")
     rows = []
     for (n, m, p) in test:
