@@ -77,19 +77,31 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
     //   forward  y'_j = alpha_j y'_{j-1} + y_j: lane-local scan from 0, then
     //            y'_k = loc_k + P_k * p  with P_k = alpha_{j0} ... alpha_{j0+k}
     //            and p the group-exclusive prefix (the value entering the lane);
-    //   backward x_j = delta_j x_{j+1} + eps_j, mirrored with suffix products D_k.
-    float P[IT], D[IT];
+    //   backward x_j = delta_j x_{j+1} + eps_j, mirrored with suffix products.
+    // The lane's items are scanned as two independent half chains (H = IT/2
+    // items each, twice the instruction-level parallelism of one chain); the
+    // halves are joined with their slope products:
+    //   Q[k] = alpha_{j0+h0} ... alpha_{j0+k}   (h0 = 0 for the first half, H for the second)
+    //   E[k] = delta_{j0+k} ... delta_{j0+h1}   (h1 = H-1 for the first half, IT-1 for the second)
+    constexpr int H = IT / 2;
+    float Q[IT], E[IT];
     {
         float pr = 1.f;
 #pragma unroll
-        for (int k = 0; k < IT; ++k) P[k] = pr = pr * al[k];
+        for (int k = 0; k < H; ++k) Q[k] = pr = pr * al[k];
         pr = 1.f;
 #pragma unroll
-        for (int k = IT - 1; k >= 0; --k) D[k] = pr = pr * de[k];
+        for (int k = H; k < IT; ++k) Q[k] = pr = pr * al[k];
+        pr = 1.f;
+#pragma unroll
+        for (int k = IT - 1; k >= H; --k) E[k] = pr = pr * de[k];
+        pr = 1.f;
+#pragma unroll
+        for (int k = H - 1; k >= 0; --k) E[k] = pr = pr * de[k];
     }
     float raf[5], rab[5];  // slope of the running inclusive map before each shuffle round
     {
-        float af = P[IT - 1], ab = D[0];
+        float af = Q[H - 1] * Q[IT - 1], ab = E[0] * E[H];
 #pragma unroll
         for (int r = 0; r < 5; ++r) {
             const int off = 1 << r;
@@ -104,10 +116,14 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
         }
     }
     for (int64_t t = 0; t < numT; ++t) {
-        // (x) forward
-        float g = 0.f;
+        // (x) forward: half chains from 0, lane total g = gB + Q_B * gA
+        float gA = 0.f, gB = 0.f;
 #pragma unroll
-        for (int k = 0; k < IT; ++k) yv[k] = g = fmaf(al[k], g, yv[k]);
+        for (int k = 0; k < H; ++k) {
+            yv[k] = gA = fmaf(al[k], gA, yv[k]);
+            yv[H + k] = gB = fmaf(al[H + k], gB, yv[H + k]);
+        }
+        float g = fmaf(Q[IT - 1], gA, gB);
 #pragma unroll
         for (int r = 0; r < 5; ++r) {
             const int off = 1 << r;
@@ -118,12 +134,20 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
         }
         float p = __shfl_up_sync(0xffffffffu, g, 1, G);
         if (gl == 0) p = 0.f;
+        const float vA = fmaf(Q[H - 1], p, gA);  // y' at the end of the first half
 #pragma unroll
-        for (int k = 0; k < IT; ++k) yv[k] = fmaf(P[k], p, yv[k]) * ib[k];  // eps_j = y'_j / beta_j
-        // (.) backward
-        float h = 0.f;
+        for (int k = 0; k < H; ++k) {
+            yv[k] = fmaf(Q[k], p, yv[k]) * ib[k];  // eps_j = y'_j / beta_j
+            yv[H + k] = fmaf(Q[H + k], vA, yv[H + k]) * ib[H + k];
+        }
+        // (.) backward: half chains from 0 (from each half's right end)
+        float hA = 0.f, hB = 0.f;
 #pragma unroll
-        for (int k = IT - 1; k >= 0; --k) yv[k] = h = fmaf(de[k], h, yv[k]);
+        for (int k = H - 1; k >= 0; --k) {
+            yv[k] = hA = fmaf(de[k], hA, yv[k]);
+            yv[H + k] = hB = fmaf(de[H + k], hB, yv[H + k]);
+        }
+        float h = fmaf(E[0], hB, hA);
 #pragma unroll
         for (int r = 0; r < 5; ++r) {
             const int off = 1 << r;
@@ -134,8 +158,12 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
         }
         float u = __shfl_down_sync(0xffffffffu, h, 1, G);
         if (gl == G - 1) u = 0.f;
+        const float xB = fmaf(E[H], u, hB);  // x at the start of the second half
 #pragma unroll
-        for (int k = 0; k < IT; ++k) yv[k] = fmaf(D[k], u, yv[k]);
+        for (int k = 0; k < H; ++k) {
+            yv[H + k] = fmaf(E[H + k], u, yv[H + k]);
+            yv[k] = fmaf(E[k], xB, yv[k]);
+        }
     }
     if (vec) {
 #pragma unroll
