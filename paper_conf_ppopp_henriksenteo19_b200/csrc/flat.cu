@@ -529,13 +529,18 @@ cudaError_t launch_segred_rows512(const SegArgs& a) {
     });
 }
 
+// A warp per row combines its P piece partials (lanes stride over the pieces,
+// a shuffle tree joins them): no single thread walks hundreds of partials.
 template <typename T, int OP>
 __global__ void __launch_bounds__(256) flat_red_split_fix(const T* __restrict__ part, T* __restrict__ out, int64_t n,
                                                           int P, T d) {
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-        T r = d;
-        for (int p = 0; p < P; ++p) r = combine<OP>(r, part[i * P + p]);
-        out[i] = r;
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += nw) {
+        T r = identity<OP, T>();
+        for (int p = lane; p < P; p += 32) r = combine<OP>(r, part[i * P + p]);
+        r = warp_reduce<OP>(r);
+        if (lane == 0) out[i] = combine<OP>(d, r);
     }
 }
 
@@ -617,8 +622,8 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
     __shared__ alignas(8) uint64_t full[kScanSlots], empty[kScanSlots];
     __shared__ SlotMeta meta[kScanSlots];
     __shared__ uint32_t s_tag;
-    __shared__ T s_wval[FB / 32];
-    __shared__ uint32_t s_wflag[FB / 32];
+    __shared__ T s_wval[2][FB / 32];  // double-buffered by item parity: no barrier between phase-1 tiles
+    __shared__ uint32_t s_wflag[2][FB / 32];
     __shared__ int s_lbterm[FB / 32];
     __shared__ T s_lbval[FB / 32];
     unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | done:32}
@@ -726,7 +731,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
                 local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
                 uint32_t exf, aggf;
                 T exv, aggv;
-                cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+                cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[vi & 1], s_wflag[vi & 1]);
                 // everyone's items are in registers (the barrier inside the scan): free the slot
                 if (t == 0) {
                     if (pend_slot >= 0) {  // a phase-3 store before this phase-1 run
@@ -738,7 +743,6 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
                 }
                 run_v = aggf ? aggv : combine<OP>(run_v, aggv);
                 run_f |= aggf;
-                consumer_sync();  // s_wval reuse
             }
             if (t == 0)
                 st_relaxed_u64(&status[c], pack_status(tag, (run_f || !carry_needed) ? ST_P : ST_A, run_f,
@@ -805,7 +809,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(
             local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
             uint32_t exf, aggf;
             T exv, aggv;
-            cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
+            cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[vi & 1], s_wflag[vi & 1]);
             {
                 const T carry_t = exf ? exv : combine<OP>(carry, exv);
                 const int lim = min(tp.nx0, tp.nvalid);
@@ -912,7 +916,7 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
             ks<<<(unsigned)(a.n * P), kSplitThreads, 0, a.stream>>>((const T*)a.in, a.m, P, head, d);
             cudaError_t e = cudaGetLastError();
             if (e != cudaSuccess) return e;
-            const int g2 = (int)std::min<int64_t>(ceil_div(a.n, 256), (int64_t)sm_count() * 4);
+            const int g2 = (int)std::min<int64_t>(ceil_div(a.n, 8), (int64_t)sm_count() * 16);
             flat_red_split_fix<T, OP><<<g2, 256, 0, a.stream>>>(head, (T*)a.out, a.n, P, d);
             return cudaGetLastError();
         }
