@@ -508,7 +508,11 @@ cudaError_t launch_segred_rows512(const SegArgs& a) {
             attr[0].val.clusterDim.z = 1;
             cfg.attrs = attr;
             cfg.numAttrs = 1;
-            auto kc = segred_cluster_kernel<T, OP, F, kSplitThreads>;
+            // very few rows (<= 4): 16-CTA clusters of 1024-thread CTAs (B200: n = 2 / 4
+            // 145 / 79 us -> 83 / 51 us; n = 8 is faster with 512 threads: 49 vs 60 us)
+            const bool big = C == 16 && a.n * 32 <= (int64_t)sm_count();
+            if (big) cfg.blockDim = dim3(1024);
+            auto kc = big ? segred_cluster_kernel<T, OP, F, 1024> : segred_cluster_kernel<T, OP, F, kSplitThreads>;
             if (C > 8) cudaFuncSetAttribute(kc, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);  // opt-in
             cudaError_t e = cudaLaunchKernelEx(&cfg, kc, (const T*)a.in, (T*)a.out, a.m, bits_to<T>(a.ne_bits));
             if (e != cudaSuccess && C > 8) {  // 16-CTA clusters refused: the portable size
