@@ -59,6 +59,10 @@ def lib() -> ctypes.CDLL:
             "oracle_redomap2": [_vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int],
             "oracle_tridag": [_vp, _vp, _vp, _vp, _vp, _c_i64, _c_i64, _c_i64, _vp],
             "oracle_lvc": [_vp] * 10 + [_c_i64] * 4 + [_vp],
+            "oracle_segred2_i32": [_vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int, _c_int, ctypes.c_int32,
+                                   ctypes.c_int32],
+            "oracle_segred2_f32": [_vp, _vp, _c_i64, _c_i64, _c_i64, _c_int, _c_int, _c_int, ctypes.c_double,
+                                   ctypes.c_double],
             "oracle_segarg_i32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int],
             "oracle_segarg_f32": [_vp, _vp, _vp, _c_i64, _c_i64, _c_int],
             "oracle_segred_irr_i32": [_vp, _vp, _vp, _c_i64, _c_int, _c_int, ctypes.c_int32],
@@ -276,3 +280,21 @@ def segarg(x: np.ndarray, which: str = "min"):
     fn = lib().oracle_segarg_i32 if x.dtype == np.int32 else lib().oracle_segarg_f32
     _check(fn(_ptr(x), _ptr(val), _ptr(idx), n, m, 1 if which == "max" else 0))
     return val, idx
+
+
+def segred2(x: np.ndarray, op_o: str = "sum", op_i: str = "max", f: str = "id", d_o=None, d_i=None):
+    """Nested reduce (G9's e_rec): out[i] = d_o (+)_j (d_i (x)_q f(x[i,j,q]))
+    over an [n][m][k] array; (+) = op_o, (x) = op_i."""
+    x = np.ascontiguousarray(x)
+    n, m, k = x.shape
+    if x.dtype == np.int32:
+        do = canonical_ne(op_o, "i32") if d_o is None else int(d_o)
+        di = canonical_ne(op_i, "i32") if d_i is None else int(d_i)
+        out = np.empty(n, np.int32)
+        _check(lib().oracle_segred2_i32(_ptr(x), _ptr(out), n, m, k, OPS[op_o], OPS[op_i], MAPS[f], _i32(do), _i32(di)))
+        return out
+    do = canonical_ne(op_o, "f32") if d_o is None else float(np.float32(d_o))
+    di = canonical_ne(op_i, "f32") if d_i is None else float(np.float32(d_i))
+    out = np.empty(n, np.float64)
+    _check(lib().oracle_segred2_f32(_ptr(x), _ptr(out), n, m, k, OPS[op_o], OPS[op_i], MAPS[f], do, di))
+    return out

@@ -560,3 +560,25 @@ def test_segarg_numpy_and_closed_forms(orc):
     assert (orc.segarg(big, "min")[1] == 0).all()
     v, i = orc.segarg(np.zeros((3, 0), np.float32), "max")
     assert (i == -1).all() and np.isneginf(v).all()
+
+
+# ---------------------------------------- segred2: nested reduce (G9 e_rec, NEXT-2)
+
+
+def test_segred2_composition_and_closed_forms(orc):
+    # the nest = the row oracle applied twice (inner over k, outer over m)
+    x = gen.generate("I32_FULL", 71, 5 * 6 * 7).numpy().reshape(5, 6, 7)
+    for op_o, op_i in (("sum", "max"), ("xor", "sum"), ("min", "and"), ("prod", "or")):
+        inner = orc.segred(np.ascontiguousarray(x.reshape(30, 7)), op_i, "sq", 3).reshape(5, 6)
+        want = orc.segred(np.ascontiguousarray(inner), op_o, "id", -2)
+        np.testing.assert_array_equal(orc.segred2(x, op_o, op_i, "sq", -2, 3), want)
+    # same operator at both levels = one flat reduce of each [m*k] row (associativity)
+    np.testing.assert_array_equal(orc.segred2(x, "sum", "sum"), orc.segred(np.ascontiguousarray(x.reshape(5, 42)), "sum"))
+    # closed form: x[i][j][q] = q -> sum over j of max over q = m*(k-1)
+    q = np.tile(np.arange(7, dtype=np.int32), (4, 3, 1))
+    np.testing.assert_array_equal(orc.segred2(q, "sum", "max"), np.full(4, 3 * 6))
+    # empty levels: k = 0 -> every g = d_i; m = 0 -> d_o
+    np.testing.assert_array_equal(orc.segred2(np.zeros((2, 3, 0), np.int32), "sum", "max", d_i=5), [15, 15])
+    np.testing.assert_array_equal(orc.segred2(np.zeros((2, 0, 4), np.int32), "sum", "max", d_o=9), [9, 9])
+    xf = gen.generate("F32_SIGNED", 72, 3 * 8 * 9).numpy().reshape(3, 8, 9)
+    np.testing.assert_allclose(orc.segred2(xf, "sum", "max"), xf.astype(np.float64).max(axis=2).sum(axis=1), rtol=1e-12)
