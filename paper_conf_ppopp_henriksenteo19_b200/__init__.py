@@ -31,7 +31,8 @@ MAPS = {"id": 0, "sq": 1, "abs": 2}
 VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3, "row_top": 4, "row_middle": 5}
 VERSION_NAMES = {v: k for k, v in VERSIONS.items()}
 SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4",
-         "segred.irr", "segscan.irr", "segarg.b4", "redomap2.f32.row", "redomap2.bf16.row")
+         "segred.irr", "segscan.irr", "segarg.b4", "redomap2.f32.row", "redomap2.bf16.row",
+         "segred2.b4")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -64,6 +65,7 @@ _SIGS = {
     "ifl_segscan_seeded": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_colred": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_colscan": ([_vp, _vp, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
+    "ifl_segred2": ([_vp, _vp, _i64, _i64, _i64, _int, _int, _int, _int, _vp, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segarg": ([_vp, _vp, _vp, _i64, _i64, _int, _int, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segred_irr": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
     "ifl_segscan_irr": ([_vp, _vp, _vp, _i64, _i64, _i64, _int, _int, _int, _vp, _int, _vp, _sz, _vp, _vp], _int),
@@ -319,6 +321,32 @@ def colred(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stre
 def colscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False):
     """out[i,j] = ne (+) f(x[0,j]) (+) ... (+) f(x[i,j]) -- column-wise inclusive scan (G4 with scan)."""
     return _col(True, x, op, f, ne, version, out, ws, stream, return_choice)
+
+
+# ------------------------------------------------------------- segred2
+
+
+def segred2(x, op_o="sum", op_i="max", f="id", ne_o=None, ne_i=None, version="auto", out=None, ws=None,
+            stream=None, return_choice=False):
+    """Nested reduce over an [n][m][k] tensor (G9's e_rec):
+    out[i] = ne_o (+)_j (ne_i (x)_q f(x[i,j,q])), (+) = op_o, (x) = op_i."""
+    if x.dim() != 3 or not x.is_contiguous() or not x.is_cuda:
+        raise ValueError("expected a contiguous [n][m][k] CUDA tensor")
+    dt = _TORCH_DT.get(x.dtype)
+    if dt not in ("i32", "f32"):
+        raise TypeError(f"unsupported dtype {x.dtype}")
+    n, m, k = x.shape
+    if out is None:
+        out = torch.empty(n, dtype=x.dtype, device=x.device)
+    wb = lib().ifl_workspace_bytes(b"segred2", n, m, k, DTYPES[dt], VERSIONS[version])
+    if ws is None and wb:
+        ws = workspace(wb, x.device, "seg2")
+    c = ifl_choice()
+    rc = lib().ifl_segred2(x.data_ptr(), out.data_ptr(), n, m, k, DTYPES[dt], OPS[op_o], OPS[op_i], MAPS[f],
+                           _ne_buf(ne_o, dt), _ne_buf(ne_i, dt), VERSIONS[version], _ptr(ws),
+                           0 if ws is None else ws.numel() * ws.element_size(), _stream(stream), ctypes.byref(c))
+    _check(rc, "ifl_segred2")
+    return (out, _choice_out(c)) if return_choice else out
 
 
 # -------------------------------------------------------------- segarg

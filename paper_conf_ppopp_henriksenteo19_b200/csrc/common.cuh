@@ -130,6 +130,7 @@ struct Acc<OP_SUM, float> {
         const float y = __fsub_rn(x, c);
         const float t = __fadd_rn(s, y);
         c = __fsub_rn(__fsub_rn(t, s), y);
+        if (!isfinite(c)) c = 0.0f;  // an infinite term: the sum is +-inf (or NaN), no compensation
         s = t;
     }
     __device__ __forceinline__ float get() const { return s; }

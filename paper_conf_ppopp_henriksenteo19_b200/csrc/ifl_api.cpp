@@ -40,7 +40,7 @@ constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE ke
 
 const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
                               "colred.b4", "colscan.b4", "segred.irr", "segscan.irr", "segarg.b4",
-                              "redomap2.f32.row", "redomap2.bf16.row"};
+                              "redomap2.f32.row", "redomap2.bf16.row", "segred2.b4"};
 
 struct Table {
     std::mutex mu;
@@ -301,6 +301,12 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
     if (strcmp(entry, "redomap2") == 0) return ifl::redomap2_ws_bytes(n, m, p, version);
     if (strcmp(entry, "colred") == 0 || strcmp(entry, "colscan") == 0) return ifl::col_ws_bytes(n, m, version);
     if (strcmp(entry, "segarg") == 0) return ifl::arg_ws_bytes(n, m, version);
+    if (strcmp(entry, "segred2") == 0) {  // (n, m, k): V_FLAT's inner results + the larger flat workspace
+        if (version != IFL_V_FLAT && version != IFL_AUTO) return 0;
+        if (mul_overflows(n, m) || mul_overflows(n * m, p)) return 0;
+        return (((size_t)(n * m) * 4 + 255) & ~(size_t)255) +
+               std::max(n * m * p > 0 ? ifl::flat_ws_bytes(n * m * p) : 0, n * m > 0 ? ifl::flat_ws_bytes(n * m) : 0);
+    }
     if (strcmp(entry, "segred_irr") == 0 || strcmp(entry, "segscan_irr") == 0) return ifl::irr_ws_bytes(m, version);
     if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
     if (strcmp(entry, "lvc") == 0)  // (numX, numY): the coefficient scans of both sites
@@ -449,6 +455,44 @@ int ifl_irr_inspect(const int64_t* offsets, int64_t n, int64_t total, void* ws16
                                 "off[n] = total = %lld; got off[n] = %lld)", (long long)total, (long long)last);
     if (max_len) *max_len = (int64_t)res[0];
     return IFL_OK;
+}
+
+int ifl_segred2(const void* in, void* out, int64_t n, int64_t m, int64_t k, int dt, int op_o, int op_i, int f,
+                const void* ne_o, const void* ne_i, int version, void* ws, size_t ws_bytes, void* stream,
+                ifl_choice* choice) {
+    const char* what = "ifl_segred2";
+    if (n < 0 || m < 0 || k < 0) return fail(IFL_EINVAL, "%s: negative size", what);
+    if (mul_overflows(n, m) || mul_overflows(n * m, k) || mul_overflows(n * m * k, 4))
+        return fail(IFL_EINVAL, "%s: size overflow", what);
+    int rc = validate_seg(false, in, out, n, m * k, dt, op_i, f, version, what);
+    if (rc) return rc;
+    rc = validate_seg(false, in, out, n, m * k, dt, op_o, IFL_F_ID, version, what);
+    if (rc) return rc;
+    if (overlap(in, (size_t)(n * m * k) * 4, out, (size_t)n * 4)) return fail(IFL_EINVAL, "%s: out overlaps in", what);
+    uint32_t bo = canonical_bits(dt, op_o), bi = canonical_bits(dt, op_i);
+    if (ne_o) memcpy(&bo, ne_o, 4);
+    if (ne_i) memcpy(&bi, ne_i, 4);
+    ifl_choice c;
+    select_version("segred2.b4", n, m, 0, true, &c);  // Par_top = n, Par_mid = n*min(m, 1024) (R3)
+    if (version != IFL_AUTO) c.version = version;
+    if (choice) *choice = c;
+    if (n == 0) return IFL_OK;
+    cudaStream_t st = (cudaStream_t)stream;
+    if (m == 0) return cuda_status(ifl::launch_fill(out, n, bo, st), what);
+    if (c.version == IFL_V_FLAT) {
+        // G9 flattened: segred^1 over the [n*m][k] inner segments, then over [n][m]
+        const size_t tb = ((size_t)(n * m) * 4 + 255) & ~(size_t)255;
+        const size_t need = ifl_workspace_bytes("segred2", n, m, k, dt, IFL_V_FLAT);
+        if (!ws || ws_bytes < need)
+            return fail(IFL_EWORKSPACE, "%s: V_FLAT needs %zu workspace bytes, got %zu", what, need, ws_bytes);
+        void* tmp = ws;
+        void* fws = (char*)ws + tb;
+        rc = ifl_segred(in, tmp, n * m, k, dt, op_i, f, &bi, IFL_AUTO, fws, ws_bytes - tb, stream, nullptr);
+        if (rc) return rc;
+        return ifl_segred(tmp, out, n, m, dt, op_o, IFL_F_ID, &bo, IFL_AUTO, fws, ws_bytes - tb, stream, nullptr);
+    }
+    ifl::Seg2Args a{in, out, n, m, k, dt, op_o, op_i, f, bo, bi, st};
+    return cuda_status(ifl::launch_seg2(a, c.version), what);
 }
 
 int ifl_segarg(const void* in, void* val, int32_t* idx, int64_t n, int64_t m, int dt, int which, int version,

@@ -53,6 +53,17 @@ size_t col_ws_bytes(int64_t n, int64_t m, int version);
 cudaError_t launch_col(const SegArgs& a, bool scan, int version);
 constexpr int64_t kColGroup = 8;  // threads per column in V_MIDDLE (reading R3's group size)
 
+// Nested reduce [n][m][k] (seg2.cu): out[i] = d_o (+)_j (d_i (x)_q f(x[i][j][q])).
+struct Seg2Args {
+    const void* in;
+    void* out;
+    int64_t n, m, k;
+    int dt, op_o, op_i, f;
+    uint32_t ne_o, ne_i;
+    cudaStream_t stream;
+};
+cudaError_t launch_seg2(const Seg2Args& a, int version);  // V_TOP / V_MIDDLE (V_FLAT: two segreds, ifl_api.cpp)
+
 // Tuple-valued per-row argmin / argmax (arg.cu).
 struct ArgArgs {
     const void* in;

@@ -387,3 +387,11 @@ def test_mm_tree_guard(L):
         assert L.ifl_redomap2(256, 512, 1024, 64, 10000, 4, 1, 1, 5, None, 0, None, None) == ifl.IFL_ENOTFIT
     finally:
         ifl.reset_thresholds()
+
+
+def test_segred2_validation(L):
+    assert L.ifl_segred2(256, 512, -1, 2, 2, 1, 0, 3, 0, None, None, -1, None, 0, None, None) == ifl.IFL_EINVAL
+    assert L.ifl_segred2(256, 512, 2, 2, 2, 1, 4, 0, 0, None, None, -1, None, 0, None, None) == ifl.IFL_EUNSUPPORTED
+    assert L.ifl_segred2(1 << 20, 1 << 30, 4, 64, 64, 1, 0, 3, 0, None, None, 2, None, 0, None, None) == ifl.IFL_EWORKSPACE
+    assert L.ifl_segred2(256, 512, 0, 4, 4, 1, 0, 3, 0, None, None, -1, None, 0, None, None) == 0
+    assert ifl.workspace_bytes("segred2", 4, 64, 64, version="flat") >= 4 * 64 * 4
