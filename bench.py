@@ -429,7 +429,7 @@ def main():
                     help="skip the per-shape forced-version timings (for the ncu launch list of the timed region)")
     ap.add_argument("--thresholds", default=None)
     ap.add_argument("--detail", default=os.path.join(ROOT, "gpurun_out", "bench_detail.json"))
-    ap.add_argument("--suite", default="sweep", choices=["sweep", "config0", "redomap2", "tridag", "dist", "lvc", "col", "irr", "arg", "mmtree"],
+    ap.add_argument("--suite", default="sweep", choices=["sweep", "config0", "redomap2", "tridag", "dist", "lvc", "col", "irr", "arg", "mmtree", "seg2"],
                     help="sweep = the contract line (configs[1]); the others measure one more SURVEY 8(a) row")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)

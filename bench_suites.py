@@ -327,6 +327,67 @@ def suite_col():
     return line
 
 
+# -------------------------------------------------------------------- segred2
+
+
+def seg2_shapes(lg):
+    out = []
+    for a in range(0, lg + 1, 2):  # n = 2^a, the rest split between m and k
+        r = lg - a
+        out.append((1 << a, 1 << (r // 2), 1 << (r - r // 2)))
+    return out
+
+
+def suite_seg2():
+    """NEXT-2 (ii): the nested reduce (G9's e_rec),
+    sum of per-segment maxima over [n][m][k] f32 with n*m*k = 2^26; thresholds
+    from ifl_tune_search over forced-version timings of the 2^25 / 2^27 sets."""
+    hbm, _, src = peaks()
+    ifl.reset_thresholds()
+
+    def run(lg, seed, versions):
+        x = gen.generate("F32_SIGNED", seed, 1 << lg, "cuda")
+        out = torch.empty(1 << lg, device="cuda")
+        res = []
+        for (n, m, k) in seg2_shapes(lg):
+            xv = x.view(n, m, k)
+            ws = ifl.workspace(ifl.workspace_bytes("segred2", n, m, k), "cuda", "seg2")
+            r = {"n": n, "m": m, "k": k}
+            for v in versions:
+                if v == "top" and n < 4096:
+                    r[v] = None  # a few threads walking 2^14+ elements each: cannot win (P:380)
+                    continue
+                r[v] = gtime(lambda: ifl.segred2(xv, "sum", "max", version=v, out=out[:n], ws=ws)) * 1e3
+            if "auto" in versions:
+                r["chosen"] = ifl.segred2(xv, "sum", "max", out=out[:n], ws=ws, return_choice=True)[1].version
+            res.append(r)
+        return res
+
+    pt, pm, tbl = [], [], []
+    for lg in (25, 27):
+        for r in run(lg, 30 + lg, ("top", "middle", "flat")):
+            c = ifl.select("segred2.b4", r["n"], r["m"])
+            pt.append(c.par_top)
+            pm.append(c.par_mid)
+            tbl.append([float("inf") if r[v] is None else r[v] for v in ("top", "middle", "flat")])
+    a, b, npaths = ifl.tune_search(pt, pm, tbl, cost=1)
+    ifl.set_thresholds("segred2.b4", a, b)
+    rows = run(26, 2, ("top", "middle", "flat", "auto"))
+    for r in rows:
+        best = min(r[v] for v in ("top", "middle", "flat") if r[v] is not None)
+        r["best_over_auto"] = round(best / r["auto"], 4)
+        r["GBps"] = round((4 * r["n"] * r["m"] * r["k"] + 4 * r["n"]) / (r["auto"] * 1e-6) / 1e9, 1)
+    tot = sum(4 * r["n"] * r["m"] * r["k"] + 4 * r["n"] for r in rows) / (sum(r["auto"] for r in rows) * 1e-6) / 1e9
+    line = base_line("nested reduce (sum of per-segment max) GB/s over [n][m][k] shapes", round(tot, 1), "GB/s",
+                     {"workload": "SURVEY 8(f) NEXT-2 (ii): f32, n*m*k = 2^26, n = 4^0..4^13", "thresholds":
+                      {"t_top": a, "t_intra": b, "paths": npaths}})
+    line["min_shape_best_over_auto"] = min(r["best_over_auto"] for r in rows)
+    line["roofline"] = {"bound": "hbm", "kernel": "segred2 sweep (AUTO)", "achieved": round(tot, 1), "peak": hbm,
+                        "unit": "GB/s", "frac": round(tot / hbm, 4), "traffic": None, "peak_source": src}
+    line["shapes"] = rows
+    return line
+
+
 # -------------------------------------------------------------------- mmtree
 
 
@@ -569,4 +630,5 @@ def suite_dist():
 
 
 SUITES = {"config0": suite_config0, "redomap2": suite_redomap2, "tridag": suite_tridag, "dist": suite_dist,
-          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr, "arg": suite_arg, "mmtree": suite_mmtree}
+          "lvc": suite_lvc, "col": suite_col, "irr": suite_irr, "arg": suite_arg, "mmtree": suite_mmtree,
+          "seg2": suite_seg2}
