@@ -448,14 +448,54 @@ __global__ void __launch_bounds__(1024) segred_mid_kernel(const T* __restrict__ 
     if (g == 0 && i < n) out[i] = combine<OP>(d, acc);
 }
 
+// Aligned rows (m % 4 == 0, 16-byte aligned base) of at most 16*G elements:
+// every thread owns <= 4 128-bit vectors of its row, all issued before the
+// first combine, with 32-bit index arithmetic and no scalar head/tail loops.
+// B200, n*m = 2^26 f32, m = 32..4096: 39-41 us (6.6-6.9 TB/s) against
+// 45-48 us for the generic kernel below.  Taking two or four slabs of rows
+// per CTA (8/16 loads in flight) measured slower (44-55 us).
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(512) segred_mid_vec_kernel(const T* __restrict__ in, T* __restrict__ out,
+                                                             int64_t n, int m, T d, int G) {
+    __shared__ T red[32];
+    using V = typename Vec4<T>::type;
+    const int g = threadIdx.x % G;
+    const int64_t i = (int64_t)blockIdx.x * (blockDim.x / G) + threadIdx.x / G;
+    const int nvec = m >> 2;
+    const T* row = in + i * m;
+    V q[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+        if (i < n && g + u * G < nvec) q[u] = ldg_stream4(row + 4 * (g + u * G));
+    T acc = identity<OP, T>();
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+        if (i < n && g + u * G < nvec) {
+            T e[4];
+            unpack4<T>(q[u], e);
+            acc = combine<OP>(acc, combine<OP>(combine<OP>(apply_map<F>(e[0]), apply_map<F>(e[1])),
+                                               combine<OP>(apply_map<F>(e[2]), apply_map<F>(e[3]))));
+        }
+    acc = group_reduce<OP>(acc, G, red);
+    if (g == 0 && i < n) out[i] = combine<OP>(d, acc);
+}
+
 cudaError_t launch_segred_mid(const SegArgs& a) {
     if (a.m >= 8192) return launch_segred_rows512(a);  // one 512-thread group per row (flat.cu)
+    const int G = mid_group_size(a.m);
+    const int B = G > 256 ? G : 256;
+    const int64_t grid = ceil_div(a.n, B / G);
+    if (a.m > 0 && a.m % 4 == 0 && ((uintptr_t)a.in & 15u) == 0 && a.m <= 16 * (int64_t)G)
+        return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+            using T = decltype(tt);
+            constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+            segred_mid_vec_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>(
+                (const T*)a.in, (T*)a.out, a.n, (int)a.m, bits_to<T>(a.ne_bits), G);
+            return cudaGetLastError();
+        });
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
-        const int G = mid_group_size(a.m);
-        const int B = G > 256 ? G : 256;
-        const int64_t grid = ceil_div(a.n, B / G);
         segred_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>((const T*)a.in, (T*)a.out, a.n, a.m,
                                                                         bits_to<T>(a.ne_bits), G);
         return cudaGetLastError();

@@ -233,3 +233,18 @@ def test_segred_long_rows_split_and_cluster(ifl, orc, dt, version):
             x, xd = gen_for(op, dt, 17, n, m, misalign=mis)
             got = ifl.segred(xd, op, "sq" if op != "prod" else "id", ne=(2 if dt == "i32" else 0.5), version=version)
             assert_parity(orc, x, got, False, op, "sq" if op != "prod" else "id", 2 if dt == "i32" else 0.5, dt)
+
+
+@pytest.mark.parametrize("f", ["id", "sq", "abs"])
+def test_middle_aligned_rows(ifl, orc, f):
+    """V_MIDDLE's vector kernel (m % 4 == 0, aligned, m <= 16*G): every group
+    size G = 1..512 (rows of 4..8188), ragged n, all ops, d applied once."""
+    for dt, ops in (("i32", OPS_I), ("f32", OPS_F)):
+        for op in ops:
+            for (n, m) in [(37, 4), (9, 12), (300, 16), (129, 20), (65, 64), (17, 100), (5, 256),
+                           (3, 2048), (7, 4096), (2, 8188)]:
+                x, xd = gen_for(op, dt, 5, n, m)
+                got = ifl.segred(xd, op, f, version="middle")
+                assert_parity(orc, x, got, False, op, f, None, dt)
+    x, xd = gen_for("sum", "i32", 6, 11, 4096)
+    assert_parity(orc, x, ifl.segred(xd, "max", "abs", ne=-3, version="middle"), False, "max", "abs", -3, "i32")
