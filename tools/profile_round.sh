@@ -23,7 +23,7 @@ cap() {  # name op version n m kernel-regex
 cap segscan_flat_n1      segscan flat   1        67108864 flat_scan
 cap segscan_flat_n4096   segscan flat   4096     16384    flat_scan
 cap segred_flat_n1       segred  flat   1        67108864 flat_red_kernel
-cap segred_middle_n1024  segred  middle 1024     65536    segred_mid
+cap segred_middle_n2e16  segred  middle 65536    1024     segred_mid_vec
 cap segscan_middle_n2e18 segscan middle 262144   256      segscan_mid
 cap segred_top_n2e24     segred  top    16777216 4        top_small
 cap segscan_top_n2e23    segscan top    8388608  8        top_warp

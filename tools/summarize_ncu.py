@@ -36,14 +36,14 @@ with open(f"profiles/{tag}_ncu_launches_summary.csv", "w") as fp:
 # ---- full captures
 ALG = {  # algorithmic bytes of the captured launch
     "segscan_flat_n1": 8 * 2**26, "segscan_flat_n4096": 8 * 2**26, "segred_flat_n1": 4 * (2**26 + 1),
-    "segred_middle_n1024": 4 * (2**26 + 1024), "segscan_middle_n2e18": 8 * 2**26,
+    "segred_middle_n2e16": 4 * (2**26 + 65536), "segscan_middle_n2e18": 8 * 2**26,
     "segred_top_n2e24": 4 * (2**26 + 2**24), "segscan_top_n2e23": 8 * 2**26,
     "redomap2_tc_8192": 2 * (2 * 8192 * 8192) + 4 * 8192 * 8192, "redomap2_flat_n1": 2 * (2 * 2**30) + 4,
     "tridag_middle_large": 8 * 65536 * 256, "tridag_flat_large": 8 * 65536 * 256,
     "lvc_outer_large": 2 * 8 * 256 * 256 * 256,  # one read + one write per element for the whole loop
     "colred_flat_n2e20": 4 * 2**26, "colscan_top_n4": 8 * 2**26, "colscan_flat_n2e26": 8 * 2**26,
 }
-GROUP = {"segscan_flat_n1": "segscan_flat", "segred_flat_n1": "segred_flat", "segred_middle_n1024": "segred_middle",
+GROUP = {"segscan_flat_n1": "segscan_flat", "segred_flat_n1": "segred_flat", "segred_middle_n2e16": "segred_middle",
          "segscan_middle_n2e18": "segscan_middle", "segred_top_n2e24": "segred_top", "segscan_top_n2e23": "segscan_top",
          "redomap2_tc_8192": "redomap2_tc", "redomap2_flat_n1": "redomap2_flat", "tridag_middle_large": "tridag_middle",
          "tridag_flat_large": "tridag_flat", "lvc_outer_large": "lvc_outer", "colred_flat_n2e20": "colred_flat",
