@@ -18,8 +18,9 @@ ap = argparse.ArgumentParser()
 ap.add_argument("ks", type=int, nargs="*", default=[18, 20, 21, 22, 23, 24])
 ap.add_argument("--ops", default="segred,segscan")
 ap.add_argument("--versions", default="top,middle,flat")
+ap.add_argument("--log2n", type=int, default=26)
 a = ap.parse_args()
-N = 1 << 26
+N = 1 << a.log2n
 xs = [gen.generate("F32_UNIT", 2, N, device="cuda"), gen.generate("F32_UNIT", 3, N, device="cuda")]
 out = torch.empty(N, device="cuda")
 ws = ifl.workspace(ifl.workspace_bytes("segscan", 1, N), "cuda")
