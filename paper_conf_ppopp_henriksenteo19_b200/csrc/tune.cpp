@@ -361,6 +361,23 @@ bool hopeless(Kind k, const int64_t* s, int v) {
     return false;
 }
 
+// Capture one forced call into an executable graph (nullptr when it cannot be
+// captured: no capture stream, or a version that synchronises or reads back).
+cudaGraphExec_t capture_call(Kind k, const int64_t* s, int v, char* scratch, cudaStream_t cs) {
+    if (!cs || cudaStreamBeginCapture(cs, cudaStreamCaptureModeThreadLocal) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return nullptr;
+    }
+    const int r = run_forced(k, s, v, scratch, cs);
+    cudaGraph_t g = nullptr;
+    const cudaError_t ce = cudaStreamEndCapture(cs, &g);
+    cudaGraphExec_t ge = nullptr;
+    if (r != IFL_OK || ce != cudaSuccess || !g || cudaGraphInstantiate(&ge, g, 0) != cudaSuccess) ge = nullptr;
+    if (g) cudaGraphDestroy(g);
+    (void)cudaGetLastError();
+    return ge;
+}
+
 }  // namespace
 
 extern "C" size_t ifl_tune_scratch_bytes(const char* site, const int64_t* shapes, int nshapes) {
@@ -387,6 +404,11 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     std::vector<int64_t> ptop(nshapes), pmid(nshapes), pchain(tree ? nshapes * 4 : 0);
     cudaEvent_t e0, e1;
     if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess) return IFL_ECUDA;
+    cudaStream_t cs = nullptr;  // capture stream (the caller's may be the uncapturable legacy stream)
+    if (cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking) != cudaSuccess) {
+        (void)cudaGetLastError();
+        cs = nullptr;
+    }
     int rc = IFL_OK;
     for (int i = 0; i < nshapes && rc == IFL_OK; ++i) {
         const int64_t* s = shapes + i * ar;
@@ -437,15 +459,24 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
             // back-to-back calls alternating two input copies instead moved the
             // tuned thresholds away from the 2^26 test sweep's best -- 5.37 vs
             // 5.60 TB/s -- so it is one call per rep.)
+            // The call is replayed as a CUDA graph when it can be captured, so a
+            // multi-kernel version is not charged eager launch gaps the graph-
+            // replayed program does not pay (B200: FLAT segred's two kernels
+            // vs MIDDLE's one at n = 8 flipped the R3 guard); otherwise eager.
+            cudaGraphExec_t ge = capture_call(k, s, v, (char*)scratch, cs);
             std::vector<float> ms(reps);
             for (int q = 0; q < reps; ++q) {
                 flush_l2(flush, st, q);  // evict the L2 (untimed)
                 cudaEventRecord(e0, st);
-                run_forced(k, s, v, (char*)scratch, st);
+                if (ge)
+                    cudaGraphLaunch(ge, st);
+                else
+                    run_forced(k, s, v, (char*)scratch, st);
                 cudaEventRecord(e1, st);
                 cudaEventSynchronize(e1);
                 cudaEventElapsedTime(&ms[q], e0, e1);
             }
+            if (ge) cudaGraphExecDestroy(ge);
             std::sort(ms.begin(), ms.end());
             table[i * NV + slot] = ms[reps / 2];
             best_ms = std::min(best_ms, (double)ms[reps / 2]);
@@ -453,6 +484,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     }
     cudaEventDestroy(e0);
     cudaEventDestroy(e1);
+    if (cs) cudaStreamDestroy(cs);
     if (rc != IFL_OK) return rc;
     if (cost_table) std::copy(table.begin(), table.end(), cost_table);
     if (tree) {
