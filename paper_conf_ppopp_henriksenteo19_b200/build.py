@@ -29,6 +29,9 @@ NVCC = shutil.which("nvcc") or "/usr/local/cuda/bin/nvcc"
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + CSRC, "-I" + os.path.join(ROOT, "include")]
 CUFLAGS = ARCH + COMMON + ["-lineinfo", "--expt-relaxed-constexpr", "-Xptxas", "-warn-spills"]
+# experiment builds only: extra -D flags for a tagged variant (IFL_BUILD_EXTRA="-DX=1 ...")
+if _TAG:
+    CUFLAGS = CUFLAGS + os.environ.get("IFL_BUILD_EXTRA", "").split()
 
 
 def _headers():
@@ -57,8 +60,14 @@ def build(force: bool = False, jobs: int | None = None, verbose: bool = False, e
     hdr = max(os.path.getmtime(h) for h in _headers())
     todo = []
     objs = []
+    only = os.environ.get("IFL_BUILD_ONLY", "").split() if _TAG else []  # experiment builds: recompile these only
+    main_obj = os.path.join(PKG, "build_obj")
     for s in srcs:
         o = os.path.join(OBJ, os.path.basename(s) + ".o")
+        if only and os.path.basename(s) not in only:
+            o = os.path.join(main_obj, os.path.basename(s) + ".o")  # the product build's object
+            objs.append(o)
+            continue
         objs.append(o)
         if force or _stale(s, o, hdr):
             todo.append((s, o))
