@@ -197,13 +197,16 @@ def tune_search_chain(par, cost_table, cost: int = 0):
 _WS: dict = {}
 
 
-def workspace(nbytes: int, device=None, key: str = "default") -> torch.Tensor:
+def workspace(nbytes: int, device=None, key: str = "default", stream=None) -> torch.Tensor:
     """A zero-initialised, reusable device workspace (the flat kernels leave it
-    re-armed for the next call, so it is zeroed only when first allocated)."""
+    re-armed for the next call, so it is zeroed only when first allocated).
+    One cache per (device, key, stream): the conveniences below key it by entry
+    point, so segred partials never land in a segscan status region, and two
+    streams never share one workspace (ifl.h forbids concurrent use)."""
     if nbytes == 0:
         return None
     dev = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
-    k = (dev, key)
+    k = (dev, key, 0 if stream is None else int(stream))
     w = _WS.get(k)
     if w is None or w.numel() < nbytes:
         w = torch.zeros(max(nbytes, 1 << 20), dtype=torch.uint8, device=dev)
@@ -256,7 +259,7 @@ def _seg(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws
     entry = "segscan" if scan else "segred"
     wb = lib().ifl_workspace_bytes(_b(entry), n, m, 0, DTYPES[dt], VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, x.device)
+        ws = workspace(wb, x.device, entry, _stream(stream))
     c = ifl_choice()
     args = (x.data_ptr(), out.data_ptr(), n, m, DTYPES[dt], OPS[op], MAPS[f], _ne_buf(ne, dt))
     tail = (VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel() * ws.element_size(),
@@ -304,7 +307,7 @@ def _col(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws
     entry = "colscan" if scan else "colred"
     wb = lib().ifl_workspace_bytes(_b(entry), n, m, 0, DTYPES[dt], VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, x.device, "col")
+        ws = workspace(wb, x.device, entry, _stream(stream))
     c = ifl_choice()
     fn = lib().ifl_colscan if scan else lib().ifl_colred
     rc = fn(x.data_ptr(), out.data_ptr(), n, m, DTYPES[dt], OPS[op], MAPS[f], _ne_buf(ne, dt), VERSIONS[version],
@@ -340,7 +343,7 @@ def segred2(x, op_o="sum", op_i="max", f="id", ne_o=None, ne_i=None, version="au
         out = torch.empty(n, dtype=x.dtype, device=x.device)
     wb = lib().ifl_workspace_bytes(b"segred2", n, m, k, DTYPES[dt], VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, x.device, "seg2")
+        ws = workspace(wb, x.device, "segred2", _stream(stream))
     c = ifl_choice()
     rc = lib().ifl_segred2(x.data_ptr(), out.data_ptr(), n, m, k, DTYPES[dt], OPS[op_o], OPS[op_i], MAPS[f],
                            _ne_buf(ne_o, dt), _ne_buf(ne_i, dt), VERSIONS[version], _ptr(ws),
@@ -365,7 +368,7 @@ def segarg(x, which="min", version="auto", out=None, ws=None, stream=None, retur
                                             torch.empty(n, dtype=torch.int32, device=x.device))
     wb = lib().ifl_workspace_bytes(b"segarg", n, m, 0, DTYPES[dt], VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, x.device, "arg")
+        ws = workspace(wb, x.device, "segarg", _stream(stream))
     c = ifl_choice()
     rc = lib().ifl_segarg(x.data_ptr(), val.data_ptr(), idx.data_ptr(), n, m, DTYPES[dt], 1 if which == "max" else 0,
                           VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel() * ws.element_size(),
@@ -401,7 +404,7 @@ def _irr(scan, x, offsets, op, f, ne, version, max_len, out, ws, stream, return_
     entry = "segscan_irr" if scan else "segred_irr"
     wb = lib().ifl_workspace_bytes(_b(entry), n, total, 0, DTYPES[dt], VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, x.device, "irr")
+        ws = workspace(wb, x.device, entry, _stream(stream))
     c = ifl_choice()
     fn = lib().ifl_segscan_irr if scan else lib().ifl_segred_irr
     rc = fn(x.data_ptr(), out.data_ptr(), offsets.data_ptr(), n, total, int(max_len), DTYPES[dt], OPS[op], MAPS[f],
@@ -440,7 +443,7 @@ def redomap2(A, B, b_kmajor=True, version="auto", out=None, ws=None, stream=None
         out = torch.empty((n, p), dtype=torch.float32, device=A.device)
     wb = lib().ifl_workspace_bytes(b"redomap2", n, m, p, DTYPES[dt], VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, A.device, "redomap2")
+        ws = workspace(wb, A.device, "redomap2", _stream(stream))
     c = ifl_choice()
     rc = lib().ifl_redomap2(A.data_ptr(), B.data_ptr(), out.data_ptr(), n, m, p, DTYPES[dt], int(b_kmajor),
                             VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel(), _stream(stream),
@@ -464,7 +467,7 @@ def tridag(a, b, c, y, version="auto", out=None, ws=None, stream=None, return_ch
         out = torch.empty_like(y)
     wb = lib().ifl_workspace_bytes(b"tridag", S, L, R, 1, VERSIONS[version])
     if ws is None and wb:
-        ws = workspace(wb, y.device, "tridag")
+        ws = workspace(wb, y.device, "tridag", _stream(stream))
     ch = ifl_choice()
     rc = lib().ifl_tridag(a.data_ptr(), b.data_ptr(), c.data_ptr(), y.data_ptr(), out.data_ptr(), S, L, R,
                           VERSIONS[version], _ptr(ws), 0 if ws is None else ws.numel(), _stream(stream),
@@ -489,7 +492,7 @@ def lvc(xsss, ysss, xcoef, ycoef, numT: int, version="auto", ws=None, stream=Non
         raise ValueError("ysss must be [numS][numY][numX]")
     wb = lib().ifl_workspace_bytes(b"lvc", numX, numY, 0, 1, -1)
     if ws is None and wb:
-        ws = workspace(wb, xsss.device, "lvc")
+        ws = workspace(wb, xsss.device, "lvc", _stream(stream))
     ch = ifl_choice()
     rc = lib().ifl_lvc(*(t.data_ptr() for t in ts), numS, int(numT), numX, numY, VERSIONS[version], _ptr(ws),
                        0 if ws is None else ws.numel(), _stream(stream), ctypes.byref(ch))

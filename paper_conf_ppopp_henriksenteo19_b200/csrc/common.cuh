@@ -109,6 +109,24 @@ __device__ __forceinline__ typename Vec4<T>::type ldg_stream4(const T* p) {
 template <typename T>
 __device__ __forceinline__ T ldg1(const T* p) { return __ldg(p); }
 
+// Coherent (weak, non-.nc) loads for kernels whose input may alias their output
+// (in-place scans, ifl.h): ld.global.nc requires memory that the kernel does not
+// write, so the scan kernels read through these instead.
+template <typename T>
+__device__ __forceinline__ typename Vec4<T>::type ld_coh4(const T* p) {
+    typename Vec4<T>::type r;
+    if constexpr (std::is_same<T, int>::value) {
+        asm volatile("ld.global.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
+    } else {
+        asm volatile("ld.global.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+                     : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p) : "memory");
+    }
+    return r;
+}
+template <typename T>
+__device__ __forceinline__ T ld_coh1(const T* p) { return *p; }
+
 // Running (+)-accumulator.  For f32 sums it is Kahan-compensated, so a long
 // sequential chain (a thread-per-segment walk over m ~ 2^26 elements) stays
 // within the 1e-5 relative parity bound; every other (+) is exact or
@@ -279,7 +297,7 @@ __host__ __device__ constexpr int64_t ceil_div(int64_t a, int64_t b) { return (a
 // warps per CTA (the tile is 32 * (M + 4) words per warp).
 __host__ __device__ constexpr int top_tile_warps(int M) { return M <= 32 ? 8 : 4; }
 template <typename T, int OP, int F, int M, bool SCAN>
-__global__ void __launch_bounds__(32 * top_tile_warps(M)) top_tile_kernel(const T* __restrict__ in, T* __restrict__ out,
+__global__ void __launch_bounds__(32 * top_tile_warps(M)) top_tile_kernel(const T* in, T* out,
                                                                           int64_t n, T d, const T* __restrict__ seed) {
     using V = typename Vec4<T>::type;
     constexpr int S = M + 4, W4 = M / 4, WPC = top_tile_warps(M);  // row stride (words), words per row
@@ -294,7 +312,7 @@ __global__ void __launch_bounds__(32 * top_tile_warps(M)) top_tile_kernel(const 
 #pragma unroll
     for (int u = 0; u < W4; ++u) {
         const int q4 = lane + 32 * u;  // 16-byte word of the block
-        if (q4 < rows * W4) q[u] = ldg_stream4(src + 4 * q4);
+        if (q4 < rows * W4) q[u] = SCAN ? ld_coh4(src + 4 * q4) : ldg_stream4(src + 4 * q4);  // scans may be in place
     }
 #pragma unroll
     for (int u = 0; u < W4; ++u) {

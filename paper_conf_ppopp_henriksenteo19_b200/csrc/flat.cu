@@ -3,11 +3,10 @@
 //
 // The flat index space [0, n*m) is cut into tiles of kFlatTile = 256 x 20
 // elements.  Segment starts are arithmetic (multiples of m): no flag array is
-// read, and d is combined into every segment's first element.  Both kernels
+// read, and d is combined into every segment's first element.  The kernels
 // are persistent (grid = resident CTAs) and stream tiles through a ring of
-// shared-memory slots (kRedSlots / kScanSlots) filled by the TMA engine (cp.async.bulk +
-// mbarrier), so loads for the next tiles are in flight while a tile is
-// processed.  Per tile:
+// shared-memory slots filled by the TMA engine (cp.async.bulk + mbarrier), so
+// loads for the next tiles are in flight while a tile is processed.  Per tile:
 //   * thread t takes its 20 consecutive elements (5 conflict-free LDS.128: the
 //     80-byte stride is an odd multiple of 16 B).  A thread whose items hold
 //     no segment boundary (the common case once m exceeds a few dozen) takes a
@@ -20,14 +19,17 @@
 //           (the open segment at its end, or the whole tile) in the workspace;
 //   pass 2  every segment that crosses tiles ta < tb is
 //           out = tail[ta] (+) tail[ta+1..tb-1] (+) head[tb]   (a tree reduce).
-// segscan (L2-blocked two-phase, see flat_scan_kernel): chunks of kChunkTiles
-//   tiles; a chunk's aggregate is computed in a first pass whose data stays in
-//   L2, a CTA-wide look-back over chunk status words (aggregate / inclusive
-//   prefix, segment flag, epoch tag; relaxed loads -- the word is
-//   self-contained) gives its carry, and the scan pass re-reads it from L2 and
-//   stores each tile from its ring slot with the TMA engine (cp.async.bulk
-//   shared->global).  The workspace is re-armed by the last CTA (counter
-//   reset, epoch bump), so no per-call memset is needed.
+//   Rows of >= 8192 elements: uniform row pieces (flat_red_split_kernel).
+// segscan:
+//   * tiles that all begin at a segment start (m divides the tile): the
+//     single-pass engine (flat_scan_dlb_kernel), no inter-tile dependence;
+//   * otherwise the job-ring engine (flat_scan_jr_kernel): reduce-then-scan
+//     desynchronised into jobs -- job k aggregates chunk k from DRAM and scans
+//     chunk k - lag from L2 -- so no look-back ever waits on a status written
+//     moments ago (under a saturated memory system a status store and the
+//     poll that sees it take microseconds: DESIGN.md section 5).
+//   Status words carry an epoch tag; the last CTA re-arms the workspace
+//   (counter reset, epoch bump), so no per-call memset is needed.
 // Workspace: [header 256 B][status: 8 B/tile][head: 4 B/tile][tail: 4 B/tile].
 #include <string.h>
 
@@ -593,273 +595,7 @@ __device__ __forceinline__ void local_seg_scan(T (&v)[FI], const ThreadPos& tp, 
     }
 }
 
-// L2-blocked two-phase segscan, warp-specialised.  Persistent CTAs,
-// co-resident by cooperative launch, own chunks of kChunkTiles consecutive
-// tiles statically (chunk c = round * grid + blockIdx).  Per chunk:
-//   phase 1  (only if the next chunk continues a segment into it) stream the
-//            chunk with an L2 evict_last policy and fold the tile aggregates
-//            into the chunk aggregate; publish it;
-//   look-back (only if the chunk does not begin a segment) over the chunk
-//            aggregates, CTA-wide, bounded arithmetically to the chunk holding
-//            the last segment start -- at most one round back;
-//   phase 3  stream the chunk again (evict_first: the round, ~48 MB, is still
-//            in the 126 MB L2, so DRAM sees one read and one write per
-//            element), scan with the running carry, store each tile from its
-//            ring slot with the TMA engine.
-// Warp 8 is the producer: it walks the CTA's item sequence (phase-1 tiles ++
-// phase-3 tiles, chunk after chunk), waits for a ring slot to be released
-// (mbarrier `empty`), writes the slot's metadata and issues the TMA load
-// (completion on `full`).  Warps 0-7 consume; they synchronise among
-// themselves with a named barrier, so the producer never stalls them and the
-// 64-bit tile arithmetic stays off their critical path.  Status words carry
-// an epoch tag; the last CTA to finish bumps the epoch (one 64-bit
-// {epoch | done} word), so no per-call memset is needed.
-#ifndef IFL_CHUNK_TILES
-#define IFL_CHUNK_TILES 8
-#endif
-constexpr int kChunkTiles = IFL_CHUNK_TILES;
-constexpr int kScanThreads = FB + 32;
-#ifndef IFL_SCAN_SLOTS
-#define IFL_SCAN_SLOTS 3  // 60 KB ring: three CTAs (27 warps) per SM
-#endif
-#ifndef IFL_SCAN_MINB
-#define IFL_SCAN_MINB 3
-#endif
-constexpr int kScanSlots = IFL_SCAN_SLOTS;
-
-template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kScanThreads, IFL_SCAN_MINB) flat_scan_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
-                                                                    uint8_t* ws, int num_tiles, int num_chunks,
-                                                                    bool tma_in, bool tma_out, const T* __restrict__ seed) {
-    extern __shared__ __align__(128) uint8_t smem_raw[];
-    T* ring = reinterpret_cast<T*>(smem_raw);
-    __shared__ alignas(8) uint64_t full[kScanSlots], empty[kScanSlots];
-    __shared__ SlotMeta meta[kScanSlots];
-    __shared__ uint32_t s_tag;
-    __shared__ T s_wval[2][FB / 32];  // double-buffered by item parity: no barrier between phase-1 tiles
-    __shared__ uint32_t s_wflag[2][FB / 32];
-    __shared__ int s_lbterm[FB / 32];
-    __shared__ T s_lbval[FB / 32];
-    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | done:32}
-    uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int G = gridDim.x;
-    const int64_t chunk_elems = (int64_t)kChunkTiles * FT;
-    auto need_carry = [&](int c) { return c > 0 && ((int64_t)c * chunk_elems) % m != 0; };
-    auto need_agg = [&](int c) { return need_carry(c + 1) && c + 1 < num_chunks; };
-    auto chunk_tiles = [&](int c) { return min(kChunkTiles, num_tiles - c * kChunkTiles); };
-
-    if (t == 0) {
-        s_tag = status_tag(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)));
-        for (int q = 0; q < kScanSlots; ++q) {
-            mbar_init(&full[q], 1);
-            mbar_init(&empty[q], 1);
-        }
-        fence_mbar_init();
-    }
-    __syncthreads();
-
-    if (w == FB / 32) {
-        // ================= producer warp (one lane)
-        if (lane == 0) {
-            const uint64_t pol_keep = policy_evict_last(), pol_stream = policy_evict_first();
-            int wv = 0;
-            for (int c = blockIdx.x; c < num_chunks; c += G) {
-                const int L = chunk_tiles(c);
-                const int t0 = c * kChunkTiles;
-                // tile metadata advanced incrementally (no 64-bit division per tile)
-                const int64_t cbase = (int64_t)t0 * FT;
-                for (int ph = need_agg(c) ? 1 : 3; ph <= 3; ph += 2) {
-                    int64_t pos = cbase % m, seg = cbase / m;
-                    for (int j = 0; j < L; ++j, ++wv) {
-                        const int sl = wv % kScanSlots;
-                        if (wv >= kScanSlots) mbar_wait(&empty[sl], ((wv / kScanSlots) - 1) & 1);
-                        SlotMeta& sm = meta[sl];
-                        const int tile = t0 + j;
-                        sm.tile = tile;
-                        sm.cnt = (int)std::min((int64_t)FT, N - (int64_t)tile * FT);
-                        sm.pos = pos;
-                        sm.seg = seg;
-                        if (tma_in && sm.cnt == FT) {
-                            mbar_arrive_expect_tx(&full[sl], FT * sizeof(T));
-                            bulk_g2s_hint(ring + sl * FT, in + (int64_t)tile * FT, FT * sizeof(T), &full[sl],
-                                          ph == 1 ? pol_keep : pol_stream);
-                        } else {
-                            mbar_arrive_expect_tx(&full[sl], 0);  // consumers copy it themselves
-                        }
-                        pos += FT;
-                        if (pos >= m) {  // m > FT: at most one wrap; otherwise divide (32-bit range)
-                            if (m > FT) {
-                                pos -= m;
-                                seg += 1;
-                            } else {
-                                seg += pos / m;
-                                pos %= m;
-                            }
-                        }
-                    }
-                }
-            }
-        }
-        return;
-    }
-
-    // ================= consumer warps 0-7
-    const uint32_t tag = s_tag;
-    uint32_t phase_bits = 0;
-    int vi = 0;
-    int pend_slot = -1;  // slot whose bulk store may still be reading smem (thread 0)
-    auto release = [&](int sl) { mbar_arrive_expect_tx(&empty[sl], 0); };
-    auto acquire = [&](int sl, T* buf, const SlotMeta& sm) {
-        mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
-        phase_bits ^= 1u << sl;
-        if (!(tma_in && sm.cnt == FT)) {  // partial / misaligned tile: cooperative copy
-            const int64_t base = (int64_t)sm.tile * FT;
-            for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
-            consumer_sync();
-        }
-    };
-    for (int c = blockIdx.x; c < num_chunks; c += G) {
-        const int L = chunk_tiles(c);
-        const bool agg_needed = need_agg(c), carry_needed = need_carry(c);
-        // ---- phase 1
-        uint32_t run_f = 0;
-        T run_v = identity<OP, T>();
-        if (agg_needed) {
-            for (int j = 0; j < L; ++j, ++vi) {
-                const int sl = vi % kScanSlots;
-                T* buf = ring + sl * FT;
-                mbar_wait(&full[sl], (phase_bits >> sl) & 1u);  // meta is valid once the slot is full
-                const SlotMeta sm = meta[sl];
-                phase_bits ^= 1u << sl;
-                if (!(tma_in && sm.cnt == FT)) {
-                    const int64_t base = (int64_t)sm.tile * FT;
-                    for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
-                    consumer_sync();
-                }
-                const ThreadPos tp = thread_pos(sm, m);
-                T v[FI];
-                load_items(buf, v);
-                bool hs;
-                T acc;
-                local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
-                uint32_t exf, aggf;
-                T exv, aggv;
-                cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[vi & 1], s_wflag[vi & 1]);
-                // everyone's items are in registers (the barrier inside the scan): free the slot
-                if (t == 0) {
-                    if (pend_slot >= 0) {  // a phase-3 store before this phase-1 run
-                        bulk_wait_read0();
-                        release(pend_slot);
-                        pend_slot = -1;
-                    }
-                    release(sl);
-                }
-                run_v = aggf ? aggv : combine<OP>(run_v, aggv);
-                run_f |= aggf;
-            }
-            if (t == 0)
-                st_relaxed_u64(&status[c], pack_status(tag, (run_f || !carry_needed) ? ST_P : ST_A, run_f,
-                                                       to_bits(run_v)));
-        }
-        // ---- look-back over preceding chunk aggregates (chunks cs .. c-1)
-        T carry = identity<OP, T>();
-        if (carry_needed) {
-            const int64_t cstart = (int64_t)c * chunk_elems;
-            const int cs = (int)((((cstart - 1) / m) * m) / chunk_elems);
-            int pred = c - 1;
-            while (true) {
-                const int idx = pred - t;
-                uint64_t word = 0;
-                if (idx >= cs) {
-                    do {
-                        word = ld_relaxed_u64(&status[idx]);  // self-contained word: no acquire needed
-                    } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
-                }
-                const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
-                const uint32_t tb = __ballot_sync(0xffffffffu, term);
-                if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
-                consumer_sync();
-                int stop = FB;
-#pragma unroll
-                for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
-                T val = (t <= stop && idx >= cs) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
-#pragma unroll
-                for (int off = 1; off < 32; off <<= 1) {  // ordered: higher lane = older chunk
-                    const T older = __shfl_down_sync(0xffffffffu, val, off);
-                    if (lane + off < 32) val = combine<OP>(older, val);
-                }
-                if (lane == 0) s_lbval[w] = val;
-                consumer_sync();
-                T win = identity<OP, T>();
-#pragma unroll
-                for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
-                carry = combine<OP>(win, carry);
-                consumer_sync();
-                if (stop < FB) break;
-                pred -= FB;
-            }
-            if (agg_needed && !run_f && t == 0)
-                st_relaxed_u64(&status[c], pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, run_v))));
-        }
-        // ---- phase 3
-        for (int j = 0; j < L; ++j, ++vi) {
-            const int sl = vi % kScanSlots;
-            T* buf = ring + sl * FT;
-            mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
-            const SlotMeta sm = meta[sl];
-            phase_bits ^= 1u << sl;
-            if (!(tma_in && sm.cnt == FT)) {
-                const int64_t base = (int64_t)sm.tile * FT;
-                for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
-                consumer_sync();
-            }
-            const int64_t base = (int64_t)sm.tile * FT;
-            const ThreadPos tp = thread_pos(sm, m);
-            T v[FI];
-            load_items(buf, v);
-            bool hs;
-            T acc;
-            local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
-            uint32_t exf, aggf;
-            T exv, aggv;
-            cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[vi & 1], s_wflag[vi & 1]);
-            {
-                const T carry_t = exf ? exv : combine<OP>(carry, exv);
-                const int lim = min(tp.nx0, tp.nvalid);
-#pragma unroll
-                for (int k = 0; k < FI; ++k)
-                    if (k < lim) v[k] = combine<OP>(carry_t, v[k]);
-            }
-            carry = aggf ? aggv : combine<OP>(carry, aggv);
-            store_items(buf, v);
-            const bool bulk = tma_out && sm.cnt == FT;
-            if (bulk) fence_proxy_async_smem();
-            consumer_sync();
-            if (bulk) {
-                if (t == 0) bulk_s2g_hint(out + base, buf, FT * sizeof(T), policy_evict_first());
-            } else {
-                for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
-                consumer_sync();
-            }
-            if (t == 0) {
-                bulk_commit();  // one group per phase-3 item (empty for cooperative stores)
-                if (pend_slot >= 0) {
-                    bulk_wait_read1();  // the previous item's store has read its slot
-                    release(pend_slot);
-                }
-                pend_slot = sl;
-            }
-        }
-    }
-    if (t == 0) {
-        bulk_wait0();
-        if (pend_slot >= 0) release(pend_slot);
-        __threadfence();
-        const unsigned long long old = atomicAdd(ctr, 1ull);
-        if ((uint32_t)old == (uint32_t)G - 1) atomicAdd(ctr, (1ull << 32) - (unsigned long long)G);
-    }
-}
+constexpr int kScanThreads = FB + 32;  // 8 consumer warps + 1 producer warp
 
 // Single-pass segmented scan with decoupled look-back over dynamically claimed
 // tiles (one global read and one global write per element, no second pass).
@@ -943,14 +679,13 @@ __device__ __forceinline__ T cta_lookback_w(const uint64_t* status, uint32_t tag
 #ifndef IFL_DLB_LBW
 #define IFL_DLB_LBW 1
 #endif
-#ifndef IFL_SCAN_DLB
-#define IFL_SCAN_DLB 0
-#endif
+// Used for tile-aligned segments only (no look-back): 2 slots x 4 CTAs per SM
+// (B200, n*m = 2^26 f32, m = 32..1024: 81-83 us = a copy's speed; 3 x 3: 82-91)
 #ifndef IFL_DLB_SLOTS
-#define IFL_DLB_SLOTS 4
+#define IFL_DLB_SLOTS 2
 #endif
 #ifndef IFL_DLB_MINB
-#define IFL_DLB_MINB 2
+#define IFL_DLB_MINB 4
 #endif
 constexpr int kDlbSlots = IFL_DLB_SLOTS;
 
@@ -1084,737 +819,6 @@ __global__ void __launch_bounds__(kScanThreads, IFL_DLB_MINB) flat_scan_dlb_kern
 }
 
 // ---------------------------------------------------------------------------
-// Aggregate-ahead segmented scan ("AR" engine).  The single-pass look-back
-// scan above is bound by the L2 round trip of its look-back under a saturated
-// memory system (every tile of a long segment waits for its predecessors'
-// statuses); the L2-blocked scan pays a grid-wide phase change per round.
-// Here the two halves of reduce-then-scan run CONCURRENTLY in different CTAs
-// of one persistent grid, over chunks of kArChunkTiles tiles:
-//   * aggregator CTAs (blockIdx < #SMs) claim chunks in order and reduce only
-//     what a successor needs -- the chunk's part after its last segment start
-//     (all of it for long segments) -- with L2::evict_last loads, publishing
-//     the segmented aggregate (an inclusive prefix when the chunk holds a
-//     segment start).  Flow control keeps them at most kArLag chunks ahead of
-//     the scanners, so the data they pull in is still in L2;
-//   * scanner CTAs claim chunks in the same order; the producer warp waits
-//     for the chunk's aggregate (its data is then in L2) and streams its tiles
-//     through the TMA ring; the consumers first resolve the chunk carry by a
-//     CTA-wide look-back over chunk statuses -- every aggregate is already
-//     published, so this is one round trip -- publish the chunk's inclusive
-//     prefix, then scan the tiles with a running carry and store each from its
-//     slot with a TMA bulk store.
-// DRAM sees one read (aggregators, or scanners for chunk prefixes that no
-// successor needs) and one write per element, reads and writes overlapped.
-#ifndef IFL_AR_CHUNK_TILES
-#define IFL_AR_CHUNK_TILES 8
-#endif
-#ifndef IFL_AR_LAG
-#define IFL_AR_LAG 160
-#endif
-#ifndef IFL_AR_SLOTS
-#define IFL_AR_SLOTS 3
-#endif
-#ifndef IFL_AR_AGG_PER_SM
-#define IFL_AR_AGG_PER_SM 1
-#endif
-#ifndef IFL_AR_MINB
-#define IFL_AR_MINB 3
-#endif
-constexpr int kArChunkTiles = IFL_AR_CHUNK_TILES;
-constexpr int kArLag = IFL_AR_LAG;
-constexpr int kArSlots = IFL_AR_SLOTS;
-
-template <typename T>
-__device__ __forceinline__ typename Vec4<T>::type ldg_keep4(const T* p, uint64_t pol) {
-    typename Vec4<T>::type r;
-    if constexpr (std::is_same<T, int>::value) {
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0,%1,%2,%3}, [%4], %5;"
-                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p), "l"(pol));
-    } else {
-        asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
-                     : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "l"(p), "l"(pol));
-    }
-    return r;
-}
-
-// CTA-wide reduction of f over src[a, b) with 8 independent 128-bit loads per
-// thread in flight, L2::evict_last; the total is valid in thread 0.
-template <typename T, int OP, int F, int NT, int U = 8>
-__device__ __forceinline__ T cta_reduce_keep(const T* __restrict__ src, int64_t a, int64_t b, T* red, uint64_t pol) {
-    using V = typename Vec4<T>::type;
-    T acc4[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
-    int64_t h = (int64_t)(((16u - ((uint32_t)(uintptr_t)(src + a) & 15u)) & 15u) / sizeof(T));
-    if (h > b - a) h = b - a;
-    for (int64_t k = a + threadIdx.x; k < a + h; k += NT) acc4[0] = combine<OP>(acc4[0], apply_map<F>(src[k]));
-    const T* body = src + a + h;
-    const int64_t nv = (b - a - h) >> 2;
-    int64_t v = threadIdx.x;
-    for (; v + (U - 1) * NT < nv; v += U * NT) {
-        V q[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) q[u] = ldg_keep4(body + 4 * (v + u * NT), pol);
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-            T e[4];
-            unpack4<T>(q[u], e);
-#pragma unroll
-            for (int c = 0; c < 4; ++c) acc4[c] = combine<OP>(acc4[c], apply_map<F>(e[c]));
-        }
-    }
-    for (; v < nv; v += NT) {
-        T e[4];
-        unpack4<T>(ldg_keep4(body + 4 * v, pol), e);
-#pragma unroll
-        for (int c = 0; c < 4; ++c) acc4[c] = combine<OP>(acc4[c], apply_map<F>(e[c]));
-    }
-    for (int64_t k = a + h + 4 * nv + threadIdx.x; k < b; k += NT) acc4[1] = combine<OP>(acc4[1], apply_map<F>(src[k]));
-    T acc = warp_reduce<OP>(combine<OP>(combine<OP>(acc4[0], acc4[1]), combine<OP>(acc4[2], acc4[3])));
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = acc;
-    __syncthreads();
-    T r = identity<OP, T>();
-    if (threadIdx.x < 32) {
-        r = threadIdx.x < NT / 32 ? red[threadIdx.x] : identity<OP, T>();
-        r = warp_reduce<OP>(r);
-    }
-    __syncthreads();  // red is reused by the next chunk
-    return r;
-}
-
-#ifdef IFL_AR_PROF
-__device__ unsigned long long g_ar_prof[16];
-#define PROF_T0(v) const long long v = clock64()
-#define PROF_ADD(acc, v) acc += (unsigned long long)(clock64() - v)
-#else
-#define PROF_T0(v)
-#define PROF_ADD(acc, v)
-#endif
-
-__device__ __forceinline__ void bulk_prefetch_l2(const void* p, uint32_t bytes, uint64_t pol) {
-    asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(p), "r"(bytes), "l"(pol)
-                 : "memory");
-}
-#ifndef IFL_AR_PF
-#define IFL_AR_PF 0
-#endif
-
-struct ArMeta {
-    int tile;   // -1: no more work
-    int cnt;
-    int chunk;  // chunk of the tile
-    int j;      // tile index inside its chunk
-    int64_t pos, seg;
-};
-
-template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kScanThreads, IFL_AR_MINB) flat_scan_ar_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
-                                                                    uint8_t* ws, int num_tiles, int num_chunks,
-                                                                    int num_agg, bool tma_in, bool tma_out,
-                                                                    const T* __restrict__ seed) {
-    extern __shared__ __align__(128) uint8_t smem_raw[];
-    T* ring = reinterpret_cast<T*>(smem_raw);
-    __shared__ alignas(8) uint64_t full[kArSlots], empty[kArSlots];
-    __shared__ ArMeta meta[kArSlots];
-    __shared__ uint32_t s_tag;
-    __shared__ T s_wval[2][FB / 32];
-    __shared__ uint32_t s_wflag[2][FB / 32];
-    __shared__ int s_lbterm[FB / 32];
-    __shared__ T s_lbval[FB / 32 + 1];
-    __shared__ int s_claim;
-    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | done:32}
-    unsigned* scan_ctr = reinterpret_cast<unsigned*>(ws + 8);
-    unsigned* agg_ctr = reinterpret_cast<unsigned*>(ws + 12);
-    uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    const int G = gridDim.x;
-    const int64_t CH = (int64_t)kArChunkTiles * FT;
-    if (t == 0) s_tag = status_tag(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)));
-#ifdef IFL_AR_PROF
-    unsigned long long pa[16] = {};
-    const long long t_start = clock64();
-#endif
-
-    if ((int)blockIdx.x < num_agg) {
-        // ====================== aggregator
-        // warp 8 (lane 0) claims chunks (flow control: at most kArLag chunks
-        // ahead of the scanners) and streams the tiles covering the chunk's
-        // needed range [lo, ce) through the TMA ring (L2::evict_last);
-        // warps 0-7 reduce each tile's part of the range from shared memory.
-        if (t == 0) {
-            for (int q = 0; q < kArSlots; ++q) {
-                mbar_init(&full[q], 1);
-                mbar_init(&empty[q], FB / 32);
-            }
-            fence_mbar_init();
-        }
-        __syncthreads();
-        const uint32_t tag = s_tag;
-        if (w == FB / 32) {
-            if (lane == 0) {
-                const uint64_t pol = policy_evict_last();
-                int wv = 0;
-                while (true) {
-                    const int c = (int)atomicAdd(agg_ctr, 1u);
-                    PROF_T0(tf);
-                    if (c < num_chunks)
-                        while ((int)ld_relaxed_u32(scan_ctr) + kArLag < c) __nanosleep(128);
-                    PROF_ADD(pa[5], tf);
-                    if (c >= num_chunks) {
-                        const int sl = wv % kArSlots;
-                        if (wv >= kArSlots) mbar_wait(&empty[sl], ((wv / kArSlots) - 1) & 1);
-                        meta[sl].tile = -1;
-                        mbar_arrive_expect_tx(&full[sl], 0);
-                        break;
-                    }
-                    if (IFL_AR_PF > 0 && tma_in && c + IFL_AR_PF < num_chunks) {
-                        // pull a chunk further ahead into L2 (no smem, no completion): the
-                        // ring loads of this CTA and the scanners' loads then hit L2
-                        const int64_t pb = (int64_t)(c + IFL_AR_PF) * CH, pe = std::min(N, pb + CH);
-                        const uint32_t bytes = (uint32_t)(((pe - pb) * (int64_t)sizeof(T)) & ~(int64_t)15);
-                        if (bytes) bulk_prefetch_l2(in + pb, bytes, pol);
-                    }
-                    const int64_t cb = (int64_t)c * CH, ce = std::min(N, cb + CH);
-                    const int64_t ls = ((ce - 1) / m) * m;
-                    const int64_t lo = ls >= cb ? ls : cb;
-                    const int ta = (int)(lo / FT), tb = (int)((ce - 1) / FT);
-                    for (int tile = ta; tile <= tb; ++tile, ++wv) {
-                        const int sl = wv % kArSlots;
-                        PROF_T0(te);
-                        if (wv >= kArSlots) mbar_wait(&empty[sl], ((wv / kArSlots) - 1) & 1);
-                        PROF_ADD(pa[6], te);
-                        ArMeta& sm = meta[sl];
-                        sm.tile = tile;
-                        sm.cnt = (int)std::min((int64_t)FT, N - (int64_t)tile * FT);
-                        sm.chunk = c;
-                        sm.j = (tile == tb ? 2 : 0) | (tile == ta ? 1 : 0);  // bit 1: last tile of the range
-                        sm.pos = std::max<int64_t>(0, lo - (int64_t)tile * FT);  // range inside the tile: [pos, seg)
-                        sm.seg = std::min<int64_t>(sm.cnt, ce - (int64_t)tile * FT);
-                        if (tma_in && sm.cnt == FT) {
-                            mbar_arrive_expect_tx(&full[sl], FT * sizeof(T));
-                            bulk_g2s_hint(ring + sl * FT, in + (int64_t)tile * FT, FT * sizeof(T), &full[sl], pol);
-                        } else {
-                            mbar_arrive_expect_tx(&full[sl], 0);
-                        }
-                    }
-                }
-            }
-        } else {
-            uint32_t phase_bits = 0;
-            T acc = identity<OP, T>();
-            for (int i = 0;; ++i) {
-                const int sl = i % kArSlots;
-                const T* buf = ring + sl * FT;
-                PROF_T0(tw);
-                mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
-                PROF_ADD(pa[7], tw);
-                phase_bits ^= 1u << sl;
-                const ArMeta am = meta[sl];
-                if (am.tile < 0) break;
-                const int64_t base = (int64_t)am.tile * FT;
-                const int a0 = (int)am.pos, a1 = (int)am.seg;
-                if (tma_in && am.cnt == FT) {
-                    for (int k = a0 + t; k < a1; k += FB) acc = combine<OP>(acc, apply_map<F>(buf[k]));
-                } else {
-                    for (int k = a0 + t; k < a1; k += FB) acc = combine<OP>(acc, apply_map<F>(in[base + k]));
-                }
-                __syncwarp();
-                if (lane == 0) mbar_arrive_expect_tx(&empty[sl], 0);  // this warp is done with the slot
-                if (am.j & 2) {  // last tile of the chunk's range: CTA total, publish
-                    T r = warp_reduce<OP>(acc);
-                    if (lane == 0) s_lbval[w] = r;
-                    consumer_sync();
-                    if (t == 0) {
-                        r = identity<OP, T>();
-#pragma unroll
-                        for (int k = 0; k < FB / 32; ++k) r = combine<OP>(r, s_lbval[k]);
-                        const int64_t cb = (int64_t)am.chunk * CH, ce = std::min(N, cb + CH);
-                        const int64_t ls = ((ce - 1) / m) * m;
-                        const bool flag = ls >= cb;
-                        const T dseg = seed ? seed[ls / m] : d;
-                        const T val = flag ? combine<OP>(dseg, r) : r;
-                        st_relaxed_u64(&status[am.chunk], pack_status(tag, flag ? ST_P : ST_A, flag ? 1u : 0u, to_bits(val)));
-                    }
-                    consumer_sync();
-                    acc = identity<OP, T>();
-                }
-            }
-        }
-    } else {
-        // ====================== scanner
-        if (t == 0) {
-            for (int q = 0; q < kArSlots; ++q) {
-                mbar_init(&full[q], 1);
-                mbar_init(&empty[q], 1);
-            }
-            fence_mbar_init();
-        }
-        __syncthreads();
-        const uint32_t tag = s_tag;
-        if (w == FB / 32) {
-            // ---------------- producer warp (one lane)
-            if (lane == 0) {
-                const uint64_t pol = policy_evict_first();
-                int wv = 0;
-                while (true) {
-                    const int c = (int)atomicAdd(scan_ctr, 1u);
-                    if (c >= num_chunks) {
-                        const int sl = wv % kArSlots;
-                        if (wv >= kArSlots) mbar_wait(&empty[sl], ((wv / kArSlots) - 1) & 1);
-                        meta[sl].tile = -1;
-                        mbar_arrive_expect_tx(&full[sl], 0);
-                        break;
-                    }
-                    // the chunk's aggregate is published: its data has been pulled into L2
-                    PROF_T0(ts);
-                    while ((uint32_t)(ld_relaxed_u64(&status[c]) >> 35) != tag) __nanosleep(64);
-                    PROF_ADD(pa[3], ts);
-                    const int t0 = c * kArChunkTiles;
-                    const int L = min(kArChunkTiles, num_tiles - t0);
-                    int64_t pos = ((int64_t)t0 * FT) % m, seg = ((int64_t)t0 * FT) / m;
-                    for (int j = 0; j < L; ++j, ++wv) {
-                        const int sl = wv % kArSlots;
-                        PROF_T0(te);
-                        if (wv >= kArSlots) mbar_wait(&empty[sl], ((wv / kArSlots) - 1) & 1);
-                        PROF_ADD(pa[4], te);
-                        ArMeta& sm = meta[sl];
-                        const int tile = t0 + j;
-                        sm.tile = tile;
-                        sm.cnt = (int)std::min((int64_t)FT, N - (int64_t)tile * FT);
-                        sm.chunk = c;
-                        sm.j = j;
-                        sm.pos = pos;
-                        sm.seg = seg;
-                        if (tma_in && sm.cnt == FT) {
-                            mbar_arrive_expect_tx(&full[sl], FT * sizeof(T));
-                            bulk_g2s_hint(ring + sl * FT, in + (int64_t)tile * FT, FT * sizeof(T), &full[sl], pol);
-                        } else {
-                            mbar_arrive_expect_tx(&full[sl], 0);
-                        }
-                        pos += FT;
-                        if (pos >= m) {
-                            if (m > FT) {
-                                pos -= m;
-                                seg += 1;
-                            } else {
-                                seg += pos / m;
-                                pos %= m;
-                            }
-                        }
-                    }
-                }
-            }
-        } else {
-            // ---------------- consumer warps 0-7
-            uint32_t phase_bits = 0;
-            int pend_slot = -1;
-            T carry = identity<OP, T>();
-            for (int i = 0;; ++i) {
-                const int sl = i % kArSlots;
-                T* buf = ring + sl * FT;
-                PROF_T0(tw);
-                mbar_wait(&full[sl], (phase_bits >> sl) & 1u);
-                PROF_ADD(pa[0], tw);
-                phase_bits ^= 1u << sl;
-                const ArMeta am = meta[sl];
-                if (t == 0 && pend_slot >= 0) {
-                    PROF_T0(tb);
-                    bulk_wait_read0();
-                    PROF_ADD(pa[9], tb);
-                    mbar_arrive_expect_tx(&empty[pend_slot], 0);
-                    pend_slot = -1;
-                }
-                if (am.tile < 0) break;
-                PROF_T0(tl);
-                if (am.j == 0) {
-                    // chunk carry-in: CTA-wide look-back over the chunk statuses
-                    const int c = am.chunk;
-                    const int64_t cb = (int64_t)c * CH;
-                    carry = identity<OP, T>();
-                    if (cb % m != 0) {
-                        const int cs = (int)(((cb / m) * m) / CH);  // chunk holding the segment's start
-                        int pred = c - 1;
-                        while (true) {
-                            const int idx = pred - t;
-                            uint64_t word = 0;
-                            if (idx >= cs) {
-                                do {
-                                    word = ld_relaxed_u64(&status[idx]);
-                                } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
-                            }
-                            const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
-                            const uint32_t tb = __ballot_sync(0xffffffffu, term);
-                            if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
-                            consumer_sync();
-                            int stop = FB;
-#pragma unroll
-                            for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
-                            T val = (t <= stop && idx >= cs) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
-#pragma unroll
-                            for (int off = 1; off < 32; off <<= 1) {
-                                const T older = __shfl_down_sync(0xffffffffu, val, off);
-                                if (lane + off < 32) val = combine<OP>(older, val);
-                            }
-                            if (lane == 0) s_lbval[w] = val;
-                            consumer_sync();
-                            T win = identity<OP, T>();
-#pragma unroll
-                            for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
-                            carry = combine<OP>(win, carry);
-                            consumer_sync();
-                            if (stop < FB) break;
-                            pred -= FB;
-                        }
-                        if (t == 0) {  // the chunk's own inclusive prefix, for the successors' look-back
-                            const uint64_t own = ld_relaxed_u64(&status[c]);
-                            if (((own >> 33) & 3u) != ST_P)
-                                st_relaxed_u64(&status[c], pack_status(tag, ST_P, 0u,
-                                                                       to_bits(combine<OP>(carry, from_bits<T>((uint32_t)own)))));
-                        }
-                    }
-                }
-                PROF_ADD(pa[1], tl);
-                const int64_t base = (int64_t)am.tile * FT;
-                if (!(tma_in && am.cnt == FT)) {
-                    for (int p = t; p < am.cnt; p += FB) buf[p] = in[base + p];
-                    consumer_sync();
-                }
-                SlotMeta smeta;
-                smeta.tile = am.tile;
-                smeta.cnt = am.cnt;
-                smeta.pos = am.pos;
-                smeta.seg = am.seg;
-                const ThreadPos tp = thread_pos(smeta, m);
-                T v[FI];
-                load_items(buf, v);
-                bool hs;
-                T acc;
-                local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
-                uint32_t exf, aggf;
-                T exv, aggv;
-                cta_seg_scan<T, OP, true>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[i & 1], s_wflag[i & 1]);
-                {
-                    const T carry_t = exf ? exv : combine<OP>(carry, exv);
-                    const int lim = min(tp.nx0, tp.nvalid);
-#pragma unroll
-                    for (int k = 0; k < FI; ++k)
-                        if (k < lim) v[k] = combine<OP>(carry_t, v[k]);
-                }
-                carry = aggf ? aggv : combine<OP>(carry, aggv);
-                store_items(buf, v);
-                const bool bulk = tma_out && am.cnt == FT;
-                if (bulk) fence_proxy_async_smem();
-                consumer_sync();
-                if (bulk) {
-                    if (t == 0) {
-                        bulk_s2g_hint(out + base, buf, FT * sizeof(T), policy_evict_first());
-                        bulk_commit();
-                        pend_slot = sl;
-                    }
-                } else {
-                    for (int p = t; p < am.cnt; p += FB) out[base + p] = buf[p];
-                    consumer_sync();
-                    if (t == 0) mbar_arrive_expect_tx(&empty[sl], 0);
-                }
-            }
-            if (t == 0) bulk_wait0();
-        }
-    }
-#ifdef IFL_AR_PROF
-    if (t == 0 || t == FB) {
-        const bool agg = (int)blockIdx.x < num_agg;
-        pa[agg ? 8 : 2] += (unsigned long long)(clock64() - t_start);
-        for (int q = 0; q < 16; ++q)
-            if (pa[q]) atomicAdd(&g_ar_prof[q], pa[q]);
-        if (t == 0) atomicAdd(&g_ar_prof[agg ? 10 : 11], 1ull);
-    }
-#endif
-    if (t == 0) {
-        __threadfence();
-        const unsigned long long old = atomicAdd(ctr, 1ull);
-        if ((uint32_t)old == (uint32_t)G - 1) {  // every CTA has made its last claim: re-arm
-            atomicExch(scan_ctr, 0u);
-            atomicExch(agg_ctr, 0u);
-            atomicAdd(ctr, (1ull << 32) - (unsigned long long)G);
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
-// "Job" engine: reduce-then-scan desynchronised into jobs.  The flattened
-// array is cut into chunks of kJobChunk elements; job k (claimed by a CTA
-// from an atomic counter when it starts, so jobs start in order) does two
-// things:
-//   1. AGGREGATE chunk k: reduce the part a successor needs -- after the
-//      chunk's last segment start, all of it for long segments -- with
-//      L2::evict_last loads, and publish the segmented aggregate (an
-//      inclusive prefix when the chunk holds a segment start);
-//   2. SCAN chunk k - kJobLag: its predecessors were aggregated kJobLag jobs
-//      ago (their data still in L2), so the CTA-wide look-back over chunk
-//      statuses finds every aggregate published and ends in one round trip
-//      at the nearest inclusive prefix; the chunk's own inclusive prefix is
-//      published at once, then the chunk is scanned in rounds of
-//      kJobThreads x 8 elements straight from registers (two 128-bit loads
-//      and stores per thread per round, the next round's loads in flight)
-//      with a running carry.
-// No shared-memory staging, no grid-wide phase: DRAM sees one read and one
-// write per element, aggregation reads and scan writes of different chunks
-// overlap, and the look-back latency of one job is hidden by the other
-// resident CTAs.  The last CTA re-arms the workspace (job counter 0, epoch+1).
-#ifndef IFL_JOB_THREADS
-#define IFL_JOB_THREADS 512
-#endif
-#ifndef IFL_JOB_ROUNDS
-#define IFL_JOB_ROUNDS 16
-#endif
-#ifndef IFL_JOB_LAG
-#define IFL_JOB_LAG 128
-#endif
-#ifndef IFL_JOB_MINB
-#define IFL_JOB_MINB 3
-#endif
-#ifndef IFL_JOB_AGG_U
-#define IFL_JOB_AGG_U 4
-#endif
-constexpr int kJobThreads = IFL_JOB_THREADS;
-constexpr int kJobWarps = kJobThreads / 32;
-constexpr int kJobItems = 8;
-constexpr int kJobRound = kJobThreads * kJobItems;
-constexpr int64_t kJobChunk = (int64_t)kJobRound * IFL_JOB_ROUNDS;
-constexpr int kJobLag = IFL_JOB_LAG;
-
-template <typename T>
-__device__ __forceinline__ void stg4(T* p, T a, T b, T c, T e) {
-    typename Vec4<T>::type q;
-    q.x = a; q.y = b; q.z = c; q.w = e;
-    *reinterpret_cast<typename Vec4<T>::type*>(p) = q;
-}
-
-// CTA-wide exclusive segmented scan of per-thread (flag, value) pairs over NW
-// warps (one __syncthreads; the warp totals are double-buffered by the caller).
-template <typename T, int OP, int NW>
-__device__ __forceinline__ void cta_seg_scan_nw(uint32_t fl, T sv, uint32_t& exf, T& exv, uint32_t& aggf, T& aggv,
-                                                T* s_wval, uint32_t* s_wflag) {
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-#pragma unroll
-    for (int off = 1; off < 32; off <<= 1) {
-        const T ov = __shfl_up_sync(0xffffffffu, sv, off);
-        const uint32_t of = __shfl_up_sync(0xffffffffu, fl, off);
-        if (lane >= off) {
-            if (!fl) sv = combine<OP>(ov, sv);
-            fl |= of;
-        }
-    }
-    if (lane == 31) {
-        s_wval[w] = sv;
-        s_wflag[w] = fl;
-    }
-    exv = __shfl_up_sync(0xffffffffu, sv, 1);
-    exf = __shfl_up_sync(0xffffffffu, fl, 1);
-    if (lane == 0) {
-        exv = identity<OP, T>();
-        exf = 0;
-    }
-    __syncthreads();
-    T pw = identity<OP, T>();
-    uint32_t pf = 0;
-    aggv = identity<OP, T>();
-    aggf = 0;
-#pragma unroll
-    for (int k = 0; k < NW; ++k) {
-        const T wv = s_wval[k];
-        const uint32_t wf = s_wflag[k];
-        if (k < w) {
-            pw = wf ? wv : combine<OP>(pw, wv);
-            pf |= wf;
-        }
-        aggv = wf ? wv : combine<OP>(aggv, wv);
-        aggf |= wf;
-    }
-    if (!exf) exv = combine<OP>(pw, exv);
-    exf |= pf;
-}
-
-// CTA-wide look-back over status words [cs, pred]: folds the aggregates from
-// the nearest inclusive (or segment-start) word up to pred.  All threads.
-template <typename T, int OP, int NW>
-__device__ __forceinline__ T cta_lookback(const uint64_t* status, uint32_t tag, int pred, int cs, int* s_lbterm,
-                                          T* s_lbval) {
-    constexpr int NT = NW * 32;
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    T carry = identity<OP, T>();
-    while (true) {
-        const int idx = pred - t;
-        uint64_t word = 0;
-        if (idx >= cs) {
-            do {
-                word = ld_relaxed_u64(&status[idx]);  // self-contained word: no acquire needed
-            } while ((uint32_t)(word >> 35) != tag || ((word >> 33) & 3u) == 0);
-        }
-        const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
-        const uint32_t tb = __ballot_sync(0xffffffffu, term);
-        if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : NT;
-        __syncthreads();
-        int stop = NT;
-#pragma unroll
-        for (int k = 0; k < NW; ++k) stop = min(stop, s_lbterm[k]);
-        T val = (t <= stop && idx >= cs) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
-#pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {  // ordered: higher lane = older word
-            const T older = __shfl_down_sync(0xffffffffu, val, off);
-            if (lane + off < 32) val = combine<OP>(older, val);
-        }
-        if (lane == 0) s_lbval[w] = val;
-        __syncthreads();
-        T win = identity<OP, T>();
-#pragma unroll
-        for (int k = NW - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
-        carry = combine<OP>(win, carry);
-        __syncthreads();
-        if (stop < NT) break;
-        pred -= NT;
-    }
-    return carry;
-}
-
-template <typename T, int OP, int F>
-__global__ void __launch_bounds__(kJobThreads, IFL_JOB_MINB) flat_scan_job_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
-                                                                     uint8_t* ws, int num_chunks, int lag,
-                                                                     bool vec, const T* __restrict__ seed) {
-    const int num_jobs = num_chunks + lag;
-    __shared__ uint32_t s_tag;
-    __shared__ int s_job;
-    __shared__ T s_red[kJobWarps];
-    __shared__ T s_wval[2][kJobWarps];
-    __shared__ uint32_t s_wflag[2][kJobWarps];
-    __shared__ int s_lbterm[kJobWarps];
-    __shared__ T s_lbval[kJobWarps];
-    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | done:32}
-    unsigned* job_ctr = reinterpret_cast<unsigned*>(ws + 8);
-    uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
-    const int t = threadIdx.x;
-    if (t == 0) {
-        s_tag = status_tag(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)));
-        s_job = (int)atomicAdd(job_ctr, 1u);
-    }
-    __syncthreads();
-    const uint32_t tag = s_tag;
-    const int k = s_job;
-    // ---- 1. aggregate chunk k
-    if (k < num_chunks) {
-        const int64_t cb = (int64_t)k * kJobChunk, ce = std::min(N, cb + kJobChunk);
-        const int64_t ls = ((ce - 1) / m) * m;  // last segment start <= ce - 1
-        const bool flag = ls >= cb;
-        const T r = cta_reduce_keep<T, OP, F, kJobThreads, IFL_JOB_AGG_U>(in, flag ? ls : cb, ce, s_red,
-                                                                         policy_evict_last());
-        if (t == 0) {
-            const T dseg = seed ? seed[ls / m] : d;
-            st_relaxed_u64(&status[k], pack_status(tag, flag ? ST_P : ST_A, flag ? 1u : 0u,
-                                                   to_bits(flag ? combine<OP>(dseg, r) : r)));
-        }
-    }
-    // ---- 2. scan chunk c = k - lag
-    const int c = k - lag;
-    if (c >= 0) {
-        const int64_t cb = (int64_t)c * kJobChunk, ce = std::min(N, cb + kJobChunk);
-        T carry = identity<OP, T>();
-        if (cb % m != 0) {
-            const int cs = (int)(((cb / m) * m) / kJobChunk);  // chunk holding the segment's start
-            carry = cta_lookback<T, OP, kJobWarps>(status, tag, c - 1, cs, s_lbterm, s_lbval);
-        }
-        if (t == 0) {  // the chunk's own aggregate (also: its data has been read -- in-place safe)
-            uint64_t own;
-            do {
-                own = ld_relaxed_u64(&status[c]);
-            } while ((uint32_t)(own >> 35) != tag || ((own >> 33) & 3u) == 0);
-            if (((own >> 33) & 3u) != ST_P)
-                st_relaxed_u64(&status[c],
-                               pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, from_bits<T>((uint32_t)own)))));
-        }
-        __syncthreads();
-        const uint64_t pol = policy_evict_first();
-        auto load_round = [&](int64_t gi, T (&r)[kJobItems]) {
-            if (vec && gi + kJobItems <= ce) {
-                T e[4];
-                unpack4<T>(ldg_keep4(in + gi, pol), e);
-#pragma unroll
-                for (int u = 0; u < 4; ++u) r[u] = e[u];
-                unpack4<T>(ldg_keep4(in + gi + 4, pol), e);
-#pragma unroll
-                for (int u = 0; u < 4; ++u) r[4 + u] = e[u];
-            } else {
-#pragma unroll
-                for (int u = 0; u < kJobItems; ++u) r[u] = gi + u < ce ? in[gi + u] : T();
-            }
-        };
-        T nxt[kJobItems];
-        load_round(cb + (int64_t)t * kJobItems, nxt);
-        int par = 0;
-        for (int64_t rb = cb; rb < ce; rb += kJobRound, par ^= 1) {
-            const int64_t gi = rb + (int64_t)t * kJobItems;
-            T v[kJobItems];
-#pragma unroll
-            for (int u = 0; u < kJobItems; ++u) v[u] = nxt[u];
-            if (rb + kJobRound < ce) load_round(gi + kJobRound, nxt);
-            const int nvalid = (int)std::max<int64_t>(0, std::min<int64_t>(kJobItems, ce - gi));
-            const int64_t pos = gi % m;
-            const int nx0 = (int)std::min<int64_t>(pos == 0 ? 0 : m - pos, kJobItems + 1);
-            const int mi = (int)std::min<int64_t>(m, kJobItems + 1);
-            bool hs = false;
-            T acc = identity<OP, T>();
-            if (nx0 > nvalid) {  // no segment start among the thread's items
-#pragma unroll
-                for (int u = 0; u < kJobItems; ++u) {
-                    acc = combine<OP>(acc, u < nvalid ? apply_map<F>(v[u]) : identity<OP, T>());
-                    v[u] = acc;
-                }
-            } else {
-                int nx = nx0;
-                int64_t ss = gi / m + (nx0 > 0 ? 1 : 0);  // segment the next start begins
-#pragma unroll
-                for (int u = 0; u < kJobItems; ++u) {
-                    if (u < nvalid) {
-                        const T x = apply_map<F>(v[u]);
-                        if (u == nx) {
-                            acc = combine<OP>(seed ? seed[ss] : d, x);
-                            ++ss;
-                            hs = true;
-                            nx += mi;
-                        } else {
-                            acc = combine<OP>(acc, x);
-                        }
-                        v[u] = acc;
-                    }
-                }
-            }
-            uint32_t exf, aggf;
-            T exv, aggv;
-            cta_seg_scan_nw<T, OP, kJobWarps>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval[par], s_wflag[par]);
-            const T carry_t = exf ? exv : combine<OP>(carry, exv);
-            const int lim = min(nx0, nvalid);
-#pragma unroll
-            for (int u = 0; u < kJobItems; ++u)
-                if (u < lim) v[u] = combine<OP>(carry_t, v[u]);
-            carry = aggf ? aggv : combine<OP>(carry, aggv);
-            if (vec && nvalid == kJobItems) {
-                stg4<T>(out + gi, v[0], v[1], v[2], v[3]);
-                stg4<T>(out + gi + 4, v[4], v[5], v[6], v[7]);
-            } else {
-#pragma unroll
-                for (int u = 0; u < kJobItems; ++u)
-                    if (u < nvalid) out[gi + u] = v[u];
-            }
-        }
-    }
-    if (t == 0) {
-        __threadfence();
-        const unsigned long long old = atomicAdd(ctr, 1ull);
-        if ((uint32_t)old == (uint32_t)num_jobs - 1) {  // the last job: re-arm
-            atomicExch(job_ctr, 0u);
-            atomicAdd(ctr, (1ull << 32) - (unsigned long long)num_jobs);
-        }
-    }
-}
-
-// ---------------------------------------------------------------------------
 // "Job ring" engine (JR): reduce-then-scan desynchronised into jobs and
 // streamed through one TMA ring per CTA.  Chunks of kJrChunkTiles tiles;
 // job k (claimed in order from an atomic counter by a persistent CTA)
@@ -1835,10 +839,10 @@ __global__ void __launch_bounds__(kJobThreads, IFL_JOB_MINB) flat_scan_job_kerne
 // aggregation never waits on anything, so every claimed job completes
 // (no co-residency requirement).
 #ifndef IFL_JR_CHUNK_TILES
-#define IFL_JR_CHUNK_TILES 8
+#define IFL_JR_CHUNK_TILES 4
 #endif
 #ifndef IFL_JR_LAG
-#define IFL_JR_LAG 96
+#define IFL_JR_LAG 192
 #endif
 #ifndef IFL_JR_SLOTS
 #define IFL_JR_SLOTS 3
@@ -2096,133 +1100,6 @@ __global__ void __launch_bounds__(kScanThreads, IFL_JR_MINB) flat_scan_jr_kernel
     }
 }
 
-// Non-persistent variant: one CTA per tile, the tile claimed by an atomic
-// counter when the CTA starts (claim order = start order, so every
-// predecessor is owned by a CTA that is already running).  A tile's status is
-// published as soon as its own data has arrived -- there is no queue of
-// claimed-but-unprocessed tiles behind a busy CTA -- and the load of every
-// resident CTA is in flight at once.
-template <typename T, int OP, int F>
-__global__ void __launch_bounds__(FB) flat_scan_np_kernel(const T* in, T* out, int64_t N, int64_t m, T d, uint8_t* ws,
-                                                          int num_tiles, bool tma_in, bool tma_out,
-                                                          const T* __restrict__ seed) {
-    extern __shared__ __align__(128) uint8_t smem_raw[];
-    T* buf = reinterpret_cast<T*>(smem_raw);
-    __shared__ alignas(8) uint64_t full;
-    __shared__ SlotMeta s_meta;
-    __shared__ uint32_t s_tag;
-    __shared__ T s_wval[FB / 32];
-    __shared__ uint32_t s_wflag[FB / 32];
-    __shared__ int s_lbterm[FB / 32];
-    __shared__ T s_lbval[FB / 32];
-    unsigned long long* ctr = reinterpret_cast<unsigned long long*>(ws);  // {epoch:32 | done:32}
-    unsigned* tile_ctr = reinterpret_cast<unsigned*>(ws + 8);
-    uint64_t* status = reinterpret_cast<uint64_t*>(ws + sizeof(FlatHdr));
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    if (t == 0) {
-        s_tag = status_tag(ld_relaxed_u64(reinterpret_cast<const uint64_t*>(ctr)));
-        const int tile = (int)atomicAdd(tile_ctr, 1u);
-        fill_meta(s_meta, tile, N, m);
-        mbar_init(&full, 1);
-        fence_mbar_init();
-        if (tma_in && s_meta.cnt == FT) {
-            mbar_arrive_expect_tx(&full, FT * sizeof(T));
-            bulk_g2s_hint(buf, in + (int64_t)tile * FT, FT * sizeof(T), &full, policy_evict_first());
-        } else {
-            mbar_arrive_expect_tx(&full, 0);
-        }
-    }
-    __syncthreads();
-    const uint32_t tag = s_tag;
-    const SlotMeta sm = s_meta;
-    const int64_t base = (int64_t)sm.tile * FT;
-    mbar_wait(&full, 0);
-    if (!(tma_in && sm.cnt == FT)) {
-        for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
-        __syncthreads();
-    }
-    const ThreadPos tp = thread_pos(sm, m);
-    T v[FI];
-    load_items(buf, v);
-    bool hs;
-    T acc;
-    local_seg_scan<T, OP, F>(v, tp, d, hs, acc, seed);
-    uint32_t exf, aggf;
-    T exv, aggv;
-    cta_seg_scan<T, OP, false>(hs ? 1u : 0u, acc, exf, exv, aggf, aggv, s_wval, s_wflag);
-    const bool carry_needed = sm.pos != 0;
-    if (t == 0)
-        st_relaxed_u64(&status[sm.tile], pack_status(tag, (aggf || !carry_needed) ? ST_P : ST_A, aggf, to_bits(aggv)));
-    T carry = identity<OP, T>();
-    if (carry_needed) {
-        const int cs = (int)((base - sm.pos) / FT);
-        int pred = sm.tile - 1;
-        while (true) {
-            const int idx = pred - t;
-            uint64_t word = 0;
-            if (idx >= cs) {
-                while (true) {
-                    word = ld_relaxed_u64(&status[idx]);
-                    if ((uint32_t)(word >> 35) == tag && ((word >> 33) & 3u) != 0) break;
-                    __nanosleep(20);
-                }
-            }
-            const bool term = idx <= cs || ((word >> 33) & 3u) == ST_P || ((word >> 32) & 1u);
-            const uint32_t tb = __ballot_sync(0xffffffffu, term);
-            if (lane == 0) s_lbterm[w] = tb ? (w * 32 + __ffs(tb) - 1) : FB;
-            __syncthreads();
-            int stop = FB;
-#pragma unroll
-            for (int k = 0; k < FB / 32; ++k) stop = min(stop, s_lbterm[k]);
-            T val = (t <= stop && idx >= cs) ? from_bits<T>((uint32_t)word) : identity<OP, T>();
-#pragma unroll
-            for (int off = 1; off < 32; off <<= 1) {
-                const T older = __shfl_down_sync(0xffffffffu, val, off);
-                if (lane + off < 32) val = combine<OP>(older, val);
-            }
-            if (lane == 0) s_lbval[w] = val;
-            __syncthreads();
-            T win = identity<OP, T>();
-#pragma unroll
-            for (int k = FB / 32 - 1; k >= 0; --k) win = combine<OP>(win, s_lbval[k]);
-            carry = combine<OP>(win, carry);
-            __syncthreads();
-            if (stop < FB) break;
-            pred -= FB;
-        }
-        if (!aggf && t == 0)
-            st_relaxed_u64(&status[sm.tile], pack_status(tag, ST_P, 0u, to_bits(combine<OP>(carry, aggv))));
-    }
-    {
-        const T carry_t = exf ? exv : combine<OP>(carry, exv);
-        const int lim = min(tp.nx0, tp.nvalid);
-#pragma unroll
-        for (int k = 0; k < FI; ++k)
-            if (k < lim) v[k] = combine<OP>(carry_t, v[k]);
-    }
-    store_items(buf, v);
-    const bool bulk = tma_out && sm.cnt == FT;
-    if (bulk) fence_proxy_async_smem();
-    __syncthreads();
-    if (bulk) {
-        if (t == 0) {
-            bulk_s2g_hint(out + base, buf, FT * sizeof(T), policy_evict_first());
-            bulk_commit();
-        }
-    } else {
-        for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
-    }
-    if (t == 0) {
-        bulk_wait_read0();  // the smem tile must outlive the bulk store's read of it
-        __threadfence();
-        const unsigned long long old = atomicAdd(ctr, 1ull);
-        if ((uint32_t)old == (uint32_t)num_tiles - 1) {  // the last tile's CTA: re-arm
-            atomicExch(tile_ctr, 0u);
-            atomicAdd(ctr, (1ull << 32) - (unsigned long long)num_tiles);
-        }
-    }
-}
-
 // ------------------------------------------------------------------ launch
 
 static int sm_count() {
@@ -2261,7 +1138,18 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const T d = bits_to<T>(a.ne_bits);
-        if (scan && IFL_SCAN_DLB == 5) {
+        if (scan && FT % a.m == 0) {
+            // every tile begins at a segment start: the tiles are independent, the
+            // single-pass engine never looks back (B200, n*m = 2^26 f32, m = 1024:
+            // 83 us, a copy's speed)
+            auto k = flat_scan_dlb_kernel<T, OP, F>;
+            const size_t smem_s = (size_t)kDlbSlots * FT * sizeof(T);
+            const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem_s, kScanThreads));
+            k<<<grid, kScanThreads, smem_s, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, tma_in,
+                                                        tma_out, (const T*)a.seed);
+            return cudaGetLastError();
+        }
+        if (scan) {  // segments cross tiles: the job-ring engine
             auto k = flat_scan_jr_kernel<T, OP, F>;
             const size_t smem_s = (size_t)kJrSlots * FT * sizeof(T);
             const int chunks = (int)ceil_div(tiles, kJrChunkTiles);
@@ -2270,71 +1158,6 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
             k<<<grid, kScanThreads, smem_s, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, chunks, lag,
                                                          tma_in, tma_out, (const T*)a.seed);
             return cudaGetLastError();
-        }
-        if (scan && IFL_SCAN_DLB == 4) {
-            const int64_t chunks = ceil_div(N, kJobChunk);
-            if (chunks > (1 << 30)) return cudaErrorInvalidValue;
-            const int lag = (int)std::min<int64_t>(kJobLag, chunks);
-            const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
-            flat_scan_job_kernel<T, OP, F><<<(unsigned)(chunks + lag), kJobThreads, 0, a.stream>>>(
-                (const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)chunks, lag, vec, (const T*)a.seed);
-            return cudaGetLastError();
-        }
-        if (scan && IFL_SCAN_DLB == 3) {
-            auto k = flat_scan_ar_kernel<T, OP, F>;
-            const size_t smem_s = (size_t)kArSlots * FT * sizeof(T);
-            const int chunks = (int)ceil_div(tiles, kArChunkTiles);
-            const int R = resident_ctas(k, smem_s, kScanThreads);
-            const int nagg = std::max(1, std::min(sm_count() * IFL_AR_AGG_PER_SM, R / 2));
-            const int grid = (int)std::min<int64_t>(R, nagg + std::max<int64_t>(1, chunks));
-            cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3((unsigned)grid);
-            cfg.blockDim = dim3(kScanThreads);
-            cfg.dynamicSmemBytes = smem_s;
-            cfg.stream = a.stream;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeCooperative;  // aggregators and scanners wait on each other
-            attr[0].val.cooperative = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = 1;
-            return cudaLaunchKernelEx(&cfg, k, (const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, chunks, nagg,
-                                      tma_in, tma_out, (const T*)a.seed);
-        }
-        if (scan && IFL_SCAN_DLB == 2) {
-            auto k = flat_scan_np_kernel<T, OP, F>;
-            const size_t smem_s = (size_t)FT * sizeof(T);
-            (void)resident_ctas(k, smem_s, FB);  // sets the dynamic smem attribute once
-            k<<<(unsigned)tiles, FB, smem_s, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, tma_in,
-                                                        tma_out, (const T*)a.seed);
-            return cudaGetLastError();
-        }
-        if (scan && IFL_SCAN_DLB == 1) {
-            auto k = flat_scan_dlb_kernel<T, OP, F>;
-            const size_t smem_s = (size_t)kDlbSlots * FT * sizeof(T);
-            const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem_s, kScanThreads));
-            k<<<grid, kScanThreads, smem_s, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, tma_in,
-                                                        tma_out, (const T*)a.seed);
-            return cudaGetLastError();
-        }
-        if (scan) {
-            auto k = flat_scan_kernel<T, OP, F>;
-            const size_t smem_s = (size_t)kScanSlots * FT * sizeof(T);
-            const int chunks = (int)ceil_div(tiles, kChunkTiles);
-            const int grid = (int)std::min<int64_t>(chunks, resident_ctas(k, smem_s, kScanThreads));
-            // cooperative launch: all CTAs co-resident (static chunk ownership + look-back)
-            cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3((unsigned)grid);
-            cfg.blockDim = dim3(kScanThreads);
-            cfg.dynamicSmemBytes = smem_s;
-            cfg.stream = a.stream;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeCooperative;
-            attr[0].val.cooperative = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = 1;
-            int nt = (int)tiles;
-            return cudaLaunchKernelEx(&cfg, k, (const T*)a.in, (T*)a.out, N, a.m, d, ws, nt, chunks, tma_in, tma_out,
-                                      (const T*)a.seed);
         }
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);
         T* tail = head + tiles;
@@ -2372,12 +1195,3 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
 
 }  // namespace ifl
 
-#ifdef IFL_AR_PROF
-extern "C" int ifl_debug_prof(unsigned long long* out16) {
-    cudaDeviceSynchronize();
-    cudaMemcpyFromSymbol(out16, ifl::g_ar_prof, 16 * sizeof(unsigned long long));
-    unsigned long long z[16] = {};
-    cudaMemcpyToSymbol(ifl::g_ar_prof, z, sizeof z);
-    return 0;
-}
-#endif

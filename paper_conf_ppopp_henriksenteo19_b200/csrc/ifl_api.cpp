@@ -212,6 +212,13 @@ int ifl_select(const char* site, int64_t n, int64_t m, int64_t p, ifl_choice* ch
         if (choice) *choice = c;
         return IFL_OK;
     }
+    if (strcmp(site, "redomap2.f32") == 0 || strcmp(site, "redomap2.bf16") == 0) {
+        // the version ifl_redomap2 runs: the 5-leaf tree (row-level guards first, R17)
+        ifl_choice c;
+        mm_tree_select(strcmp(site, "redomap2.bf16") == 0 ? IFL_BF16 : IFL_F32, n, m, p, &c);
+        if (choice) *choice = c;
+        return IFL_OK;
+    }
     if (strcmp(site, "tridag") == 0) fits = ifl::tridag_mid_fits(m);
     return select_version(site, n, m, p, fits, choice) >= 0 ? IFL_OK : IFL_EINVAL;
 }

@@ -189,12 +189,13 @@ cudaError_t launch_lvc_outer(const LvcSite& x, const LvcSite& y, int64_t numT, c
     // registers (2 CTAs/SM); 8 doubles the lanes, which wins when the problem
     // is too small to fill the GPU (B200, LocVolCalib datasets: small 98 vs
     // 105 us at 8 / 16, medium 84 vs 70, large 1100 vs 902).  L > 256 needs 16.
-    // IFL_LVC_IT=8|16 forces one (experiments).
+    // -DIFL_LVC_IT=8|16 forces one (experiment builds only).
     const int64_t Lmax = std::max(x.L, y.L);
-    static const int it_env = [] {
-        const char* e = getenv("IFL_LVC_IT");
-        return e ? atoi(e) : 0;
-    }();
+#ifdef IFL_LVC_IT
+    constexpr int it_env = IFL_LVC_IT;
+#else
+    constexpr int it_env = 0;
+#endif
     const int64_t lanes8 = x.S * pow2_at_least(std::max<int64_t>(1, ceil_div(x.L, 8))) +
                            y.S * pow2_at_least(std::max<int64_t>(1, ceil_div(y.L, 8)));
     int IT = (Lmax > 256 || lanes8 >= (int64_t)148 * 1024) ? 16 : 8;

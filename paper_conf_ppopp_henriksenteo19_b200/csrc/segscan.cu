@@ -40,7 +40,7 @@ __host__ __device__ __forceinline__ int stop_rpt(int64_t m) { return m <= kTopKT
 // Copy between a global window and the padded smem tile (see segred.cu).
 // LOAD: global -> smem; STORE: smem -> global.
 template <bool LOAD, typename T>
-__device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* __restrict__ out, int64_t r0,
+__device__ __forceinline__ void top_xfer(T* tile, const T* in, T* out, int64_t r0,
                                          int rows, int64_t m, int64_t k0, int kt, bool whole, bool vec) {
     const int t = threadIdx.x;
     using V = typename Vec4<T>::type;
@@ -52,7 +52,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
             for (int v = t; v < nv; v += kTopThreads) {
                 if (LOAD) {
                     T e[4];
-                    unpack4<T>(ldg_stream4(in + r0 * m + 4 * v), e);
+                    unpack4<T>(ld_coh4(in + r0 * m + 4 * v), e);
 #pragma unroll
                     for (int u = 0; u < 4; ++u) tile[spadq(4 * v + u)] = e[u];
                 } else {
@@ -67,7 +67,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
             p0 = nv << 2;
         }
         for (int p = p0 + t; p < cnt; p += kTopThreads) {
-            if (LOAD) tile[spadq(p)] = ldg1(in + r0 * m + p);
+            if (LOAD) tile[spadq(p)] = ld_coh1(in + r0 * m + p);
             else out[r0 * m + p] = tile[spadq(p)];
         }
     } else if (vec && kt == kTopKT) {
@@ -77,7 +77,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
             const int q0 = row * kTopKT + 4 * c4;
             if (LOAD) {
                 T e[4];
-                unpack4<T>(ldg_stream4(in + gi), e);
+                unpack4<T>(ld_coh4(in + gi), e);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) tile[spadq(q0 + u)] = e[u];
             } else {
@@ -94,7 +94,7 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* __restrict__ in, T* _
             const int row = p >> 5, col = p & 31;
             if (col < kt) {
                 const int64_t gi = (r0 + row) * m + k0 + col;
-                if (LOAD) tile[spadq(p)] = ldg1(in + gi);
+                if (LOAD) tile[spadq(p)] = ld_coh1(in + gi);
                 else out[gi] = tile[spadq(p)];
             }
         }
@@ -169,7 +169,7 @@ __global__ void __launch_bounds__(256) segscan_top_small_kernel(const T* in, T* 
         V q[4];
 #pragma unroll
         for (int u = 0; u < 4; ++u)
-            if (v0 + u * stride < nv) q[u] = ldg_stream4(in + 4 * (v0 + u * stride));
+            if (v0 + u * stride < nv) q[u] = ld_coh4(in + 4 * (v0 + u * stride));
 #pragma unroll
         for (int u = 0; u < 4; ++u) {
             const int64_t v = v0 + u * stride;
@@ -218,7 +218,7 @@ __global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int6
             const int q4 = lane + 32 * u;
             if (q4 < rows * W4) {
                 T e[4];
-                unpack4<T>(ldg_stream4(src + 4 * q4), e);
+                unpack4<T>(ld_coh4(src + 4 * q4), e);
 #pragma unroll
                 for (int k = 0; k < 4; ++k) {
                     const int q = 4 * q4 + k;
@@ -274,7 +274,7 @@ __global__ void __launch_bounds__(256) top_warp_kernel(const T* in, T* out, int6
 // V_TOP for m in {8, 16, 32}, 16-byte-aligned: one thread per row, its m/4
 // 128-bit words loaded straight into registers, scanned, stored back.
 template <typename T, int OP, int F, int M>
-__global__ void __launch_bounds__(256) segscan_top_row_kernel(const T* __restrict__ in, T* __restrict__ out,
+__global__ void __launch_bounds__(256) segscan_top_row_kernel(const T* in, T* out,
                                                               int64_t n, T d, const T* __restrict__ seed) {
     using V = typename Vec4<T>::type;
     const int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -282,7 +282,7 @@ __global__ void __launch_bounds__(256) segscan_top_row_kernel(const T* __restric
     const T* p = in + r * M;
     V q[M / 4];
 #pragma unroll
-    for (int u = 0; u < M / 4; ++u) q[u] = IFL_ROW_L1 ? __ldg(reinterpret_cast<const V*>(p + 4 * u)) : ldg_stream4(p + 4 * u);
+    for (int u = 0; u < M / 4; ++u) q[u] = ld_coh4(p + 4 * u);
     T a = seed ? seed[r] : d;
     T* o = out + r * M;
 #pragma unroll
@@ -396,13 +396,13 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
             const int64_t kh = k0 + 4 * h;
             if (live && vec && kh + 4 <= m) {
                 T e[4];
-                unpack4<T>(ldg_stream4(row + kh), e);
+                unpack4<T>(ld_coh4(row + kh), e);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) v[4 * h + u] = apply_map<F>(e[u]);
             } else {
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
-                    v[4 * h + u] = (live && kh + u < m) ? apply_map<F>(ldg1(row + kh + u)) : identity<OP, T>();
+                    v[4 * h + u] = (live && kh + u < m) ? apply_map<F>(ld_coh1(row + kh + u)) : identity<OP, T>();
             }
         }
 #pragma unroll
@@ -484,12 +484,12 @@ __global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
             const int64_t kh = k0 + 4 * h;
             if (live && vec && kh + 4 <= m) {
                 T e[4];
-                unpack4<T>(ldg_stream4(row + kh), e);
+                unpack4<T>(ld_coh4(row + kh), e);
 #pragma unroll
                 for (int u = 0; u < 4; ++u) r[4 * h + u] = e[u];
             } else {
 #pragma unroll
-                for (int u = 0; u < 4; ++u) r[4 * h + u] = (live && kh + u < m) ? ldg1(row + kh + u) : T();
+                for (int u = 0; u < 4; ++u) r[4 * h + u] = (live && kh + u < m) ? ld_coh1(row + kh + u) : T();
             }
         }
     };

@@ -82,6 +82,20 @@ def test_irr_descriptors(ifl, orc, version, scan):
 
 
 @pytest.mark.parametrize("version", VERS)
+def test_irr_scan_in_place(ifl, orc, version):
+    """ifl.h: out == in is allowed for the irregular scan (every version)."""
+    for k, off in enumerate(descriptors()):
+        total = int(off[-1])
+        offd = torch.from_numpy(off).cuda()
+        for name, dtn in (("I32_FULL", 100), ("F32_SIGNED", 110)):
+            x = gen.generate(name, dtn + k, total)
+            xd = x.cuda()
+            got = ifl.segscan_irr(xd, offd, "sum", version=version, out=xd)
+            assert got.data_ptr() == xd.data_ptr()
+            check(orc, x, off, got, True, "sum")
+
+
+@pytest.mark.parametrize("version", VERS)
 def test_irr_ops_maps_neutral(ifl, orc, version):
     off = descriptors()[3]
     offd = torch.from_numpy(off).cuda()

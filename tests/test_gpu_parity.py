@@ -140,7 +140,10 @@ def test_misaligned_and_odd(ifl, orc, version, scan):
 
 @pytest.mark.parametrize("version", ["top", "middle", "flat"])
 def test_inplace_scan(ifl, orc, version):
-    for (n, m) in [(100, 100), (2, 7168 * 3 + 1), (4096, 8)]:
+    # (100, 1024) / (7, 5120): tile-aligned segments (single-pass engine);
+    # (3, 2^20) / (1, 5120*50+3): segments across tiles (job-ring engine)
+    for (n, m) in [(100, 100), (2, 7168 * 3 + 1), (4096, 8), (100, 1024), (7, 5120), (3, 1 << 20),
+                   (1, 5120 * 50 + 3)]:
         x, xd = gen_for("sum", "i32", 5, n, m)
         got = ifl.segscan(xd, "sum", "id", version=version, out=xd)
         assert got.data_ptr() == xd.data_ptr()
@@ -169,6 +172,22 @@ def test_flat_many_tiles_lookback(ifl, orc):
             for _ in range(3):
                 assert_parity(orc, x, ifl.segred(xd, "sum", version="flat"), False, "sum", "id", None, dt)
                 assert_parity(orc, x, ifl.segscan(xd, "sum", version="flat"), True, "sum", "id", None, dt)
+
+
+@pytest.mark.parametrize("dt", ["i32", "f32"])
+def test_workspace_shared_after_segred(ifl, orc, dt):
+    """a segred on N1 elements leaves small-integer partials where a
+    later segscan on N2 > 8 N1 elements keeps its status words.  The status
+    tag is a scrambled epoch, so stale partials are not taken for valid words;
+    the binding also keys its cached workspaces by entry point."""
+    ws = torch.zeros(ifl.workspace_bytes("segscan", 1, 1 << 22), dtype=torch.uint8, device="cuda")
+    small = torch.ones(64, 5121, dtype=torch.int32 if dt == "i32" else torch.float32, device="cuda")
+    for _ in range(3):
+        ifl.segred(small * 2, "sum", version="flat", ws=ws)  # partials 2, 4, ... 10242
+        for (n, m) in [(1, 1 << 22), (4, 1 << 20), (1000, 4000)]:
+            x, xd = gen_for("sum", dt, 8, n, m)
+            assert_parity(orc, x, ifl.segscan(xd, "sum", version="flat", ws=ws), True, "sum", "id", None, dt)
+            ifl.segred(xd, "sum", version="flat", ws=ws)
 
 
 def test_config0_int32_1024x1024(ifl, orc):

@@ -1,5 +1,6 @@
 import sys, torch, numpy as np
-sys.path.insert(0, "/root/repo")
+import os
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import ifl_inputs as gen, paper_conf_ppopp_henriksenteo19_b200 as ifl
 lg, mean = int(sys.argv[1]), float(sys.argv[2])
 n = max(1, (1 << lg) // int(mean))
