@@ -539,6 +539,59 @@ def test_irr_numpy_cumsum_and_brute_force(orc):
         assert (np.abs(got - want) <= 1e-12 * (ab + 1)).all()
 
 
+def test_irr_f32_scan_against_numpy_and_fsum(orc):
+    """oracle_segscan_irr_f32 (unpinned): per segment, the scan is
+    d + numpy's float64 cumsum of f(x), its last element is math.fsum of the
+    segment, min/max scans are numpy's accumulate, and absum restarts at every
+    segment (a value carried across a boundary, or absum not reset, fails)."""
+    rng = np.random.default_rng(5)
+    for trial in range(6):
+        lens = rng.integers(0, 12, size=rng.integers(1, 50)).astype(np.int64)
+        lens[rng.integers(0, len(lens))] = 0                               # at least one empty segment
+        off = np.r_[0, np.cumsum(lens)]
+        xf = gen.generate("F32_SIGNED", 90 + trial, int(off[-1])).numpy()
+        for f, fx in (("id", xf.astype(np.float64)), ("sq", (xf * xf).astype(np.float32).astype(np.float64)),
+                      ("abs", np.abs(xf).astype(np.float64))):
+            for d in (None, 1.5):
+                dd = 0.0 if d is None else d
+                got, ab = orc.seg_irr(xf, off, True, "sum", f, d, with_absum=True)
+                for i in range(len(lens)):
+                    a, b = off[i], off[i + 1]
+                    if a == b:
+                        continue
+                    seg = fx[a:b]
+                    np.testing.assert_allclose(got[a:b], dd + np.cumsum(seg), rtol=0, atol=1e-12 * (1 + np.abs(seg).sum()))
+                    assert abs(got[b - 1] - math.fsum([dd] + list(seg))) <= 1e-12 * (1 + np.abs(seg).sum())
+                    np.testing.assert_allclose(ab[a:b], np.cumsum(np.abs(seg)), rtol=1e-15, atol=0)
+        for op, acc in (("min", np.minimum.accumulate), ("max", np.maximum.accumulate)):
+            got = orc.seg_irr(xf, off, True, op)
+            for i in range(len(lens)):
+                a, b = off[i], off[i + 1]
+                if a < b:
+                    np.testing.assert_array_equal(got[a:b], acc(xf[a:b].astype(np.float64)))
+
+
+def test_f32_reverse_scan(orc):
+    """The reversed scan (tridag's back-substitution direction):
+    out[i][j] = d (+) f(x[i][m-1]) (+) ... (+) f(x[i][j]) -- numpy's cumsum of the
+    reversed row, reversed back; closed form m - j for ones; min/max by
+    numpy's accumulate; absum is the reversed prefix of |f(x)|."""
+    for (n, m) in [(1, 1), (3, 17), (5, 1000)]:
+        ones = np.ones((n, m), np.float32)
+        np.testing.assert_array_equal(orc.segscan(ones, "sum", reverse=True), np.tile(np.arange(m, 0, -1.0), (n, 1)))
+        x = gen.matrix("F32_SIGNED", 33, n, m).numpy()
+        got, ab = orc.segscan(x, "sum", "id", d=0.25, reverse=True, with_absum=True)
+        want = 0.25 + np.cumsum(x[:, ::-1].astype(np.float64), axis=1)[:, ::-1]
+        np.testing.assert_allclose(got, want, rtol=0, atol=1e-12 * (1 + np.abs(x).sum()))
+        np.testing.assert_allclose(ab, np.cumsum(np.abs(x[:, ::-1]).astype(np.float64), axis=1)[:, ::-1], rtol=1e-14)
+        for op, acc in (("min", np.minimum.accumulate), ("max", np.maximum.accumulate)):
+            np.testing.assert_array_equal(orc.segscan(x, op, reverse=True),
+                                          acc(x[:, ::-1].astype(np.float64), axis=1)[:, ::-1])
+        xi = gen.matrix("I32_FULL", 34, n, m).numpy()
+        np.testing.assert_array_equal(orc.segscan(xi, "sum", reverse=True),
+                                      _wrap(np.cumsum(xi[:, ::-1].astype(np.int64), axis=1)[:, ::-1]))
+
+
 # ------------------------------------------- segarg: tuple-valued (+) (NEXT-3)
 
 
@@ -552,6 +605,16 @@ def test_segarg_numpy_and_closed_forms(orc):
     xf = gen.matrix("F32_SIGNED", 52, 20, 31).numpy()
     v, i = orc.segarg(xf, "min")
     np.testing.assert_array_equal(i, np.argmin(xf, axis=1))
+    # f32 argmax (unpinned): numpy's first occurrence, on data with
+    # many ties (values rounded to 1/8) and on plain signed data
+    xt = (np.round(gen.matrix("F32_SIGNED", 53, 40, 57).numpy() * 8) / 8).astype(np.float32)
+    for xx in (xf, xt):
+        for which, npf in (("max", np.argmax), ("min", np.argmin)):
+            v, i = orc.segarg(xx, which)
+            np.testing.assert_array_equal(i, npf(xx, axis=1))
+            np.testing.assert_array_equal(v, xx[np.arange(xx.shape[0]), i])
+    inc = np.tile(np.arange(9, dtype=np.float32), (3, 1))                  # increasing: argmax = last
+    assert (orc.segarg(inc, "max")[1] == 8).all() and (orc.segarg(-inc, "max")[1] == 0).all()
     # closed forms: decreasing rows -> last index; constant rows -> index 0; empty rows -> (d, -1)
     dec = np.tile(np.arange(9, 0, -1, dtype=np.int32), (3, 1))
     assert (orc.segarg(dec, "min")[1] == 8).all() and (orc.segarg(dec, "max")[1] == 0).all()
