@@ -234,12 +234,12 @@ def _choice_out(c: ifl_choice) -> Choice:
 
 
 def _seg(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws, stream, return_choice,
-         seed=None):
+         seed=None, reverse=False):
     host = not x.is_cuda
     if host:  # end-to-end path: pinned host -> device -> host
         xd = x.to("cuda", non_blocking=True)
         sd = None if seed is None else seed.to("cuda", non_blocking=True)
-        r = _seg(scan, xd, op, f, ne, version, None, ws, stream, return_choice, sd)
+        r = _seg(scan, xd, op, f, ne, version, None, ws, stream, return_choice, sd, reverse)
         if return_choice:
             r, c = r
         o = torch.empty(r.shape, dtype=r.dtype, pin_memory=True) if out is None else out
@@ -270,7 +270,7 @@ def _seg(scan: bool, x: torch.Tensor, op: str, f: str, ne, version: str, out, ws
         rc = lib().ifl_segscan_seeded(*args[:7], seed.data_ptr(), *tail)
         entry = "segscan_seeded"
     elif scan:
-        rc = lib().ifl_segscan(*args, 0, *tail)
+        rc = lib().ifl_segscan(*args, 1 if reverse else 0, *tail)
     else:
         rc = lib().ifl_segred(*args, *tail)
     _check(rc, "ifl_" + entry)
@@ -283,13 +283,16 @@ def segred(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stre
 
 
 def segscan(x, op="sum", f="id", ne=None, version="auto", out=None, ws=None, stream=None, return_choice=False,
-            seed=None):
+            seed=None, reverse=False):
     """Inclusive per-row scanomap (example P:116).  ``seed``
     (an [n] tensor) replaces ne row by row: out[i,j] = seed[i] (+) f(x[i,0])
-    (+) ... (+) f(x[i,j]) -- the carry-in of a column block (ifl_segscan_seeded)."""
+    (+) ... (+) f(x[i,j]) -- the carry-in of a column block (ifl_segscan_seeded).
+    ``reverse``: out[i,j] = ne (+) f(x[i,m-1]) (+) ... (+) f(x[i,j])."""
     if seed is not None and ne is not None:
         raise ValueError("pass either ne or seed")
-    return _seg(True, x, op, f, ne, version, out, ws, stream, return_choice, seed)
+    if seed is not None and reverse:
+        raise ValueError("seeded scans run forward only")
+    return _seg(True, x, op, f, ne, version, out, ws, stream, return_choice, seed, reverse)
 
 
 # ----------------------------------------------------------- colred / colscan

@@ -692,7 +692,7 @@ constexpr int kDlbSlots = IFL_DLB_SLOTS;
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(kScanThreads, IFL_DLB_MINB) flat_scan_dlb_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
                                                                       uint8_t* ws, int num_tiles, bool tma_in,
-                                                                      bool tma_out, const T* __restrict__ seed) {
+                                                                      bool tma_out, const T* __restrict__ seed, bool rev) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
     __shared__ alignas(8) uint64_t full[kDlbSlots], empty[kDlbSlots];
@@ -761,7 +761,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_DLB_MINB) flat_scan_dlb_kern
         if (sm.tile < 0) break;
         const int64_t base = (int64_t)sm.tile * FT;
         if (!(tma_in && sm.cnt == FT)) {
-            for (int p = t; p < sm.cnt; p += FB) buf[p] = in[base + p];
+            for (int p = t; p < sm.cnt; p += FB) buf[p] = in[rev ? N - 1 - (base + p) : base + p];
             consumer_sync();
         }
         const ThreadPos tp = thread_pos(sm, m);
@@ -802,7 +802,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_DLB_MINB) flat_scan_dlb_kern
                 pend_slot = sl;
             }
         } else {
-            for (int p = t; p < sm.cnt; p += FB) out[base + p] = buf[p];
+            for (int p = t; p < sm.cnt; p += FB) out[rev ? N - 1 - (base + p) : base + p] = buf[p];
             consumer_sync();
             if (t == 0) mbar_arrive_expect_tx(&empty[sl], 0);
         }
@@ -873,7 +873,7 @@ __device__ __forceinline__ void mbar_arrive_cnt(uint64_t* bar, uint32_t cnt) {
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(kScanThreads, IFL_JR_MINB) flat_scan_jr_kernel(const T* in, T* out, int64_t N, int64_t m, T d,
                                                                     uint8_t* ws, int num_tiles, int num_chunks, int lag,
-                                                                    bool tma_in, bool tma_out, const T* __restrict__ seed) {
+                                                                    bool tma_in, bool tma_out, const T* __restrict__ seed, bool rev) {
     extern __shared__ __align__(128) uint8_t smem_raw[];
     T* ring = reinterpret_cast<T*>(smem_raw);
     __shared__ alignas(8) uint64_t full[kJrSlots], empty[kJrSlots];
@@ -1002,7 +1002,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_JR_MINB) flat_scan_jr_kernel
                 if (in_smem) {
                     for (int q = jm.a0 + t; q < jm.a1; q += FB) acc_a = combine<OP>(acc_a, apply_map<F>(buf[q]));
                 } else {
-                    for (int q = jm.a0 + t; q < jm.a1; q += FB) acc_a = combine<OP>(acc_a, apply_map<F>(in[base + q]));
+                    for (int q = jm.a0 + t; q < jm.a1; q += FB) acc_a = combine<OP>(acc_a, apply_map<F>(in[rev ? N - 1 - (base + q) : base + q]));
                 }
                 __syncwarp();
                 if (lane == 0) mbar_arrive_cnt(&empty[sl], 1);  // this warp is done with the slot
@@ -1047,7 +1047,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_JR_MINB) flat_scan_jr_kernel
                 consumer_sync();
             }
             if (!in_smem) {
-                for (int p = t; p < jm.cnt; p += FB) buf[p] = in[base + p];
+                for (int p = t; p < jm.cnt; p += FB) buf[p] = in[rev ? N - 1 - (base + p) : base + p];
                 consumer_sync();
             }
             SlotMeta smeta;
@@ -1083,7 +1083,7 @@ __global__ void __launch_bounds__(kScanThreads, IFL_JR_MINB) flat_scan_jr_kernel
                     pend_slot = sl;
                 }
             } else {
-                for (int p = t; p < jm.cnt; p += FB) out[base + p] = buf[p];
+                for (int p = t; p < jm.cnt; p += FB) out[rev ? N - 1 - (base + p) : base + p] = buf[p];
                 consumer_sync();
                 if (t == 0) mbar_arrive_cnt(&empty[sl], NCW);
             }
@@ -1131,8 +1131,11 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
     const int64_t N = a.n * a.m;
     const int64_t tiles = ceil_div(N, kFlatTile);
     if (tiles > 0x3fffffffLL) return cudaErrorInvalidValue;
-    const bool tma_in = ((uintptr_t)a.in % 16) == 0;
-    const bool tma_out = ((uintptr_t)a.out % 16) == 0;
+    // reverse scans: the flat index space mirrored (element k is physical n*m-1-k:
+    // rows reversed, in reverse order -- the same regular segments), read and
+    // written by the engines' cooperative (non-TMA) paths
+    const bool tma_in = !a.rev && ((uintptr_t)a.in % 16) == 0;
+    const bool tma_out = !a.rev && ((uintptr_t)a.out % 16) == 0;
     uint8_t* ws = (uint8_t*)a.ws;
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
@@ -1146,7 +1149,7 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
             const size_t smem_s = (size_t)kDlbSlots * FT * sizeof(T);
             const int grid = (int)std::min<int64_t>(tiles, resident_ctas(k, smem_s, kScanThreads));
             k<<<grid, kScanThreads, smem_s, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, tma_in,
-                                                        tma_out, (const T*)a.seed);
+                                                        tma_out, (const T*)a.seed, a.rev);
             return cudaGetLastError();
         }
         if (scan) {  // segments cross tiles: the job-ring engine
@@ -1156,7 +1159,7 @@ cudaError_t launch_flat(const SegArgs& a, bool scan) {
             const int lag = std::min(IFL_JR_LAG, chunks);
             const int grid = (int)std::min<int64_t>(resident_ctas(k, smem_s, kScanThreads), chunks + lag);
             k<<<grid, kScanThreads, smem_s, a.stream>>>((const T*)a.in, (T*)a.out, N, a.m, d, ws, (int)tiles, chunks, lag,
-                                                         tma_in, tma_out, (const T*)a.seed);
+                                                         tma_in, tma_out, (const T*)a.seed, a.rev);
             return cudaGetLastError();
         }
         T* head = reinterpret_cast<T*>(ws + sizeof(FlatHdr) + (size_t)tiles * 8);

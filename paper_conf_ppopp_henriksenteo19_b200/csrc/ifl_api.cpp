@@ -329,7 +329,7 @@ int ifl_workspace_init(void* ws, size_t ws_bytes, void* stream) {
 
 static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f,
                    const void* ne, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice,
-                   const void* seed = nullptr) {
+                   const void* seed = nullptr, bool rev = false) {
     const char* what = seed ? "ifl_segscan_seeded" : scan ? "ifl_segscan" : "ifl_segred";
     int rc = validate_seg(scan, in, out, n, m, dt, op, f, version, what);
     if (rc) return rc;
@@ -354,7 +354,7 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
         return cuda_status(ifl::launch_fill(out, n, bits, (cudaStream_t)stream), what);
     }
     (void)v;
-    ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream, seed};
+    ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream, seed, rev};
     cudaError_t e;
     switch (c.version) {
     case IFL_V_TOP: e = scan ? ifl::launch_segscan_top(a) : ifl::launch_segred_top(a); break;
@@ -550,8 +550,8 @@ int ifl_segred(const void* in, void* out, int64_t n, int64_t m, int dt, int op, 
 
 int ifl_segscan(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* ne, int reverse,
                 int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice) {
-    if (reverse) return fail(IFL_EUNSUPPORTED, "ifl_segscan: reverse scans are not exposed");
-    return run_seg(true, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice);
+    if (reverse != 0 && reverse != 1) return fail(IFL_EINVAL, "ifl_segscan: reverse must be 0 or 1");
+    return run_seg(true, in, out, n, m, dt, op, f, ne, version, ws, ws_bytes, stream, choice, nullptr, reverse == 1);
 }
 
 int ifl_segscan_seeded(const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, const void* seed,

@@ -20,6 +20,7 @@ struct SegArgs {
     size_t ws_bytes;
     cudaStream_t stream;
     const void* seed = nullptr;  // segscan: per-row d (device [n]) or NULL = ne_bits for every row
+    bool rev = false;            // segscan: reversed scan (row read from its last element)
 };
 
 // Flat engine tile geometry (flat.cu).  ws layout: 256-byte header then one

@@ -41,7 +41,15 @@ __host__ __device__ __forceinline__ int stop_rpt(int64_t m) { return m <= kTopKT
 // LOAD: global -> smem; STORE: smem -> global.
 template <bool LOAD, typename T>
 __device__ __forceinline__ void top_xfer(T* tile, const T* in, T* out, int64_t r0,
-                                         int rows, int64_t m, int64_t k0, int kt, bool whole, bool vec) {
+                                         int rows, int64_t m, int64_t k0, int kt, bool whole, bool vec,
+                                         bool rev = false) {
+    // rev (reverse scans): logical column c of a row is physical column m-1-c
+    // (vec is false then: the scalar paths below do the mirroring)
+    auto ph = [&](int64_t g) -> int64_t {
+        if (!rev) return g;
+        const int64_t r = g / m;
+        return r * m + (m - 1 - (g - r * m));
+    };
     const int t = threadIdx.x;
     using V = typename Vec4<T>::type;
     if (whole) {
@@ -67,8 +75,8 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* in, T* out, int64_t r
             p0 = nv << 2;
         }
         for (int p = p0 + t; p < cnt; p += kTopThreads) {
-            if (LOAD) tile[spadq(p)] = ld_coh1(in + r0 * m + p);
-            else out[r0 * m + p] = tile[spadq(p)];
+            if (LOAD) tile[spadq(p)] = ld_coh1(in + ph(r0 * m + p));
+            else out[ph(r0 * m + p)] = tile[spadq(p)];
         }
     } else if (vec && kt == kTopKT) {
         for (int v = t; v < rows * 8; v += kTopThreads) {
@@ -94,8 +102,8 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* in, T* out, int64_t r
             const int row = p >> 5, col = p & 31;
             if (col < kt) {
                 const int64_t gi = (r0 + row) * m + k0 + col;
-                if (LOAD) tile[spadq(p)] = ld_coh1(in + gi);
-                else out[gi] = tile[spadq(p)];
+                if (LOAD) tile[spadq(p)] = ld_coh1(in + ph(gi));
+                else out[ph(gi)] = tile[spadq(p)];
             }
         }
     }
@@ -103,7 +111,8 @@ __device__ __forceinline__ void top_xfer(T* tile, const T* in, T* out, int64_t r
 
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T* out, int64_t n, int64_t m, T d,
-                                                                  bool vec, const T* __restrict__ seed) {
+                                                                  bool vec, const T* __restrict__ seed,
+                                                                  bool rev = false) {
     __shared__ T tile[kTopWords];
     const int t = threadIdx.x;
     const int rpt = stop_rpt(m);
@@ -113,7 +122,7 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
         const int64_t r0 = b * rows_blk;
         const int rows = (int)min(rows_blk, n - r0);
         if (m <= kTopKT) {
-            top_xfer<true>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
+            top_xfer<true>(tile, in, out, r0, rows, m, 0, (int)m, true, vec, rev);
             __syncthreads();
             const int mm = (int)m;
             for (int j = 0; j < rpt; ++j) {
@@ -127,13 +136,13 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
                 }
             }
             __syncthreads();
-            top_xfer<false>(tile, in, out, r0, rows, m, 0, (int)m, true, vec);
+            top_xfer<false>(tile, in, out, r0, rows, m, 0, (int)m, true, vec, rev);
             __syncthreads();
         } else {
             Acc<OP, T> a((seed && t < rows) ? seed[r0 + t] : d);
             for (int64_t k0 = 0; k0 < m; k0 += kTopKT) {
                 const int kt = (int)min((int64_t)kTopKT, m - k0);
-                top_xfer<true>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+                top_xfer<true>(tile, in, out, r0, rows, m, k0, kt, false, vec, rev);
                 __syncthreads();
                 if (t < rows) {
                     if (kt == kTopKT) {
@@ -150,7 +159,7 @@ __global__ void __launch_bounds__(kTopThreads) segscan_top_kernel(const T* in, T
                     }
                 }
                 __syncthreads();
-                top_xfer<false>(tile, in, out, r0, rows, m, k0, kt, false, vec);
+                top_xfer<false>(tile, in, out, r0, rows, m, k0, kt, false, vec, rev);
                 __syncthreads();
             }
         }
@@ -316,7 +325,8 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const T* seed = (const T*)a.seed;
-        const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) &&
+        // reverse scans take the generic kernel's scalar (mirroring) paths
+        const bool vec = !a.rev && ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) &&
                          (a.m <= kTopKT || a.m % 4 == 0);
         if (vec && (a.m == 1 || a.m == 2 || a.m == 4)) {
             const int64_t nv = ceil_div(a.n * a.m, 4);
@@ -360,7 +370,7 @@ cudaError_t launch_segscan_top(const SegArgs& a) {
         }
         const int64_t nblk = ceil_div(a.n, (int64_t)kTopThreads * stop_rpt(a.m));
         segscan_top_kernel<T, OP, F><<<stop_grid(nblk), kTopThreads, 0, a.stream>>>(
-            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec, seed);
+            (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), vec, seed, a.rev);
         return cudaGetLastError();
     });
 }
@@ -377,7 +387,7 @@ int midscan_group_size(int64_t m) {
 
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, int64_t n, int64_t m, T d, int G,
-                                                           bool vec, const T* __restrict__ seed) {
+                                                           bool vec, const T* __restrict__ seed, bool rev = false) {
     __shared__ T wtot[2][32];
     using V = typename Vec4<T>::type;
     const int g = threadIdx.x % G;
@@ -386,7 +396,10 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
     const bool live = i < n;
     const T* row = in + (live ? i * m : 0);
     T* orow = out + (live ? i * m : 0);
-    T carry = (seed && live) ? seed[i] : d;
+    // running carry across rounds: Kahan-compensated for f32 sums (a row of
+    // 4 x 10^8 elements adds 10^5 round totals into it; plain f32 drifts past
+    // the 1e-5 * sum|f(x)| bound)
+    Acc<OP, T> carry((seed && live) ? seed[i] : d);
     int par = 0;
     for (int64_t base = 0; base < m; base += (int64_t)G * kMidItems, par ^= 1) {
         const int64_t k0 = base + (int64_t)g * kMidItems;
@@ -402,7 +415,7 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
             } else {
 #pragma unroll
                 for (int u = 0; u < 4; ++u)
-                    v[4 * h + u] = (live && kh + u < m) ? apply_map<F>(ld_coh1(row + kh + u)) : identity<OP, T>();
+                    v[4 * h + u] = (live && kh + u < m) ? apply_map<F>(ld_coh1(row + (rev ? m - 1 - (kh + u) : kh + u))) : identity<OP, T>();
             }
         }
 #pragma unroll
@@ -432,7 +445,7 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
             }
             ex = combine<OP>(before, ex);
         }
-        const T pre = combine<OP>(carry, ex);
+        const T pre = combine<OP>(carry.get(), ex);
 #pragma unroll
         for (int u = 0; u < kMidItems; ++u) v[u] = combine<OP>(pre, v[u]);
         if (live) {
@@ -446,11 +459,11 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
                 } else {
 #pragma unroll
                     for (int u = 0; u < 4; ++u)
-                        if (kh + u < m) orow[kh + u] = v[4 * h + u];
+                        if (kh + u < m) orow[rev ? m - 1 - (kh + u) : kh + u] = v[4 * h + u];
                 }
             }
         }
-        carry = combine<OP>(carry, total);
+        carry.add(total);
     }
 }
 
@@ -463,7 +476,7 @@ __global__ void __launch_bounds__(1024) segscan_mid_kernel(const T* in, T* out, 
 template <typename T, int OP, int F>
 __global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
     segscan_mid_multi_kernel(const T* in, T* out, int64_t n, int64_t m, T d, int G, bool vec,
-                             const T* __restrict__ seed) {
+                             const T* __restrict__ seed, bool rev = false) {
     __shared__ T wtot[2][32];
     using V = typename Vec4<T>::type;
     const int g = threadIdx.x % G;
@@ -472,7 +485,10 @@ __global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
     const bool live = i < n;
     const T* row = in + (live ? i * m : 0);
     T* orow = out + (live ? i * m : 0);
-    T carry = (seed && live) ? seed[i] : d;
+    // running carry across rounds: Kahan-compensated for f32 sums (a row of
+    // 4 x 10^8 elements adds 10^5 round totals into it; plain f32 drifts past
+    // the 1e-5 * sum|f(x)| bound)
+    Acc<OP, T> carry((seed && live) ? seed[i] : d);
     int par = 0;
     const int64_t step = (int64_t)G * kMidItems;
     // raw items of one round (two 128-bit halves, each vectorised when whole; f applied at use,
@@ -489,7 +505,7 @@ __global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
                 for (int u = 0; u < 4; ++u) r[4 * h + u] = e[u];
             } else {
 #pragma unroll
-                for (int u = 0; u < 4; ++u) r[4 * h + u] = (live && kh + u < m) ? ld_coh1(row + kh + u) : T();
+                for (int u = 0; u < 4; ++u) r[4 * h + u] = (live && kh + u < m) ? ld_coh1(row + (rev ? m - 1 - (kh + u) : kh + u)) : T();
             }
         }
     };
@@ -531,7 +547,7 @@ __global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
             }
             ex = combine<OP>(before, ex);
         }
-        const T pre = combine<OP>(carry, ex);
+        const T pre = combine<OP>(carry.get(), ex);
 #pragma unroll
         for (int u = 0; u < kMidItems; ++u) v[u] = combine<OP>(pre, v[u]);
         if (live) {
@@ -545,11 +561,11 @@ __global__ void __launch_bounds__(IFL_MIDSCAN_GMAX, IFL_MULTI_MINB)
                 } else {
 #pragma unroll
                     for (int u = 0; u < 4; ++u)
-                        if (kh + u < m) orow[kh + u] = v[4 * h + u];
+                        if (kh + u < m) orow[rev ? m - 1 - (kh + u) : kh + u] = v[4 * h + u];
                 }
             }
         }
-        carry = combine<OP>(carry, total);
+        carry.add(total);
     }
 }
 
@@ -559,14 +575,14 @@ cudaError_t launch_segscan_mid(const SegArgs& a) {
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         const int G = midscan_group_size(a.m);
         const int B = G > 256 ? G : 256;
-        const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) && (a.m % 4 == 0);
+        const bool vec = !a.rev && ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) && (a.m % 4 == 0);
         const int64_t grid = ceil_div(a.n, B / G);
         if (a.m > (int64_t)G * kMidItems)  // several rounds per row: pipelined loads
             segscan_mid_multi_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>(
-                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), G, vec, (const T*)a.seed);
+                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), G, vec, (const T*)a.seed, a.rev);
         else
             segscan_mid_kernel<T, OP, F><<<(unsigned)grid, B, 0, a.stream>>>(
-                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), G, vec, (const T*)a.seed);
+                (const T*)a.in, (T*)a.out, a.n, a.m, bits_to<T>(a.ne_bits), G, vec, (const T*)a.seed, a.rev);
         return cudaGetLastError();
     });
 }

@@ -71,8 +71,9 @@ def test_validation_errors(L):
     assert _segred(L, 4096, 4096 + 8, 4, 4) == E         # out overlaps in
     # segscan: in place is fine (validated only), partial overlap is not
     assert L.ifl_segscan(4096, 4096 + 4, 4, 4, 1, 0, 0, None, 0, -1, None, 0, None, None) == E
-    assert L.ifl_segscan(4096, 4096, 4, 4, 1, 0, 0, None, 1, -1, None, 0, None, None) == ifl.IFL_EUNSUPPORTED
-    assert "overlap" in L.ifl_last_error().decode() or "reverse" in L.ifl_last_error().decode()
+    assert L.ifl_segscan(4096, 4096, 4, 4, 1, 0, 0, None, 2, -1, None, 0, None, None) == E  # reverse is 0 or 1
+    assert "reverse" in L.ifl_last_error().decode()
+    assert L.ifl_segscan(4096, 4096, 0, 4, 1, 0, 0, None, 1, -1, None, 0, None, None) == 0   # reverse, n = 0: no-op
 
 
 def test_empty_n_is_noop(L):

@@ -267,3 +267,41 @@ def test_middle_aligned_rows(ifl, orc, f):
                 assert_parity(orc, x, got, False, op, f, None, dt)
     x, xd = gen_for("sum", "i32", 6, 11, 4096)
     assert_parity(orc, x, ifl.segred(xd, "max", "abs", ne=-3, version="middle"), False, "max", "abs", -3, "i32")
+
+
+@pytest.mark.parametrize("version", VERS)
+@pytest.mark.parametrize("dt", ["i32", "f32"])
+def test_reverse_scan(ifl, orc, version, dt):
+    """reverse = 1: out[i][j] = d (+) f(x[i][m-1]) (+) ... (+) f(x[i][j]) (ifl.h),
+    every version (TOP / MIDDLE mirror rows, FLAT mirrors the flat index space:
+    tile-aligned and job-ring engines), ragged shapes, misaligned and in place."""
+    shapes = [(1, 1), (5, 3), (33, 64), (7, 1000), (3, 5120), (2, 50001), (200, 1024), (1, 5120 * 13 + 7)]
+    ops = OPS_I if dt == "i32" else OPS_F
+    for (n, m) in shapes:
+        for op in ops:
+            x, xd = gen_for(op, dt, 21, n, m)
+            got = ifl.segscan(xd, op, "sq" if op == "sum" else "id", ne=(3 if dt == "i32" else 0.5) if op == "sum" else None,
+                              version=version, reverse=True)
+            d = (3 if dt == "i32" else 0.5) if op == "sum" else None
+            f = "sq" if op == "sum" else "id"
+            if dt == "i32":
+                np.testing.assert_array_equal(got.cpu().numpy(), orc.segscan(x.numpy(), op, f, d, reverse=True))
+            else:
+                want, ab = orc.segscan(x.numpy(), op, f, d, reverse=True, with_absum=True)
+                g = got.cpu().numpy().astype(np.float64)
+                if op in ("min", "max"):
+                    np.testing.assert_array_equal(g, want)
+                elif op == "sum":
+                    assert (np.abs(g - want) <= 1e-5 * (ab + 0.5)).all()
+                else:
+                    assert (np.abs(g - want) <= (m + 2) * 2.0**-23 * np.abs(want) + 1e-30).all()
+        # misaligned input/output and in place
+        x, xd = gen_for("sum", dt, 22, n, m, misalign=True)
+        want = orc.segscan(x.numpy(), "sum", reverse=True, with_absum=dt == "f32")
+        got = ifl.segscan(xd, "sum", version=version, reverse=True)
+        got2 = ifl.segscan(xd, "sum", version=version, reverse=True, out=xd)
+        for g in (got, got2):
+            if dt == "i32":
+                np.testing.assert_array_equal(g.cpu().numpy(), want)
+            else:
+                assert (np.abs(g.cpu().numpy() - want[0]) <= 1e-5 * want[1]).all()
