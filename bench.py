@@ -147,7 +147,7 @@ def run_ours(args, rank, world, device):
             scratch = torch.empty(scratch_bytes, dtype=torch.uint8, device=device)
             scratch.view(-1)[: (scratch_bytes // 4) * 4].view(torch.float32).copy_(
                 gen.generate("F32_UNIT", 4, scratch_bytes // 4, device=device))
-            a, b, tbl = ifl.tune(site, train, reps=3, cost=1, scratch=scratch)
+            a, b, tbl = ifl.tune(site, train, reps=7, cost=1, scratch=scratch)
             tuned[site] = {"t_top": a, "t_intra": b}
             del scratch
         log(f"[bench] tuned in {time.time() - t0:.1f}s: {tuned}")
@@ -352,6 +352,7 @@ def run_ours(args, rank, world, device):
                "note": "pinned host input copied in once per shape and shared by segred+segscan"}
 
     res = {
+        "x": xs[0], "ws": ws,
         "value": value, "total_ms": total_ms, "step_ms": step_ms, "step_bytes": step_bytes, "table": table,
         "ratios": ratios, "fixed_tot": fixed_tot, "auto_tot": auto_tot, "tuned": tuned, "clocks": ck,
         "dom": dom, "achieved": achieved, "peak": pk, "traffic": traffic, "e2e": e2e, "groups": groups,
@@ -360,7 +361,206 @@ def run_ours(args, rank, world, device):
     return res
 
 
+# ------------------------------------------------- N > 1: the sharded sweep
+
+
+def sharded_shapes(world: int, rank: int, log2n: int = LOG2_N):
+    """The weak-scaled sweep over N GPUs (dist.py): global shape
+    [2^k][world * 2^log2n / 2^k], split by the device-level guard -- rows when
+    2^k >= world (outer: no collective), else every row's columns (inner: one
+    all_reduce of the n partials for segred; all_gather of block totals and a
+    seeded local scan for segscan).  Every rank's block holds exactly 2^log2n
+    elements.  Returns (n_g, m_g, plan, (n_local, m_local)) per shape."""
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    out = []
+    for k in range(log2n + 1):
+        ng, mg = 1 << k, (world << log2n) >> k
+        plan = dist.plan_segred(ng, mg, world, rank)
+        loc = (plan.hi - plan.lo, mg) if plan.mode == "outer" else (ng, plan.hi - plan.lo)
+        assert loc[0] * loc[1] == 1 << log2n, (ng, mg, plan)
+        out.append((ng, mg, plan, loc))
+    return out
+
+
+def sharded_step(x, shapes, local_segred=None, local_segscan=None):
+    """One step of the sharded sweep on this rank: segred_dist + segscan_dist
+    per shape over the rank's resident block x (2^log2n elements)."""
+    from paper_conf_ppopp_henriksenteo19_b200 import dist
+    outs = []
+    for ng, mg, plan, (nl, ml) in shapes:
+        xb = x.view(nl, ml)
+        outs.append(dist.segred_dist(xb, ng, mg, "sum", "id", None, plan=plan, local_segred=local_segred))
+        outs.append(dist.segscan_dist(xb, ng, mg, "sum", "id", None, plan=plan, local_segred=local_segred,
+                                      local_segscan=local_segscan))
+    return outs
+
+
+def run_sharded(args, rank, world, device):
+    import torch
+    import torch.distributed as td
+
+    import ifl_inputs as gen
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+
+    torch.cuda.set_device(device)
+    ifl.reset_thresholds()
+    if args.thresholds:
+        ifl.load_thresholds(args.thresholds)
+    N = 1 << LOG2_N
+    shapes = sharded_shapes(world, rank)
+    step_bytes = sum(bytes_segred(ng, mg) + bytes_segscan(ng, mg) for ng, mg, _, _ in shapes)  # global
+    # each rank's block: the global flat index space offset by its share (counter-based generator)
+    xs = [gen.generate("F32_UNIT", 2 + c, N, device=device) for c in range(2)]
+    stream = torch.cuda.current_stream()
+    for c in range(2):  # warm every kernel and collective outside capture
+        sharded_step(xs[c], shapes)
+    torch.cuda.synchronize()
+    # our kernel launches per step: one eager step under the profiler, kernels of namespace ifl::
+    launches = None
+    try:
+        from torch.profiler import ProfilerActivity, profile
+        with profile(activities=[ProfilerActivity.CUDA]) as prof:
+            sharded_step(xs[0], shapes)
+            torch.cuda.synchronize()
+        launches = sum(1 for ev in prof.events() if "ifl::" in ev.name)
+    except Exception as e:  # profiler unavailable: leave the count out rather than guess
+        log(f"[bench] kernel count unavailable: {e}")
+    graphs, mode = [], "cuda-graph"
+    try:
+        for c in range(2):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                sharded_step(xs[c], shapes)
+            graphs.append(g)
+        torch.cuda.synchronize()
+    except Exception as e:  # NCCL capture refused: eager steps (host launch gaps included)
+        log(f"[bench] graph capture of the sharded step failed ({type(e).__name__}: {e}); eager")
+        graphs, mode = [], "eager"
+        torch.cuda.synchronize()
+
+    def step(i):
+        if graphs:
+            graphs[i % 2].replay()
+        else:
+            sharded_step(xs[i % 2], shapes)
+
+    for i in range(args.warmup):
+        step(i)
+    torch.cuda.synchronize()
+    td.barrier()
+    torch.cuda.synchronize()
+    clocks = Clocks(device)
+    clocks.start()
+    time.sleep(0.3)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for i in range(args.steps):
+        step(i)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ck = clocks.stop()
+    td.barrier()
+    torch.cuda.synchronize()
+    t = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=device)
+    td.all_reduce(t, op=td.ReduceOp.MAX)
+    total_ms = float(t.item())
+    # the collectives' share: the same step with the device-level exchange removed
+    # (inner-plan shapes computed locally only), timed the same way
+    def local_only(i):
+        for _, _, _, (nl, ml) in shapes:
+            xb = xs[i % 2].view(nl, ml)
+            ifl.segred(xb, "sum")
+            ifl.segscan(xb, "sum")
+
+    for i in range(2):
+        local_only(i)
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for i in range(args.steps):
+        local_only(i)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    tl = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=device)
+    td.all_reduce(tl, op=td.ReduceOp.MAX)
+    # e2e: pinned host block in, the sharded step, every result out
+    hx = torch.empty(N, dtype=torch.float32, pin_memory=True)
+    hx.copy_(xs[0])
+    dx = torch.empty(N, dtype=torch.float32, device=device)
+    td.barrier()
+    torch.cuda.synchronize()
+    esteps = max(1, min(args.steps, 3))
+    e0.record(stream)
+    h2d = d2h = 0
+    for i in range(esteps):
+        dx.copy_(hx, non_blocking=True)
+        outs = sharded_step(dx, shapes)
+        hos = [o.to("cpu", non_blocking=True) for o in outs]
+        if i == 0:
+            h2d += N * 4
+            d2h += sum(o.numel() * o.element_size() for o in outs)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    del hos
+    te = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=device)
+    td.all_reduce(te, op=td.ReduceOp.MAX)
+    return {
+        "value": step_bytes * args.steps / (total_ms / 1e3) / 1e9, "total_ms": total_ms, "step_bytes": step_bytes,
+        "clocks": ck, "mode": mode, "local_ms": float(tl.item()),
+        "e2e": {"value": round(step_bytes * esteps / (float(te.item()) / 1e3) / 1e9, 2), "unit": "GB/s",
+                "h2d_bytes_per_step": h2d * world, "d2h_bytes_per_step": d2h * world,
+                "note": "every rank: its pinned host block in, the sharded step, its results out"},
+        "launches": None if launches is None else launches * args.steps,
+    }
+
+
 # ------------------------------------------------------------ CPU oracle
+
+
+def host_info():
+    """The host the CPU oracle runs on (core count and model)."""
+    model = ""
+    try:
+        with open("/proc/cpuinfo") as fp:
+            for line in fp:
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+    except OSError:
+        pass
+    return {"host_cpus": os.cpu_count(), "affinity_cpus": len(os.sched_getaffinity(0)), "cpu_model": model}
+
+
+def parity_sample(x, ws):
+    """Every timed AUTO call's output checked against the CPU oracle
+    (SURVEY 8(d) "every timed run's output is parity-checked"): each of the 54
+    calls of the step is run once more exactly as timed, and its first and last
+    rows are compared with the oracle's (f32 sum: |g - r| <= 1e-5 * sum|x|)."""
+    import numpy as np
+    import torch
+
+    import oracle
+    import paper_conf_ppopp_henriksenteo19_b200 as ifl
+    N = 1 << LOG2_N
+    out = torch.empty(N, dtype=torch.float32, device=x.device)
+    checked = failed = 0
+    worst = 0.0
+    for (n, m) in shapes():
+        xv = x.view(n, m)
+        rows = sorted({0, n - 1})
+        xr = xv[rows].cpu().numpy()
+        for kind in ("segred", "segscan"):
+            if kind == "segred":
+                got = ifl.segred(xv, out=out[:n], ws=ws)[rows].cpu().numpy()
+                want, ab = oracle.segred(xr, "sum", with_absum=True)
+            else:
+                got = ifl.segscan(xv, out=out.view(n, m), ws=ws)[rows].cpu().numpy()
+                want, ab = oracle.segscan(xr, "sum", with_absum=True)
+            err = np.abs(got.astype(np.float64) - want) / np.maximum(ab, 1e-30)
+            checked += 1
+            worst = max(worst, float(err.max()))
+            failed += int((err > 1e-5).any())
+    return {"calls_checked": checked, "failed": failed, "rows": "first and last row of every AUTO call",
+            "bar": "|g - r| <= 1e-5 * sum|f(x)| per element (C3)", "worst_rel_to_bound_base": worst}
 
 
 def oracle_sample(step_index: int = 0):
@@ -406,7 +606,8 @@ def run_reference(args, rank, world):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(secs / args.steps * 1e3, 2),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": "configs[1] fp32 segmented redomap sweep n*m=2^26 (bounded sample, CPU oracle)"},
-        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
+                         **host_info()},
         "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     return line
@@ -416,7 +617,11 @@ def run_reference(args, rank, world):
 
 
 def main():
-    os.environ.setdefault("NCCL_DEBUG", "WARN")  # keep NCCL's banner off the JSON stdout
+    # NCCL's communicator INIT lines (rank count, transports) go to stderr,
+    # where the driver can read them; stdout keeps the one JSON line
+    os.environ.setdefault("NCCL_DEBUG", "INFO")
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+    os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=5)
@@ -458,15 +663,46 @@ def main():
         import torch.distributed as td
         torch.cuda.set_device(local)
         td.init_process_group("nccl", device_id=torch.device("cuda", local))
+    if world > 1:
+        r = run_sharded(args, rank, world, local)
+        if rank == 0:
+            pk = peaks()
+            line = {
+                "metric": METRIC, "value": round(r["value"], 2), "unit": "GB/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(r["total_ms"] / args.steps, 4),
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f32",
+                "data": "synthetic",
+                "config": {
+                    "workload": f"configs[1] sweep weak-scaled over {world} GPUs: global [2^k][{world}*2^26/2^k], "
+                                "k=0..26, segred+segscan (+, f=id) through dist.py's device-level guard (row split, "
+                                "or column split + one all_reduce / all_gather when 2^k < GPUs)",
+                    "n_times_m_per_gpu": 1 << LOG2_N, "shapes": LOG2_N + 1,
+                    "l2": "per-GPU blocks 256 MiB > 126 MB L2; two resident copies alternate per step",
+                    "parallelism": f"dp{world} (device-level G3: outer split / inner split + NCCL)",
+                    "step": r["mode"],
+                },
+                "frac_of_8TBps": round(r["value"] / world / NOMINAL_HBM_GBS, 4),
+                "frac_of_measured_hbm": round(r["value"] / world / pk["hbm_gbs"], 4),
+                "collective_share": round(max(0.0, 1.0 - r["local_ms"] / r["total_ms"]), 4),
+                "roofline": None, "cpu_baseline": None, "e2e": r["e2e"], "gpu_launches": r["launches"],
+                "clocks": r["clocks"],
+            }
+            print(json.dumps(line), flush=True)
+        import torch.distributed as td
+        td.barrier()
+        td.destroy_process_group()
+        return
     r = run_ours(args, rank, world, local)
     if rank == 0:
         import numpy as np
         pk = r["peak"]
         cpu = None
+        parity = None
         if not args.no_cpu and world == 1:
             v, dt, sample = oracle_sample()
             cpu = {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
-                   "seconds": round(dt, 2)}
+                   "seconds": round(dt, 2), **host_info()}
+            parity = parity_sample(r["x"], r["ws"])
         best_fixed = min(r["fixed_tot"].values())
         line = {
             "metric": METRIC,
@@ -498,6 +734,7 @@ def main():
                          "peak": pk["hbm_gbs"], "unit": "GB/s", "frac": round(r["achieved"] / pk["hbm_gbs"], 4),
                          "traffic": r["traffic"], "peak_source": pk["source"]},
             "cpu_baseline": cpu,
+            "parity": parity,
             "e2e": r["e2e"],
             "gpu_launches": r["launches"],
             "clocks": r["clocks"],

@@ -103,7 +103,7 @@ def suite_redomap2():
         train = mm_shapes(ktrain)
         need = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data, len(train))
         scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
-        a, b, tbl = ifl.tune(site, train, reps=3, cost=1, scratch=scratch)
+        a, b, tbl = ifl.tune(site, train, reps=7, cost=1, scratch=scratch)
         tuned[site] = {"t_top": a, "t_intra": b}
         del scratch
         for k in ks:
@@ -166,7 +166,7 @@ def suite_tridag():
     train = [s for ds in ("small", "large") for s in sites(ds)[0]]
     need = ifl.lib().ifl_tune_scratch_bytes(b"tridag", np.asarray(train, np.int64).ctypes.data, len(train))
     scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
-    a_, b_, tbl = ifl.tune("tridag", train, reps=3, cost=1, scratch=scratch)
+    a_, b_, tbl = ifl.tune("tridag", train, reps=7, cost=1, scratch=scratch)
     del scratch
     rows = []
     for ds in ("small", "medium", "large"):
@@ -230,10 +230,10 @@ def suite_lvc():
     train = [s for ds in ("small", "large") for s in sites(ds)[0]]
     need = ifl.lib().ifl_tune_scratch_bytes(b"tridag", np.asarray(train, np.int64).ctypes.data, len(train))
     scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
-    ifl.tune("tridag", train, reps=3, cost=1, scratch=scratch)
+    ifl.tune("tridag", train, reps=7, cost=1, scratch=scratch)
     del scratch
     ltrain = [(S, 8, X, Y) for (S, T, X, Y) in gen.LVC_DATASETS.values()]
-    t0, _, ltbl = ifl.tune("lvc", ltrain, reps=3, cost=1)
+    t0, _, ltbl = ifl.tune("lvc", ltrain, reps=7, cost=1)
     rows = []
     for ds, (S, T, X, Y) in gen.LVC_DATASETS.items():
         (ax, bx, cx), (ay, by, cy), xs, ys = gen.lvc_problem(17, S, X, Y, "cuda")
@@ -288,7 +288,7 @@ def suite_col():
         need = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data, len(train))
         scratch = torch.empty(need, dtype=torch.uint8, device="cuda")
         scratch.view(-1)[: (need // 4) * 4].view(torch.float32).copy_(gen.generate("F32_UNIT", 4, need // 4, "cuda"))
-        a, b, _ = ifl.tune(site, train, reps=3, cost=1, scratch=scratch)
+        a, b, _ = ifl.tune(site, train, reps=7, cost=1, scratch=scratch)
         del scratch
         tuned[site] = {"t_top": a, "t_intra": b}
     N = 1 << L2N

@@ -25,6 +25,35 @@
 
 namespace {
 
+// Minimax cost (cost = 1): paths whose worst slowdown is within 1 % of the
+// best achievable one are a measurement tie (per-shape medians of a few reps
+// move that much from box to box), and among them the smallest sum of
+// runtimes wins -- so a near-equal worst shape no longer decides the versions
+// of all the other shapes.  Two passes (optimum first, then the tie set), so
+// ties cannot chain.  cost = 0 (the paper's sum): exact minimum.
+constexpr double kTieTol = 0.01;
+
+struct PathCost {
+    double primary, sum;
+    size_t order;  // first enumeration position (deterministic tie-break)
+};
+
+template <typename Map>
+typename Map::const_iterator pick_path(const Map& memo, int cost) {
+    double best = std::numeric_limits<double>::infinity();
+    for (auto& kv : memo) best = std::min(best, kv.second.first.primary);
+    const double lim = cost == 1 ? best * (1.0 + kTieTol) : best;
+    auto pick = memo.end();
+    for (auto it = memo.begin(); it != memo.end(); ++it) {
+        const PathCost& c = it->second.first;
+        if (c.primary > lim) continue;
+        if (pick == memo.end() || c.sum < pick->second.first.sum ||
+            (c.sum == pick->second.first.sum && c.order < pick->second.first.order))
+            pick = it;
+    }
+    return pick;
+}
+
 std::vector<int64_t> candidates(std::vector<int64_t> v) {
     std::sort(v.begin(), v.end());
     v.erase(std::unique(v.begin(), v.end()), v.end());
@@ -54,33 +83,28 @@ extern "C" int ifl_tune_search(const int64_t* par_top, const int64_t* par_mid, c
     for (int s = 0; s < nshapes; ++s)
         for (int v = 0; v < 3; ++v) best[s] = std::min(best[s], cost_table[s * 3 + v]);
 
-    std::map<std::vector<int>, std::pair<double, double>> memo;  // path -> (primary, sum)
-    double bp = std::numeric_limits<double>::infinity(), bs = bp;
-    int64_t btop = ct.back(), bintra = ci.back();
+    // path -> (cost, thresholds of its first enumeration)
+    std::map<std::vector<int>, std::pair<PathCost, std::pair<int64_t, int64_t>>> memo;
     for (int64_t a : ct) {
         for (int64_t b : ci) {
             std::vector<int> path(nshapes);
             for (int s = 0; s < nshapes; ++s)
                 path[s] = pt[s] >= a ? IFL_V_TOP : (pm[s] >= b ? IFL_V_MIDDLE : IFL_V_FLAT);
-            auto it = memo.find(path);
-            if (it == memo.end()) {
-                double sum = 0, worst = 0;
-                for (int s = 0; s < nshapes; ++s) {
-                    const double c = cost_table[s * 3 + path[s]];
-                    sum += c;
-                    worst = std::max(worst, c / best[s]);
-                }
-                it = memo.emplace(path, std::make_pair(cost == 0 ? sum : worst, sum)).first;
+            if (memo.count(path)) continue;
+            double sum = 0, worst = 0;
+            for (int s = 0; s < nshapes; ++s) {
+                const double c = cost_table[s * 3 + path[s]];
+                sum += c;
+                worst = std::max(worst, c / best[s]);
             }
-            const double p = it->second.first, s = it->second.second;
-            if (p < bp || (p == bp && s < bs)) {
-                bp = p;
-                bs = s;
-                btop = a;
-                bintra = b;
-            }
+            memo.emplace(path, std::make_pair(PathCost{cost == 0 ? sum : worst, sum, memo.size()},
+                                              std::make_pair(a, b)));
         }
     }
+    auto it = pick_path(memo, cost);
+    const double bp = it == memo.end() ? std::numeric_limits<double>::infinity() : it->second.first.primary;
+    const int64_t btop = it == memo.end() ? ct.back() : it->second.second.first;
+    const int64_t bintra = it == memo.end() ? ci.back() : it->second.second.second;
     if (t_top) *t_top = btop;
     if (t_intra) *t_intra = bintra;
     if (n_paths) *n_paths = (int)memo.size();
@@ -101,28 +125,19 @@ struct ChainSearch {
     int ns, G, kind;
     std::vector<std::vector<int64_t>> cand;
     std::vector<double> best;
-    std::map<std::vector<int>, std::pair<double, double>> memo;
+    std::map<std::vector<int>, std::pair<PathCost, std::vector<int64_t>>> memo;  // path -> (cost, thresholds)
     std::vector<int> path;
-    std::vector<int64_t> cur, bt;
-    double bp = std::numeric_limits<double>::infinity(), bs = std::numeric_limits<double>::infinity();
+    std::vector<int64_t> cur;
 
     void eval() {
-        auto it = memo.find(path);
-        if (it == memo.end()) {
-            double sum = 0, worst = 0;
-            for (int s = 0; s < ns; ++s) {
-                const double c = cost[s * (G + 1) + path[s]];
-                sum += c;
-                worst = std::max(worst, c / best[s]);
-            }
-            it = memo.emplace(path, std::make_pair(kind == 0 ? sum : worst, sum)).first;
+        if (memo.count(path)) return;
+        double sum = 0, worst = 0;
+        for (int s = 0; s < ns; ++s) {
+            const double c = cost[s * (G + 1) + path[s]];
+            sum += c;
+            worst = std::max(worst, c / best[s]);
         }
-        const double p = it->second.first, q = it->second.second;
-        if (p < bp || (p == bp && q < bs)) {
-            bp = p;
-            bs = q;
-            bt = cur;
-        }
+        memo.emplace(path, std::make_pair(PathCost{kind == 0 ? sum : worst, sum, memo.size()}, cur));
     }
     void rec(int k, int left) {
         if (k == G || left == 0) {
@@ -172,12 +187,12 @@ extern "C" int ifl_tune_search_chain(const int64_t* par, const double* cost_tabl
         for (int v = 0; v <= G; ++v) cs.best[s] = std::min(cs.best[s], cost_table[s * (G + 1) + v]);
     cs.path.assign(nshapes, -1);
     cs.cur.assign(G, INT64_MAX);
-    cs.bt.assign(G, INT64_MAX);
     cs.rec(0, nshapes);
+    auto it = pick_path(cs.memo, cost);
     if (thresholds)
-        for (int k = 0; k < G; ++k) thresholds[k] = cs.bt[k];
+        for (int k = 0; k < G; ++k) thresholds[k] = it == cs.memo.end() ? INT64_MAX : it->second.second[k];
     if (n_paths) *n_paths = (int)cs.memo.size();
-    return std::isfinite(cs.bp) ? IFL_OK : IFL_ENOTFIT;
+    return (it != cs.memo.end() && std::isfinite(it->second.first.primary)) ? IFL_OK : IFL_ENOTFIT;
 }
 
 namespace {

@@ -237,6 +237,23 @@ def test_fig5_duplicate_paths_memoised(L):
     ifl.reset_thresholds()
 
 
+def test_tune_search_minimax_tie_tolerance(L):
+    """cost = 1: a path whose worst slowdown is within 1 % of the optimum is a
+    tie and the smaller sum of runtimes wins; beyond 1 % the minimax decides.
+    Two shapes with the same Par share a version: FLAT for both costs a worst
+    slowdown of 1.001 (sum 11.0), MIDDLE for both 1.005 (sum 10.995)."""
+    pt = pm = [5, 5]
+    table = [[9.0, 1.005, 1.0], [99.0, 9.99, 10.0]]
+    a, b, _ = ifl.tune_search(pt, pm, table, cost=1)
+    ifl.set_thresholds("segred.b4", a, b)
+    assert ifl.select("segred.b4", 5, 1).version == "middle"
+    table2 = [[9.0, 1.05, 1.0], [99.0, 9.99, 10.0]]  # MIDDLE's worst is now 5 % off: not a tie
+    a, b, _ = ifl.tune_search(pt, pm, table2, cost=1)
+    ifl.set_thresholds("segred.b4", a, b)
+    assert ifl.select("segred.b4", 5, 1).version == "flat"
+    ifl.reset_thresholds()
+
+
 def test_tune_search_minimax_cost(L):
     # cost 1 = max slowdown vs best; cost 0 = sum (P:372) -- can disagree.
     pt = [1, 100]
@@ -325,7 +342,7 @@ def _chain_brute(par, cost, kind):
         v = sorted(set(int(x) for x in v))
         return [v[0]] + [v[i] + 1 for i in range(len(v) - 1)] + [2**63 - 1]
     best = cost.min(axis=1)
-    res = None
+    keys = []
     for th in itertools.product(*[cands(par[:, k]) for k in range(G)]):
         leaf = []
         for s in range(ns):
@@ -336,9 +353,13 @@ def _chain_brute(par, cost, kind):
                     break
             leaf.append(lf)
         c = [cost[s, leaf[s]] for s in range(ns)]
-        key = (sum(c) if kind == 0 else max(ci / bi for ci, bi in zip(c, best)), sum(c))
-        res = key if res is None or key < res else res
-    return res
+        keys.append((sum(c) if kind == 0 else max(ci / bi for ci, bi in zip(c, best)), sum(c)))
+    if kind == 0:
+        return min(keys)
+    # minimax with the 1 % tie rule of tune.cpp: the smallest sum among paths
+    # whose worst slowdown is within 1 % of the optimum
+    opt = min(k[0] for k in keys)
+    return min((k for k in keys if k[0] <= opt * 1.01), key=lambda k: k[1])
 
 
 @pytest.mark.parametrize("G", [1, 2, 3, 4])

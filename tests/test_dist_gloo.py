@@ -298,3 +298,72 @@ def test_colred_lvc_irr_dist_world2():
         bad = [r for r in res if not r[-1]]
         assert not bad, (rank, bad[:5])
         assert len(res) > 20
+
+
+def _bench_worker(rank, world, port, q):
+    """bench.py's N > 1 step (the weak-scaled sweep through dist.py), gloo on
+    CPU with the oracle standing in for the GPU library: every rank's results
+    equal the oracle on the global [2^k][world * 2^L / 2^k] arrays."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    td.init_process_group("gloo", rank=rank, world_size=world)
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+    import oracle
+    results = []
+
+    def local_scan(x, op, f, ne, seed):
+        xn = x.numpy()
+        if seed is not None:
+            return torch.from_numpy(oracle.segscan_seeded(xn, seed.numpy(), op, f).astype(xn.dtype))
+        return torch.from_numpy(np.ascontiguousarray(oracle.segscan(xn, op, f, ne).astype(xn.dtype)))
+    try:
+        L = 6
+        shapes = bench.sharded_shapes(world, rank, log2n=L)
+        # the global array of every shape: world blocks of 2^L int32, rank r's block at r * 2^L
+        G = gen.generate("I32_FULL", 17, world << L)
+        mine = G[rank << L:(rank + 1) << L].contiguous()
+        outs = bench.sharded_step(mine, shapes, local_segred=_oracle_local, local_segscan=local_scan)
+        for i, (ng, mg, plan, (nl, ml)) in enumerate(shapes):
+            # rank r's block: rows [lo, hi) (outer) or columns [lo, hi) of every row (inner) of the global array
+            blocks = []
+            for r in range(world):
+                p = __import__("paper_conf_ppopp_henriksenteo19_b200.dist", fromlist=["x"]).plan_segred(ng, mg, world, r)
+                blocks.append((p, G[r << L:(r + 1) << L]))
+            X = np.zeros((ng, mg), np.int32)
+            for p, b in blocks:
+                if p.mode == "outer":
+                    X[p.lo:p.hi] = b.numpy().reshape(p.hi - p.lo, mg)
+                else:
+                    X[:, p.lo:p.hi] = b.numpy().reshape(ng, p.hi - p.lo)
+            red, scan = outs[2 * i].numpy(), outs[2 * i + 1].numpy()
+            want_red, want_scan = oracle.segred(X, "sum"), oracle.segscan(X, "sum")
+            if plan.mode == "outer":
+                ok = np.array_equal(red, want_red[plan.lo:plan.hi]) and np.array_equal(
+                    scan, want_scan[plan.lo:plan.hi])
+            else:
+                ok = np.array_equal(red, want_red) and np.array_equal(scan, want_scan[:, plan.lo:plan.hi])
+            results.append((plan.mode, ng, mg, bool(ok)))
+        q.put((rank, results))
+    except Exception:
+        import traceback
+        q.put((rank, [("error", traceback.format_exc(), False)]))
+    finally:
+        td.destroy_process_group()
+
+
+def test_bench_sharded_step_world2():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bench_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+    for rank, rows in res:
+        bad = [r for r in rows if not r[-1]]
+        assert not bad, f"rank {rank}: {bad[:5]}"
+        assert any(r[0] == "outer" for r in rows) and any(r[0] == "inner" for r in rows)
