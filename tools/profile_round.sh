@@ -20,8 +20,9 @@ cap() {  # name op version n m kernel-regex
     -o gpurun_out/ncu/$1 python tools/prof_one.py --op $2 --version $3 --n $4 --m $5 ${7:-} > /dev/null 2>&1
   echo "$1 rc=$?"
 }
-cap segscan_flat_n1      segscan flat   1        67108864 flat_scan
-cap segscan_flat_n4096   segscan flat   4096     16384    flat_scan
+cap segscan_flat_n1      segscan flat   1        67108864 flat_scan_jr
+cap segscan_flat_n4096   segscan flat   4096     16384    flat_scan_jr
+cap segscan_flat_n65536  segscan flat   65536    1024     flat_scan_dlb
 cap segred_flat_n1       segred  flat   1        67108864 flat_red_kernel
 cap segred_middle_n2e16  segred  middle 65536    1024     segred_mid_vec
 cap segscan_middle_n2e18 segscan middle 262144   256      segscan_mid

@@ -35,7 +35,7 @@ with open(f"profiles/{tag}_ncu_launches_summary.csv", "w") as fp:
 
 # ---- full captures
 ALG = {  # algorithmic bytes of the captured launch
-    "segscan_flat_n1": 8 * 2**26, "segscan_flat_n4096": 8 * 2**26, "segred_flat_n1": 4 * (2**26 + 1),
+    "segscan_flat_n1": 8 * 2**26, "segscan_flat_n4096": 8 * 2**26, "segscan_flat_n65536": 8 * 2**26, "segred_flat_n1": 4 * (2**26 + 1),
     "segred_middle_n2e16": 4 * (2**26 + 65536), "segscan_middle_n2e18": 8 * 2**26,
     "segred_top_n2e24": 4 * (2**26 + 2**24), "segscan_top_n2e23": 8 * 2**26,
     "redomap2_tc_8192": 2 * (2 * 8192 * 8192) + 4 * 8192 * 8192, "redomap2_flat_n1": 2 * (2 * 2**30) + 4,
@@ -43,14 +43,14 @@ ALG = {  # algorithmic bytes of the captured launch
     "lvc_outer_large": 2 * 8 * 256 * 256 * 256,  # one read + one write per element for the whole loop
     "colred_flat_n2e20": 4 * 2**26, "colscan_top_n4": 8 * 2**26, "colscan_flat_n2e26": 8 * 2**26,
 }
-GROUP = {"segscan_flat_n1": "segscan_flat", "segred_flat_n1": "segred_flat", "segred_middle_n2e16": "segred_middle",
+GROUP = {"segscan_flat_n1": "segscan_flat", "segscan_flat_n65536": "segscan_flat_dlb", "segred_flat_n1": "segred_flat", "segred_middle_n2e16": "segred_middle",
          "segscan_middle_n2e18": "segscan_middle", "segred_top_n2e24": "segred_top", "segscan_top_n2e23": "segscan_top",
          "redomap2_tc_8192": "redomap2_tc", "redomap2_flat_n1": "redomap2_flat", "tridag_middle_large": "tridag_middle",
          "tridag_flat_large": "tridag_flat", "lvc_outer_large": "lvc_outer", "colred_flat_n2e20": "colred_flat",
          "colscan_top_n4": "colscan_top", "colscan_flat_n2e26": "colscan_flat",
          "segred_irr_flat_m1k": "segred_irr_flat", "segscan_irr_flat_m1k": "segscan_irr_flat"}
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
-        "dram__throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_sector_hit_rate.pct",
+        "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "lts__t_sector_hit_rate.pct",
         "sm__warps_active.avg.pct_of_peak_sustained_active", "smsp__issue_active.avg.pct_of_peak_sustained_active",
         "launch__registers_per_thread", "launch__grid_size", "launch__block_size",
         "smsp__average_warps_issue_stalled_long_scoreboard_per_issue_active.ratio",
@@ -58,8 +58,11 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
 traffic = {}
 md = [f"# ncu summary ({tag})\n", "Full-set captures (`--set full --clock-control none`, one launch each, "
       "cold cache), from `tools/profile_round.sh`.  traffic = dram read + write; alg = algorithmic bytes "
-      "(SURVEY 8(d)).\n", "| capture | kernel | time | DRAM read | DRAM write | traffic / alg | DRAM % peak | "
-      "L2 hit % | warps active % | issue active % |", "|---|---|---|---|---|---|---|---|---|---|"]
+      "(SURVEY 8(d)).  DRAM % = gpu__dram_throughput (of ncu's DRAM peak); tensor % = "
+      "sm__pipe_tensor_cycles_active (of active cycles) / bf16 dense op rate (of peak, elapsed).\n",
+      "| capture | kernel | time | DRAM read | DRAM write | traffic / alg | DRAM % peak | "
+      "L2 hit % | warps active % | issue active % | tensor pipe % | bf16 MMA % |",
+      "|---|---|---|---|---|---|---|---|---|---|---|---|"]
 for f in sorted(glob.glob(os.path.join(src, "*.raw.csv"))):
     name = os.path.basename(f).replace(".raw.csv", "")
     with open(f) as fp:
@@ -84,10 +87,12 @@ for f in sorted(glob.glob(os.path.join(src, "*.raw.csv"))):
     ratio = (rdb + wrb) / alg if alg else float("nan")
     kern = d.get("Kernel Name", "?").split("(")[0].replace("void ", "")
     md.append(f"| {name} | `{kern}` | {t_us:.1f} us | {rdb / 1e6:.1f} MB | {wrb / 1e6:.1f} MB | {ratio:.3f} | "
-              f"{num('dram__throughput.avg.pct_of_peak_sustained_elapsed'):.1f} | "
+              f"{num('gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed'):.1f} | "
               f"{num('lts__t_sector_hit_rate.pct'):.1f} | "
               f"{num('sm__warps_active.avg.pct_of_peak_sustained_active'):.1f} | "
-              f"{num('smsp__issue_active.avg.pct_of_peak_sustained_active'):.1f} |")
+              f"{num('smsp__issue_active.avg.pct_of_peak_sustained_active'):.1f} | "
+              f"{num('sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active'):.1f} | "
+              f"{num('sm__ops_path_tensor_op_hmma_src_bf16_dst_fp32_sparsity_off.avg.pct_of_peak_sustained_elapsed'):.1f} |")
     if name in GROUP:
         traffic[GROUP[name]] = {"capture": name, "dram_bytes_per_launch": rdb + wrb, "algorithmic_bytes": alg,
                                 "ratio": round(ratio, 4), "ncu_time_us": round(t_us, 2)}
