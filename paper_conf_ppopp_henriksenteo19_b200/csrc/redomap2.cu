@@ -71,80 +71,6 @@ __global__ void __launch_bounds__(256) transpose_kernel(const Tin* __restrict__ 
         if (j0 + r < p && k0 + tx < m) Bt[(j0 + r) * m + k0 + tx] = tile[tx][r];
 }
 
-// --------------------------------------------------------------- V_FLAT
-
-constexpr int kFlatMmThreads = 256;
-
-int64_t mm_flat_splits(int64_t n, int64_t m, int64_t p) {
-    const int64_t outs = n * p;
-    const int64_t want = ceil_div((int64_t)148 * 8, outs);          // fill the GPU
-    const int64_t maxs = std::max<int64_t>(1, ceil_div(m, 4096));   // >= 4096 k per split
-    return std::max<int64_t>(1, std::min(want, maxs));
-}
-
-template <typename Tin, bool VEC>
-__global__ void __launch_bounds__(kFlatMmThreads) mm_flat_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
-                                                                 float* __restrict__ C, float* __restrict__ part,
-                                                                 int64_t n, int64_t m, int64_t p, int64_t kchunk,
-                                                                 int nsplit) {
-    __shared__ float red[kFlatMmThreads / 32];
-    constexpr int E = VecE<Tin>::E;
-    const int64_t o = (int64_t)blockIdx.y + (int64_t)blockIdx.z * gridDim.y;
-    if (o >= n * p) return;
-    const int64_t i = o / p, j = o - i * p;
-    const int split = blockIdx.x;
-    const int64_t k0 = split * kchunk, k1 = std::min(m, k0 + kchunk);
-    const Tin* a = A + i * m;
-    const Tin* b = Bt + j * m;
-    float acc[4] = {0.f, 0.f, 0.f, 0.f};
-    int64_t k = k0 + (int64_t)threadIdx.x * E;
-    if (VEC) {
-        for (; k + E + (int64_t)kFlatMmThreads * E <= k1; k += 2 * (int64_t)kFlatMmThreads * E) {
-            float x0[E], y0[E], x1[E], y1[E];
-            load16(a + k, x0);
-            load16(b + k, y0);
-            load16(a + k + kFlatMmThreads * E, x1);
-            load16(b + k + kFlatMmThreads * E, y1);
-#pragma unroll
-            for (int e = 0; e < E; ++e) {
-                acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
-                acc[(e + 2) & 3] = fmaf(x1[e], y1[e], acc[(e + 2) & 3]);
-            }
-        }
-        for (; k + E <= k1; k += (int64_t)kFlatMmThreads * E) {
-            float x0[E], y0[E];
-            load16(a + k, x0);
-            load16(b + k, y0);
-#pragma unroll
-            for (int e = 0; e < E; ++e) acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
-        }
-        // ragged tail of the chunk (fewer than E elements per thread slot)
-        const int64_t tail0 = k1 - ((k1 - k0) % E);
-        for (int64_t kk = tail0 + threadIdx.x; kk < k1; kk += kFlatMmThreads) acc[0] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[0]);
-    } else {
-        for (int64_t kk = k0 + threadIdx.x; kk < k1; kk += kFlatMmThreads)
-            acc[kk & 3] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[kk & 3]);
-    }
-    float s = (acc[0] + acc[1]) + (acc[2] + acc[3]);
-    s = warp_reduce<OP_SUM>(s);
-    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        float r = 0.f;
-        for (int w = 0; w < kFlatMmThreads / 32; ++w) r += red[w];
-        if (nsplit == 1) C[o] = r;
-        else part[o * nsplit + split] = r;
-    }
-}
-
-__global__ void mm_flat_finalize(const float* __restrict__ part, float* __restrict__ C, int64_t outs, int nsplit) {
-    for (int64_t o = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; o < outs; o += (int64_t)gridDim.x * blockDim.x) {
-        float r = 0.f;
-        for (int s = 0; s < nsplit; ++s) r += part[o * nsplit + s];
-        C[o] = r;
-    }
-}
-
 // ------------------------------------------------------------- V_MIDDLE
 
 template <typename Tin, bool VEC>
@@ -317,10 +243,299 @@ cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* par
 
 static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 
-// V_FLAT's SIMT form: tiny n*p -> one CTA per (output, k-chunk) dot product;
-// otherwise 32x32 output tiles split along k until the GPU is full.
+// V_FLAT's register-blocked split-K engine for skinny outputs (n*p <= 4096,
+// the degenerate end of the Fig 2 family): grid = (k-chunks,
+// RI x RJ output tiles).  Each thread walks its k positions of the chunk in
+// 8-byte vectors of the RI rows of A and of B (B^T rows, or for B given as
+// yss [m][p] the RJ-wide slices of yss's rows -- no transposition pass),
+// staged through an S-deep cp.async pipeline in THREAD-PRIVATE shared-memory
+// slots (each thread consumes only its own copies: no CTA barrier in the
+// loop, and S-1 stages of loads in flight without holding registers), and
+// accumulates the RI x RJ partial dot products in registers (bf16 widened to
+// f32 exactly).  Every element of A and B is read from DRAM once per output
+// tile row / column; the CTA reduces its partials (shuffles + smem) into one
+// partial tile, and mm_splitk_finalize sums the chunks in a fixed order.
+constexpr int kSkinnyThreads = 256;
+constexpr int kSkinnyStageBytes = 128 * 1024;  // pipeline depth: as many stages as fit 128 KB (3..12)
+constexpr int64_t kSkinnyMaxOuts = 4096;
+
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// 8 bytes of Tin -> E floats
+template <typename Tin>
+__device__ __forceinline__ void unpack8(uint2 u, float (&o)[8 / sizeof(Tin)]) {
+    if constexpr (std::is_same<Tin, float>::value) {
+        o[0] = __uint_as_float(u.x);
+        o[1] = __uint_as_float(u.y);
+    } else {
+        o[0] = __uint_as_float(u.x << 16);
+        o[1] = __uint_as_float(u.x & 0xffff0000u);
+        o[2] = __uint_as_float(u.y << 16);
+        o[3] = __uint_as_float(u.y & 0xffff0000u);
+    }
+}
+
+// Shared-memory words per thread per stage: RI A vectors + the B data of one
+// k-vector (KMAJ: RJ vectors; row-major: E slices of RJ elements, in units
+// of min(8, RJ * sizeof) bytes).
+template <typename Tin, int RI, int RJ, bool KMAJ>
+struct SkinnyGeom {
+    static constexpr int E = 8 / (int)sizeof(Tin);
+    static constexpr int SLICE = RJ * (int)sizeof(Tin);        // bytes of one row-major B slice
+    static constexpr int UNIT = SLICE >= 8 ? 8 : 4;            // cp.async size (row-major needs SLICE >= 4)
+    static constexpr int BU = KMAJ ? RJ : E * (SLICE / UNIT);  // B copies per k-vector
+    static constexpr int BWORDS = KMAJ ? RJ : E * ((SLICE + 7) / 8);  // 8-byte smem words of B
+    static constexpr int WORDS = RI + BWORDS;
+    static constexpr int S0 = kSkinnyStageBytes / (WORDS * kSkinnyThreads * 8);
+    static constexpr int S = S0 < 3 ? 3 : S0 > 12 ? 12 : S0;  // cp.async stages
+    static constexpr size_t SMEM = (size_t)S * WORDS * kSkinnyThreads * 8;
+};
+
+template <typename Tin, int RI, int RJ, bool KMAJ>
+__global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __restrict__ A, const Tin* __restrict__ B,
+                                                                   float* __restrict__ part, int64_t n, int64_t m,
+                                                                   int64_t p, int64_t kchunk, int tiles_j) {
+    using Gm = SkinnyGeom<Tin, RI, RJ, KMAJ>;
+    constexpr int E = Gm::E, NW = kSkinnyThreads / 32, S = Gm::S;
+    extern __shared__ __align__(16) uint2 sbuf[];  // [S][WORDS][threads]
+    __shared__ float red[NW][RI * RJ];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int tile = blockIdx.y;
+    const int64_t i0 = (int64_t)(tile / tiles_j) * RI, j0 = (int64_t)(tile % tiles_j) * RJ;
+    const int64_t k0 = (int64_t)blockIdx.x * kchunk, k1 = std::min(m, k0 + kchunk);
+    const int64_t stride = (int64_t)kSkinnyThreads * E;
+    const int nit = (int)ceil_div(std::max<int64_t>(0, k1 - k0), stride);
+    const Tin* ar[RI];
+#pragma unroll
+    for (int r = 0; r < RI; ++r) ar[r] = A + std::min(i0 + r, n - 1) * m;  // rows past n: clamped, dropped at the end
+    const Tin* br[RJ];
+#pragma unroll
+    for (int c = 0; c < RJ; ++c) br[c] = B + std::min(j0 + c, p - 1) * m;  // KMAJ rows of B^T
+    auto slot = [&](int st, int word) -> uint2* { return sbuf + ((size_t)st * Gm::WORDS + word) * kSkinnyThreads + t; };
+    auto issue = [&](int it) {
+        const int64_t k = k0 + (int64_t)it * stride + (int64_t)t * E;
+        if (it < nit && k < k1) {
+            const int st = it % S;
+#pragma unroll
+            for (int r = 0; r < RI; ++r) cp_async8(slot(st, r), ar[r] + k);
+            if constexpr (KMAJ) {
+#pragma unroll
+                for (int c = 0; c < RJ; ++c) cp_async8(slot(st, RI + c), br[c] + k);
+            } else {
+#pragma unroll
+                for (int e = 0; e < E; ++e) {
+                    const char* src = reinterpret_cast<const char*>(B + (k + e) * p + j0);
+                    char* dst = reinterpret_cast<char*>(slot(st, RI + e * ((Gm::SLICE + 7) / 8)));
+#pragma unroll
+                    for (int u = 0; u < Gm::SLICE / Gm::UNIT; ++u) {
+                        // consecutive 8-byte words of a slice are kSkinnyThreads words apart
+                        char* d = dst + (size_t)((u * Gm::UNIT) / 8) * kSkinnyThreads * 8 + (u * Gm::UNIT) % 8;
+                        if constexpr (Gm::UNIT == 8) cp_async8(d, src + u * 8);
+                        else cp_async4(d, src + u * 4);
+                    }
+                }
+            }
+        }
+        cp_async_commit();  // (possibly empty) group per iteration keeps the wait count uniform
+    };
+    float acc[RI][RJ];
+#pragma unroll
+    for (int r = 0; r < RI; ++r)
+#pragma unroll
+        for (int c = 0; c < RJ; ++c) acc[r][c] = 0.f;
+#pragma unroll
+    for (int s = 0; s < S - 1; ++s) issue(s);
+    for (int it = 0; it < nit; ++it) {
+        issue(it + S - 1);
+        cp_async_wait<S - 1>();  // this thread's copies of iteration it have landed
+        const int64_t k = k0 + (int64_t)it * stride + (int64_t)t * E;
+        if (k >= k1) continue;
+        const int st = it % S;
+        float a[RI][E], b[RJ][E];
+#pragma unroll
+        for (int r = 0; r < RI; ++r) unpack8<Tin>(*slot(st, r), a[r]);
+        if constexpr (KMAJ) {
+#pragma unroll
+            for (int c = 0; c < RJ; ++c) unpack8<Tin>(*slot(st, RI + c), b[c]);
+        } else {
+#pragma unroll
+            for (int e = 0; e < E; ++e) {
+                const uint2* q = slot(st, RI + e * ((Gm::SLICE + 7) / 8));
+#pragma unroll
+                for (int c = 0; c < RJ; ++c) {
+                    const int byte = c * (int)sizeof(Tin);
+                    const uint2 wd = q[(size_t)(byte / 8) * kSkinnyThreads];
+                    const uint32_t h = (byte % 8) < 4 ? wd.x : wd.y;
+                    if constexpr (std::is_same<Tin, float>::value) b[c][e] = __uint_as_float(h);
+                    else b[c][e] = __uint_as_float((byte % 4) == 0 ? (h << 16) : (h & 0xffff0000u));
+                }
+            }
+        }
+#pragma unroll
+        for (int e = 0; e < E; ++e)
+#pragma unroll
+            for (int r = 0; r < RI; ++r)
+#pragma unroll
+                for (int c = 0; c < RJ; ++c) acc[r][c] = fmaf(a[r][e], b[c][e], acc[r][c]);
+    }
+    cp_async_wait<0>();
+#pragma unroll
+    for (int r = 0; r < RI; ++r)
+#pragma unroll
+        for (int c = 0; c < RJ; ++c) {
+            const float v = warp_reduce<OP_SUM>(acc[r][c]);
+            if (lane == 0) red[w][r * RJ + c] = v;
+        }
+    __syncthreads();
+    if (t < RI * RJ) {
+        float s = 0.f;
+#pragma unroll
+        for (int q = 0; q < NW; ++q) s += red[q][t];
+        const int64_t i = i0 + t / RJ, j = j0 + t % RJ;
+        if (i < n && j < p) part[(int64_t)blockIdx.x * n * p + i * p + j] = s;
+    }
+}
+
+// Scalar form (misaligned operands or m not a multiple of the vector width).
+template <typename Tin, int RI, int RJ, bool KMAJ>
+__global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const Tin* __restrict__ A,
+                                                                          const Tin* __restrict__ B,
+                                                                          float* __restrict__ part, int64_t n,
+                                                                          int64_t m, int64_t p, int64_t kchunk,
+                                                                          int tiles_j) {
+    constexpr int NW = kSkinnyThreads / 32;
+    __shared__ float red[NW][RI * RJ];
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int tile = blockIdx.y;
+    const int64_t i0 = (int64_t)(tile / tiles_j) * RI, j0 = (int64_t)(tile % tiles_j) * RJ;
+    const int64_t k0 = (int64_t)blockIdx.x * kchunk, k1 = std::min(m, k0 + kchunk);
+    float acc[RI][RJ];
+#pragma unroll
+    for (int r = 0; r < RI; ++r)
+#pragma unroll
+        for (int c = 0; c < RJ; ++c) acc[r][c] = 0.f;
+    for (int64_t k = k0 + t; k < k1; k += kSkinnyThreads) {
+        float a[RI], b[RJ];
+#pragma unroll
+        for (int r = 0; r < RI; ++r) a[r] = to_f(__ldg(A + std::min(i0 + r, n - 1) * m + k));
+#pragma unroll
+        for (int c = 0; c < RJ; ++c) {
+            const int64_t j = std::min(j0 + c, p - 1);
+            b[c] = to_f(KMAJ ? __ldg(B + j * m + k) : __ldg(B + k * p + j));
+        }
+#pragma unroll
+        for (int r = 0; r < RI; ++r)
+#pragma unroll
+            for (int c = 0; c < RJ; ++c) acc[r][c] = fmaf(a[r], b[c], acc[r][c]);
+    }
+#pragma unroll
+    for (int r = 0; r < RI; ++r)
+#pragma unroll
+        for (int c = 0; c < RJ; ++c) {
+            const float v = warp_reduce<OP_SUM>(acc[r][c]);
+            if (lane == 0) red[w][r * RJ + c] = v;
+        }
+    __syncthreads();
+    if (t < RI * RJ) {
+        float s = 0.f;
+#pragma unroll
+        for (int q = 0; q < NW; ++q) s += red[q][t];
+        const int64_t i = i0 + t / RJ, j = j0 + t % RJ;
+        if (i < n && j < p) part[(int64_t)blockIdx.x * n * p + i * p + j] = s;
+    }
+}
+
+// Where the engine is V_FLAT's form: f32 up to 4096 outputs; bf16 up to 256
+// (beyond, the tcgen05 split-K tiles win: B200, k = 30 family, n = p = 32 / 64:
+// 63 / 32 us vs 96 / 104 us for this FMA-bound engine)
+static bool skinny_ok(int64_t n, int64_t p, bool bf16) { return n * p <= (bf16 ? 256 : kSkinnyMaxOuts); }
+static int skinny_r(int64_t x) { return x >= 8 ? 8 : x >= 4 ? 4 : x >= 2 ? 2 : 1; }
+// k-chunks: one wave of CTAs (one per SM: the pipelines take ~128 KB of
+// shared memory) over all output tiles, >= 2 vector rounds per chunk
+static int64_t skinny_kchunk(int64_t n, int64_t m, int64_t p) {
+    const int64_t tiles = ceil_div(n, skinny_r(n)) * ceil_div(p, skinny_r(p));
+    const int64_t want = std::max<int64_t>(1, (int64_t)148 / tiles);
+    int64_t kc = std::max<int64_t>((int64_t)kSkinnyThreads * 8, ceil_div(m, want));
+    return ceil_div(kc, 8) * 8;  // a multiple of every vector width
+}
+static int64_t skinny_splits(int64_t n, int64_t m, int64_t p) { return ceil_div(m, skinny_kchunk(n, m, p)); }
+
+template <typename Tin, int RI, int RJ, bool KMAJ>
+static cudaError_t launch_skinny_k(const Tin* A, const Tin* B, float* dst, int64_t n, int64_t m, int64_t p,
+                                   int64_t kc, int64_t splits, int tj, int64_t tiles, cudaStream_t s) {
+    using Gm = SkinnyGeom<Tin, RI, RJ, KMAJ>;
+    constexpr int E = Gm::E;
+    // cp.async needs 8-byte aligned rows (KMAJ) / UNIT-aligned B slices (row-major)
+    bool vec = ((uintptr_t)A % 8 == 0) && (m % E == 0);
+    if (KMAJ) vec = vec && ((uintptr_t)B % 8 == 0);
+    else vec = vec && Gm::SLICE >= 4 && ((uintptr_t)B % Gm::UNIT == 0) && ((p * (int64_t)sizeof(Tin)) % Gm::UNIT == 0) &&
+               (p % RJ == 0);
+    dim3 g((unsigned)splits, (unsigned)tiles);
+    if (vec) {
+        const size_t smem = Gm::SMEM;
+        auto k = mm_skinny_kernel<Tin, RI, RJ, KMAJ>;
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            attr = true;
+        }
+        k<<<g, kSkinnyThreads, smem, s>>>(A, B, dst, n, m, p, kc, tj);
+    } else {
+        mm_skinny_scalar_kernel<Tin, RI, RJ, KMAJ><<<g, kSkinnyThreads, 0, s>>>(A, B, dst, n, m, p, kc, tj);
+    }
+    return cudaGetLastError();
+}
+
+template <typename Tin, int RI, int RJ>
+static cudaError_t launch_skinny_rr(const Tin* A, const Tin* B, float* C, float* part, int64_t n, int64_t m, int64_t p,
+                                    bool kmajor, cudaStream_t s) {
+    const int64_t kc = skinny_kchunk(n, m, p), splits = ceil_div(m, kc);
+    const int tj = (int)ceil_div(p, RJ);
+    const int64_t tiles = ceil_div(n, RI) * tj;
+    float* dst = splits == 1 ? C : part;
+    cudaError_t e = kmajor ? launch_skinny_k<Tin, RI, RJ, true>(A, B, dst, n, m, p, kc, splits, tj, tiles, s)
+                           : launch_skinny_k<Tin, RI, RJ, false>(A, B, dst, n, m, p, kc, splits, tj, tiles, s);
+    if (e != cudaSuccess || splits == 1) return e;
+    const int64_t outs = n * p;
+    mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, s>>>(part, C, outs,
+                                                                                                   (int)splits);
+    return cudaGetLastError();
+}
+
+template <typename Tin, int RI>
+static cudaError_t launch_skinny_r(const Tin* A, const Tin* B, float* C, float* part, int64_t n, int64_t m, int64_t p,
+                                   bool kmajor, cudaStream_t s) {
+    switch (skinny_r(p)) {
+    case 8: return launch_skinny_rr<Tin, RI, 8>(A, B, C, part, n, m, p, kmajor, s);
+    case 4: return launch_skinny_rr<Tin, RI, 4>(A, B, C, part, n, m, p, kmajor, s);
+    case 2: return launch_skinny_rr<Tin, RI, 2>(A, B, C, part, n, m, p, kmajor, s);
+    default: return launch_skinny_rr<Tin, RI, 1>(A, B, C, part, n, m, p, kmajor, s);
+    }
+}
+
+template <typename Tin>
+static cudaError_t launch_skinny(const Tin* A, const Tin* B, float* C, float* part, int64_t n, int64_t m, int64_t p,
+                                 bool kmajor, cudaStream_t s) {
+    switch (skinny_r(n)) {
+    case 8: return launch_skinny_r<Tin, 8>(A, B, C, part, n, m, p, kmajor, s);
+    case 4: return launch_skinny_r<Tin, 4>(A, B, C, part, n, m, p, kmajor, s);
+    case 2: return launch_skinny_r<Tin, 2>(A, B, C, part, n, m, p, kmajor, s);
+    default: return launch_skinny_r<Tin, 1>(A, B, C, part, n, m, p, kmajor, s);
+    }
+}
+
+
+// V_FLAT's SIMT form beyond the skinny engine: 32x32 output tiles split along
+// k until the GPU is full.
 constexpr int kFlatTileBM = 32, kFlatTileBK = 32;
-static bool flat_use_dot(int64_t n, int64_t p) { return n * p <= 16; }
 static int64_t simt_flat_splits(int64_t n, int64_t m, int64_t p) {
     const int64_t tiles = ceil_div(n, kFlatTileBM) * ceil_div(p, kFlatTileBM);
     const int64_t nk = ceil_div(m, kFlatTileBK);
@@ -334,7 +549,7 @@ size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
     size_t b = align256((size_t)m * p * 4);
     size_t part = 0;
     if (version == 2 || version == -1) {
-        part = std::max(part, (size_t)n * p * mm_flat_splits(n, m, p) * 4);
+        if (skinny_ok(n, p, false)) part = std::max(part, (size_t)n * p * skinny_splits(n, m, p) * 4);
         part = std::max(part, (size_t)n * p * simt_flat_splits(n, m, p) * 4);
         part = std::max(part, (size_t)n * p * tc_splits(n, m, p, true) * 4);
     }
@@ -359,6 +574,9 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     const Tin* A = (const Tin*)a.A;
     const Tin* Bt = (const Tin*)a.B;
     char* ws = (char*)a.ws;
+    if (version == 2 && skinny_ok(a.n, a.p, std::is_same<Tin, __nv_bfloat16>::value) && a.m > 0)
+        // V_FLAT, skinny outputs: either B layout, no transposition pass
+        return launch_skinny<Tin>(A, Bt, a.C, (float*)ws, a.n, a.m, a.p, a.b_kmajor != 0, a.stream);
     size_t used = 0;
     if (!a.b_kmajor) {  // yss [m][p] -> yss^T [p][m]
         Tin* t = (Tin*)ws;
@@ -381,21 +599,6 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     constexpr bool kBf16 = std::is_same<Tin, __nv_bfloat16>::value;
     const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, Bt);
     if (version == 2) {  // ---- V_FLAT: every level parallel (split-K)
-        if (flat_use_dot(a.n, a.p)) {
-            const int64_t s = mm_flat_splits(a.n, a.m, a.p);
-            int64_t kchunk = ceil_div(a.m, s);
-            kchunk = ceil_div(kchunk, (int64_t)E) * E;  // keep vector alignment of every chunk
-            const int nsplit = (int)ceil_div(a.m, kchunk);
-            const int64_t gy = std::min<int64_t>(outs, 65535), gz = ceil_div(outs, gy);
-            dim3 g((unsigned)nsplit, (unsigned)gy, (unsigned)gz);
-            if (vec) mm_flat_kernel<Tin, true><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
-            else mm_flat_kernel<Tin, false><<<g, kFlatMmThreads, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kchunk, nsplit);
-            cudaError_t e = cudaGetLastError();
-            if (e != cudaSuccess || nsplit == 1) return e;
-            mm_flat_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 8), 256, 0, a.stream>>>(
-                part, a.C, outs, nsplit);
-            return cudaGetLastError();
-        }
         // bf16: 128x256 tensor-core tiles split along k (even a mostly empty
         // tile beats SIMT here); f32: SIMT 32x32 (16x16 when skinny) tiles
         if (tc)

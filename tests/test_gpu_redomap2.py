@@ -143,3 +143,29 @@ def test_redomap2_row_middle_notfit_and_tree(ifl, orc):
             assert ch.version in ("row_top", "row_middle", "top", "middle", "flat")
     finally:
         ifl.reset_thresholds()
+
+
+SKINNY = [(1, 1, 1), (1, 4096, 1), (3, 1000003, 5), (8, 1 << 20, 8), (7, 5000, 3), (16, 300001, 16), (5, 64, 40),
+          (64, 20000, 64), (1, 1 << 22, 2), (33, 9999, 2)]
+
+
+@pytest.mark.parametrize("dt", ["f32", "bf16"])
+@pytest.mark.parametrize("kmajor", [True, False])
+def test_flat_skinny_engine(ifl, orc, dt, kmajor):
+    """V_FLAT's split-K register-block engine (n*p <= 4096 f32 / <= 256 bf16):
+    both B layouts read in place (no transposition), odd n and p (partial
+    register tiles), m not a multiple of the vector width, misaligned
+    operands (the scalar form), and k split across many CTAs."""
+    tdt = torch.float32 if dt == "f32" else torch.bfloat16
+    for (n, m, p) in SKINNY:
+        A, Bt = operands(dt, n, m, p, seed=40)
+        A, Bt = A.to(tdt), Bt.to(tdt)
+        B = Bt if kmajor else Bt.t().contiguous()
+        C = ifl.redomap2(A.cuda(), B.cuda(), b_kmajor=kmajor, version="flat")
+        check(orc, A, Bt, C)
+        # misaligned A (offset by one element): scalar engine
+        buf = torch.empty(n * m + 1, dtype=tdt, device="cuda")
+        Am = buf[1:].view(n, m)
+        Am.copy_(A.cuda())
+        C2 = ifl.redomap2(Am, B.cuda(), b_kmajor=kmajor, version="flat")
+        check(orc, A, Bt, C2)
