@@ -44,6 +44,11 @@ def gtime(fn, R=4, reps=3):
     return statistics.median(ts)
 
 
+NOMINAL_HBM = 8000.0  # GB/s (north_star "~8 TB/s")
+# f32 FMA (CUDA cores) peak: 148 SMs x 128 FMA/clk x 2 flop x 1.965 GHz
+FMA_TFLOPS = 148 * 128 * 2 * 1.965e9 / 1e12
+
+
 def peaks():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(p):
@@ -95,12 +100,12 @@ def suite_redomap2():
     hbm, tc_peak, src = peaks()
     rows = []
     tuned = {}
-    for dt, tdt, site, ktrain, ks in (("bf16", torch.bfloat16, "redomap2.bf16", 25, (30,)),
-                                      ("f32", torch.float32, "redomap2.f32", 23, (25,))):
-        # P:138 protocol (tune on a smaller constant-work family, test on a
-        # larger one); on B200 k = 20 is launch-bound and L2-resident, so the
-        # training family is k = 25 (bf16) / 23 (f32), testing k = 30 / 25
-        train = mm_shapes(ktrain)
+    for dt, tdt, site, ktrain, ks in (("bf16", torch.bfloat16, "redomap2.bf16", (28, 31), (30,)),
+                                      ("f32", torch.float32, "redomap2.f32", (23, 27), (25,))):
+        # P:138 protocol (tune on other constant-work families than the test
+        # one): training families bracket the test size, as for the sweep --
+        # k = 28 and 31 (bf16) / 23 and 27 (f32), testing k = 30 / 25
+        train = [s for kt in ktrain for s in mm_shapes(kt)]
         need = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data, len(train))
         scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
         a, b, tbl = ifl.tune(site, train, reps=7, cost=1, scratch=scratch)
@@ -123,6 +128,19 @@ def suite_redomap2():
                 r["best_over_auto"] = best / r["auto"]
                 r["flops"] = 2.0 * n * m * p
                 r["bytes"] = (2 if dt == "bf16" else 4) * (n * m + m * p) + 4 * n * p
+                # per-shape roofline: max(bytes / HBM, flops / tensor or FMA peak)
+                fpeak = tc_peak if dt == "bf16" else FMA_TFLOPS
+                r["auto_GBps"] = r["bytes"] / (r["auto"] * 1e-6) / 1e9
+                r["frac_of_8TBps"] = r["auto_GBps"] / NOMINAL_HBM
+                r["frac_of_measured_hbm"] = r["auto_GBps"] / hbm
+                r["roofline_us"] = max(r["bytes"] / (hbm * 1e9), r["flops"] / (fpeak * 1e12)) * 1e6
+                r["frac_of_roofline"] = r["roofline_us"] / r["auto"]
+                # B given as yss [m][p] (b_kmajor = 0), AUTO: read in place by V_FLAT
+                if r["chosen"] == "flat":
+                    Bm = Bt.t().contiguous()
+                    r["auto_rowmajor_B"] = gtime(lambda: ifl.redomap2(A, Bm, b_kmajor=False, out=C, ws=ws)) * 1e3
+                    r["rowmajor_over_kmajor"] = r["auto_rowmajor_B"] / r["auto"]
+                    del Bm
                 rows.append(r)
                 del A, Bt, C
     # dense bf16 square (tensor-core roofline)
@@ -139,8 +157,14 @@ def suite_redomap2():
     line = base_line("map-map-redomap (matmul-shaped) sweep throughput, configs[2] k=30 bf16",
                      round(tot_b / (tot_t * 1e-6) / 1e9, 1), "GB/s",
                      {"workload": "configs[2]: A[2^a][2^(k-2a)] x B[2^(k-2a)][2^a], test k=30 (bf16) / 25 (f32), "
-                                  "tuned on k=25 / 23 (P:138 protocol)", "thresholds": tuned}, dtype="bf16")
+                                  "tuned on k=28+31 / 23+27 (P:138 protocol)", "thresholds": tuned}, dtype="bf16")
     line["min_shape_best_over_auto"] = round(min(r["best_over_auto"] for r in rows), 4)
+    k30 = [r for r in rows if r["dt"] == "bf16" and r["k"] == 30]
+    line["k30_per_shape"] = [{"n": r["n"], "m": r["m"], "chosen": r["chosen"], "auto_us": round(r["auto"], 1),
+                              "GBps": round(r["auto_GBps"]), "frac_of_8TBps": round(r["frac_of_8TBps"], 3),
+                              "frac_of_roofline": round(r["frac_of_roofline"], 3),
+                              "rowmajor_over_kmajor": round(r.get("rowmajor_over_kmajor", float("nan")), 3)}
+                             for r in k30]
     top = sq[8192]
     line["roofline"] = {"bound": "tensor", "kernel": "mm_top_tc_kernel (8192^3 bf16)",
                         "achieved": round(top["TFLOPs"], 1), "peak": tc_peak, "unit": "TFLOP/s",

@@ -1004,8 +1004,8 @@ __global__ void __launch_bounds__(kScanThreads, IFL_JR_MINB) flat_scan_jr_kernel
                 } else {
                     for (int q = jm.a0 + t; q < jm.a1; q += FB) acc_a = combine<OP>(acc_a, apply_map<F>(in[rev ? N - 1 - (base + q) : base + q]));
                 }
-                __syncwarp();
-                if (lane == 0) mbar_arrive_cnt(&empty[sl], 1);  // this warp is done with the slot
+                consumer_sync();  // every consumer warp is done with the slot
+                if (t == 0) mbar_arrive_cnt(&empty[sl], NCW);
                 if (jm.flags & 1) {  // last tile of the range: CTA total, publish
                     T r = warp_reduce<OP>(acc_a);
                     if (lane == 0) s_lbval[w] = r;

@@ -458,11 +458,15 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const 
 // 63 / 32 us vs 96 / 104 us for this FMA-bound engine)
 static bool skinny_ok(int64_t n, int64_t p, bool bf16) { return n * p <= (bf16 ? 256 : kSkinnyMaxOuts); }
 static int skinny_r(int64_t x) { return x >= 8 ? 8 : x >= 4 ? 4 : x >= 2 ? 2 : 1; }
-// k-chunks: one wave of CTAs (one per SM: the pipelines take ~128 KB of
-// shared memory) over all output tiles, >= 2 vector rounds per chunk
+// k-chunks: one wave of CTAs over all output tiles (as many per SM as the
+// pipeline's shared memory allows), >= 2 vector rounds per chunk
 static int64_t skinny_kchunk(int64_t n, int64_t m, int64_t p) {
     const int64_t tiles = ceil_div(n, skinny_r(n)) * ceil_div(p, skinny_r(p));
-    const int64_t want = std::max<int64_t>(1, (int64_t)148 / tiles);
+    // CTAs per SM the pipeline's shared memory allows (K-major words; >= 1, <= 4)
+    const int words = skinny_r(n) + skinny_r(p);
+    const int S = std::min(12, std::max(3, kSkinnyStageBytes / (words * kSkinnyThreads * 8)));
+    const int occ = std::min(4, std::max(1, (200 * 1024) / (S * words * kSkinnyThreads * 8)));
+    const int64_t want = std::max<int64_t>(1, (int64_t)148 * occ / tiles);
     int64_t kc = std::max<int64_t>((int64_t)kSkinnyThreads * 8, ceil_div(m, want));
     return ceil_div(kc, 8) * 8;  // a multiple of every vector width
 }
@@ -576,7 +580,8 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     char* ws = (char*)a.ws;
     if (version == 2 && skinny_ok(a.n, a.p, std::is_same<Tin, __nv_bfloat16>::value) && a.m > 0)
         // V_FLAT, skinny outputs: either B layout, no transposition pass
-        return launch_skinny<Tin>(A, Bt, a.C, (float*)ws, a.n, a.m, a.p, a.b_kmajor != 0, a.stream);
+        // (yss with a single column is the same memory as its transpose)
+        return launch_skinny<Tin>(A, Bt, a.C, (float*)ws, a.n, a.m, a.p, a.b_kmajor != 0 || a.p == 1, a.stream);
     size_t used = 0;
     if (!a.b_kmajor) {  // yss [m][p] -> yss^T [p][m]
         Tin* t = (Tin*)ws;
