@@ -140,15 +140,17 @@ def run_ours(args, rank, world, device):
     tuned = {}
     if not args.no_tune:
         t0 = time.time()
+        # the 4-leaf chain (TOP, MIDDLE, CLUSTER, FLAT; reading R18) per site
         for site in ("segred.b4", "segscan.b4"):
             train = [s for lg in (25, 27) for s in shapes(lg)]
-            scratch_bytes = ifl.lib().ifl_tune_scratch_bytes(site.encode(), np.asarray(train, np.int64).ctypes.data,
+            tsite = site + ".tree"
+            scratch_bytes = ifl.lib().ifl_tune_scratch_bytes(tsite.encode(), np.asarray(train, np.int64).ctypes.data,
                                                              len(train))
             scratch = torch.empty(scratch_bytes, dtype=torch.uint8, device=device)
             scratch.view(-1)[: (scratch_bytes // 4) * 4].view(torch.float32).copy_(
                 gen.generate("F32_UNIT", 4, scratch_bytes // 4, device=device))
-            a, b, tbl = ifl.tune(site, train, reps=7, cost=1, scratch=scratch)
-            tuned[site] = {"t_top": a, "t_intra": b}
+            a, b, tbl = ifl.tune(tsite, train, reps=7, cost=1, scratch=scratch)
+            tuned[site] = {"t_top": a, "t_intra": b, "t_cluster": ifl.get_thresholds(site + ".cl")[0]}
             del scratch
         log(f"[bench] tuned in {time.time() - t0:.1f}s: {tuned}")
         if rank == 0:  # reused by the ncu launch-list pass (--no-tune --thresholds)
@@ -158,7 +160,8 @@ def run_ours(args, rank, world, device):
         ifl.load_thresholds(args.thresholds)
         for site in ("segred.b4", "segscan.b4"):
             a, b = ifl.get_thresholds(site)
-            tuned[site] = {"t_top": a, "t_intra": b, "from": os.path.basename(args.thresholds)}
+            tuned[site] = {"t_top": a, "t_intra": b, "t_cluster": ifl.get_thresholds(site + ".cl")[0],
+                           "from": os.path.basename(args.thresholds)}
 
     # ---- resident inputs: two copies > L2, alternate per step
     xs = [gen.generate("F32_UNIT", 2 + rank * 101, N, device=device),
@@ -260,16 +263,26 @@ def run_ours(args, rank, world, device):
 
     auto_ms = {(k, n): time_call(k, n, m, "auto") for k, n, m in calls}
     per_call_ms = [auto_ms[(k, n)] for k, n, m in calls]
+    VS = ("top", "middle", "cluster", "flat")
+
+    def forced_time(kind, n, m, v):
+        try:
+            return time_call(kind, n, m, v)
+        except ifl.IflError as e:  # V_CLUSTER segscan on rows past its fit: not a runnable version there
+            if e.code != ifl.IFL_ENOTFIT:
+                raise
+            return float("inf")
+
     if args.no_forced:  # launch-list runs: only the contract region
-        forced = {(k, n, v): auto_ms[(k, n)] for k, n, m in calls for v in ("top", "middle", "flat")}
+        forced = {(k, n, v): auto_ms[(k, n)] for k, n, m in calls for v in VS}
     else:
-        forced = {(k, n, v): time_call(k, n, m, v) for k, n, m in calls for v in ("top", "middle", "flat")}
+        forced = {(k, n, v): forced_time(k, n, m, v) for k, n, m in calls for v in VS}
     table = []
     ratios = []
-    fixed_tot = {v: 0.0 for v in ("top", "middle", "flat")}
+    fixed_tot = {v: 0.0 for v in VS}
     auto_tot = 0.0
     for kind, n, m in calls:
-        tv = {v: forced[(kind, n, v)] for v in ("top", "middle", "flat")}
+        tv = {v: forced[(kind, n, v)] for v in VS}
         best = min(tv.values())
         ta = auto_ms[(kind, n)]
         b = bytes_segred(n, m) if kind == "segred" else bytes_segscan(n, m)
@@ -278,7 +291,9 @@ def run_ours(args, rank, world, device):
             fixed_tot[v] += tv[v]
         auto_tot += ta
         table.append({"op": kind, "n": n, "m": m, "chosen": choices[(kind, n)], "auto_us": ta * 1e3,
-                      "top_us": tv["top"] * 1e3, "middle_us": tv["middle"] * 1e3, "flat_us": tv["flat"] * 1e3,
+                      "top_us": tv["top"] * 1e3, "middle_us": tv["middle"] * 1e3,
+                      "cluster_us": tv["cluster"] * 1e3 if tv["cluster"] != float("inf") else None,
+                      "flat_us": tv["flat"] * 1e3,
                       "best_single": min(tv, key=tv.get), "best_over_auto": best / ta,
                       "auto_GBps": b / (ta / 1e3) / 1e9, "frac_of_8TBps": b / (ta / 1e3) / 1e9 / NOMINAL_HBM_GBS})
 
@@ -290,18 +305,18 @@ def run_ours(args, rank, world, device):
         for kind in ("segred", "segscan"):
             ks = [(n, m) for k2, n, m in calls if k2 == kind]
             site = kind + ".b4"
-            pt, pm, tbl = [], [], []
+            par, tbl = [], []
             for (n, m) in ks:
                 c = ifl.select(site, n, m)
-                pt.append(c.par_top)
-                pm.append(c.par_mid)
-                tbl.append([forced[(kind, n, v)] for v in ("top", "middle", "flat")])
-            a, b, _ = ifl.tune_search(pt, pm, tbl, cost=1)
+                par.append([c.par_top, c.par_mid, n * min(m, 8192)])
+                tbl.append([min(forced[(kind, n, v)], 1e30) for v in VS])
+            th, _ = ifl.tune_search_chain(par, tbl, cost=1)
             ratios_k = []
-            for (n, m), ptop, pmid, row in zip(ks, pt, pm, tbl):
-                v = 0 if ptop >= a else (1 if pmid >= b else 2)
+            for pr, row in zip(par, tbl):
+                v = next((q for q in range(3) if pr[q] >= th[q]), 3)
                 ratios_k.append(min(row) / row[v])
-            g3_best[kind] = {"t_top": a, "t_intra": b, "min_shape_best_over_chosen": round(min(ratios_k), 4)}
+            g3_best[kind] = {"t_top": th[0], "t_intra": th[1], "t_cluster": th[2],
+                             "min_shape_best_over_chosen": round(min(ratios_k), 4)}
 
     # ---- dominant kernel roofline (CUDA-event durations on the launch stream)
     groups = {}

@@ -492,49 +492,13 @@ __global__ void __launch_bounds__(NT) segred_cluster_kernel(const T* __restrict_
 static int sm_count();
 
 // V_MIDDLE for rows of >= 8192 elements: a 512-thread CTA per row (the group
-// size V_MIDDLE already uses there), 4 independent 128-bit loads per thread.
+// size V_MIDDLE already uses there; 1024 threads when rows are fewer than two
+// per SM), 4 independent 128-bit loads per thread.
 cudaError_t launch_segred_rows512(const SegArgs& a) {
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
         if (a.n > 0x7fffffffLL) return cudaErrorInvalidValue;
-        // few rows (< 2 per SM): a cluster of C CTAs (512 threads) per row, C a
-        // power of two <= 16 chosen so n*C CTAs fill the GPU (B200: n = 2^5..2^8
-        // rows of 2^18..2^21 elements at 6.4-6.6 TB/s; non-power-of-two C and
-        // 1024-thread CTAs measured slower)
-        const int64_t target = (int64_t)sm_count() * 4;
-        int64_t C = 1;
-        while (C * 2 <= 8 && C * 2 * a.n <= target && C * 2 * 8192 <= a.m) C *= 2;
-        // 16-CTA clusters only while 8-CTA ones leave over half the SMs idle
-        // (measured: 16 rows x 16 CTAs 40.9 us vs x 8 48.1; 32 rows x 16 46.7 vs x 8 40.4)
-        if (C == 8 && 16 * a.n <= (int64_t)sm_count() * 2 && 16 * 8192 <= a.m) C = 16;
-        if (a.n < 2 * sm_count() && C >= 2) {
-            cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3((unsigned)(a.n * C));
-            cfg.blockDim = dim3(kSplitThreads);
-            cfg.stream = a.stream;
-            cudaLaunchAttribute attr[1];
-            attr[0].id = cudaLaunchAttributeClusterDimension;
-            attr[0].val.clusterDim.x = (unsigned)C;
-            attr[0].val.clusterDim.y = 1;
-            attr[0].val.clusterDim.z = 1;
-            cfg.attrs = attr;
-            cfg.numAttrs = 1;
-            // very few rows (<= 4): 16-CTA clusters of 1024-thread CTAs (B200: n = 2 / 4
-            // 145 / 79 us -> 83 / 51 us; n = 8 is faster with 512 threads: 49 vs 60 us)
-            const bool big = C == 16 && a.n * 32 <= (int64_t)sm_count();
-            if (big) cfg.blockDim = dim3(1024);
-            auto kc = big ? segred_cluster_kernel<T, OP, F, 1024> : segred_cluster_kernel<T, OP, F, kSplitThreads>;
-            if (C > 8) cudaFuncSetAttribute(kc, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);  // opt-in
-            cudaError_t e = cudaLaunchKernelEx(&cfg, kc, (const T*)a.in, (T*)a.out, a.m, bits_to<T>(a.ne_bits));
-            if (e != cudaSuccess && C > 8) {  // 16-CTA clusters refused: the portable size
-                (void)cudaGetLastError();
-                attr[0].val.clusterDim.x = 8;
-                cfg.gridDim = dim3((unsigned)(a.n * 8));
-                e = cudaLaunchKernelEx(&cfg, kc, (const T*)a.in, (T*)a.out, a.m, bits_to<T>(a.ne_bits));
-            }
-            return e;
-        }
         if (a.n < 2 * sm_count())
             flat_red_split_kernel<T, OP, F, true, 1024><<<(unsigned)a.n, 1024, 0, a.stream>>>(
                 (const T*)a.in, a.m, 1, (T*)a.out, bits_to<T>(a.ne_bits));
@@ -542,6 +506,181 @@ cudaError_t launch_segred_rows512(const SegArgs& a) {
             flat_red_split_kernel<T, OP, F, true><<<(unsigned)a.n, kSplitThreads, 0, a.stream>>>(
                 (const T*)a.in, a.m, 1, (T*)a.out, bits_to<T>(a.ne_bits));
         return cudaGetLastError();
+    });
+}
+
+// ----------------------------------------------------------------- V_CLUSTER
+// The thread-block cluster as a hardware level between the CTA and the grid
+// (P:346's hierarchy extended): a cluster of C CTAs is the
+// group of one segment, its CTAs combine through distributed shared memory.
+
+// Cluster size for a segred row: a power of two <= 16 so that n*C CTAs fill
+// the GPU with pieces of >= 4096 elements (B200: n = 2^5..2^8 rows of
+// 2^18..2^21 elements at 6.4-6.6 TB/s; 16-CTA clusters only while 8-CTA ones
+// leave over half the SMs idle: 16 rows x 16 CTAs 40.9 us vs x 8 48.1).
+static int64_t cluster_size_red(int64_t n, int64_t m) {
+    const int64_t target = (int64_t)sm_count() * 4;
+    int64_t C = 1;
+    while (C * 2 <= 8 && C * 2 * n <= target && C * 2 * 4096 <= m) C *= 2;
+    if (C == 8 && 16 * n <= (int64_t)sm_count() * 2 && 16 * 4096 <= m) C = 16;
+    return C;
+}
+
+template <typename K, typename... Args>
+static cudaError_t launch_clustered(K kernel, int64_t rows, int64_t C, int threads, size_t smem, cudaStream_t st,
+                                    Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)(rows * C));
+    cfg.blockDim = dim3(threads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = (unsigned)C;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    if (C > 8) cudaFuncSetAttribute(kernel, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);  // opt-in
+    return cudaLaunchKernelEx(&cfg, kernel, args...);
+}
+
+cudaError_t launch_segred_cluster(const SegArgs& a) {
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        int64_t C = cluster_size_red(a.n, a.m);
+        if (a.n * C > 0x7fffffffLL) return cudaErrorInvalidValue;
+        // very few rows (<= 4): 16-CTA clusters of 1024-thread CTAs (B200: n = 2 / 4
+        // 145 / 79 us -> 83 / 51 us; n = 8 is faster with 512 threads: 49 vs 60 us)
+        const bool big = C == 16 && a.n * 32 <= (int64_t)sm_count();
+        auto kc = big ? segred_cluster_kernel<T, OP, F, 1024> : segred_cluster_kernel<T, OP, F, kSplitThreads>;
+        cudaError_t e = launch_clustered(kc, a.n, C, big ? 1024 : kSplitThreads, 0, a.stream, (const T*)a.in,
+                                         (T*)a.out, a.m, bits_to<T>(a.ne_bits));
+        if (e != cudaSuccess && C > 8) {  // 16-CTA clusters refused: the portable size
+            (void)cudaGetLastError();
+            e = launch_clustered(kc, a.n, 8, big ? 1024 : kSplitThreads, 0, a.stream, (const T*)a.in, (T*)a.out, a.m,
+                                 bits_to<T>(a.ne_bits));
+        }
+        return e;
+    });
+}
+
+// segscan on the cluster level: CTA r of a row's cluster holds piece r of the
+// row in shared memory (read once, f applied), reduces it, and after a cluster
+// barrier takes its carry-in = d (+) totals of CTAs 0..r-1 through DSMEM; it
+// then scans its piece from shared memory and stores it -- one read and one
+// write per element.  Each thread scans a contiguous run of the piece (padded
+// layout p + p/32: conflict-light strided runs).  Fit: a piece of at most
+// kClPieceMax elements per CTA, 16 CTAs per cluster at most.
+constexpr int kClThreads = 512;
+constexpr int64_t kClPieceMax = 40960;  // 160 KB of f32 (+ padding) per CTA
+
+__device__ __forceinline__ int clpad(int p) { return p + (p >> 5); }
+
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(kClThreads) segscan_cluster_kernel(const T* in, T* out, int64_t m, T d,
+                                                                     const T* __restrict__ seed, bool rev) {
+    extern __shared__ __align__(16) uint8_t cl_raw[];
+    T* piece = reinterpret_cast<T*>(cl_raw);
+    __shared__ T red[kClThreads / 32];
+    __shared__ T cta_total, s_carry;
+    unsigned rank, csize;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+    asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(csize));
+    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
+    const int64_t row = blockIdx.x / csize;
+    const int64_t len = ceil_div(ceil_div(m, (int64_t)csize), 4) * 4;
+    const int64_t a = std::min(m, (int64_t)rank * len), b = std::min(m, a + len);
+    const int L = (int)(b - a);
+    const T* src = in + row * m;
+    T* dst = out + row * m;
+    for (int p = t; p < L; p += kClThreads) piece[clpad(p)] = apply_map<F>(src[rev ? m - 1 - (a + p) : a + p]);
+    __syncthreads();
+    const int CL = (L + kClThreads - 1) / kClThreads;
+    const int lo = min(L, t * CL), hi = min(L, lo + CL);
+    T s = identity<OP, T>();
+    for (int k = lo; k < hi; ++k) s = combine<OP>(s, piece[clpad(k)]);
+    // CTA exclusive scan of the thread sums
+    T inc = s;
+#pragma unroll
+    for (int off = 1; off < 32; off <<= 1) {
+        const T o = __shfl_up_sync(0xffffffffu, inc, off);
+        if (lane >= off) inc = combine<OP>(o, inc);
+    }
+    if (lane == 31) red[w] = inc;
+    T ex = __shfl_up_sync(0xffffffffu, inc, 1);
+    if (lane == 0) ex = identity<OP, T>();
+    __syncthreads();
+    T before = identity<OP, T>(), tot = identity<OP, T>();
+#pragma unroll
+    for (int q = 0; q < kClThreads / 32; ++q) {
+        if (q < w) before = combine<OP>(before, red[q]);
+        tot = combine<OP>(tot, red[q]);
+    }
+    ex = combine<OP>(before, ex);
+    if (t == 0) cta_total = tot;
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+    if (t == 0) {
+        T c = seed ? seed[row] : d;
+        const uint32_t local = (uint32_t)__cvta_generic_to_shared(&cta_total);
+        for (unsigned q = 0; q < rank; ++q) {
+            uint32_t remote, bits;
+            asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(remote) : "r"(local), "r"(q));
+            asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(bits) : "r"(remote) : "memory");
+            c = combine<OP>(c, from_bits<T>(bits));
+        }
+        s_carry = c;
+    }
+    __syncthreads();
+    T run = combine<OP>(s_carry, ex);
+    for (int k = lo; k < hi; ++k) {
+        run = combine<OP>(run, piece[clpad(k)]);
+        piece[clpad(k)] = run;
+    }
+    __syncthreads();
+    for (int p = t; p < L; p += kClThreads) dst[rev ? m - 1 - (a + p) : a + p] = piece[clpad(p)];
+    // keep every CTA's shared memory alive until the higher ranks have read its total
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+// Cluster size for a segscan row: the smallest power of two whose pieces fit,
+// grown (<= 16) while the clusters leave SMs idle and pieces stay >= 2048.
+// 0 = does not fit (m > 16 * kClPieceMax).
+int64_t cluster_size_scan(int64_t n, int64_t m) {
+    int64_t C = 1;
+    while (C <= 16 && C * kClPieceMax < m) C *= 2;
+    if (C > 16) return 0;
+    while (C * 2 <= 16 && n * C < 2 * (int64_t)sm_count() && m / (C * 2) >= 2048) C *= 2;
+    return C;
+}
+
+cudaError_t launch_segscan_cluster(const SegArgs& a) {
+    const int64_t C = cluster_size_scan(a.n, a.m);
+    if (C == 0) return cudaErrorNotSupported;
+    if (a.n * C > 0x7fffffffLL) return cudaErrorInvalidValue;
+    return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
+        using T = decltype(tt);
+        constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
+        const int64_t len = ceil_div(ceil_div(a.m, C), 4) * 4;
+        const size_t smem = (size_t)(len + len / 32 + 1) * sizeof(T);
+        auto k = segscan_cluster_kernel<T, OP, F>;
+        static bool attr = false;
+        if (!attr) {
+            cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)((kClPieceMax + kClPieceMax / 32 + 1) * sizeof(T)));
+            attr = true;
+        }
+        cudaError_t e = launch_clustered(k, a.n, C, kClThreads, smem, a.stream, (const T*)a.in, (T*)a.out, a.m,
+                                         bits_to<T>(a.ne_bits), (const T*)a.seed, a.rev);
+        if (e != cudaSuccess && C > 8) {  // 16-CTA clusters refused: this row does not fit 8 pieces
+            (void)cudaGetLastError();
+            if (8 * kClPieceMax < a.m) return cudaErrorNotSupported;
+            const int64_t len8 = ceil_div(ceil_div(a.m, (int64_t)8), 4) * 4;
+            e = launch_clustered(k, a.n, 8, kClThreads, (size_t)(len8 + len8 / 32 + 1) * sizeof(T), a.stream,
+                                 (const T*)a.in, (T*)a.out, a.m, bits_to<T>(a.ne_bits), (const T*)a.seed, a.rev);
+        }
+        return e;
     });
 }
 

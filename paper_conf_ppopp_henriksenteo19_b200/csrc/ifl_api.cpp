@@ -40,7 +40,8 @@ constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE ke
 
 const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
                               "colred.b4", "colscan.b4", "segred.irr", "segscan.irr", "segarg.b4",
-                              "redomap2.f32.row", "redomap2.bf16.row", "segred2.b4"};
+                              "redomap2.f32.row", "redomap2.bf16.row", "segred2.b4", "segred.b4.cl",
+                              "segscan.b4.cl"};
 
 struct Table {
     std::mutex mu;
@@ -49,9 +50,9 @@ struct Table {
     Table() { reset(); }
     void reset() {
         thr.clear();
-        for (const char* s : kSites)  // the matmul row level is off until tuned (reading R17)
-            thr[s] = strstr(s, ".row") ? std::make_pair(INT64_MAX, INT64_MAX)
-                                       : std::make_pair(kDefaultThreshold, kDefaultThreshold);
+        for (const char* s : kSites)  // the matmul row level and the cluster level are off until tuned (R17, R18)
+            thr[s] = (strstr(s, ".row") || strstr(s, ".cl")) ? std::make_pair(INT64_MAX, INT64_MAX)
+                                                               : std::make_pair(kDefaultThreshold, kDefaultThreshold);
         par_mode = 1;
     }
 };
@@ -115,6 +116,28 @@ int select_version(const char* site, int64_t n, int64_t m, int64_t p, bool mid_f
     return v;
 }
 
+// The cluster level of the segred / segscan guard chain (reading R18):
+// after TOP and MIDDLE fail, Par_cl = n * min(m, 8192) (R3's utilized
+// parallelism: a cluster of up to 16 x 512 threads per segment) >= t_cl picks
+// V_CLUSTER when it fits, else V_FLAT.
+void cluster_guard(bool scan, int64_t n, int64_t m, ifl_choice* c) {
+    if (c->version != IFL_V_FLAT) return;
+    int64_t tcl, unused;
+    int mode;
+    {
+        Table& T = table();
+        std::lock_guard<std::mutex> g(T.mu);
+        auto it = T.thr.find(scan ? "segscan.b4.cl" : "segred.b4.cl");
+        tcl = it->second.first;
+        unused = it->second.second;
+        mode = T.par_mode;
+    }
+    (void)unused;
+    const int64_t pcl = mode == 1 ? sat_mul(n, std::min(m, ifl::kClusterBmax)) : sat_mul(n, m);
+    const bool fits = !scan || ifl::cluster_size_scan(n, m) != 0;
+    if (pcl >= tcl && fits) c->version = IFL_V_CLUSTER;
+}
+
 // Irregular segments: G3 with the inspector's imbalance measure.
 // Par_top = total / max_len (longest-segment equivalents: what a thread per
 // segment really runs in parallel), or n when max_len is unknown (0);
@@ -164,7 +187,7 @@ bool overlap(const void* a, size_t an, const void* b, size_t bn) {
 }
 
 int validate_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int dt, int op, int f, int version,
-                 const char* what) {
+                 const char* what, bool cluster_ok = false) {
     if (n < 0 || m < 0) return fail(IFL_EINVAL, "%s: negative size n=%lld m=%lld", what, (long long)n, (long long)m);
     if (mul_overflows(n, m) || mul_overflows(n * m, 4))
         return fail(IFL_EINVAL, "%s: n*m overflows int64", what);
@@ -172,7 +195,8 @@ int validate_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, int
     if (op < IFL_SUM || op > IFL_XOR) return fail(IFL_EINVAL, "%s: bad op %d", what, op);
     if (dt == IFL_F32 && op > IFL_MAX) return fail(IFL_EUNSUPPORTED, "%s: bitwise op on f32", what);
     if (f < IFL_F_ID || f > IFL_F_ABS) return fail(IFL_EINVAL, "%s: bad map %d", what, f);
-    if (version < IFL_AUTO || version > IFL_V_FLAT) return fail(IFL_EINVAL, "%s: bad version %d", what, version);
+    if ((version < IFL_AUTO || version > IFL_V_FLAT) && !(cluster_ok && version == IFL_V_CLUSTER))
+        return fail(IFL_EINVAL, "%s: bad version %d", what, version);
     if (n > 0 && m > 0 && in == nullptr) return fail(IFL_EINVAL, "%s: in is NULL", what);
     if ((scan ? n * m : n) > 0 && out == nullptr) return fail(IFL_EINVAL, "%s: out is NULL", what);
     if (((uintptr_t)in % 4) || ((uintptr_t)out % 4)) return fail(IFL_EINVAL, "%s: pointers not element-aligned", what);
@@ -220,6 +244,13 @@ int ifl_select(const char* site, int64_t n, int64_t m, int64_t p, ifl_choice* ch
         return IFL_OK;
     }
     if (strcmp(site, "tridag") == 0) fits = ifl::tridag_mid_fits(m);
+    if (strcmp(site, "segred.b4") == 0 || strcmp(site, "segscan.b4") == 0) {  // the 4-leaf chain (R18)
+        ifl_choice c;
+        select_version(site, n, m, p, true, &c);
+        cluster_guard(strncmp(site, "segscan", 7) == 0, n, m, &c);
+        if (choice) *choice = c;
+        return IFL_OK;
+    }
     return select_version(site, n, m, p, fits, choice) >= 0 ? IFL_OK : IFL_EINVAL;
 }
 
@@ -331,7 +362,7 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
                    const void* ne, int version, void* ws, size_t ws_bytes, void* stream, ifl_choice* choice,
                    const void* seed = nullptr, bool rev = false) {
     const char* what = seed ? "ifl_segscan_seeded" : scan ? "ifl_segscan" : "ifl_segred";
-    int rc = validate_seg(scan, in, out, n, m, dt, op, f, version, what);
+    int rc = validate_seg(scan, in, out, n, m, dt, op, f, version, what, true);
     if (rc) return rc;
     const size_t ob = (size_t)(scan ? n * m : n) * 4, ib = (size_t)(n * m) * 4;
     if (scan) {
@@ -346,8 +377,11 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
     const char* site = scan ? "segscan.b4" : "segred.b4";
     ifl_choice c;
     const int v = select_version(site, n, m, 0, true, &c);
+    cluster_guard(scan, n, m, &c);
     if (version != IFL_AUTO) c.version = version;
     if (choice) *choice = c;
+    if (c.version == IFL_V_CLUSTER && scan && n * m > 0 && ifl::cluster_size_scan(n, m) == 0)
+        return fail(IFL_ENOTFIT, "%s: V_CLUSTER keeps a row in 16 shared-memory pieces (m <= 655360)", what);
     if (n == 0) return IFL_OK;
     if (m == 0) {  // reduce of an empty list is d; scan of it is empty
         if (scan) return IFL_OK;
@@ -359,6 +393,7 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
     switch (c.version) {
     case IFL_V_TOP: e = scan ? ifl::launch_segscan_top(a) : ifl::launch_segred_top(a); break;
     case IFL_V_MIDDLE: e = scan ? ifl::launch_segscan_mid(a) : ifl::launch_segred_mid(a); break;
+    case IFL_V_CLUSTER: e = scan ? ifl::launch_segscan_cluster(a) : ifl::launch_segred_cluster(a); break;
     default: {
         const size_t need = ifl::flat_ws_bytes(n * m);
         if (!ws || ws_bytes < need)

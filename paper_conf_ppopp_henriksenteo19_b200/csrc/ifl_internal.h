@@ -37,6 +37,11 @@ cudaError_t launch_segscan_top(const SegArgs& a);
 cudaError_t launch_segscan_mid(const SegArgs& a);
 cudaError_t launch_flat(const SegArgs& a, bool scan);
 cudaError_t launch_segred_rows512(const SegArgs& a);  // V_MIDDLE segred, m >= 8192 (flat.cu)
+// V_CLUSTER (flat.cu): a thread-block cluster per segment, DSMEM combine
+cudaError_t launch_segred_cluster(const SegArgs& a);
+cudaError_t launch_segscan_cluster(const SegArgs& a);  // cudaErrorNotSupported when a row does not fit
+int64_t cluster_size_scan(int64_t n, int64_t m);       // 0: a row does not fit 16 pieces
+constexpr int64_t kClusterBmax = 8192;                 // Par_cl = n * min(m, 8192) (reading R18)
 cudaError_t launch_fill(void* out, int64_t count, uint32_t bits, cudaStream_t s);
 
 // Group size (threads per segment) used by the V_MIDDLE kernels.

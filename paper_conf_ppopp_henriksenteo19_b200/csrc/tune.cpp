@@ -197,7 +197,8 @@ extern "C" int ifl_tune_search_chain(const int64_t* par, const double* cost_tabl
 
 namespace {
 
-enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_COLRED, K_COLSCAN, K_TREE_F32, K_TREE_BF16, K_BAD };
+enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_COLRED, K_COLSCAN, K_TREE_F32, K_TREE_BF16,
+            K_SEGRED_CL, K_SEGSCAN_CL, K_BAD };
 
 Kind kind_of(const char* site) {
     if (!site) return K_BAD;
@@ -211,13 +212,26 @@ Kind kind_of(const char* site) {
     if (!strcmp(site, "colscan.b4")) return K_COLSCAN;
     if (!strcmp(site, "redomap2.f32.tree")) return K_TREE_F32;
     if (!strcmp(site, "redomap2.bf16.tree")) return K_TREE_BF16;
+    if (!strcmp(site, "segred.b4.tree")) return K_SEGRED_CL;
+    if (!strcmp(site, "segscan.b4.tree")) return K_SEGSCAN_CL;
     return K_BAD;
 }
 
-Kind mm_of(Kind k) { return k == K_TREE_F32 ? K_MM_F32 : k == K_TREE_BF16 ? K_MM_BF16 : k; }
+// the 4-leaf segred / segscan chain (TOP, MIDDLE, CLUSTER, FLAT; reading R18)
+// runs the plain site's calls with one more forced version
+Kind mm_of(Kind k) {
+    return k == K_TREE_F32 ? K_MM_F32 : k == K_TREE_BF16 ? K_MM_BF16 : k == K_SEGRED_CL ? K_SEGRED
+         : k == K_SEGSCAN_CL ? K_SEGSCAN : k;
+}
 bool is_tree(Kind k) { return k == K_TREE_F32 || k == K_TREE_BF16; }
+bool is_cl(Kind k) { return k == K_SEGRED_CL || k == K_SEGSCAN_CL; }
 
-int arity(Kind k) { return (k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN) ? 2 : k == K_LVC ? 4 : 3; }
+int arity(Kind k) {
+    return (k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN || k == K_SEGRED_CL || k == K_SEGSCAN_CL)
+               ? 2
+           : k == K_LVC ? 4
+                        : 3;
+}
 
 size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 int64_t ceil_div_i64(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -412,11 +426,12 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     if (cudaMemsetAsync(flush, 0, kFlushBytes, st) != cudaSuccess) return IFL_ECUDA;  // valid floats, once
     // the matmul tree sites time five leaves (ROW_TOP, ROW_MIDDLE, TOP, MIDDLE,
     // FLAT) and search a chain of four guards; every other site three versions
-    const bool tree = is_tree(k);
-    const int NV = tree ? 5 : 3;
+    const bool tree = is_tree(k), cl = is_cl(k);
+    const int NV = tree ? 5 : cl ? 4 : 3;
     static const int kTreeVersion[5] = {IFL_V_ROW_TOP, IFL_V_ROW_MIDDLE, IFL_V_TOP, IFL_V_MIDDLE, IFL_V_FLAT};
+    static const int kClVersion[4] = {IFL_V_TOP, IFL_V_MIDDLE, IFL_V_CLUSTER, IFL_V_FLAT};
     std::vector<double> table(nshapes * NV, std::numeric_limits<double>::infinity());
-    std::vector<int64_t> ptop(nshapes), pmid(nshapes), pchain(tree ? nshapes * 4 : 0);
+    std::vector<int64_t> ptop(nshapes), pmid(nshapes), pchain(tree ? nshapes * 4 : cl ? nshapes * 3 : 0);
     cudaEvent_t e0, e1;
     if (cudaEventCreate(&e0) != cudaSuccess || cudaEventCreate(&e1) != cudaSuccess) return IFL_ECUDA;
     cudaStream_t cs = nullptr;  // capture stream (the caller's may be the uncapturable legacy stream)
@@ -428,7 +443,9 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     for (int i = 0; i < nshapes && rc == IFL_OK; ++i) {
         const int64_t* s = shapes + i * ar;
         ifl_choice c;
-        const char* psite = tree ? (k == K_TREE_F32 ? "redomap2.f32" : "redomap2.bf16") : site;
+        const char* psite = tree ? (k == K_TREE_F32 ? "redomap2.f32" : "redomap2.bf16")
+                          : cl ? (k == K_SEGRED_CL ? "segred.b4" : "segscan.b4")
+                               : site;
         ifl_select(psite, s[0], s[1], ar == 3 && k != K_TRIDAG ? s[2] : 0, &c);
         if (k == K_LVC) c.par_mid = 0;  // one guard: Par = numS
         ptop[i] = c.par_top;
@@ -438,6 +455,11 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
             pchain[i * 4 + 1] = s[0] * std::min<int64_t>(s[2], 8) * 32;
             pchain[i * 4 + 2] = c.par_top;
             pchain[i * 4 + 3] = c.par_mid;
+        }
+        if (cl) {  // Par of the three guards: n, n*min(m,1024), n*min(m,8192) (par mode 0: n*m)
+            pchain[i * 3 + 0] = c.par_top;
+            pchain[i * 3 + 1] = c.par_mid;
+            pchain[i * 3 + 2] = ifl_get_par_mode() == 1 ? s[0] * std::min<int64_t>(s[1], ifl::kClusterBmax) : s[0] * s[1];
         }
         // zero this shape's workspace (the tail of its scratch layout); the
         // input region keeps the caller's data
@@ -452,7 +474,7 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         double best_ms = std::numeric_limits<double>::infinity();
         for (int vv = 0; vv < NV; ++vv) {
             const int slot = NV - 1 - vv;                     // table column
-            const int v = tree ? kTreeVersion[slot] : slot;  // version run
+            const int v = tree ? kTreeVersion[slot] : cl ? kClVersion[slot] : slot;  // version run
             if (hopeless(k, s, v)) continue;  // stays +inf: unavailable to the search
             flush_l2(flush, st);
             cudaEventRecord(e0, st);
@@ -519,6 +541,18 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         rc = ifl_set_thresholds(bf ? "redomap2.bf16.row" : "redomap2.f32.row", th[0], th[1]);
         if (rc != IFL_OK) return rc;
         return ifl_set_thresholds(bf ? "redomap2.bf16" : "redomap2.f32", th[2], th[3]);
+    }
+    if (cl) {
+        int64_t th[3];
+        int np;
+        rc = ifl_tune_search_chain(pchain.data(), table.data(), nshapes, 3, cost, th, &np);
+        if (rc != IFL_OK) return rc;
+        if (t_top) *t_top = th[0];
+        if (t_intra) *t_intra = th[1];
+        const bool sc = k == K_SEGSCAN_CL;
+        rc = ifl_set_thresholds(sc ? "segscan.b4.cl" : "segred.b4.cl", th[2], th[2]);
+        if (rc != IFL_OK) return rc;
+        return ifl_set_thresholds(sc ? "segscan.b4" : "segred.b4", th[0], th[1]);
     }
     int64_t a, b;
     int np;

@@ -107,10 +107,29 @@ def test_redomap2_tridag_validation(L):
 def test_default_thresholds_are_2_pow_15(L):
     ifl.reset_thresholds()
     for s in ifl.SITES:
-        if s.endswith(".row"):  # the matmul row level is off until tuned (reading R17)
+        if s.endswith((".row", ".cl")):  # the matmul row level / the cluster level are off until tuned (R17, R18)
             assert ifl.get_thresholds(s) == (2**63 - 1, 2**63 - 1)
         else:
             assert ifl.get_thresholds(s) == (2**15, 2**15)
+
+
+@pytest.mark.parametrize("site", ["segred.b4", "segscan.b4"])
+def test_cluster_level_guard_chain(L, site):
+    """Reading R18: TOP -> MIDDLE -> CLUSTER -> FLAT; Par_cl = n*min(m, 8192);
+    the cluster level is off by default (the paper's three versions), and a
+    segscan row that does not fit 16 shared-memory pieces never takes it."""
+    ifl.reset_thresholds()
+    assert ifl.select(site, 4, 1 << 20).version == "flat"               # default: no cluster leaf
+    ifl.set_thresholds(site, 1 << 20, 1 << 30)                           # TOP / MIDDLE guards fail below
+    ifl.set_thresholds(site + ".cl", 1 << 15, 0)
+    assert ifl.select(site, 4, 1 << 19).version == "cluster"             # Par_cl = 4 * 8192 >= 2^15
+    assert ifl.select(site, 3, 1 << 19).version == "flat"                # 3 * 8192 < 2^15
+    assert ifl.select(site, 64, 100).version == "flat"                   # 64 * 100 < 2^15
+    assert ifl.select(site, 1 << 20, 4).version == "top"                 # the outer guard still first
+    if site == "segscan.b4":
+        assert ifl.select(site, 4, 16 * 40960 + 4).version == "flat"     # does not fit: never CLUSTER
+        assert ifl.select(site, 4, 16 * 40960).version == "cluster"
+    ifl.reset_thresholds()
 
 
 @pytest.mark.parametrize("site", ["segred.b4", "segscan.b4"])

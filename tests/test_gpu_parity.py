@@ -13,7 +13,7 @@ import ifl_inputs as gen
 
 pytestmark = pytest.mark.gpu
 
-VERS = ["top", "middle", "flat", "auto"]
+VERS = ["top", "middle", "cluster", "flat", "auto"]
 TINY = [0, 1, 2, 3, 5, 8, 31, 32, 33, 127, 1024, 4097]
 
 
@@ -159,6 +159,8 @@ def test_f32_exact_all_versions_bitwise(ifl, orc, scan):
         x, xd = make("F32_EXACT", 3, n, m)
         want = (orc.segscan if scan else orc.segred)(x.numpy(), "sum")
         for v in VERS:
+            if v == "cluster" and scan and m > 16 * 40960:
+                continue  # a cluster-per-row scan does not fit rows this long (IFL_ENOTFIT, test_cluster_level)
             got = fn(xd, "sum", "id", version=v).cpu().numpy()
             np.testing.assert_array_equal(got, want.astype(np.float32), err_msg=v)
 
@@ -305,3 +307,31 @@ def test_reverse_scan(ifl, orc, version, dt):
                 np.testing.assert_array_equal(g.cpu().numpy(), want)
             else:
                 assert (np.abs(g.cpu().numpy() - want[0]) <= 1e-5 * want[1]).all()
+
+
+def test_cluster_level(ifl, orc):
+    """V_CLUSTER (reading R18): cluster sizes 1..16 across row lengths, a
+    segscan row at the fit limit and one past it (IFL_ENOTFIT), and AUTO
+    taking the cluster leaf once its threshold is set."""
+    for (n, m) in [(1, 16 * 40960), (3, 300007), (8, 1 << 20), (40, 70000), (700, 5000)]:
+        for dt in ("i32", "f32"):
+            x, xd = gen_for("sum", dt, 31, n, m)
+            assert_parity(orc, x, ifl.segred(xd, "sum", "sq", version="cluster"), False, "sum", "sq", None, dt)
+            assert_parity(orc, x, ifl.segscan(xd, "sum", "sq", version="cluster"), True, "sum", "sq", None, dt)
+            got = ifl.segscan(xd, "max", version="cluster", reverse=True)
+            want = orc.segscan(x.numpy(), "max", reverse=True)
+            np.testing.assert_array_equal(got.cpu().numpy(), want.astype(got.cpu().numpy().dtype))
+    x, xd = gen_for("sum", "i32", 32, 2, 16 * 40960 + 4)
+    with pytest.raises(ifl.IflError) as e:
+        ifl.segscan(xd, version="cluster")
+    assert e.value.code == ifl.IFL_ENOTFIT
+    assert_parity(orc, x, ifl.segred(xd, "sum", version="cluster"), False, "sum", "id", None, "i32")
+    try:
+        ifl.set_thresholds("segscan.b4", 1 << 40, 1 << 40)
+        ifl.set_thresholds("segscan.b4.cl", 1, 1)
+        x, xd = gen_for("sum", "f32", 33, 16, 100000)
+        got, ch = ifl.segscan(xd, return_choice=True)
+        assert ch.version == "cluster"
+        assert_parity(orc, x, got, True, "sum", "id", None, "f32")
+    finally:
+        ifl.reset_thresholds()

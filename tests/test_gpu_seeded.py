@@ -11,7 +11,7 @@ import ifl_inputs as gen
 
 pytestmark = pytest.mark.gpu
 
-VERS = ["top", "middle", "flat", "auto"]
+VERS = ["top", "middle", "cluster", "flat", "auto"]
 SHAPES = [(7, 1), (9, 2), (13, 4), (45, 8), (70, 16), (33, 32), (50, 33), (300, 100), (3, 7000), (2, 30001),
           (1, 200000), (4000, 37)]
 
