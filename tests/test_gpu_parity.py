@@ -317,6 +317,8 @@ def test_cluster_level(ifl, orc):
         for dt in ("i32", "f32"):
             x, xd = gen_for("sum", dt, 31, n, m)
             assert_parity(orc, x, ifl.segred(xd, "sum", "sq", version="cluster"), False, "sum", "sq", None, dt)
+            if m > 16 * 40960:
+                continue  # segred only: a cluster-per-row scan keeps the row in shared memory
             assert_parity(orc, x, ifl.segscan(xd, "sum", "sq", version="cluster"), True, "sum", "sq", None, dt)
             got = ifl.segscan(xd, "max", version="cluster", reverse=True)
             want = orc.segscan(x.numpy(), "max", reverse=True)
