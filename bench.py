@@ -140,9 +140,14 @@ def run_ours(args, rank, world, device):
     tuned = {}
     if not args.no_tune:
         t0 = time.time()
-        # the 4-leaf chain (TOP, MIDDLE, CLUSTER, FLAT; reading R18) per site
+        # V_MIDDLE's group size first (the tuned tile/group-size dimension, reading
+        # R19; shapes whose rows a group can hold), then the 4-leaf chain (TOP,
+        # MIDDLE, CLUSTER, FLAT; reading R18) per site
         for site in ("segred.b4", "segscan.b4"):
             train = [s for lg in (25, 27) for s in shapes(lg)]
+            gtrain = [s for s in train if s[1] <= 8192]
+            g, _, _ = ifl.tune(site + ".midg", gtrain, reps=7, cost=1)
+            tuned[site + ".midg"] = {"group_shift": g - 8}
             tsite = site + ".tree"
             scratch_bytes = ifl.lib().ifl_tune_scratch_bytes(tsite.encode(), np.asarray(train, np.int64).ctypes.data,
                                                              len(train))
@@ -161,6 +166,7 @@ def run_ours(args, rank, world, device):
         for site in ("segred.b4", "segscan.b4"):
             a, b = ifl.get_thresholds(site)
             tuned[site] = {"t_top": a, "t_intra": b, "t_cluster": ifl.get_thresholds(site + ".cl")[0],
+                           "group_shift": ifl.get_thresholds(site + ".midg")[0] - 8,
                            "from": os.path.basename(args.thresholds)}
 
     # ---- resident inputs: two copies > L2, alternate per step

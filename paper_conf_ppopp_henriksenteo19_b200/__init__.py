@@ -32,7 +32,7 @@ VERSIONS = {"auto": -1, "top": 0, "middle": 1, "flat": 2, "outer": 3, "row_top":
 VERSION_NAMES = {v: k for k, v in VERSIONS.items()}
 SITES = ("segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc", "colred.b4", "colscan.b4",
          "segred.irr", "segscan.irr", "segarg.b4", "redomap2.f32.row", "redomap2.bf16.row",
-         "segred2.b4", "segred.b4.cl", "segscan.b4.cl")
+         "segred2.b4", "segred.b4.cl", "segscan.b4.cl", "segred.b4.midg", "segscan.b4.midg")
 
 _TORCH_DT = {torch.int32: "i32", torch.float32: "f32", torch.bfloat16: "bf16"}
 
@@ -518,7 +518,7 @@ def tune(site: str, shapes, reps: int = 5, cost: int = 0, scratch: torch.Tensor 
         scratch = torch.zeros(need, dtype=torch.uint8, device="cuda")
     if sh.ndim != 2 or sh.shape[1] != (2 if site.startswith(("seg", "col")) else 4 if site == "lvc" else 3):
         raise ValueError(f"{site}: shapes must be tuples of the site's arity")
-    nv = (5 if site.startswith("redomap2") else 4) if site.endswith(".tree") else 3
+    nv = (5 if site.startswith("redomap2") else 4) if site.endswith(".tree") else 5 if site.endswith(".midg") else 3
     tbl = np.zeros(ns * nv, np.float64)
     a, b = ctypes.c_int64(), ctypes.c_int64()
     _check(lib().ifl_tune(_b(site), sh.ctypes.data, ns, reps, cost, scratch.data_ptr(), scratch.numel(),

@@ -41,7 +41,10 @@ constexpr int64_t kBmax = 1024;                  // largest CTA of a V_MIDDLE ke
 const char* const kSites[] = {"segred.b4", "segscan.b4", "redomap2.f32", "redomap2.bf16", "tridag", "lvc",
                               "colred.b4", "colscan.b4", "segred.irr", "segscan.irr", "segarg.b4",
                               "redomap2.f32.row", "redomap2.bf16.row", "segred2.b4", "segred.b4.cl",
-                              "segscan.b4.cl"};
+                              "segscan.b4.cl", "segred.b4.midg", "segscan.b4.midg"};
+// ".midg" sites hold V_MIDDLE's group-size exponent, biased: t_top = 8 + shift
+// (group size x 2^shift, shift in [-3, 3]; reading R19)
+constexpr int64_t kMidgBias = 8;
 
 struct Table {
     std::mutex mu;
@@ -51,7 +54,8 @@ struct Table {
     void reset() {
         thr.clear();
         for (const char* s : kSites)  // the matmul row level and the cluster level are off until tuned (R17, R18)
-            thr[s] = (strstr(s, ".row") || strstr(s, ".cl")) ? std::make_pair(INT64_MAX, INT64_MAX)
+            thr[s] = strstr(s, ".midg")                        ? std::make_pair(kMidgBias, (int64_t)0)
+                     : (strstr(s, ".row") || strstr(s, ".cl")) ? std::make_pair(INT64_MAX, INT64_MAX)
                                                                : std::make_pair(kDefaultThreshold, kDefaultThreshold);
         par_mode = 1;
     }
@@ -389,6 +393,11 @@ static int run_seg(bool scan, const void* in, void* out, int64_t n, int64_t m, i
     }
     (void)v;
     ifl::SegArgs a{in, out, n, m, dt, op, f, bits, ws, ws_bytes, (cudaStream_t)stream, seed, rev};
+    {
+        int64_t g, unused;
+        ifl_get_thresholds(scan ? "segscan.b4.midg" : "segred.b4.midg", &g, &unused);
+        a.gshift = (int)std::max<int64_t>(-3, std::min<int64_t>(3, g - kMidgBias));
+    }
     cudaError_t e;
     switch (c.version) {
     case IFL_V_TOP: e = scan ? ifl::launch_segscan_top(a) : ifl::launch_segred_top(a); break;

@@ -21,6 +21,7 @@ struct SegArgs {
     cudaStream_t stream;
     const void* seed = nullptr;  // segscan: per-row d (device [n]) or NULL = ne_bits for every row
     bool rev = false;            // segscan: reversed scan (row read from its last element)
+    int gshift = 0;              // V_MIDDLE group size x 2^gshift (the tuned group-size dimension, R19)
 };
 
 // Flat engine tile geometry (flat.cu).  ws layout: 256-byte header then one

@@ -13,6 +13,8 @@
 //            tree -- the level-0 reduction of P:346-358.
 #include <string.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 #include "dispatch.cuh"
 #include "ifl_internal.h"
@@ -482,7 +484,8 @@ __global__ void __launch_bounds__(512) segred_mid_vec_kernel(const T* __restrict
 
 cudaError_t launch_segred_mid(const SegArgs& a) {
     if (a.m >= 8192) return launch_segred_rows512(a);  // one 512-thread group per row (flat.cu)
-    const int G = mid_group_size(a.m);
+    const int G0 = mid_group_size(a.m);
+    const int G = std::max(1, std::min(IFL_MID_GMAX, a.gshift >= 0 ? G0 << a.gshift : G0 >> -a.gshift));
     const int B = G > 256 ? G : 256;
     const int64_t grid = ceil_div(a.n, B / G);
     if (a.m > 0 && a.m % 4 == 0 && ((uintptr_t)a.in & 15u) == 0 && a.m <= 16 * (int64_t)G)

@@ -12,6 +12,8 @@
 //            round total to the next round.
 #include <string.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 #include "dispatch.cuh"
 #include "ifl_internal.h"
@@ -570,7 +572,8 @@ cudaError_t launch_segscan_mid(const SegArgs& a) {
     return dispatch_all(a.dt, a.op, a.f, [&](auto tt, auto opc, auto fc) -> cudaError_t {
         using T = decltype(tt);
         constexpr int OP = decltype(opc)::value, F = decltype(fc)::value;
-        const int G = midscan_group_size(a.m);
+        const int G0 = midscan_group_size(a.m);
+        const int G = std::max(1, std::min(IFL_MIDSCAN_GMAX, a.gshift >= 0 ? G0 << a.gshift : G0 >> -a.gshift));
         const int B = G > 256 ? G : 256;
         const bool vec = !a.rev && ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0) && (a.m % 4 == 0);
         const int64_t grid = ceil_div(a.n, B / G);

@@ -198,7 +198,7 @@ extern "C" int ifl_tune_search_chain(const int64_t* par, const double* cost_tabl
 namespace {
 
 enum Kind { K_SEGRED, K_SEGSCAN, K_MM_F32, K_MM_BF16, K_TRIDAG, K_LVC, K_COLRED, K_COLSCAN, K_TREE_F32, K_TREE_BF16,
-            K_SEGRED_CL, K_SEGSCAN_CL, K_BAD };
+            K_SEGRED_CL, K_SEGSCAN_CL, K_SEGRED_MIDG, K_SEGSCAN_MIDG, K_BAD };
 
 Kind kind_of(const char* site) {
     if (!site) return K_BAD;
@@ -214,20 +214,24 @@ Kind kind_of(const char* site) {
     if (!strcmp(site, "redomap2.bf16.tree")) return K_TREE_BF16;
     if (!strcmp(site, "segred.b4.tree")) return K_SEGRED_CL;
     if (!strcmp(site, "segscan.b4.tree")) return K_SEGSCAN_CL;
+    if (!strcmp(site, "segred.b4.midg")) return K_SEGRED_MIDG;
+    if (!strcmp(site, "segscan.b4.midg")) return K_SEGSCAN_MIDG;
     return K_BAD;
 }
 
 // the 4-leaf segred / segscan chain (TOP, MIDDLE, CLUSTER, FLAT; reading R18)
 // runs the plain site's calls with one more forced version
 Kind mm_of(Kind k) {
-    return k == K_TREE_F32 ? K_MM_F32 : k == K_TREE_BF16 ? K_MM_BF16 : k == K_SEGRED_CL ? K_SEGRED
-         : k == K_SEGSCAN_CL ? K_SEGSCAN : k;
+    return k == K_TREE_F32 ? K_MM_F32 : k == K_TREE_BF16 ? K_MM_BF16 : (k == K_SEGRED_CL || k == K_SEGRED_MIDG) ? K_SEGRED
+         : (k == K_SEGSCAN_CL || k == K_SEGSCAN_MIDG) ? K_SEGSCAN : k;
 }
+bool is_midg(Kind k) { return k == K_SEGRED_MIDG || k == K_SEGSCAN_MIDG; }
 bool is_tree(Kind k) { return k == K_TREE_F32 || k == K_TREE_BF16; }
 bool is_cl(Kind k) { return k == K_SEGRED_CL || k == K_SEGSCAN_CL; }
 
 int arity(Kind k) {
-    return (k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN || k == K_SEGRED_CL || k == K_SEGSCAN_CL)
+    return (k == K_SEGRED || k == K_SEGSCAN || k == K_COLRED || k == K_COLSCAN || k == K_SEGRED_CL || k == K_SEGSCAN_CL ||
+            k == K_SEGRED_MIDG || k == K_SEGSCAN_MIDG)
                ? 2
            : k == K_LVC ? 4
                         : 3;
@@ -426,8 +430,11 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
     if (cudaMemsetAsync(flush, 0, kFlushBytes, st) != cudaSuccess) return IFL_ECUDA;  // valid floats, once
     // the matmul tree sites time five leaves (ROW_TOP, ROW_MIDDLE, TOP, MIDDLE,
     // FLAT) and search a chain of four guards; every other site three versions
-    const bool tree = is_tree(k), cl = is_cl(k);
-    const int NV = tree ? 5 : cl ? 4 : 3;
+    const bool tree = is_tree(k), cl = is_cl(k), midg = is_midg(k);
+    // ".midg" sites: the V_MIDDLE group size is the tuned dimension -- slots
+    // 0..4 are group-size exponents -2..+2 of the MIDDLE version (reading R19)
+    const int NV = tree ? 5 : cl ? 4 : midg ? 5 : 3;
+    const char* gsite = k == K_SEGSCAN_MIDG ? "segscan.b4.midg" : "segred.b4.midg";
     static const int kTreeVersion[5] = {IFL_V_ROW_TOP, IFL_V_ROW_MIDDLE, IFL_V_TOP, IFL_V_MIDDLE, IFL_V_FLAT};
     static const int kClVersion[4] = {IFL_V_TOP, IFL_V_MIDDLE, IFL_V_CLUSTER, IFL_V_FLAT};
     std::vector<double> table(nshapes * NV, std::numeric_limits<double>::infinity());
@@ -474,7 +481,8 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         double best_ms = std::numeric_limits<double>::infinity();
         for (int vv = 0; vv < NV; ++vv) {
             const int slot = NV - 1 - vv;                     // table column
-            const int v = tree ? kTreeVersion[slot] : cl ? kClVersion[slot] : slot;  // version run
+            const int v = tree ? kTreeVersion[slot] : cl ? kClVersion[slot] : midg ? (int)IFL_V_MIDDLE : slot;
+            if (midg) ifl_set_thresholds(gsite, 8 + (slot - 2), 0);  // this slot's group size
             if (hopeless(k, s, v)) continue;  // stays +inf: unavailable to the search
             flush_l2(flush, st);
             cudaEventRecord(e0, st);
@@ -541,6 +549,31 @@ extern "C" int ifl_tune(const char* site, const int64_t* shapes, int nshapes, in
         rc = ifl_set_thresholds(bf ? "redomap2.bf16.row" : "redomap2.f32.row", th[0], th[1]);
         if (rc != IFL_OK) return rc;
         return ifl_set_thresholds(bf ? "redomap2.bf16" : "redomap2.f32", th[2], th[3]);
+    }
+    if (midg) {  // one exponent for the site: the paper's sum of runtimes, or the minimax with the 1 % tie rule
+        std::vector<double> best(nshapes, std::numeric_limits<double>::infinity());
+        for (int i = 0; i < nshapes; ++i)
+            for (int q = 0; q < NV; ++q) best[i] = std::min(best[i], table[i * NV + q]);
+        std::vector<double> prim(NV), sum(NV, 0.0);
+        for (int q = 0; q < NV; ++q) {
+            double worst = 0;
+            for (int i = 0; i < nshapes; ++i) {
+                sum[q] += table[i * NV + q];
+                worst = std::max(worst, table[i * NV + q] / best[i]);
+            }
+            prim[q] = cost == 0 ? sum[q] : worst;
+        }
+        const double opt = *std::min_element(prim.begin(), prim.end());
+        int pick = 2;  // the untuned group size unless another one is better
+        for (int q = 0; q < NV; ++q) {
+            const bool tie = cost == 1 ? prim[q] <= opt * (1.0 + kTieTol) : prim[q] == opt;
+            const bool pick_tie = cost == 1 ? prim[pick] <= opt * (1.0 + kTieTol) : prim[pick] == opt;
+            if (tie && (!pick_tie || sum[q] < sum[pick])) pick = q;
+        }
+        if (!std::isfinite(prim[pick])) return IFL_ENOTFIT;
+        if (t_top) *t_top = 8 + (pick - 2);
+        if (t_intra) *t_intra = 0;
+        return ifl_set_thresholds(gsite, 8 + (pick - 2), 0);
     }
     if (cl) {
         int64_t th[3];

@@ -109,6 +109,8 @@ def test_default_thresholds_are_2_pow_15(L):
     for s in ifl.SITES:
         if s.endswith((".row", ".cl")):  # the matmul row level / the cluster level are off until tuned (R17, R18)
             assert ifl.get_thresholds(s) == (2**63 - 1, 2**63 - 1)
+        elif s.endswith(".midg"):  # V_MIDDLE group-size exponent 0, biased by 8 (R19)
+            assert ifl.get_thresholds(s) == (8, 0)
         else:
             assert ifl.get_thresholds(s) == (2**15, 2**15)
 

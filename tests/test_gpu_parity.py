@@ -337,3 +337,25 @@ def test_cluster_level(ifl, orc):
         assert_parity(orc, x, got, True, "sum", "id", None, "f32")
     finally:
         ifl.reset_thresholds()
+
+
+def test_middle_group_size_dimension(ifl, orc):
+    """Reading R19: V_MIDDLE's group size x 2^shift (shift -3..3, the tuned
+    tile/group-size dimension) keeps every result; the tuner site picks one."""
+    try:
+        for shift in range(-3, 4):
+            ifl.set_thresholds("segred.b4.midg", 8 + shift, 0)
+            ifl.set_thresholds("segscan.b4.midg", 8 + shift, 0)
+            for (n, m) in [(37, 4), (65, 64), (17, 100), (5, 1024), (3, 4096), (9, 3001)]:
+                for dt in ("i32", "f32"):
+                    x, xd = gen_for("sum", dt, 40, n, m)
+                    assert_parity(orc, x, ifl.segred(xd, "sum", version="middle"), False, "sum", "id", None, dt)
+                    assert_parity(orc, x, ifl.segscan(xd, "sum", version="middle"), True, "sum", "id", None, dt)
+        ifl.reset_thresholds()
+        train = [(1 << k, 1 << (20 - k)) for k in range(10, 21, 2)]
+        for site in ("segred.b4.midg", "segscan.b4.midg"):
+            t, u, tbl = ifl.tune(site, train, reps=2, cost=1)
+            assert 6 <= t <= 10 and u == 0 and tbl.shape == (len(train), 5)
+            assert ifl.get_thresholds(site) == (t, 0)
+    finally:
+        ifl.reset_thresholds()
