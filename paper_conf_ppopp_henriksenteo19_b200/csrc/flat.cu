@@ -595,7 +595,19 @@ __global__ void __launch_bounds__(kClThreads) segscan_cluster_kernel(const T* in
     const int L = (int)(b - a);
     const T* src = in + row * m;
     T* dst = out + row * m;
-    for (int p = t; p < L; p += kClThreads) piece[clpad(p)] = apply_map<F>(src[rev ? m - 1 - (a + p) : a + p]);
+    using V = typename Vec4<T>::type;
+    // 128-bit loads when the piece starts 16-byte aligned (pieces are multiples of 4 elements)
+    const bool vec = !rev && (((uintptr_t)(src + a)) & 15u) == 0 && (L & 3) == 0;
+    if (vec) {
+        for (int q = t; q < (L >> 2); q += kClThreads) {
+            T e[4];
+            unpack4<T>(ld_coh4(src + a + 4 * q), e);
+#pragma unroll
+            for (int u = 0; u < 4; ++u) piece[clpad(4 * q + u)] = apply_map<F>(e[u]);
+        }
+    } else {
+        for (int p = t; p < L; p += kClThreads) piece[clpad(p)] = apply_map<F>(src[rev ? m - 1 - (a + p) : a + p]);
+    }
     __syncthreads();
     const int CL = (L + kClThreads - 1) / kClThreads;
     const int lo = min(L, t * CL), hi = min(L, lo + CL);
@@ -639,7 +651,18 @@ __global__ void __launch_bounds__(kClThreads) segscan_cluster_kernel(const T* in
         piece[clpad(k)] = run;
     }
     __syncthreads();
-    for (int p = t; p < L; p += kClThreads) dst[rev ? m - 1 - (a + p) : a + p] = piece[clpad(p)];
+    if (vec && (((uintptr_t)(dst + a)) & 15u) == 0) {
+        for (int q = t; q < (L >> 2); q += kClThreads) {
+            V o;
+            o.x = piece[clpad(4 * q)];
+            o.y = piece[clpad(4 * q + 1)];
+            o.z = piece[clpad(4 * q + 2)];
+            o.w = piece[clpad(4 * q + 3)];
+            *reinterpret_cast<V*>(dst + a + 4 * q) = o;
+        }
+    } else {
+        for (int p = t; p < L; p += kClThreads) dst[rev ? m - 1 - (a + p) : a + p] = piece[clpad(p)];
+    }
     // keep every CTA's shared memory alive until the higher ranks have read its total
     asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
