@@ -23,13 +23,15 @@ cap() {  # name op version n m kernel-regex
 cap segscan_flat_n1      segscan flat   1        67108864 flat_scan_jr
 cap segscan_flat_n4096   segscan flat   4096     16384    flat_scan_jr
 cap segscan_flat_n65536  segscan flat   65536    1024     flat_scan_dlb
-cap segred_flat_n1       segred  flat   1        67108864 flat_red_kernel
+cap segred_flat_n1       segred  flat   1        67108864 flat_red_split_kernel
+cap segred_flat_n4096    segred  flat   4096     16384    flat_red_split_kernel
+cap segred_cluster_n16   segred  cluster 16      4194304  segred_cluster
 cap segred_middle_n2e16  segred  middle 65536    1024     segred_mid_vec
 cap segscan_middle_n2e18 segscan middle 262144   256      segscan_mid
 cap segred_top_n2e24     segred  top    16777216 4        top_small
 cap segscan_top_n2e23    segscan top    8388608  8        top_warp
 cap redomap2_tc_8192     redomap2 top   8192     8192     mm_top_tc "--p 8192 --dt bf16"
-cap redomap2_flat_n1     redomap2 flat  1        1073741824 mm_top_tc "--p 1 --dt bf16"
+cap redomap2_flat_n8     redomap2 flat  8        16777216 mm_skinny "--p 8 --dt bf16"
 cap tridag_middle_large  tridag  middle 65536    256      tridag_mid "--p 256"
 cap tridag_flat_large    tridag  flat   65536    256      tridag_flat16 "--p 256"
 cap lvc_outer_large      lvc     outer  256      256      lvc_outer "--p 256"

@@ -39,13 +39,16 @@ ALG = {  # algorithmic bytes of the captured launch
     "segred_middle_n2e16": 4 * (2**26 + 65536), "segscan_middle_n2e18": 8 * 2**26,
     "segred_top_n2e24": 4 * (2**26 + 2**24), "segscan_top_n2e23": 8 * 2**26,
     "redomap2_tc_8192": 2 * (2 * 8192 * 8192) + 4 * 8192 * 8192, "redomap2_flat_n1": 2 * (2 * 2**30) + 4,
+    "redomap2_flat_n8": 2 * (16 * 2**24) + 4 * 64, "segred_flat_n4096": 4 * (2**26 + 4096),
+    "segred_cluster_n16": 4 * (2**26 + 16),
     "tridag_middle_large": 8 * 65536 * 256, "tridag_flat_large": 8 * 65536 * 256,
     "lvc_outer_large": 2 * 8 * 256 * 256 * 256,  # one read + one write per element for the whole loop
     "colred_flat_n2e20": 4 * 2**26, "colscan_top_n4": 8 * 2**26, "colscan_flat_n2e26": 8 * 2**26,
 }
 GROUP = {"segscan_flat_n1": "segscan_flat", "segscan_flat_n65536": "segscan_flat_dlb", "segred_flat_n1": "segred_flat", "segred_middle_n2e16": "segred_middle",
          "segscan_middle_n2e18": "segscan_middle", "segred_top_n2e24": "segred_top", "segscan_top_n2e23": "segscan_top",
-         "redomap2_tc_8192": "redomap2_tc", "redomap2_flat_n1": "redomap2_flat", "tridag_middle_large": "tridag_middle",
+         "redomap2_tc_8192": "redomap2_tc", "redomap2_flat_n1": "redomap2_flat", "redomap2_flat_n8": "redomap2_flat",
+         "segred_cluster_n16": "segred_cluster", "tridag_middle_large": "tridag_middle",
          "tridag_flat_large": "tridag_flat", "lvc_outer_large": "lvc_outer", "colred_flat_n2e20": "colred_flat",
          "colscan_top_n4": "colscan_top", "colscan_flat_n2e26": "colscan_flat",
          "segred_irr_flat_m1k": "segred_irr_flat", "segscan_irr_flat_m1k": "segscan_irr_flat"}
