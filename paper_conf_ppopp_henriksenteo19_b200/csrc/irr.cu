@@ -35,11 +35,7 @@ namespace {
 constexpr int kIrrThreads = 256;
 constexpr int kIrrItems = 16;
 constexpr int64_t kIrrTile = (int64_t)kIrrThreads * kIrrItems;
-// offsets of a tile's segment range staged in (dynamic) shared memory: room
-// for 2x the tile's average segment count, 2048..8192 entries (short
-// segments: a tile spans thousands of them, and an unstaged tile binary-
-// searches global memory)
-constexpr int kIrrSmemOffMin = 2048, kIrrSmemOffMax = 8192;
+constexpr int kIrrSmemOff = 2048;  // offsets of up to 2047 segments per tile staged in shared memory
 
 // ------------------------------------------------------------ V_TOP
 
@@ -269,8 +265,7 @@ __device__ __forceinline__ void irr_tile(int64_t tile, int64_t Tn, T (&v)[kIrrIt
                                          const int64_t* __restrict__ off, int64_t n, int64_t total, T d,
                                          const int64_t* __restrict__ tile_seg, T* __restrict__ head,
                                          T* __restrict__ tail, uint32_t* __restrict__ tflag,
-                                         const T* __restrict__ cin, bool vec, int64_t* s_off, T* s_v, uint32_t* s_f,
-                                         int soff_cap) {
+                                         const T* __restrict__ cin, bool vec, int64_t* s_off, T* s_v, uint32_t* s_f) {
     const int t = threadIdx.x;
     const int64_t base = tile * kIrrTile;
     const int cnt = (int)(total - base < kIrrTile ? total - base : kIrrTile);
@@ -278,7 +273,7 @@ __device__ __forceinline__ void irr_tile(int64_t tile, int64_t Tn, T (&v)[kIrrIt
     const int64_t s_lo = tile_seg[tile];
     const int64_t s_hi = tile + 1 < Tn ? tile_seg[tile + 1] : n - 1;
     const int64_t nseg = s_hi - s_lo + 2;  // offsets off[s_lo .. s_hi + 1]
-    const bool staged = nseg <= soff_cap;
+    const bool staged = nseg <= kIrrSmemOff;
     __syncthreads();  // s_off / s_v of the previous tile are no longer read
     if (staged)
         for (int64_t k = threadIdx.x; k < nseg; k += kIrrThreads) s_off[k] = off[s_lo + k];
@@ -407,8 +402,8 @@ __global__ void __launch_bounds__(kIrrThreads) irr_flat_kernel(const T* __restri
                                                                const int64_t* __restrict__ tile_seg,
                                                                T* __restrict__ head, T* __restrict__ tail,
                                                                uint32_t* __restrict__ tflag, const T* __restrict__ cin,
-                                                               bool vec, int soff_cap) {
-    extern __shared__ int64_t s_off[];  // soff_cap entries
+                                                               bool vec) {
+    __shared__ int64_t s_off[kIrrSmemOff];
     __shared__ T s_v[kIrrThreads / 32];
     __shared__ uint32_t s_f[kIrrThreads / 32];
     const int64_t Tn = (total + kIrrTile - 1) / kIrrTile;
@@ -422,7 +417,7 @@ __global__ void __launch_bounds__(kIrrThreads) irr_flat_kernel(const T* __restri
         int nn = 0;
         if (r + 1 < kIrrTPB && tile + 1 < Tn) nn = irr_load<T, OP>(in, total, tile + 1, vec, vn);
         irr_tile<T, OP, F, MODE>(tile, Tn, v, nval, out, off, n, total, d, tile_seg, head, tail, tflag, cin, vec, s_off,
-                                 s_v, s_f, soff_cap);
+                                 s_v, s_f);
 #pragma unroll
         for (int k = 0; k < kIrrItems; ++k) v[k] = vn[k];
         nval = nn;
@@ -539,30 +534,17 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
         if (Tn > 0x7fffffffLL) return cudaErrorInvalidValue;
-        const int64_t per_tile = a.total > 0 ? ceil_div(a.n * kIrrTile, a.total) : a.n;
-        const int cap = (int)std::max<int64_t>(kIrrSmemOffMin, std::min<int64_t>(kIrrSmemOffMax, 2 * per_tile + 64));
-        const size_t soff = (size_t)cap * sizeof(int64_t);
-        static bool attr = false;
-        if (!attr) {
-            cudaFuncSetAttribute(irr_flat_kernel<T, OP, F, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)(kIrrSmemOffMax * sizeof(int64_t)));
-            cudaFuncSetAttribute(irr_flat_kernel<T, OP, F, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)(kIrrSmemOffMax * sizeof(int64_t)));
-            cudaFuncSetAttribute(irr_flat_kernel<T, OP, F, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                 (int)(kIrrSmemOffMax * sizeof(int64_t)));
-            attr = true;
-        }
         if (scan)
-            irr_flat_kernel<T, OP, F, 1><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, soff, a.stream>>>(
-                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec, cap);
+            irr_flat_kernel<T, OP, F, 1><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
+                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
         else
-            irr_flat_kernel<T, OP, F, 0><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, soff, a.stream>>>(
-                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec, cap);
+            irr_flat_kernel<T, OP, F, 0><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
+                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
         if (!scan) return cudaGetLastError();  // crossing segments were combined atomically
         irr_tile_scan_kernel<T, OP><<<1, 1024, 0, a.stream>>>(tail, tflag, cin, Tn);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
-        irr_flat_kernel<T, OP, F, 2><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, soff, a.stream>>>(
-            in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec, cap);
+        irr_flat_kernel<T, OP, F, 2><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
+            in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
         return cudaGetLastError();
     });
 }
