@@ -112,3 +112,25 @@ def test_lvc_tune_installs_t0(ifl):
         assert ifl.get_thresholds("lvc")[0] == t0
     finally:
         ifl.reset_thresholds()
+
+
+@pytest.mark.parametrize("version", ["outer", "middle", "flat"])
+def test_lvc_step_by_step(ifl, orc, version):
+    """The per-step bar behind the numT * 1e-5 loop bound (R13), checked
+    directly: every step of the loop (one ifl_lvc step on the GPU's f32 state)
+    is within the tridag bar 1e-5 * max(1, ||x||_inf) of the oracle's exact
+    step from the same state -- the loop bound's only slack is the sum over
+    steps, and the matrices' row margin keeps step errors from growing."""
+    numS, numT, numX, numY = 2, 16, 32, 256
+    (ax, bx, cx), (ay, by, cy), xs, ys = gen.lvc_problem(21, numS, numX, numY)
+    xd, yd = xs.cuda(), ys.cuda()
+    xc = tuple(t.cuda() for t in (ax, bx, cx))
+    yc = tuple(t.cuda() for t in (ay, by, cy))
+    co = [t.numpy() for t in (ax, bx, cx, ay, by, cy)]
+    for step in range(numT):
+        x0, y0 = xd.cpu().numpy().copy(), yd.cpu().numpy().copy()
+        ifl.lvc(xd, yd, xc, yc, 1, version=version)
+        want_x, want_y = orc.lvc(*co, x0, y0, 1)
+        for got, want in ((xd.cpu().numpy(), want_x), (yd.cpu().numpy(), want_y)):
+            err = np.abs(got.astype(np.float64) - want).max()
+            assert err <= 1e-5 * max(1.0, np.abs(want).max()), f"{version} step {step}: {err:.3g}"
