@@ -349,7 +349,7 @@ size_t ifl_workspace_bytes(const char* entry, int64_t n, int64_t m, int64_t p, i
         return (((size_t)(n * m) * 4 + 255) & ~(size_t)255) +
                std::max(n * m * p > 0 ? ifl::flat_ws_bytes(n * m * p) : 0, n * m > 0 ? ifl::flat_ws_bytes(n * m) : 0);
     }
-    if (strcmp(entry, "segred_irr") == 0 || strcmp(entry, "segscan_irr") == 0) return ifl::irr_ws_bytes(m, version);
+    if (strcmp(entry, "segred_irr") == 0 || strcmp(entry, "segscan_irr") == 0) return ifl::irr_ws_bytes(n, m, version);
     if (strcmp(entry, "tridag") == 0) return ifl::tridag_ws_bytes(p > 0 ? p : n, m, version);
     if (strcmp(entry, "lvc") == 0)  // (numX, numY): the coefficient scans of both sites
         return ifl::tridag_ws_bytes(n, m, version) + ifl::tridag_ws_bytes(m, n, version);
@@ -469,7 +469,7 @@ static int run_irr(bool scan, const void* in, void* out, const int64_t* off, int
     if (n == 0) return IFL_OK;
     if (total == 0) return scan ? IFL_OK : cuda_status(ifl::launch_fill(out, n, bits, (cudaStream_t)stream), what);
     if (c.version == IFL_V_FLAT) {
-        const size_t need = ifl::irr_ws_bytes(total, IFL_V_FLAT);
+        const size_t need = ifl::irr_ws_bytes(n, total, IFL_V_FLAT);
         if (!ws || ws_bytes < need)
             return fail(IFL_EWORKSPACE, "%s: V_FLAT needs %zu workspace bytes, got %zu", what, need, ws_bytes);
     }

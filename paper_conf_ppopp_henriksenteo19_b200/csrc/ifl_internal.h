@@ -97,8 +97,8 @@ struct IrrArgs {
     size_t ws_bytes;
     cudaStream_t stream;
 };
-int64_t irr_tiles(int64_t total);
-size_t irr_ws_bytes(int64_t total, int version);
+int64_t irr_tiles(int64_t n, int64_t total);
+size_t irr_ws_bytes(int64_t n, int64_t total, int version);
 cudaError_t launch_irr(const IrrArgs& a, bool scan, int version);
 cudaError_t launch_irr_inspect(const int64_t* off, int64_t n, void* res16, cudaStream_t s);
 

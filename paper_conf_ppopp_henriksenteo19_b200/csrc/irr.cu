@@ -8,20 +8,8 @@
 //             when lengths vary: its time is set by the longest segment);
 //   V_MIDDLE  warp per segment: strided loads, shuffle reduce / warp scans
 //             with a running carry;
-//   V_FLAT    flattened over all elements: 4096-element tiles (256 threads x
-//             16 items) with per-tile segment ranges, a CTA-wide segmented
-//             scan of the thread pieces, and tile aggregates combined by a
-//             single-CTA segmented scan over tiles:
-//               pass 0  tile -> the segment holding its first element
-//                       (each segment writes its tile starts; long ones with
-//                       the whole warp); empty segments reduce to d;
-//               pass 1  per tile: complete segments written; segred: the
-//                       head / tail pieces of segments crossing tiles are
-//                       combined into their outputs atomically (done);
-//                       segscan: the tile's tail piece and flag recorded;
-//               pass 2  (segscan) exclusive segmented scan of the tile tails;
-//               pass 3  (segscan) the tile rescanned with its carry (two
-//                       reads + one write per element).
+//   V_FLAT    flattened over segments and elements together (merge path:
+//             tiles of 4096 merge items, see below).
 #include <algorithm>
 
 #include "common.cuh"
@@ -35,7 +23,6 @@ namespace {
 constexpr int kIrrThreads = 256;
 constexpr int kIrrItems = 16;
 constexpr int64_t kIrrTile = (int64_t)kIrrThreads * kIrrItems;
-constexpr int kIrrSmemOff = 2048;  // offsets of up to 2047 segments per tile staged in shared memory
 
 // ------------------------------------------------------------ V_TOP
 
@@ -106,53 +93,63 @@ __global__ void __launch_bounds__(256) irr_mid_kernel(const T* __restrict__ in, 
 }
 
 // ------------------------------------------------------------ V_FLAT
+// Merge-path decomposition (B200 design; the paper only names irregular
+// nesting as future work): the n segment ends off[1..n] and the
+// `total` element indices 0..total-1 are merged into one sequence of n + total
+// items (an end off[i+1] comes before element j when off[i+1] <= j), and every
+// tile takes kIrrTile consecutive merge items.  Every tile thus holds the same
+// amount of work whatever the length mix -- empty segments, a mean of one
+// element, or one segment of 12M elements.
+//   partition  the (segment, element) coordinates of every tile start
+//              (8 lanes per tile, 8-ary search over off);
+//   segred     pass 1 (persistent CTAs, 3 per SM): the next tile's segment
+//              ends and elements are copied into shared memory with cp.async
+//              while the current one is walked -- each thread walks 16
+//              consecutive items branch-free, a CTA-wide segmented scan of
+//              the thread pieces gives each thread's carry, complete segments
+//              are staged in place of their ends and stored coalesced; the
+//              tile records its head piece (its first segment, when that began
+//              in an earlier tile) and its open tail (flag: a segment starts
+//              in the tile);
+//              pass 2: segmented scan of the tile tails in two parallel
+//              kernels (chunk aggregates; chunk scans seeded by the preceding
+//              aggregates) that complete the head pieces, out[i] = carry (+)
+//              head;
+//   segscan    pass 1: per tile (a warp each), the reduce of its open tail
+//              only (elements after the tile's last segment start: short
+//              segments read almost nothing); pass 2: the segmented scan of
+//              the tails (cin); pass 3: the merge walk again with the tile's
+//              carry, the scanned elements staged in place and stored
+//              coalesced (two reads + one write per element when segments are
+//              long; one read + one write when they are short).
 
-// pass 0: every tile t learns the (non-empty) segment holding its first
-// element: segment i writes tile_seg[t] for each tile start inside
-// [off[i], off[i+1]) -- each tile exactly once, so no initialisation and no
-// scan are needed.  A lane whose segment covers more than two tile starts
-// hands it to its whole warp (ballot), so a long segment costs ~1/32 of its
-// tiles per lane.  Empty segments reduce to d.
-template <typename T, int OP, bool RED>
-__global__ void __launch_bounds__(256) irr_claim_kernel(const int64_t* __restrict__ off, int64_t n,
-                                                        int64_t* __restrict__ tile_seg, T* __restrict__ out, T d) {
-    const int lane = threadIdx.x & 31;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    // uniform trip count per warp so the ballots see every lane
-    const int64_t base0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) - lane;
-    for (int64_t b0 = base0; b0 < n; b0 += stride) {
-        const int64_t i = b0 + lane;
-        int64_t t0 = 0, t1 = 0;  // tile starts [t0, t1) inside segment i
-        if (i < n) {
-            const int64_t a = off[i], b = off[i + 1];
-            if (a == b) {
-                if constexpr (RED) out[i] = d;
-            } else {
-                t0 = (a + kIrrTile - 1) / kIrrTile;
-                t1 = (b + kIrrTile - 1) / kIrrTile;
-                // a segment crossing tiles is assembled by atomic combines
-                if constexpr (RED)
-                    if (a / kIrrTile != (b - 1) / kIrrTile) out[i] = identity<OP, T>();
-            }
-        }
-        const bool longseg = t1 - t0 > 2;
-        if (!longseg)
-            for (int64_t t = t0; t < t1; ++t) tile_seg[t] = i;
-        unsigned ball = __ballot_sync(0xffffffffu, longseg);
-        while (ball) {  // the warp writes each long segment's tiles together
-            const int src = __ffs(ball) - 1;
-            ball &= ball - 1;
-            const int64_t s0 = __shfl_sync(0xffffffffu, t0, src), s1 = __shfl_sync(0xffffffffu, t1, src);
-            for (int64_t t = s0 + lane; t < s1; t += 32) tile_seg[t] = b0 + src;
-        }
-    }
+// Shared-memory staging, padded so the thread-blocked walk (lanes ~16 items
+// apart) is bank-conflict-free: ends E[k] = off[i0 + k] (int64, one pad word
+// per 16), elements X[k] (one pad word per 32).
+__device__ __forceinline__ int pe(int k) { return k + (k >> 4); }
+__device__ __forceinline__ int px(int k) { return k + (k >> 5); }
+__host__ __device__ constexpr int mp_xoff(int ns) { return (((ns + 1) + ((ns + 1) >> 4) + 1) * 8 + 15) & ~15; }
+constexpr int kMpBuf = mp_xoff((int)kIrrTile) + 16 * 4;  // ns = kIrrTile, ne = 0 is the largest tile
+constexpr int kMpCtasPerSm = 3;
+constexpr size_t kMpSmem = 2 * (size_t)kMpBuf;
+
+__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
 }
+__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
 
 // CTA-wide exclusive scan of (flag, value) thread pieces under the segmented
-// operator (f1,v1).(f2,v2) = (f1|f2, f2 ? v2 : v1 (+) v2).
-template <typename T, int OP>
-__device__ __forceinline__ void irr_cta_seg_scan(uint32_t fl, T v, uint32_t& exf, T& exv, uint32_t& aggf, T& aggv,
-                                                 T* s_v, uint32_t* s_f) {
+// operator (f1,v1).(f2,v2) = (f1|f2, f2 ? v2 : v1 (+) v2), seeded with an
+// initial piece (init_f, init_v): exf/exv = everything before the thread,
+// aggf/aggv = the whole CTA.  NT threads.
+template <typename T, int OP, int NT>
+__device__ __forceinline__ void irr_cta_seg_scan(uint32_t fl, T v, uint32_t init_f, T init_v, uint32_t& exf, T& exv,
+                                                 uint32_t& aggf, T& aggv, T* s_v, uint32_t* s_f) {
     const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -174,12 +171,12 @@ __device__ __forceinline__ void irr_cta_seg_scan(uint32_t fl, T v, uint32_t& exf
         exf = 0;
     }
     __syncthreads();
-    T pw = identity<OP, T>();
-    uint32_t pf = 0;
-    aggv = identity<OP, T>();
-    aggf = 0;
+    T pw = init_v;  // the initial piece, then the warps before w
+    uint32_t pf = init_f;
+    aggv = init_v;
+    aggf = init_f;
 #pragma unroll
-    for (int k = 0; k < kIrrThreads / 32; ++k) {
+    for (int k = 0; k < NT / 32; ++k) {
         const T wv = s_v[k];
         const uint32_t wf = s_f[k];
         if (k < w) {
@@ -193,313 +190,327 @@ __device__ __forceinline__ void irr_cta_seg_scan(uint32_t fl, T v, uint32_t& exf
     exf |= pf;
 }
 
-// Shared state of one tile: its segment range and the staged offsets.
-struct IrrTile {
-    int64_t base, s_lo, s_hi;
-    int cnt;
-    bool staged;
+// partition: coord[b] = the number of segment ends among the first
+// min(b*T, n+total) merge items.  P(i) = off[i+1] + i + 1 <= D is monotone
+// (true then false); 8 lanes per tile start probe 8 evenly spaced i per round.
+__global__ void __launch_bounds__(256) irr_mp_partition_kernel(const int64_t* __restrict__ off, int64_t n,
+                                                               int64_t total, int64_t Tn, int64_t* __restrict__ coord) {
+    const int lane = threadIdx.x & 31, sub = lane & 7;
+    const unsigned gmask = 0xffu << (lane & 24);
+    const int64_t b = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
+    const bool live = b <= Tn;
+    const int64_t D = live ? min(b * kIrrTile, n + total) : 0;
+    int64_t lo = max((int64_t)0, D - total), hi = min(D, n);
+    while (__any_sync(0xffffffffu, lo < hi)) {  // uniform trip count: the ballots need every lane
+        const int64_t step = (hi - lo + 7) / 8;
+        const int64_t p = lo + step * sub;
+        const bool pr = lo < hi && p < hi && __ldg(off + p + 1) + p + 1 <= D;
+        const int c = __popc(__ballot_sync(0xffffffffu, pr) & gmask);  // true probes: sub-lanes 0..c-1
+        if (lo < hi) {
+            if (c == 0) {
+                hi = lo;  // P(lo) is false: the split is lo
+            } else {
+                hi = min(lo + step * c, hi);
+                lo = lo + step * (c - 1) + 1;
+            }
+        }
+    }
+    if (live && sub == 0) coord[b] = lo;
+}
+
+struct MpTile {
+    int64_t i0, j0;
+    int ns, ne;
 };
 
-// largest i in [lo, hi] with off[i] <= e (off[lo] <= e holds)
-__device__ __forceinline__ int64_t seg_search(const int64_t* o, int64_t lo, int64_t hi, int64_t e) {
-    while (lo < hi) {
-        const int64_t mid = (lo + hi + 1) >> 1;
-        if (o[mid] <= e) lo = mid;
-        else hi = mid - 1;
-    }
-    return lo;
+__device__ __forceinline__ MpTile mp_tile(int64_t b, int64_t i0, int64_t i1, int64_t W) {
+    MpTile t;
+    const int64_t D0 = b * kIrrTile, D1 = min(D0 + kIrrTile, W);
+    t.i0 = i0;
+    t.j0 = D0 - i0;
+    t.ns = (int)(i1 - i0);
+    t.ne = (int)((D1 - i1) - t.j0);
+    return t;
 }
 
-// *addr = *addr (+) v, atomically: the pieces of a segment that crosses tiles
-// are combined into its output in any order (every builtin (+) is associative
-// and commutative; f32 sums may differ from run to run only by association,
-// within the parity bound).
-template <int OP, typename T>
-__device__ __forceinline__ void atomic_combine(T* addr, T v) {
-    if constexpr (std::is_same<T, int>::value) {
-        if constexpr (OP == OP_SUM) { atomicAdd(addr, v); return; }
-        if constexpr (OP == OP_MIN) { atomicMin(addr, v); return; }
-        if constexpr (OP == OP_MAX) { atomicMax(addr, v); return; }
-        if constexpr (OP == OP_AND) { atomicAnd(addr, v); return; }
-        if constexpr (OP == OP_OR) { atomicOr(addr, v); return; }
-        if constexpr (OP == OP_XOR) { atomicXor(addr, v); return; }
-    } else {
-        if constexpr (OP == OP_SUM) { atomicAdd(addr, v); return; }
-    }
-    // PROD (both types), f32 MIN / MAX: compare-and-swap on the bit pattern
-    unsigned* a = reinterpret_cast<unsigned*>(addr);
-    unsigned old = *a, assumed;
-    do {
-        assumed = old;
-        const T cur = from_bits<T>(assumed);
-        old = atomicCAS(a, assumed, to_bits<T>(combine<OP>(cur, v)));
-    } while (old != assumed);
+// Issue the cp.async copies of a tile into buffer `buf` (one commit group).
+template <typename T>
+__device__ __forceinline__ void mp_issue(const T* in, const int64_t* off, const MpTile& tl, uint8_t* buf) {
+    int64_t* E = reinterpret_cast<int64_t*>(buf);
+    T* X = reinterpret_cast<T*>(buf + mp_xoff(tl.ns));
+    for (int k = threadIdx.x; k <= tl.ns; k += kIrrThreads) cp_async8(E + pe(k), off + tl.i0 + k);
+    for (int k = threadIdx.x; k < tl.ne; k += kIrrThreads) cp_async4(X + px(k), in + tl.j0 + k);
+    cp_async_commit();
 }
 
-// Load the thread's 16 items of tile `tile` (identity past the end).
-template <typename T, int OP>
-__device__ __forceinline__ int irr_load(const T* __restrict__ in, int64_t total, int64_t tile, bool vec,
-                                        T (&v)[kIrrItems]) {
-    const int64_t e0 = tile * kIrrTile + (int64_t)threadIdx.x * kIrrItems;
-    const int nval = (int)max((int64_t)0, min((int64_t)kIrrItems, total - e0));
-    if (vec && nval == kIrrItems) {
-#pragma unroll
-        for (int c = 0; c < kIrrItems / 4; ++c) {
-            T e[4];
-            unpack4<T>(ldg_stream4(in + e0 + 4 * c), e);
-#pragma unroll
-            for (int q = 0; q < 4; ++q) v[4 * c + q] = e[q];
-        }
-    } else {
-#pragma unroll
-        for (int k = 0; k < kIrrItems; ++k) v[k] = k < nval ? __ldg(in + e0 + k) : identity<OP, T>();
-    }
-    return nval;
-}
-
-// One tile.  MODE 0: segred pass 1 (complete segments -> out, head / tail /
-// flags); MODE 1: segscan pass 1 (tail / flags); MODE 2: segscan pass 3
-// (rescan with the tile's carry, write out).
-template <typename T, int OP, int F, int MODE>
-__device__ __forceinline__ void irr_tile(int64_t tile, int64_t Tn, T (&v)[kIrrItems], int nval, T* __restrict__ out,
-                                         const int64_t* __restrict__ off, int64_t n, int64_t total, T d,
-                                         const int64_t* __restrict__ tile_seg, T* __restrict__ head,
-                                         T* __restrict__ tail, uint32_t* __restrict__ tflag,
-                                         const T* __restrict__ cin, bool vec, int64_t* s_off, T* s_v, uint32_t* s_f) {
-    const int t = threadIdx.x;
-    const int64_t base = tile * kIrrTile;
-    const int cnt = (int)(total - base < kIrrTile ? total - base : kIrrTile);
-    const int64_t e0 = base + (int64_t)t * kIrrItems;
-    const int64_t s_lo = tile_seg[tile];
-    const int64_t s_hi = tile + 1 < Tn ? tile_seg[tile + 1] : n - 1;
-    const int64_t nseg = s_hi - s_lo + 2;  // offsets off[s_lo .. s_hi + 1]
-    const bool staged = nseg <= kIrrSmemOff;
-    __syncthreads();  // s_off / s_v of the previous tile are no longer read
-    if (staged)
-        for (int64_t k = threadIdx.x; k < nseg; k += kIrrThreads) s_off[k] = off[s_lo + k];
-    __syncthreads();
-    auto O = [&](int64_t i) -> int64_t { return staged ? s_off[i - s_lo] : off[i]; };
-    // segment of the first item; the walk skips empty segments
-    int64_t seg = s_lo, cur_start = 0, nxt = 0;
-    if (nval > 0) {
-        seg = staged ? s_lo + seg_search(s_off, 0, s_hi - s_lo, e0) : seg_search(off, s_lo, s_hi, e0);
-        cur_start = O(seg);
-        nxt = O(seg + 1);
-    }
-    bool has_start = false, stash = false;
-    int first_start = kIrrItems;  // item index of the thread's first segment start
-    int64_t stash_seg = -1;
-    T acc = identity<OP, T>(), stash_v = identity<OP, T>();
-    if (nval > 0 && e0 + nval <= nxt) {
-        // fast path (long segments): every item lies in segment seg; at most
-        // the first item starts it and at most the last one ends it
-        const bool st = e0 == cur_start;
-        if constexpr (MODE == 2) {
-            T r = st ? d : identity<OP, T>();
-#pragma unroll
-            for (int k = 0; k < kIrrItems; ++k)
-                if (k < nval) v[k] = r = combine<OP>(r, apply_map<F>(v[k]));
-            acc = r;
-        } else {
-            T a4[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
-#pragma unroll
-            for (int k = 0; k < kIrrItems; ++k)
-                if (k < nval) a4[k & 3] = combine<OP>(a4[k & 3], apply_map<F>(v[k]));
-            acc = combine<OP>(combine<OP>(a4[0], a4[1]), combine<OP>(a4[2], a4[3]));
-            if (st) acc = combine<OP>(d, acc);
-        }
-        has_start = st;
-        first_start = st ? 0 : kIrrItems;
-        if (e0 + nval == nxt) {
-            if (!st) {
-                stash = true;
-                stash_v = acc;
-                stash_seg = seg;
-            } else if constexpr (MODE == 0) {
-                out[seg] = acc;
-            }
-        }
-    } else
-#pragma unroll
-    for (int k = 0; k < kIrrItems; ++k) {
-        if (k < nval) {
-            const int64_t e = e0 + k;
-            while (e >= nxt) {  // next non-empty segment
-                ++seg;
-                cur_start = nxt;
-                nxt = O(seg + 1);
-            }
-            const T x = apply_map<F>(v[k]);
-            if (e == cur_start) {
-                acc = combine<OP>(d, x);
-                if (!has_start) first_start = k;
-                has_start = true;
-            } else {
-                acc = combine<OP>(acc, x);
-            }
-            if constexpr (MODE == 2) v[k] = acc;
-            if (e + 1 == nxt) {  // item ends segment seg
-                if (!has_start) {  // started before this thread
-                    stash = true;
-                    stash_v = acc;
-                    stash_seg = seg;
-                } else if constexpr (MODE == 0) {
-                    out[seg] = acc;
-                }
-            }
-        }
-    }
-    uint32_t exf, aggf;
-    T exv, aggv;
-    irr_cta_seg_scan<T, OP>(has_start ? 1u : 0u, acc, exf, exv, aggf, aggv, s_v, s_f);
-    if constexpr (MODE == 0) {
-        if (stash) {
-            const T val = combine<OP>(exv, stash_v);
-            if (exf) out[stash_seg] = val;                  // started earlier in this tile: complete
-            else atomic_combine<OP>(out + stash_seg, val);  // the head piece of a crossing segment
-        }
-        if (t == 0) {
-            // the open piece at the tile's end (from its last start, with d, or
-            // the whole tile) belongs to a segment that continues past the tile
-            const int64_t e_last = base + cnt - 1;
-            const int64_t sl = staged ? s_lo + seg_search(s_off, 0, s_hi - s_lo, e_last) : seg_search(off, s_lo, s_hi, e_last);
-            if (O(sl + 1) > e_last + 1) atomic_combine<OP>(out + sl, aggv);
-        }
-    } else if constexpr (MODE == 1) {
-        if (t == 0) {
-            tail[tile] = aggv;
-            tflag[tile] = aggf ? 1u : 0u;
-        }
-    } else {
-        // carry for the items before the thread's first start
-        const T pre = exf ? exv : combine<OP>(cin[tile], exv);
-#pragma unroll
-        for (int k = 0; k < kIrrItems; ++k)
-            if (k < first_start && k < nval) v[k] = combine<OP>(pre, v[k]);
-        if (vec && nval == kIrrItems) {
-#pragma unroll
-            for (int c = 0; c < kIrrItems / 4; ++c) {
-                typename Vec4<T>::type q;
-                q.x = v[4 * c]; q.y = v[4 * c + 1]; q.z = v[4 * c + 2]; q.w = v[4 * c + 3];
-                __stcs(reinterpret_cast<typename Vec4<T>::type*>(out + e0 + 4 * c), q);
-            }
-        } else {
-#pragma unroll
-            for (int k = 0; k < kIrrItems; ++k)
-                if (k < nval) out[e0 + k] = v[k];
-        }
-    }
-}
-
-// kIrrTPB consecutive tiles per CTA; the next tile's items are loaded while
-// the current one is processed.
-constexpr int kIrrTPB = 1;
-
-template <typename T, int OP, int F, int MODE>
-__global__ void __launch_bounds__(kIrrThreads) irr_flat_kernel(const T* __restrict__ in, T* __restrict__ out,
-                                                               const int64_t* __restrict__ off, int64_t n,
-                                                               int64_t total, T d,
-                                                               const int64_t* __restrict__ tile_seg,
-                                                               T* __restrict__ head, T* __restrict__ tail,
-                                                               uint32_t* __restrict__ tflag, const T* __restrict__ cin,
-                                                               bool vec) {
-    __shared__ int64_t s_off[kIrrSmemOff];
+// Pass 1 of segred (SCAN = false) / pass 3 of segscan (SCAN = true) over
+// tiles blockIdx.x, +gridDim.x, ... with the next tile in flight.
+// segscan: in may equal out (a tile reads and writes only its own elements;
+// cp.async reads are issued before that tile's stores).
+template <typename T, int OP, int F, bool SCAN>
+__global__ void __launch_bounds__(kIrrThreads, kMpCtasPerSm)
+    irr_mp_kernel(const T* in, T* out, const int64_t* __restrict__ off, int64_t n, int64_t total, T d,
+                  const int64_t* __restrict__ coord, T* __restrict__ tail, uint32_t* __restrict__ tflag,
+                  T* __restrict__ head, const T* __restrict__ cin, int64_t Tn) {
+    extern __shared__ __align__(16) uint8_t mp_raw[];
     __shared__ T s_v[kIrrThreads / 32];
     __shared__ uint32_t s_f[kIrrThreads / 32];
-    const int64_t Tn = (total + kIrrTile - 1) / kIrrTile;
-    const int64_t t0 = (int64_t)blockIdx.x * kIrrTPB;
-    T v[kIrrItems], vn[kIrrItems];
-    int nval = irr_load<T, OP>(in, total, t0, vec, v);
+    __shared__ int s_skip0;
+    __shared__ int s_start[kIrrThreads];
+    const int t = threadIdx.x;
+    const int64_t G = gridDim.x, W = n + total;
+    int64_t b = blockIdx.x;
+    if (b >= Tn) return;
+    MpTile cur = mp_tile(b, coord[b], coord[b + 1], W);
+    mp_issue<T>(in, off, cur, mp_raw);
+    int64_t nb = b + G, ni0 = 0, ni1 = 0;
+    if (nb < Tn) {
+        ni0 = coord[nb];
+        ni1 = coord[nb + 1];
+    }
+    for (int r = 0; b < Tn; ++r) {
+        uint8_t* buf = mp_raw + (size_t)(r & 1) * kMpBuf;
+        MpTile nxt{};
+        if (nb < Tn) {
+            nxt = mp_tile(nb, ni0, ni1, W);
+            mp_issue<T>(in, off, nxt, mp_raw + (size_t)((r + 1) & 1) * kMpBuf);
+        } else {
+            cp_async_commit();
+        }
+        // coordinates two tiles ahead, in flight during this tile
+        const int64_t nnb = nb + G;
+        int64_t pi0 = 0, pi1 = 0;
+        if (nnb < Tn) {
+            pi0 = coord[nnb];
+            pi1 = coord[nnb + 1];
+        }
+        T carry_in = identity<OP, T>();
+        if constexpr (SCAN) carry_in = cin[b];
+        cp_async_wait<1>();
+        if (t == 0) s_skip0 = 0;
+        __syncthreads();
+        // ---------------- the tile
+        int* E32 = reinterpret_cast<int*>(buf);  // low words of E
+        T* X = reinterpret_cast<T*>(buf + mp_xoff(cur.ns));
+        const int j0lo = (int)cur.j0;
+        const uint32_t start_f = reinterpret_cast<const int64_t*>(buf)[0] >= cur.j0 ? 1u : 0u;
+        const int Wt = cur.ns + cur.ne;
+        const int d0 = min(t * kIrrItems, Wt), cnt = min(d0 + kIrrItems, Wt) - d0;
+        // thread starts without a search: end k sits at merge position
+        // pos(k) = k + (its end - j0) (strictly increasing), so the thread
+        // whose first item is 16u (pos(k-1) < 16u <= pos(k)) starts at end k;
+        // threads past the last end start at ns
+        for (int k = t; k < cur.ns; k += kIrrThreads) {
+            const int pk = k + (E32[2 * pe(k + 1)] - j0lo);
+            const int pp = k == 0 ? -1 : (k - 1) + (E32[2 * pe(k)] - j0lo);
+            for (int u = (pp >> 4) + 1; u * kIrrItems <= pk; ++u) s_start[u] = k;
+        }
+        if (t * kIrrItems > (cur.ns == 0 ? -1 : (cur.ns - 1) + (E32[2 * pe(cur.ns)] - j0lo))) s_start[t] = cur.ns;
+        __syncthreads();  // (segred: also every read of the ends is done before segment values overwrite them)
+        int i = s_start[t];
+        const int ie = t + 1 < kIrrThreads ? s_start[t + 1] : cur.ns;
+        const int j_s = d0 - i;
+        T acc = identity<OP, T>();
+        int first = -1;  // segred: the thread's first segment end
+        int lead = 0;    // segscan: elements before the thread's first segment start
+        if (i == ie && cnt == kIrrItems) {  // elements only
 #pragma unroll
-    for (int r = 0; r < kIrrTPB; ++r) {
-        const int64_t tile = t0 + r;
-        if (tile >= Tn) break;
-        int nn = 0;
-        if (r + 1 < kIrrTPB && tile + 1 < Tn) nn = irr_load<T, OP>(in, total, tile + 1, vec, vn);
-        irr_tile<T, OP, F, MODE>(tile, Tn, v, nval, out, off, n, total, d, tile_seg, head, tail, tflag, cin, vec, s_off,
-                                 s_v, s_f);
+            for (int k = 0; k < kIrrItems; ++k) {
+                acc = combine<OP>(acc, apply_map<F>(X[px(j_s + k)]));
+                if constexpr (SCAN) X[px(j_s + k)] = acc;
+            }
+            lead = cnt;
+        } else if (i == ie) {
+            for (int k = 0; k < cnt; ++k) {
+                acc = combine<OP>(acc, apply_map<F>(X[px(j_s + k)]));
+                if constexpr (SCAN) X[px(j_s + k)] = acc;
+            }
+            lead = cnt;
+        } else {
+            int j = j_s;
+            bool seen = false;
+            int ce = E32[2 * pe(i + 1)] - j0lo;
 #pragma unroll
-        for (int k = 0; k < kIrrItems; ++k) v[k] = vn[k];
-        nval = nn;
+            for (int k = 0; k < kIrrItems; ++k) {
+                const bool valid = k < cnt;
+                const bool end = valid && ce <= j;
+                const bool elt = valid && !end;
+                const T nacc = combine<OP>(acc, apply_map<F>(X[px(j)]));  // j <= ne: inside the buffer
+                if constexpr (SCAN) {
+                    if (elt) X[px(j)] = nacc;
+                } else {
+                    if (end) E32[2 * pe(i + 1)] = (int)to_bits<T>(acc);
+                    first = (end && first < 0) ? i : first;
+                }
+                seen = seen || end;
+                lead += (elt && !seen) ? 1 : 0;
+                i += end ? 1 : 0;
+                const int nc = E32[2 * pe(i + 1)] - j0lo;  // i + 1 <= ns + 1: inside (used only when i < ie)
+                ce = end ? (i < ie ? nc : 0x7fffffff) : ce;
+                acc = end ? d : (elt ? nacc : acc);
+                j += elt ? 1 : 0;
+            }
+            if constexpr (SCAN) first = seen ? 0 : -1;
+        }
+        uint32_t exf, aggf;
+        T exv, aggv;
+        const T init_v = start_f ? d : (SCAN ? carry_in : identity<OP, T>());
+        irr_cta_seg_scan<T, OP, kIrrThreads>(first >= 0 ? 1u : 0u, acc, start_f, init_v, exf, exv, aggf, aggv, s_v,
+                                             s_f);
+        if constexpr (SCAN) {
+            if (lead == kIrrItems) {
+#pragma unroll
+                for (int k = 0; k < kIrrItems; ++k) X[px(j_s + k)] = combine<OP>(exv, X[px(j_s + k)]);
+            } else {
+                for (int k = 0; k < lead; ++k) X[px(j_s + k)] = combine<OP>(exv, X[px(j_s + k)]);
+            }
+            __syncthreads();
+            for (int k = t; k < cur.ne; k += kIrrThreads) __stcs(out + cur.j0 + k, X[px(k)]);
+        } else {
+            if (first >= 0) {
+                const T v = combine<OP>(exv, from_bits<T>((uint32_t)E32[2 * pe(first + 1)]));
+                if (exf) {
+                    E32[2 * pe(first + 1)] = (int)to_bits<T>(v);
+                } else {  // segment i0 began in an earlier tile: its head piece
+                    head[b] = v;
+                    s_skip0 = 1;
+                }
+            }
+            if (t == kIrrThreads - 1) tail[b] = aggv;
+            __syncthreads();
+            if (t == 0) tflag[b] = aggf | (s_skip0 ? 2u : 0u);
+            for (int k = t + s_skip0; k < cur.ns; k += kIrrThreads)
+                __stcs(out + cur.i0 + k, from_bits<T>((uint32_t)E32[2 * pe(k + 1)]));
+        }
+        __syncthreads();  // buffer free for the tile after next
+        // ----------------
+        b = nb;
+        cur = nxt;
+        nb = nnb;
+        ni0 = pi0;
+        ni1 = pi1;
+    }
+    cp_async_wait<0>();
+}
+
+// segscan pass 1 (a warp per tile): the open tail, from the start of the
+// segment open at the tile's end (off[i1], with d) or the whole tile.
+template <typename T, int OP, int F>
+__global__ void __launch_bounds__(256) irr_mp_tail_kernel(const T* __restrict__ in, const int64_t* __restrict__ off,
+                                                          int64_t n, int64_t total, T d,
+                                                          const int64_t* __restrict__ coord, T* __restrict__ tail,
+                                                          uint32_t* __restrict__ tflag, int64_t Tn) {
+    const int lane = threadIdx.x & 31;
+    const int64_t b = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (b >= Tn) return;
+    const int64_t D1 = min((b + 1) * kIrrTile, n + total);
+    const int64_t j0 = b * kIrrTile - coord[b], i1 = coord[b + 1], j1 = D1 - i1;
+    const int64_t s = __ldg(off + i1);
+    const bool started = s >= j0;
+    const int64_t a = started ? s : j0;
+    T acc[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+    int64_t k = a + lane;
+    for (; k + 96 < j1; k += 128) {
+        T x[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) x[q] = __ldg(in + k + 32 * q);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[q] = combine<OP>(acc[q], apply_map<F>(x[q]));
+    }
+    for (; k < j1; k += 32) acc[0] = combine<OP>(acc[0], apply_map<F>(__ldg(in + k)));
+    const T r = warp_reduce<OP>(combine<OP>(combine<OP>(acc[0], acc[1]), combine<OP>(acc[2], acc[3])));
+    if (lane == 0) {
+        tail[b] = started ? combine<OP>(d, r) : r;
+        tflag[b] = started ? 1u : 0u;
     }
 }
 
-// pass 2: exclusive segmented scan over the tile tails, one CTA (chunks of
-// 1024 x 8 tiles, loads in flight): cin[t] = the open segment's value
-// entering tile t (from its start, with d).
+// Segmented scan of the tile tails in two parallel kernels over chunks of
+// kTsChunk tiles.  A: each chunk's aggregate (flag, value).
+constexpr int kTsChunk = 256;
+
 template <typename T, int OP>
-__global__ void __launch_bounds__(1024) irr_tile_scan_kernel(const T* __restrict__ tail,
-                                                             const uint32_t* __restrict__ tflag, T* __restrict__ cin,
-                                                             int64_t Tn) {
-    __shared__ T s_v[32];
-    __shared__ uint32_t s_f[32];
-    constexpr int PT = 8;
-    const int t = threadIdx.x, lane = t & 31, w = t >> 5;
-    T carry = identity<OP, T>();
-    for (int64_t c0 = 0; c0 < Tn; c0 += 1024 * PT) {
-        const int64_t k0 = c0 + (int64_t)t * PT;
-        T tv[PT];
-        uint32_t tf[PT];
-#pragma unroll
-        for (int q = 0; q < PT; ++q) {
-            const bool ok = k0 + q < Tn;
-            tv[q] = ok ? tail[k0 + q] : identity<OP, T>();
-            tf[q] = ok ? (tflag[k0 + q] & 1u) : 0u;
-        }
-        uint32_t f = 0;
-        T v = identity<OP, T>();
-#pragma unroll
-        for (int q = 0; q < PT; ++q) {
-            v = tf[q] ? tv[q] : combine<OP>(v, tv[q]);
-            f |= tf[q];
-        }
-        uint32_t fl = f;
-        T inc = v;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const T ov = __shfl_up_sync(0xffffffffu, inc, o);
-            const uint32_t of = __shfl_up_sync(0xffffffffu, fl, o);
-            if (lane >= o) {
-                if (!fl) inc = combine<OP>(ov, inc);
-                fl |= of;
-            }
-        }
-        if (lane == 31) {
-            s_v[w] = inc;
-            s_f[w] = fl;
-        }
-        T ex = __shfl_up_sync(0xffffffffu, inc, 1);
-        uint32_t exf = __shfl_up_sync(0xffffffffu, fl, 1);
-        if (lane == 0) {
-            ex = identity<OP, T>();
-            exf = 0;
-        }
-        __syncthreads();
-        T pw = carry, cv = carry;  // prefix of the warps before w / of the whole chunk, from the carry
-        for (int k = 0; k < 32; ++k) {
-            if (k < w) pw = s_f[k] ? s_v[k] : combine<OP>(pw, s_v[k]);
-            cv = s_f[k] ? s_v[k] : combine<OP>(cv, s_v[k]);
-        }
-        T run = exf ? ex : combine<OP>(pw, ex);
-#pragma unroll
-        for (int q = 0; q < PT; ++q) {
-            if (k0 + q < Tn) cin[k0 + q] = run;
-            run = tf[q] ? tv[q] : combine<OP>(run, tv[q]);
-        }
-        carry = cv;
-        __syncthreads();
+__global__ void __launch_bounds__(kTsChunk) irr_mp_ts_agg_kernel(const T* __restrict__ tail,
+                                                                 const uint32_t* __restrict__ tflag,
+                                                                 T* __restrict__ cagg, uint32_t* __restrict__ cflag,
+                                                                 int64_t Tn) {
+    __shared__ T s_v[kTsChunk / 32];
+    __shared__ uint32_t s_f[kTsChunk / 32];
+    const int64_t k = (int64_t)blockIdx.x * kTsChunk + threadIdx.x;
+    const bool ok = k < Tn;
+    uint32_t exf, aggf;
+    T exv, aggv;
+    irr_cta_seg_scan<T, OP, kTsChunk>(ok ? (tflag[k] & 1u) : 0u, ok ? tail[k] : identity<OP, T>(), 0u,
+                                      identity<OP, T>(), exf, exv, aggf, aggv, s_v, s_f);
+    if (threadIdx.x == 0) {
+        cagg[blockIdx.x] = aggv;
+        cflag[blockIdx.x] = aggf;
     }
+}
+
+// B: chunk c's prefix = the segmented fold of chunks 0..c-1, then the chunk's
+// exclusive scan: cin[k] (segscan) or the head fix-ups (segred).
+template <typename T, int OP, bool SEGRED>
+__global__ void __launch_bounds__(kTsChunk) irr_mp_ts_scan_kernel(const T* __restrict__ tail,
+                                                                  const uint32_t* __restrict__ tflag,
+                                                                  const T* __restrict__ cagg,
+                                                                  const uint32_t* __restrict__ cflag,
+                                                                  T* __restrict__ cin, const T* __restrict__ head,
+                                                                  const int64_t* __restrict__ coord,
+                                                                  T* __restrict__ out, int64_t Tn) {
+    __shared__ T s_v[kTsChunk / 32];
+    __shared__ uint32_t s_f[kTsChunk / 32];
+    const int c = blockIdx.x, t = threadIdx.x;
+    // prefix over chunks [0, c): thread t folds a contiguous block of them
+    const int per = (c + kTsChunk - 1) / kTsChunk;
+    uint32_t pf = 0;
+    T pv = identity<OP, T>();
+    for (int q = 0; q < per; ++q) {
+        const int k = t * per + q;
+        if (k < c) {
+            const uint32_t f = cflag[k];
+            const T v = cagg[k];
+            pv = f ? v : combine<OP>(pv, v);
+            pf |= f;
+        }
+    }
+    uint32_t exf, aggf, pref_f;
+    T exv, aggv, pref_v;
+    irr_cta_seg_scan<T, OP, kTsChunk>(pf, pv, 0u, identity<OP, T>(), exf, exv, pref_f, pref_v, s_v, s_f);
+    __syncthreads();  // s_v / s_f reused
+    const int64_t k = (int64_t)c * kTsChunk + t;
+    const bool ok = k < Tn;
+    const uint32_t tf = ok ? tflag[k] : 0u;
+    irr_cta_seg_scan<T, OP, kTsChunk>(tf & 1u, ok ? tail[k] : identity<OP, T>(), pref_f, pref_v, exf, exv, aggf,
+                                      aggv, s_v, s_f);
+    if (!ok) return;
+    if constexpr (SEGRED) {
+        if (tf & 2u) out[coord[k]] = combine<OP>(exv, head[k]);
+    } else {
+        cin[k] = exv;
+    }
+}
+
+// the persistent kernel's > 48 KB of dynamic shared memory (once per instantiation)
+template <typename T, int OP, int F, bool SCAN>
+void mp_prepare() {
+    static const bool once = [] {
+        cudaFuncSetAttribute(irr_mp_kernel<T, OP, F, SCAN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)kMpSmem);
+        return true;
+    }();
+    (void)once;
 }
 
 }  // namespace
 
-int64_t irr_tiles(int64_t total) { return ceil_div(total, kIrrTile); }
+int64_t irr_tiles(int64_t n, int64_t total) { return ceil_div(n + total, kIrrTile); }
 
-// [tile_seg: 8 B][head: 4 B][tail: 4 B][cin: 4 B][tflag: 4 B] per tile
-size_t irr_ws_bytes(int64_t total, int version) {
+// [coords: 8 B x (Tn + 1)][tail|flag|head|cin: 4 B x Tn each][chunk agg|flag: 4 B x chunks each]
+size_t irr_ws_bytes(int64_t n, int64_t total, int version) {
     if (version != IFL_V_FLAT && version != IFL_AUTO) return 0;
-    const int64_t Tn = irr_tiles(total);
-    return (size_t)Tn * 24 + 64;
+    const int64_t Tn = irr_tiles(n, total), C = ceil_div(Tn, kTsChunk);
+    return (size_t)(Tn + 1) * 8 + (size_t)Tn * 16 + (size_t)C * 8 + 64;
 }
 
 cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
@@ -521,30 +532,44 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
             }
             return cudaGetLastError();
         }
-        const int64_t Tn = irr_tiles(a.total);
-        int64_t* tile_seg = (int64_t*)a.ws;
-        T* head = (T*)(tile_seg + Tn);
-        T* tail = head + Tn;
-        T* cin = tail + Tn;
-        uint32_t* tflag = (uint32_t*)(cin + Tn);
-        cudaError_t e;
-        const unsigned gs = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(a.n, 256), 148 * 16));
-        if (scan) irr_claim_kernel<T, OP, false><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
-        else irr_claim_kernel<T, OP, true><<<gs, 256, 0, a.stream>>>(a.off, a.n, tile_seg, out, d);
-        if ((e = cudaGetLastError()) != cudaSuccess) return e;
-        const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
+        const int64_t Tn = irr_tiles(a.n, a.total);
+        if (Tn == 0) return cudaSuccess;
         if (Tn > 0x7fffffffLL) return cudaErrorInvalidValue;
-        if (scan)
-            irr_flat_kernel<T, OP, F, 1><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
-                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
-        else
-            irr_flat_kernel<T, OP, F, 0><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
-                in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
-        if (!scan) return cudaGetLastError();  // crossing segments were combined atomically
-        irr_tile_scan_kernel<T, OP><<<1, 1024, 0, a.stream>>>(tail, tflag, cin, Tn);
+        const int64_t C = ceil_div(Tn, kTsChunk);
+        int64_t* coord = (int64_t*)a.ws;
+        T* tail = (T*)(coord + Tn + 1);
+        uint32_t* tflag = (uint32_t*)(tail + Tn);
+        T* head = (T*)(tflag + Tn);
+        T* cin = head + Tn;
+        T* cagg = cin + Tn;
+        uint32_t* cflag = (uint32_t*)(cagg + C);
+        const unsigned G = (unsigned)std::min<int64_t>(Tn, (int64_t)148 * kMpCtasPerSm);
+        cudaError_t e;
+        irr_mp_partition_kernel<<<(unsigned)ceil_div((Tn + 1) * 8, 256), 256, 0, a.stream>>>(a.off, a.n, a.total, Tn,
+                                                                                              coord);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
-        irr_flat_kernel<T, OP, F, 2><<<(unsigned)ceil_div(Tn, kIrrTPB), kIrrThreads, 0, a.stream>>>(
-            in, out, a.off, a.n, a.total, d, tile_seg, head, tail, tflag, cin, vec);
+        if (!scan) {
+            mp_prepare<T, OP, F, false>();
+            irr_mp_kernel<T, OP, F, false><<<G, kIrrThreads, kMpSmem, a.stream>>>(
+                in, out, a.off, a.n, a.total, d, coord, tail, tflag, head, cin, Tn);
+        } else {
+            irr_mp_tail_kernel<T, OP, F><<<(unsigned)ceil_div(Tn * 32, 256), 256, 0, a.stream>>>(
+                in, a.off, a.n, a.total, d, coord, tail, tflag, Tn);
+        }
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        irr_mp_ts_agg_kernel<T, OP><<<(unsigned)C, kTsChunk, 0, a.stream>>>(tail, tflag, cagg, cflag, Tn);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        if (!scan) {
+            irr_mp_ts_scan_kernel<T, OP, true><<<(unsigned)C, kTsChunk, 0, a.stream>>>(tail, tflag, cagg, cflag, cin,
+                                                                                       head, coord, out, Tn);
+            return cudaGetLastError();
+        }
+        irr_mp_ts_scan_kernel<T, OP, false><<<(unsigned)C, kTsChunk, 0, a.stream>>>(tail, tflag, cagg, cflag, cin,
+                                                                                    head, coord, out, Tn);
+        if ((e = cudaGetLastError()) != cudaSuccess) return e;
+        mp_prepare<T, OP, F, true>();
+        irr_mp_kernel<T, OP, F, true><<<G, kIrrThreads, kMpSmem, a.stream>>>(in, out, a.off, a.n, a.total, d, coord,
+                                                                            tail, tflag, head, cin, Tn);
         return cudaGetLastError();
     });
 }

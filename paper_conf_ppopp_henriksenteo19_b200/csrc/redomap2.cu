@@ -5,8 +5,9 @@
 //            (paper version 1): every (i, j, k) parallel -- the m-long dot
 //            products are split across CTAs (split-K), partials reduced in a
 //            deterministic second pass.  For degenerate shapes (n*p small).
-//   V_MIDDLE segmap^1 <i><j> (segred^0 <k> ...): a warp per output element,
-//            lanes split k, shuffle-tree reduction.
+//   V_MIDDLE segmap^1 <i><j> (segred^0 <k> ...): a group of 1-8 warps per
+//            output element (more when few outputs reduce a long k), lanes
+//            split k, shuffle-tree reduction.
 //   V_TOP    segmap^1 <i><j> (redomap sequential in k) with block tiling and
 //            register tiling (paper versions 2 and 3): a 128x128 output tile
 //            per CTA, 8x8 per thread, k-tiles double-buffered in shared
@@ -73,45 +74,62 @@ __global__ void __launch_bounds__(256) transpose_kernel(const Tin* __restrict__ 
 
 // ------------------------------------------------------------- V_MIDDLE
 
-template <typename Tin, bool VEC>
+// WPO warps per output (the group of segred^0): 1 when the outputs fill the
+// GPU, up to 8 (the whole CTA) when few outputs each reduce a long k.
+template <typename Tin, bool VEC, int WPO>
 __global__ void __launch_bounds__(256) mm_mid_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
                                                      float* __restrict__ C, int64_t n, int64_t m, int64_t p) {
-    constexpr int E = VecE<Tin>::E;
-    const int lane = threadIdx.x & 31;
-    const int64_t o = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
-    if (o >= n * p) return;
-    const int64_t i = o / p, j = o - i * p;
-    const Tin* a = A + i * m;
-    const Tin* b = Bt + j * m;
+    constexpr int E = VecE<Tin>::E, G = 32 * WPO;
+    __shared__ float red[8];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    const int gl = (w % WPO) * 32 + lane;  // lane within the group
+    const int64_t o = (int64_t)blockIdx.x * (8 / WPO) + w / WPO;
+    const bool live = o < n * p;
     float acc[4] = {0.f, 0.f, 0.f, 0.f};
-    if (VEC) {
-        int64_t k = (int64_t)lane * E;
-        for (; k + E + 32 * E <= m; k += 64 * E) {
-            float x0[E], y0[E], x1[E], y1[E];
-            load16(a + k, x0);
-            load16(b + k, y0);
-            load16(a + k + 32 * E, x1);
-            load16(b + k + 32 * E, y1);
+    if (live) {
+        const int64_t i = o / p, j = o - i * p;
+        const Tin* a = A + i * m;
+        const Tin* b = Bt + j * m;
+        if (VEC) {
+            int64_t k = (int64_t)gl * E;
+            for (; k + E + G * E <= m; k += 2 * G * E) {
+                float x0[E], y0[E], x1[E], y1[E];
+                load16(a + k, x0);
+                load16(b + k, y0);
+                load16(a + k + G * E, x1);
+                load16(b + k + G * E, y1);
 #pragma unroll
-            for (int e = 0; e < E; ++e) {
-                acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
-                acc[(e + 2) & 3] = fmaf(x1[e], y1[e], acc[(e + 2) & 3]);
+                for (int e = 0; e < E; ++e) {
+                    acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+                    acc[(e + 2) & 3] = fmaf(x1[e], y1[e], acc[(e + 2) & 3]);
+                }
             }
-        }
-        for (; k + E <= m; k += 32 * E) {
-            float x0[E], y0[E];
-            load16(a + k, x0);
-            load16(b + k, y0);
+            for (; k + E <= m; k += G * E) {
+                float x0[E], y0[E];
+                load16(a + k, x0);
+                load16(b + k, y0);
 #pragma unroll
-            for (int e = 0; e < E; ++e) acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+                for (int e = 0; e < E; ++e) acc[e & 3] = fmaf(x0[e], y0[e], acc[e & 3]);
+            }
+            for (int64_t kk = m - (m % E) + gl; kk < m; kk += G) acc[0] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[0]);
+        } else {
+            for (int64_t kk = gl; kk < m; kk += G) acc[kk & 3] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[kk & 3]);
         }
-        for (int64_t kk = m - (m % E) + lane; kk < m; kk += 32) acc[0] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[0]);
-    } else {
-        for (int64_t kk = lane; kk < m; kk += 32) acc[kk & 3] = fmaf(to_f(a[kk]), to_f(b[kk]), acc[kk & 3]);
     }
     float s = (acc[0] + acc[1]) + (acc[2] + acc[3]);
     s = warp_reduce<OP_SUM>(s);
-    if (lane == 0) C[o] = s;
+    if constexpr (WPO == 1) {
+        if (lane == 0 && live) C[o] = s;
+    } else {
+        if (lane == 0) red[w] = s;
+        __syncthreads();
+        if (live && w % WPO == 0 && lane == 0) {
+            float r = 0.f;
+#pragma unroll
+            for (int q = 0; q < WPO; ++q) r += red[w + q];
+            C[o] = r;
+        }
+    }
 }
 
 // -------------------------------------------------------- tiled SIMT kernel
@@ -632,10 +650,23 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
             part, a.C, outs, (int)splits);
         return cudaGetLastError();
     }
-    if (version == 1) {  // ---- V_MIDDLE: a warp per output
-        const int64_t grid = ceil_div(outs, 8);
-        if (vec) mm_mid_kernel<Tin, true><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
-        else mm_mid_kernel<Tin, false><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+    if (version == 1) {  // ---- V_MIDDLE: a group of warps per output
+        // group size: warps per output so that >= 148 x 32 warps run, each with
+        // >= 4 vector rounds of k
+        int wpo = 1;
+        while (wpo < 8 && outs * wpo < (int64_t)148 * 32 && a.m >= (int64_t)wpo * 2 * 32 * E * 4) wpo *= 2;
+        const int64_t grid = ceil_div(outs * wpo, 8);
+        auto go = [&](auto wc) {
+            constexpr int W = decltype(wc)::value;
+            if (vec) mm_mid_kernel<Tin, true, W><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+            else mm_mid_kernel<Tin, false, W><<<(unsigned)grid, 256, 0, a.stream>>>(A, Bt, a.C, a.n, a.m, a.p);
+        };
+        switch (wpo) {
+        case 8: go(std::integral_constant<int, 8>{}); break;
+        case 4: go(std::integral_constant<int, 4>{}); break;
+        case 2: go(std::integral_constant<int, 2>{}); break;
+        default: go(std::integral_constant<int, 1>{}); break;
+        }
         return cudaGetLastError();
     }
     // ---- V_TOP: output tiles, sequential k (tensor cores for bf16)

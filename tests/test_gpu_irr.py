@@ -38,10 +38,13 @@ def descriptors():
         list(rng.integers(0, 40, 3000)),         # short, ragged
         list(rng.integers(0, 3000, 60)),         # long, ragged
         [1] * 9000,                              # unit segments
+        [0] * 10000 + [50000] + [0] * 10000,     # one long segment between runs of empties
+        [0] * 4096 + [1] + [0] * 4095 + [2],     # merge-path tiles of ends only
     ):
         lens = np.asarray(lens, np.int64)
         out.append(np.r_[0, np.cumsum(lens)].astype(np.int64))
     out.append(gen.irregular_offsets(9, 4000, 24.0))  # Pareto tail (the bench recipe)
+    out.append(gen.irregular_offsets(13, 60000, 1.0))  # the bench's mean-1 mix (mostly empty / unit segments)
     return out
 
 
