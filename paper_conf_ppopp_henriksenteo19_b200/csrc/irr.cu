@@ -123,25 +123,13 @@ __global__ void __launch_bounds__(256) irr_mid_kernel(const T* __restrict__ in, 
 //              coalesced (two reads + one write per element when segments are
 //              long; one read + one write when they are short).
 
-// Shared-memory staging, padded so the thread-blocked walk (lanes ~16 items
-// apart) is bank-conflict-free: ends E[k] = off[i0 + k] (int64, one pad word
-// per 16), elements X[k] (one pad word per 32).
-__device__ __forceinline__ int pe(int k) { return k + (k >> 4); }
-__device__ __forceinline__ int px(int k) { return k + (k >> 5); }
-__host__ __device__ constexpr int mp_xoff(int ns) { return (((ns + 1) + ((ns + 1) >> 4) + 1) * 8 + 15) & ~15; }
-constexpr int kMpBuf = mp_xoff((int)kIrrTile) + 16 * 4;  // ns = kIrrTile, ne = 0 is the largest tile
-constexpr int kMpCtasPerSm = 3;
-constexpr size_t kMpSmem = 2 * (size_t)kMpBuf;
-
-__device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async4(void* smem, const void* gmem) {
-    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+// Shared-memory staging (int32 ends relative to the tile's first element,
+// elements), padded by one word per 32 so the thread-blocked walk (lanes ~16
+// items apart) is bank-conflict-free.
+constexpr int kMpSmem = (int)kIrrTile + (int)kIrrTile / 32 + 1;  // pd(kIrrTile) + 1
+constexpr int kMpThreads = 128, kMpItems = 32, kMpItemsLog2 = 5;
+static_assert(kMpThreads * kMpItems == kIrrTile && (1 << kMpItemsLog2) == kMpItems, "merge-path tile");
+__device__ __forceinline__ int pd(int k) { return k + (k >> 5); }
 
 // CTA-wide exclusive scan of (flag, value) thread pieces under the segmented
 // operator (f1,v1).(f2,v2) = (f1|f2, f2 ? v2 : v1 (+) v2), seeded with an
@@ -218,179 +206,181 @@ __global__ void __launch_bounds__(256) irr_mp_partition_kernel(const int64_t* __
     if (live && sub == 0) coord[b] = lo;
 }
 
-struct MpTile {
-    int64_t i0, j0;
-    int ns, ne;
-};
-
-__device__ __forceinline__ MpTile mp_tile(int64_t b, int64_t i0, int64_t i1, int64_t W) {
-    MpTile t;
-    const int64_t D0 = b * kIrrTile, D1 = min(D0 + kIrrTile, W);
-    t.i0 = i0;
-    t.j0 = D0 - i0;
-    t.ns = (int)(i1 - i0);
-    t.ne = (int)((D1 - i1) - t.j0);
-    return t;
+// Elements-only segred tiles (no segment end: the tile lies inside one
+// segment): a plain CTA reduction, float4 loads striped across the CTA from
+// the tile's 16-byte-aligned base (no shared-memory staging).
+template <typename T, int OP, int F>
+__device__ __forceinline__ void mp_elems_red(const T* __restrict__ in, int64_t j0, uint32_t start_f, T init_v,
+                                             int64_t b, T* __restrict__ tail, uint32_t* __restrict__ tflag, T* s_v,
+                                             uint32_t* s_f) {
+    const int t = threadIdx.x, R = (int)(j0 & 3);
+    const T* base = in + (j0 - R);  // group g = elements [4g, 4g + 4) of base; the tile is [R, R + kIrrTile)
+    T acc[4] = {identity<OP, T>(), identity<OP, T>(), identity<OP, T>(), identity<OP, T>()};
+    constexpr int NG = (int)kIrrTile / 4 / kMpThreads;
+    typename Vec4<T>::type u[NG];
+#pragma unroll
+    for (int q = 0; q < NG; ++q) u[q] = ldg_stream4(base + 4 * (t + kMpThreads * q));
+#pragma unroll
+    for (int q = 0; q < NG; ++q) {
+        T e[4];
+        unpack4<T>(u[q], e);
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const T m = apply_map<F>(e[c]);
+            acc[c] = (q == 0 && t == 0 && c < R) ? acc[c] : combine<OP>(acc[c], m);
+        }
+    }
+    if (R != 0 && t == 0) {  // the tile's last R elements: group kIrrTile / 4
+        T e[4];
+        unpack4<T>(ldg_stream4(base + kIrrTile), e);
+#pragma unroll
+        for (int c = 0; c < 4; ++c)
+            if (c < R) acc[c] = combine<OP>(acc[c], apply_map<F>(e[c]));
+    }
+    uint32_t exf, aggf;
+    T exv, aggv;
+    irr_cta_seg_scan<T, OP, kMpThreads>(0u, combine<OP>(combine<OP>(acc[0], acc[1]), combine<OP>(acc[2], acc[3])),
+                                        start_f, init_v, exf, exv, aggf, aggv, s_v, s_f);
+    if (t == kMpThreads - 1) {
+        tail[b] = aggv;
+        tflag[b] = aggf;
+    }
 }
 
-// Issue the cp.async copies of a tile into buffer `buf` (one commit group).
-template <typename T>
-__device__ __forceinline__ void mp_issue(const T* in, const int64_t* off, const MpTile& tl, uint8_t* buf) {
-    int64_t* E = reinterpret_cast<int64_t*>(buf);
-    T* X = reinterpret_cast<T*>(buf + mp_xoff(tl.ns));
-    for (int k = threadIdx.x; k <= tl.ns; k += kIrrThreads) cp_async8(E + pe(k), off + tl.i0 + k);
-    for (int k = threadIdx.x; k < tl.ne; k += kIrrThreads) cp_async4(X + px(k), in + tl.j0 + k);
-    cp_async_commit();
-}
-
-// Pass 1 of segred (SCAN = false) / pass 3 of segscan (SCAN = true) over
-// tiles blockIdx.x, +gridDim.x, ... with the next tile in flight.
+// Pass 1 of segred (SCAN = false) / pass 3 of segscan (SCAN = true), a tile
+// per CTA of 128 threads x 32 items (twelve CTAs per SM).  The tile's ends
+// (int32, relative to its first element) and elements share one padded
+// shared-memory array: ends at [0, ns), elements at [ns, ns + ne).
 // segscan: in may equal out (a tile reads and writes only its own elements;
-// cp.async reads are issued before that tile's stores).
+// coherent loads).
 template <typename T, int OP, int F, bool SCAN>
-__global__ void __launch_bounds__(kIrrThreads, kMpCtasPerSm)
-    irr_mp_kernel(const T* in, T* out, const int64_t* __restrict__ off, int64_t n, int64_t total, T d,
-                  const int64_t* __restrict__ coord, T* __restrict__ tail, uint32_t* __restrict__ tflag,
-                  T* __restrict__ head, const T* __restrict__ cin, int64_t Tn) {
-    extern __shared__ __align__(16) uint8_t mp_raw[];
-    __shared__ T s_v[kIrrThreads / 32];
-    __shared__ uint32_t s_f[kIrrThreads / 32];
+__global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out, const int64_t* __restrict__ off,
+                                                            int64_t n, int64_t total, T d,
+                                                            const int64_t* __restrict__ coord, T* __restrict__ tail,
+                                                            uint32_t* __restrict__ tflag, T* __restrict__ head,
+                                                            const T* __restrict__ cin, bool vec) {
+    __shared__ int s_b[kMpSmem];  // ends (segred: then segment values), then elements (bit patterns)
+    __shared__ T s_v[kMpThreads / 32];
+    __shared__ uint32_t s_f[kMpThreads / 32];
+    __shared__ int s_start[kMpThreads];
     __shared__ int s_skip0;
-    __shared__ int s_start[kIrrThreads];
     const int t = threadIdx.x;
-    const int64_t G = gridDim.x, W = n + total;
-    int64_t b = blockIdx.x;
-    if (b >= Tn) return;
-    MpTile cur = mp_tile(b, coord[b], coord[b + 1], W);
-    mp_issue<T>(in, off, cur, mp_raw);
-    int64_t nb = b + G, ni0 = 0, ni1 = 0;
-    if (nb < Tn) {
-        ni0 = coord[nb];
-        ni1 = coord[nb + 1];
+    const int64_t b = blockIdx.x;
+    const int64_t D0 = b * kIrrTile, D1 = min(D0 + kIrrTile, n + total);
+    const int64_t i0 = coord[b], i1 = coord[b + 1];
+    const int64_t j0 = D0 - i0;
+    const int ns = (int)(i1 - i0), ne = (int)((D1 - i1) - j0);
+    const uint32_t start_f = __ldg(off + i0) >= j0 ? 1u : 0u;
+    T init_v = start_f ? d : identity<OP, T>();
+    if constexpr (SCAN) {
+        if (!start_f) init_v = cin[b];
+    } else {
+        if (ns == 0 && ne == (int)kIrrTile && vec && (j0 & ~(int64_t)3) + kIrrTile + 4 <= total) {
+            mp_elems_red<T, OP, F>(in, j0, start_f, init_v, b, tail, tflag, s_v, s_f);
+            return;
+        }
     }
-    for (int r = 0; b < Tn; ++r) {
-        uint8_t* buf = mp_raw + (size_t)(r & 1) * kMpBuf;
-        MpTile nxt{};
-        if (nb < Tn) {
-            nxt = mp_tile(nb, ni0, ni1, W);
-            mp_issue<T>(in, off, nxt, mp_raw + (size_t)((r + 1) & 1) * kMpBuf);
-        } else {
-            cp_async_commit();
-        }
-        // coordinates two tiles ahead, in flight during this tile
-        const int64_t nnb = nb + G;
-        int64_t pi0 = 0, pi1 = 0;
-        if (nnb < Tn) {
-            pi0 = coord[nnb];
-            pi1 = coord[nnb + 1];
-        }
-        T carry_in = identity<OP, T>();
-        if constexpr (SCAN) carry_in = cin[b];
-        cp_async_wait<1>();
-        if (t == 0) s_skip0 = 0;
-        __syncthreads();
-        // ---------------- the tile
-        int* E32 = reinterpret_cast<int*>(buf);  // low words of E
-        T* X = reinterpret_cast<T*>(buf + mp_xoff(cur.ns));
-        const int j0lo = (int)cur.j0;
-        const uint32_t start_f = reinterpret_cast<const int64_t*>(buf)[0] >= cur.j0 ? 1u : 0u;
-        const int Wt = cur.ns + cur.ne;
-        const int d0 = min(t * kIrrItems, Wt), cnt = min(d0 + kIrrItems, Wt) - d0;
-        // thread starts without a search: end k sits at merge position
-        // pos(k) = k + (its end - j0) (strictly increasing), so the thread
-        // whose first item is 16u (pos(k-1) < 16u <= pos(k)) starts at end k;
-        // threads past the last end start at ns
-        for (int k = t; k < cur.ns; k += kIrrThreads) {
-            const int pk = k + (E32[2 * pe(k + 1)] - j0lo);
-            const int pp = k == 0 ? -1 : (k - 1) + (E32[2 * pe(k)] - j0lo);
-            for (int u = (pp >> 4) + 1; u * kIrrItems <= pk; ++u) s_start[u] = k;
-        }
-        if (t * kIrrItems > (cur.ns == 0 ? -1 : (cur.ns - 1) + (E32[2 * pe(cur.ns)] - j0lo))) s_start[t] = cur.ns;
-        __syncthreads();  // (segred: also every read of the ends is done before segment values overwrite them)
-        int i = s_start[t];
-        const int ie = t + 1 < kIrrThreads ? s_start[t + 1] : cur.ns;
-        const int j_s = d0 - i;
-        T acc = identity<OP, T>();
-        int first = -1;  // segred: the thread's first segment end
-        int lead = 0;    // segscan: elements before the thread's first segment start
-        if (i == ie && cnt == kIrrItems) {  // elements only
+    auto X = [&](int j) -> int& { return s_b[pd(ns + j)]; };
+    // ---- staging
+#pragma unroll 4
+    for (int k = t; k < ns; k += kMpThreads) s_b[pd(k)] = (int)(__ldg(off + i0 + 1 + k) - j0);
+    if constexpr (SCAN) {
+#pragma unroll 8
+        for (int k = t; k < ne; k += kMpThreads) X(k) = (int)to_bits<T>(__ldcs(in + j0 + k));
+    } else {
+#pragma unroll 8
+        for (int k = t; k < ne; k += kMpThreads) X(k) = (int)to_bits<T>(__ldg(in + j0 + k));
+    }
+    if (t == 0) s_skip0 = 0;
+    __syncthreads();
+    const int Wt = ns + ne;
+    const int d0 = min(t * kMpItems, Wt), cnt = min(d0 + kMpItems, Wt) - d0;
+    // thread starts without a search: end k sits at merge position
+    // pos(k) = k + s_b[k] (strictly increasing), so the thread whose first
+    // item is 32u (pos(k-1) < 32u <= pos(k)) starts at end k; threads past
+    // the last end start at ns
+    for (int k = t; k < ns; k += kMpThreads) {
+        const int pk = k + s_b[pd(k)];
+        const int pp = k == 0 ? -1 : (k - 1) + s_b[pd(k - 1)];
+        for (int u = (pp >> kMpItemsLog2) + 1; u * kMpItems <= pk; ++u) s_start[u] = k;  // pp >= -1: floor
+    }
+    if (t * kMpItems > (ns == 0 ? -1 : (ns - 1) + s_b[pd(ns - 1)])) s_start[t] = ns;
+    __syncthreads();  // (segred: also every read of the ends is done before segment values overwrite them)
+    int i = s_start[t];
+    const int ie = t + 1 < kMpThreads ? s_start[t + 1] : ns;
+    const int j_s = d0 - i;
+    T acc = identity<OP, T>();
+    int first = -1;  // segred: the thread's first segment end
+    int lead = 0;    // segscan: elements before the thread's first segment start
+    if (i == ie && cnt == kMpItems) {  // elements only
 #pragma unroll
-            for (int k = 0; k < kIrrItems; ++k) {
-                acc = combine<OP>(acc, apply_map<F>(X[px(j_s + k)]));
-                if constexpr (SCAN) X[px(j_s + k)] = acc;
-            }
-            lead = cnt;
-        } else if (i == ie) {
-            for (int k = 0; k < cnt; ++k) {
-                acc = combine<OP>(acc, apply_map<F>(X[px(j_s + k)]));
-                if constexpr (SCAN) X[px(j_s + k)] = acc;
-            }
-            lead = cnt;
-        } else {
-            int j = j_s;
-            bool seen = false;
-            int ce = E32[2 * pe(i + 1)] - j0lo;
-#pragma unroll
-            for (int k = 0; k < kIrrItems; ++k) {
-                const bool valid = k < cnt;
-                const bool end = valid && ce <= j;
-                const bool elt = valid && !end;
-                const T nacc = combine<OP>(acc, apply_map<F>(X[px(j)]));  // j <= ne: inside the buffer
-                if constexpr (SCAN) {
-                    if (elt) X[px(j)] = nacc;
-                } else {
-                    if (end) E32[2 * pe(i + 1)] = (int)to_bits<T>(acc);
-                    first = (end && first < 0) ? i : first;
-                }
-                seen = seen || end;
-                lead += (elt && !seen) ? 1 : 0;
-                i += end ? 1 : 0;
-                const int nc = E32[2 * pe(i + 1)] - j0lo;  // i + 1 <= ns + 1: inside (used only when i < ie)
-                ce = end ? (i < ie ? nc : 0x7fffffff) : ce;
-                acc = end ? d : (elt ? nacc : acc);
-                j += elt ? 1 : 0;
-            }
-            if constexpr (SCAN) first = seen ? 0 : -1;
+        for (int k = 0; k < kMpItems; ++k) {
+            acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j_s + k))));
+            if constexpr (SCAN) X(j_s + k) = (int)to_bits<T>(acc);
         }
-        uint32_t exf, aggf;
-        T exv, aggv;
-        const T init_v = start_f ? d : (SCAN ? carry_in : identity<OP, T>());
-        irr_cta_seg_scan<T, OP, kIrrThreads>(first >= 0 ? 1u : 0u, acc, start_f, init_v, exf, exv, aggf, aggv, s_v,
-                                             s_f);
-        if constexpr (SCAN) {
-            if (lead == kIrrItems) {
+        lead = cnt;
+    } else if (i == ie) {
+        for (int k = 0; k < cnt; ++k) {
+            acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j_s + k))));
+            if constexpr (SCAN) X(j_s + k) = (int)to_bits<T>(acc);
+        }
+        lead = cnt;
+    } else {
+        int j = j_s;
+        bool seen = false;
+        int ce = s_b[pd(i)];
 #pragma unroll
-                for (int k = 0; k < kIrrItems; ++k) X[px(j_s + k)] = combine<OP>(exv, X[px(j_s + k)]);
+        for (int k = 0; k < kMpItems; ++k) {
+            const bool valid = k < cnt;
+            const bool end = valid && ce <= j;
+            const bool elt = valid && !end;
+            const T nacc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j))));  // j <= ne: inside
+            if constexpr (SCAN) {
+                if (elt) X(j) = (int)to_bits<T>(nacc);
             } else {
-                for (int k = 0; k < lead; ++k) X[px(j_s + k)] = combine<OP>(exv, X[px(j_s + k)]);
+                if (end) s_b[pd(i)] = (int)to_bits<T>(acc);
+                first = (end && first < 0) ? i : first;
             }
-            __syncthreads();
-            for (int k = t; k < cur.ne; k += kIrrThreads) __stcs(out + cur.j0 + k, X[px(k)]);
-        } else {
-            if (first >= 0) {
-                const T v = combine<OP>(exv, from_bits<T>((uint32_t)E32[2 * pe(first + 1)]));
-                if (exf) {
-                    E32[2 * pe(first + 1)] = (int)to_bits<T>(v);
-                } else {  // segment i0 began in an earlier tile: its head piece
-                    head[b] = v;
-                    s_skip0 = 1;
-                }
-            }
-            if (t == kIrrThreads - 1) tail[b] = aggv;
-            __syncthreads();
-            if (t == 0) tflag[b] = aggf | (s_skip0 ? 2u : 0u);
-            for (int k = t + s_skip0; k < cur.ns; k += kIrrThreads)
-                __stcs(out + cur.i0 + k, from_bits<T>((uint32_t)E32[2 * pe(k + 1)]));
+            seen = seen || end;
+            lead += (elt && !seen) ? 1 : 0;
+            i += end ? 1 : 0;
+            const int nc = s_b[pd(i)];  // read only when i < ie
+            ce = end ? (i < ie ? nc : 0x7fffffff) : ce;
+            acc = end ? d : (elt ? nacc : acc);
+            j += elt ? 1 : 0;
         }
-        __syncthreads();  // buffer free for the tile after next
-        // ----------------
-        b = nb;
-        cur = nxt;
-        nb = nnb;
-        ni0 = pi0;
-        ni1 = pi1;
+        if constexpr (SCAN) first = seen ? 0 : -1;
     }
-    cp_async_wait<0>();
+    uint32_t exf, aggf;
+    T exv, aggv;
+    irr_cta_seg_scan<T, OP, kMpThreads>(first >= 0 ? 1u : 0u, acc, start_f, init_v, exf, exv, aggf, aggv, s_v, s_f);
+    if constexpr (SCAN) {
+        if (lead == kMpItems) {
+#pragma unroll
+            for (int k = 0; k < kMpItems; ++k)
+                X(j_s + k) = (int)to_bits<T>(combine<OP>(exv, from_bits<T>((uint32_t)X(j_s + k))));
+        } else {
+            for (int k = 0; k < lead; ++k)
+                X(j_s + k) = (int)to_bits<T>(combine<OP>(exv, from_bits<T>((uint32_t)X(j_s + k))));
+        }
+        __syncthreads();
+#pragma unroll 8
+        for (int k = t; k < ne; k += kMpThreads) __stcs(out + j0 + k, from_bits<T>((uint32_t)X(k)));
+    } else {
+        if (first >= 0) {
+            const T v = combine<OP>(exv, from_bits<T>((uint32_t)s_b[pd(first)]));
+            if (exf) {
+                s_b[pd(first)] = (int)to_bits<T>(v);
+            } else {  // segment i0 began in an earlier tile: its head piece
+                head[b] = v;
+                s_skip0 = 1;
+            }
+        }
+        if (t == kMpThreads - 1) tail[b] = aggv;
+        __syncthreads();
+        if (t == 0) tflag[b] = aggf | (s_skip0 ? 2u : 0u);
+        for (int k = t + s_skip0; k < ns; k += kMpThreads) __stcs(out + i0 + k, from_bits<T>((uint32_t)s_b[pd(k)]));
+    }
 }
 
 // segscan pass 1 (a warp per tile): the open tail, from the start of the
@@ -491,17 +481,6 @@ __global__ void __launch_bounds__(kTsChunk) irr_mp_ts_scan_kernel(const T* __res
     }
 }
 
-// the persistent kernel's > 48 KB of dynamic shared memory (once per instantiation)
-template <typename T, int OP, int F, bool SCAN>
-void mp_prepare() {
-    static const bool once = [] {
-        cudaFuncSetAttribute(irr_mp_kernel<T, OP, F, SCAN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             (int)kMpSmem);
-        return true;
-    }();
-    (void)once;
-}
-
 }  // namespace
 
 int64_t irr_tiles(int64_t n, int64_t total) { return ceil_div(n + total, kIrrTile); }
@@ -543,15 +522,14 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         T* cin = head + Tn;
         T* cagg = cin + Tn;
         uint32_t* cflag = (uint32_t*)(cagg + C);
-        const unsigned G = (unsigned)std::min<int64_t>(Tn, (int64_t)148 * kMpCtasPerSm);
+        const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
         cudaError_t e;
         irr_mp_partition_kernel<<<(unsigned)ceil_div((Tn + 1) * 8, 256), 256, 0, a.stream>>>(a.off, a.n, a.total, Tn,
                                                                                               coord);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
         if (!scan) {
-            mp_prepare<T, OP, F, false>();
-            irr_mp_kernel<T, OP, F, false><<<G, kIrrThreads, kMpSmem, a.stream>>>(
-                in, out, a.off, a.n, a.total, d, coord, tail, tflag, head, cin, Tn);
+            irr_mp_kernel<T, OP, F, false><<<(unsigned)Tn, kMpThreads, 0, a.stream>>>(
+                in, out, a.off, a.n, a.total, d, coord, tail, tflag, head, cin, vec);
         } else {
             irr_mp_tail_kernel<T, OP, F><<<(unsigned)ceil_div(Tn * 32, 256), 256, 0, a.stream>>>(
                 in, a.off, a.n, a.total, d, coord, tail, tflag, Tn);
@@ -567,9 +545,8 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         irr_mp_ts_scan_kernel<T, OP, false><<<(unsigned)C, kTsChunk, 0, a.stream>>>(tail, tflag, cagg, cflag, cin,
                                                                                     head, coord, out, Tn);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
-        mp_prepare<T, OP, F, true>();
-        irr_mp_kernel<T, OP, F, true><<<G, kIrrThreads, kMpSmem, a.stream>>>(in, out, a.off, a.n, a.total, d, coord,
-                                                                            tail, tflag, head, cin, Tn);
+        irr_mp_kernel<T, OP, F, true><<<(unsigned)Tn, kMpThreads, 0, a.stream>>>(in, out, a.off, a.n, a.total, d,
+                                                                                  coord, tail, tflag, head, cin, vec);
         return cudaGetLastError();
     });
 }
