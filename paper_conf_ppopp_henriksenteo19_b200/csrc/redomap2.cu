@@ -14,7 +14,9 @@
 //            memory.  bf16 inputs take the tcgen05/TMEM/TMA tensor-core kernel
 //            (redomap2_tc.cu) when the shape allows.
 // A is [n][m]; B is yss^T as [p][m] (b_kmajor = 1, the array P:122 maps over)
-// or yss as [m][p] (b_kmajor = 0: transposed into the workspace first).
+// or yss as [m][p] (b_kmajor = 0: read in place by the SIMT tile kernels and
+// the skinny engine; transposed into the workspace first for V_MIDDLE, the
+// row-level leaves and the tcgen05 kernel).
 // Inputs f32 or bf16, accumulation and C in f32.
 #include <cuda_bf16.h>
 
@@ -139,10 +141,13 @@ __global__ void __launch_bounds__(256) mm_mid_kernel(const Tin* __restrict__ A, 
 // k-tile prefetched into registers while the current one is multiplied.
 // blockIdx.z = k-split: k-tiles [z*kps, (z+1)*kps); partial tiles go to
 // part[z] when gridDim.z > 1 (V_FLAT's split-K), else straight to C.
-template <typename Tin, int BM, int BN, int BK, bool VEC>
+// BKM = false: B is yss itself, [m][p] (row-major, P:122 before the
+// transpose): its k-tile rows are read along p (coalesced, 16-byte vectors
+// when bvec) straight into the k-major shared tile -- no transposition pass.
+template <typename Tin, int BM, int BN, int BK, bool VEC, bool BKM>
 __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict__ A, const Tin* __restrict__ Bt,
                                                            float* __restrict__ C, float* __restrict__ part, int64_t n,
-                                                           int64_t m, int64_t p, int64_t kps) {
+                                                           int64_t m, int64_t p, int64_t kps, bool bvec) {
     constexpr int TM = BM / 16, TN = BN / 16;
     constexpr int EPT = BM * BK / 256;  // k-values each thread stages per tile (BM == BN)
     static_assert(BM == BN && EPT >= 1 && BK % EPT == 0, "tile config");
@@ -153,9 +158,11 @@ __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict
     const int64_t row0 = (int64_t)blockIdx.y * BM, col0 = (int64_t)blockIdx.x * BN;
     const int lr = tid / TPR, lk = (tid % TPR) * EPT;
     float ra[EPT], rb[EPT];
-    const bool arow = row0 + lr < n, brow = col0 + lr < p;
+    const bool arow = row0 + lr < n, brow = BKM && col0 + lr < p;
     const Tin* ap = A + (arow ? (row0 + lr) * m : 0);
     const Tin* bp = Bt + (brow ? (col0 + lr) * m : 0);
+    // row-major B: thread stages EPT consecutive columns of k-row bk
+    const int bk = tid / (BN / EPT), bc = (tid % (BN / EPT)) * EPT;
     const int64_t nk_all = ceil_div(m, BK);
     const int64_t kt_begin = (int64_t)blockIdx.z * kps;
     const int64_t kt_end = std::min(nk_all, kt_begin + kps);
@@ -163,6 +170,21 @@ __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict
     auto gload = [&](int64_t k0) {
         const int64_t kb = k0 + lk;
         constexpr int E = VecE<Tin>::E;
+        if constexpr (!BKM) {
+            const int64_t kr = k0 + bk, c = col0 + bc;
+            if ((EPT % E == 0) && bvec && kr < m && c + EPT <= p) {
+#pragma unroll
+                for (int h = 0; h < EPT / E; ++h) {
+                    float y[E];
+                    load16(Bt + kr * p + c + h * E, y);
+#pragma unroll
+                    for (int e = 0; e < E; ++e) rb[h * E + e] = y[e];
+                }
+            } else {
+#pragma unroll
+                for (int e = 0; e < EPT; ++e) rb[e] = (kr < m && c + e < p) ? to_f(Bt[kr * p + c + e]) : 0.f;
+            }
+        }
         if (VEC && (EPT % E == 0) && kb + EPT <= m) {
 #pragma unroll
             for (int h = 0; h < EPT / E; ++h) {
@@ -171,14 +193,16 @@ __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict
                 else
 #pragma unroll
                     for (int e = 0; e < E; ++e) x[e] = 0.f;
-                if (brow) load16(bp + kb + h * E, y);
-                else
+                if constexpr (BKM) {
+                    if (brow) load16(bp + kb + h * E, y);
+                    else
 #pragma unroll
-                    for (int e = 0; e < E; ++e) y[e] = 0.f;
+                        for (int e = 0; e < E; ++e) y[e] = 0.f;
+                }
 #pragma unroll
                 for (int e = 0; e < E; ++e) {
                     ra[h * E + e] = x[e];
-                    rb[h * E + e] = y[e];
+                    if constexpr (BKM) rb[h * E + e] = y[e];
                 }
             }
         } else {
@@ -186,7 +210,7 @@ __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict
             for (int e = 0; e < EPT; ++e) {
                 const int64_t k = kb + e;
                 ra[e] = (arow && k < m) ? to_f(ap[k]) : 0.f;
-                rb[e] = (brow && k < m) ? to_f(bp[k]) : 0.f;
+                if constexpr (BKM) rb[e] = (brow && k < m) ? to_f(bp[k]) : 0.f;
             }
         }
     };
@@ -194,7 +218,8 @@ __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict
 #pragma unroll
         for (int e = 0; e < EPT; ++e) {
             As[buf][lk + e][lr] = ra[e];
-            Bs[buf][lk + e][lr] = rb[e];
+            if constexpr (BKM) Bs[buf][lk + e][lr] = rb[e];
+            else Bs[buf][bk][bc + e] = rb[e];
         }
     };
     float acc[TM][TN];
@@ -591,6 +616,19 @@ size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
 
 bool redomap2_tc_ok(const MmArgs& a) { return a.in_dt == 2 && tc_shape_ok(a.n, a.m, a.p, a.A, a.B); }
 
+// the SIMT tile kernel for either B layout (bkm: yss^T [p][m]; else yss [m][p])
+template <typename Tin, int BM, int BK>
+static void simt_go(dim3 g, bool vec, bool bkm, bool bvec, const Tin* A, const Tin* B, float* C, float* part,
+                    int64_t n, int64_t m, int64_t p, int64_t kps, cudaStream_t s) {
+    if (bkm) {
+        if (vec) mm_tile_simt_kernel<Tin, BM, BM, BK, true, true><<<g, 256, 0, s>>>(A, B, C, part, n, m, p, kps, bvec);
+        else mm_tile_simt_kernel<Tin, BM, BM, BK, false, true><<<g, 256, 0, s>>>(A, B, C, part, n, m, p, kps, bvec);
+    } else {
+        if (vec) mm_tile_simt_kernel<Tin, BM, BM, BK, true, false><<<g, 256, 0, s>>>(A, B, C, part, n, m, p, kps, bvec);
+        else mm_tile_simt_kernel<Tin, BM, BM, BK, false, false><<<g, 256, 0, s>>>(A, B, C, part, n, m, p, kps, bvec);
+    }
+}
+
 template <typename Tin>
 static cudaError_t run_mm(int version, const MmArgs& a) {
     const Tin* A = (const Tin*)a.A;
@@ -600,8 +638,13 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
         // V_FLAT, skinny outputs: either B layout, no transposition pass
         // (yss with a single column is the same memory as its transpose)
         return launch_skinny<Tin>(A, Bt, a.C, (float*)ws, a.n, a.m, a.p, a.b_kmajor != 0 || a.p == 1, a.stream);
+    constexpr bool kBf16 = std::is_same<Tin, __nv_bfloat16>::value;
+    // tensor cores (bf16), V_MIDDLE and the row-level leaves read yss^T; the
+    // SIMT tile kernels of V_TOP / V_FLAT read either layout in place
+    const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, a.b_kmajor ? a.B : a.ws);
+    const bool direct = !a.b_kmajor && (version == 0 || version == 2) && !tc;
     size_t used = 0;
-    if (!a.b_kmajor) {  // yss [m][p] -> yss^T [p][m]
+    if (!a.b_kmajor && !direct) {  // yss [m][p] -> yss^T [p][m]
         Tin* t = (Tin*)ws;
         used = align256((size_t)a.m * a.p * sizeof(Tin));
         if (a.m * a.p > 0) {
@@ -616,11 +659,11 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     if (version == IFL_V_ROW_TOP || version == IFL_V_ROW_MIDDLE)  // row-level leaves (mm_row.cu)
         return launch_mm_row(version, A, Bt, a.C, a.n, a.m, a.p, a.in_dt, a.stream);
     constexpr int E = VecE<Tin>::E;
-    const bool vec = ((uintptr_t)A % 16 == 0) && ((uintptr_t)Bt % 16 == 0) && (a.m % E == 0);
+    const bool bkm = !direct;
+    const bool vec = ((uintptr_t)A % 16 == 0) && (!bkm || (uintptr_t)Bt % 16 == 0) && (a.m % E == 0);
+    const bool bvec = !bkm && ((uintptr_t)Bt % 16 == 0) && (a.p % E == 0);
     const int64_t outs = a.n * a.p;
     float* part = (float*)(ws + used);
-    constexpr bool kBf16 = std::is_same<Tin, __nv_bfloat16>::value;
-    const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, Bt);
     if (version == 2) {  // ---- V_FLAT: every level parallel (split-K)
         // bf16: 128x256 tensor-core tiles split along k (even a mostly empty
         // tile beats SIMT here); f32: SIMT 32x32 (16x16 when skinny) tiles
@@ -630,20 +673,11 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
         const int64_t s = simt_flat_splits(a.n, a.m, a.p);
         const int64_t nk = ceil_div(a.m, kFlatTileBK), kps = ceil_div(nk, s), splits = ceil_div(nk, kps);
         dim3 g((unsigned)ceil_div(a.p, BM), (unsigned)ceil_div(a.n, BM), (unsigned)splits);
-        if (BM == 16) {
-            if (vec)
-                mm_tile_simt_kernel<Tin, 16, 16, kFlatTileBK * 2, true><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m,
-                                                                                          a.p, ceil_div(kps, 2));
-            else
-                mm_tile_simt_kernel<Tin, 16, 16, kFlatTileBK * 2, false><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m,
-                                                                                           a.p, ceil_div(kps, 2));
-        } else if (vec) {
-            mm_tile_simt_kernel<Tin, kFlatTileBM, kFlatTileBM, kFlatTileBK, true>
-                <<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
-        } else {
-            mm_tile_simt_kernel<Tin, kFlatTileBM, kFlatTileBM, kFlatTileBK, false>
-                <<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
-        }
+        if (BM == 16)
+            simt_go<Tin, 16, kFlatTileBK * 2>(g, vec, bkm, bvec, A, Bt, a.C, part, a.n, a.m, a.p, ceil_div(kps, 2),
+                                              a.stream);
+        else
+            simt_go<Tin, kFlatTileBM, kFlatTileBK>(g, vec, bkm, bvec, A, Bt, a.C, part, a.n, a.m, a.p, kps, a.stream);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess || splits == 1) return e;
         mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, a.stream>>>(
@@ -679,8 +713,7 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
         const int64_t s32 = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / t32, nk32 / 8));
         const int64_t kps32 = ceil_div(nk32, s32), sp32 = ceil_div(nk32, kps32);
         dim3 g32((unsigned)ceil_div(a.p, 32), (unsigned)ceil_div(a.n, 32), (unsigned)sp32);
-        if (vec) mm_tile_simt_kernel<Tin, 32, 32, 32, true><<<g32, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps32);
-        else mm_tile_simt_kernel<Tin, 32, 32, 32, false><<<g32, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps32);
+        simt_go<Tin, 32, 32>(g32, vec, bkm, bvec, A, Bt, a.C, part, a.n, a.m, a.p, kps32, a.stream);
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess || sp32 == 1) return e;
         mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, a.stream>>>(
@@ -691,8 +724,7 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     const int64_t s = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / tiles, nk / 64));
     const int64_t kps = ceil_div(nk, s), splits = ceil_div(nk, kps);
     dim3 g((unsigned)ceil_div(a.p, 128), (unsigned)ceil_div(a.n, 128), (unsigned)splits);
-    if (vec) mm_tile_simt_kernel<Tin, 128, 128, 16, true><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
-    else mm_tile_simt_kernel<Tin, 128, 128, 16, false><<<g, 256, 0, a.stream>>>(A, Bt, a.C, part, a.n, a.m, a.p, kps);
+    simt_go<Tin, 128, 16>(g, vec, bkm, bvec, A, Bt, a.C, part, a.n, a.m, a.p, kps, a.stream);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess || splits == 1) return e;
     mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, a.stream>>>(part, a.C, outs,

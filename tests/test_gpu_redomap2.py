@@ -62,7 +62,10 @@ def test_redomap2_versions(ifl, orc, version, dt):
 @pytest.mark.parametrize("dt", ["f32", "bf16"])
 def test_redomap2_row_major_B(ifl, orc, version, dt):
     """B given as yss [m][p] (b_kmajor = 0): same result."""
-    for (n, m, p) in [(5, 33, 17), (200, 128, 300), (1, 5000, 2)]:
+    # the SIMT tile kernels read yss in place (R24): 32x32 / 128x128 TOP tiles,
+    # FLAT's split-K 32x32 tiles, vector and scalar (p % 4 != 0) row loads
+    for (n, m, p) in [(5, 33, 17), (200, 128, 300), (1, 5000, 2), (100, 300, 72), (1280, 32, 1280),
+                      (1100, 40, 1030), (64, 4096, 64)]:
         A, Bt = operands(dt, n, m, p, seed=9)
         B = Bt.t().contiguous()
         C = ifl.redomap2(A.cuda(), B.cuda(), b_kmajor=False, version=version)
