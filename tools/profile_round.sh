@@ -38,8 +38,8 @@ cap lvc_outer_large      lvc     outer  256      256      lvc_outer "--p 256"
 cap colred_flat_n2e20    colred  flat   1048576  64       col_red_kernel
 cap colscan_top_n4       colscan top    4        16777216 col_scan_kernel
 cap colscan_flat_n2e26   colscan flat   67108864 1        col_scan_kernel
-cap segred_irr_flat_m1k  segred_irr flat 1       1024     irr_flat_kernel
-cap segscan_irr_flat_m1k segscan_irr flat 1      1024     irr_flat_kernel
+cap segred_irr_flat_m1k  segred_irr flat 1       1024     irr_mp_kernel
+cap segscan_irr_flat_m1k segscan_irr flat 1      1024     irr_mp_kernel
 for f in gpurun_out/ncu/*.ncu-rep; do
   ncu -i $f --page raw --csv > ${f%.ncu-rep}.raw.csv 2>/dev/null
 done
