@@ -668,8 +668,14 @@ def run_reference(args, rank, world):
 
 
 def main():
+    # stdout carries the one JSON line only: native writes to file descriptor 1
+    # (NCCL prints its version banner there) are sent to stderr, Python's
+    # prints keep the original stdout
+    real_out = os.dup(1)
+    os.dup2(2, 1)
+    sys.stdout = os.fdopen(real_out, "w", buffering=1)
     # NCCL's communicator INIT lines (rank count, transports) go to stderr,
-    # where the driver can read them; stdout keeps the one JSON line
+    # where the driver can read them
     os.environ.setdefault("NCCL_DEBUG", "INFO")
     os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
     os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")

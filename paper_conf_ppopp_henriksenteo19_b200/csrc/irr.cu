@@ -180,15 +180,16 @@ __device__ __forceinline__ void irr_cta_seg_scan(uint32_t fl, T v, uint32_t init
 
 // partition: coord[b] = the number of segment ends among the first
 // min(b*T, n+total) merge items.  P(i) = off[i+1] + i + 1 <= D is monotone
-// (true then false); 8 lanes per tile start probe 8 evenly spaced i per round.
-__global__ void __launch_bounds__(256) irr_mp_partition_kernel(const int64_t* __restrict__ off, int64_t n,
-                                                               int64_t total, int64_t Tn, int64_t* __restrict__ coord) {
+// (true then false): 8 lanes probe 8 evenly spaced i per round.  A CTA owns 32
+// consecutive tile starts: two 8-lane groups first find the coordinates of
+// its first and last start over the whole descriptor, then every start is
+// searched only between them (a window of <= 32 tiles: fewer rounds, and the
+// probes of one CTA share sectors in L2 instead of 32 random DRAM walks).
+__device__ __forceinline__ int64_t mp_search8(const int64_t* __restrict__ off, int64_t D, int64_t lo, int64_t hi,
+                                              bool live) {
     const int lane = threadIdx.x & 31, sub = lane & 7;
     const unsigned gmask = 0xffu << (lane & 24);
-    const int64_t b = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 3;
-    const bool live = b <= Tn;
-    const int64_t D = live ? min(b * kIrrTile, n + total) : 0;
-    int64_t lo = max((int64_t)0, D - total), hi = min(D, n);
+    if (!live) lo = hi;
     while (__any_sync(0xffffffffu, lo < hi)) {  // uniform trip count: the ballots need every lane
         const int64_t step = (hi - lo + 7) / 8;
         const int64_t p = lo + step * sub;
@@ -203,7 +204,31 @@ __global__ void __launch_bounds__(256) irr_mp_partition_kernel(const int64_t* __
             }
         }
     }
-    if (live && sub == 0) coord[b] = lo;
+    return lo;
+}
+
+constexpr int kPartPerCta = 32;  // tile starts per CTA (8 lanes each: 256 threads)
+
+__global__ void __launch_bounds__(256) irr_mp_partition_kernel(const int64_t* __restrict__ off, int64_t n,
+                                                               int64_t total, int64_t Tn, int64_t* __restrict__ coord) {
+    __shared__ int64_t s_bound[2];
+    const int t = threadIdx.x, sub = t & 7, grp = t >> 3;
+    const int64_t W = n + total;
+    const int64_t b0 = (int64_t)blockIdx.x * kPartPerCta;
+    const int64_t bl = min(b0 + kPartPerCta, Tn);  // the CTA's starts are b0 .. bl (bl inclusive)
+    if (t < 32) {  // warp 0: groups 0 / 1 find the bounds (b0, bl) over the whole descriptor
+        const int64_t bb = grp == 0 ? b0 : bl;
+        const int64_t D = min(bb * kIrrTile, W);
+        const int64_t r = mp_search8(off, D, max((int64_t)0, D - total), min(D, n), grp < 2);
+        if (sub == 0 && grp < 2) s_bound[grp] = r;
+    }
+    __syncthreads();
+    const int64_t b = b0 + grp;
+    const bool live = b <= bl && b <= Tn;
+    const int64_t D = live ? min(b * kIrrTile, W) : 0;
+    const int64_t lo = max(s_bound[0], D - total), hi = min(s_bound[1], min(D, n));
+    const int64_t r = mp_search8(off, D, lo, max(lo, hi), live);
+    if (live && sub == 0) coord[b] = r;
 }
 
 // Elements-only segred tiles (no segment end: the tile lies inside one
@@ -312,42 +337,33 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
     T acc = identity<OP, T>();
     int first = -1;  // segred: the thread's first segment end
     int lead = 0;    // segscan: elements before the thread's first segment start
-    if (i == ie && cnt == kMpItems) {  // elements only
-#pragma unroll
-        for (int k = 0; k < kMpItems; ++k) {
-            acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j_s + k))));
-            if constexpr (SCAN) X(j_s + k) = (int)to_bits<T>(acc);
-        }
-        lead = cnt;
-    } else if (i == ie) {
-        for (int k = 0; k < cnt; ++k) {
-            acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j_s + k))));
-            if constexpr (SCAN) X(j_s + k) = (int)to_bits<T>(acc);
-        }
-        lead = cnt;
-    } else {
-        int j = j_s;
+    // the walk as runs of elements between segment ends (a thread in one
+    // segment is one run; divergent lanes cost the longest run, not the sum
+    // of both paths)
+    {
+        int j = j_s, rem = cnt;
         bool seen = false;
-        int ce = s_b[pd(i)];
-#pragma unroll
-        for (int k = 0; k < kMpItems; ++k) {
-            const bool valid = k < cnt;
-            const bool end = valid && ce <= j;
-            const bool elt = valid && !end;
-            const T nacc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j))));  // j <= ne: inside
-            if constexpr (SCAN) {
-                if (elt) X(j) = (int)to_bits<T>(nacc);
-            } else {
-                if (end) s_b[pd(i)] = (int)to_bits<T>(acc);
-                first = (end && first < 0) ? i : first;
+        while (rem > 0) {
+            const int ce = i < ie ? s_b[pd(i)] : 0x7fffffff;
+            const int run = min(ce - j, rem);  // elements before the next end
+#pragma unroll 4
+            for (int q = 0; q < run; ++q) {
+                acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j + q))));
+                if constexpr (SCAN) X(j + q) = (int)to_bits<T>(acc);
             }
-            seen = seen || end;
-            lead += (elt && !seen) ? 1 : 0;
-            i += end ? 1 : 0;
-            const int nc = s_b[pd(i)];  // read only when i < ie
-            ce = end ? (i < ie ? nc : 0x7fffffff) : ce;
-            acc = end ? d : (elt ? nacc : acc);
-            j += elt ? 1 : 0;
+            if (!seen) lead += run;
+            j += run;
+            rem -= run;
+            if (rem > 0) {  // the end of segment i0 + i
+                if constexpr (!SCAN) {
+                    s_b[pd(i)] = (int)to_bits<T>(acc);
+                    if (first < 0) first = i;
+                }
+                seen = true;
+                acc = d;
+                ++i;
+                --rem;
+            }
         }
         if constexpr (SCAN) first = seen ? 0 : -1;
     }
@@ -524,8 +540,8 @@ cudaError_t launch_irr(const IrrArgs& a, bool scan, int version) {
         uint32_t* cflag = (uint32_t*)(cagg + C);
         const bool vec = ((uintptr_t)a.in % 16 == 0) && ((uintptr_t)a.out % 16 == 0);
         cudaError_t e;
-        irr_mp_partition_kernel<<<(unsigned)ceil_div((Tn + 1) * 8, 256), 256, 0, a.stream>>>(a.off, a.n, a.total, Tn,
-                                                                                              coord);
+        irr_mp_partition_kernel<<<(unsigned)ceil_div(Tn + 1, kPartPerCta), 256, 0, a.stream>>>(a.off, a.n, a.total,
+                                                                                                 Tn, coord);
         if ((e = cudaGetLastError()) != cudaSuccess) return e;
         if (!scan) {
             irr_mp_kernel<T, OP, F, false><<<(unsigned)Tn, kMpThreads, 0, a.stream>>>(

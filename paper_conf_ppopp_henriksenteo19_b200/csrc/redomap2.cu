@@ -342,9 +342,44 @@ struct SkinnyGeom {
     static constexpr size_t SMEM = (size_t)S * WORDS * kSkinnyThreads * 8;
 };
 
+// The end of a skinny CTA: its RI x RJ dot products (thread t < RI*RJ holds
+// output t).  Without k-splits they go to C; otherwise to the partial tiles,
+// and the last CTA of the output tile to arrive (a counter per tile) sums the
+// splits' partials in split order into C -- the order of mm_splitk_finalize,
+// so the result is deterministic -- and re-arms the counter: V_FLAT's skinny
+// engine is one kernel.
+template <int RI, int RJ>
+__device__ __forceinline__ void skinny_store(float v, float* __restrict__ part, float* __restrict__ C,
+                                             unsigned* __restrict__ cnt, int64_t n, int64_t p, int64_t i0,
+                                             int64_t j0, int tile) {
+    __shared__ unsigned s_last;
+    const int t = threadIdx.x;
+    const int splits = (int)gridDim.x;
+    const int64_t i = i0 + t / RJ, j = j0 + t % RJ;
+    const bool own = t < RI * RJ && i < n && j < p;
+    if (splits == 1) {
+        if (own) C[i * p + j] = v;
+        return;
+    }
+    if (own) part[(int64_t)blockIdx.x * n * p + i * p + j] = v;
+    __threadfence();
+    __syncthreads();
+    if (t == 0) s_last = atomicAdd(cnt + tile, 1u) == (unsigned)(splits - 1) ? 1u : 0u;
+    __syncthreads();
+    if (!s_last) return;
+    __threadfence();
+    if (own) {
+        float r = 0.f;
+        for (int q = 0; q < splits; ++q) r += __ldcg(part + (int64_t)q * n * p + i * p + j);
+        C[i * p + j] = r;
+    }
+    if (t == 0) cnt[tile] = 0u;
+}
+
 template <typename Tin, int RI, int RJ, bool KMAJ>
 __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __restrict__ A, const Tin* __restrict__ B,
-                                                                   float* __restrict__ part, int64_t n, int64_t m,
+                                                                   float* __restrict__ part, float* __restrict__ C,
+                                                                   unsigned* __restrict__ cnt, int64_t n, int64_t m,
                                                                    int64_t p, int64_t kchunk, int tiles_j) {
     using Gm = SkinnyGeom<Tin, RI, RJ, KMAJ>;
     constexpr int E = Gm::E, NW = kSkinnyThreads / 32, S = Gm::S;
@@ -438,20 +473,20 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __
             if (lane == 0) red[w][r * RJ + c] = v;
         }
     __syncthreads();
-    if (t < RI * RJ) {
-        float s = 0.f;
+    float s = 0.f;
+    if (t < RI * RJ)
 #pragma unroll
         for (int q = 0; q < NW; ++q) s += red[q][t];
-        const int64_t i = i0 + t / RJ, j = j0 + t % RJ;
-        if (i < n && j < p) part[(int64_t)blockIdx.x * n * p + i * p + j] = s;
-    }
+    skinny_store<RI, RJ>(s, part, C, cnt, n, p, i0, j0, tile);
 }
 
 // Scalar form (misaligned operands or m not a multiple of the vector width).
 template <typename Tin, int RI, int RJ, bool KMAJ>
 __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const Tin* __restrict__ A,
                                                                           const Tin* __restrict__ B,
-                                                                          float* __restrict__ part, int64_t n,
+                                                                          float* __restrict__ part,
+                                                                          float* __restrict__ C,
+                                                                          unsigned* __restrict__ cnt, int64_t n,
                                                                           int64_t m, int64_t p, int64_t kchunk,
                                                                           int tiles_j) {
     constexpr int NW = kSkinnyThreads / 32;
@@ -487,13 +522,11 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const 
             if (lane == 0) red[w][r * RJ + c] = v;
         }
     __syncthreads();
-    if (t < RI * RJ) {
-        float s = 0.f;
+    float s = 0.f;
+    if (t < RI * RJ)
 #pragma unroll
         for (int q = 0; q < NW; ++q) s += red[q][t];
-        const int64_t i = i0 + t / RJ, j = j0 + t % RJ;
-        if (i < n && j < p) part[(int64_t)blockIdx.x * n * p + i * p + j] = s;
-    }
+    skinny_store<RI, RJ>(s, part, C, cnt, n, p, i0, j0, tile);
 }
 
 // Where the engine is V_FLAT's form: f32 up to 4096 outputs; bf16 up to 256
@@ -516,8 +549,9 @@ static int64_t skinny_kchunk(int64_t n, int64_t m, int64_t p) {
 static int64_t skinny_splits(int64_t n, int64_t m, int64_t p) { return ceil_div(m, skinny_kchunk(n, m, p)); }
 
 template <typename Tin, int RI, int RJ, bool KMAJ>
-static cudaError_t launch_skinny_k(const Tin* A, const Tin* B, float* dst, int64_t n, int64_t m, int64_t p,
-                                   int64_t kc, int64_t splits, int tj, int64_t tiles, cudaStream_t s) {
+static cudaError_t launch_skinny_k(const Tin* A, const Tin* B, float* part, float* C, unsigned* cnt, int64_t n,
+                                   int64_t m, int64_t p, int64_t kc, int64_t splits, int tj, int64_t tiles,
+                                   cudaStream_t s) {
     using Gm = SkinnyGeom<Tin, RI, RJ, KMAJ>;
     constexpr int E = Gm::E;
     // cp.async needs 8-byte aligned rows (KMAJ) / UNIT-aligned B slices (row-major)
@@ -534,9 +568,9 @@ static cudaError_t launch_skinny_k(const Tin* A, const Tin* B, float* dst, int64
             cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
             attr = true;
         }
-        k<<<g, kSkinnyThreads, smem, s>>>(A, B, dst, n, m, p, kc, tj);
+        k<<<g, kSkinnyThreads, smem, s>>>(A, B, part, C, cnt, n, m, p, kc, tj);
     } else {
-        mm_skinny_scalar_kernel<Tin, RI, RJ, KMAJ><<<g, kSkinnyThreads, 0, s>>>(A, B, dst, n, m, p, kc, tj);
+        mm_skinny_scalar_kernel<Tin, RI, RJ, KMAJ><<<g, kSkinnyThreads, 0, s>>>(A, B, part, C, cnt, n, m, p, kc, tj);
     }
     return cudaGetLastError();
 }
@@ -547,14 +581,10 @@ static cudaError_t launch_skinny_rr(const Tin* A, const Tin* B, float* C, float*
     const int64_t kc = skinny_kchunk(n, m, p), splits = ceil_div(m, kc);
     const int tj = (int)ceil_div(p, RJ);
     const int64_t tiles = ceil_div(n, RI) * tj;
-    float* dst = splits == 1 ? C : part;
-    cudaError_t e = kmajor ? launch_skinny_k<Tin, RI, RJ, true>(A, B, dst, n, m, p, kc, splits, tj, tiles, s)
-                           : launch_skinny_k<Tin, RI, RJ, false>(A, B, dst, n, m, p, kc, splits, tj, tiles, s);
-    if (e != cudaSuccess || splits == 1) return e;
-    const int64_t outs = n * p;
-    mm_splitk_finalize<<<(unsigned)std::min<int64_t>(ceil_div(outs, 256), 148 * 16), 256, 0, s>>>(part, C, outs,
-                                                                                                   (int)splits);
-    return cudaGetLastError();
+    // per-tile arrival counters after the partial tiles (zero at rest: the last CTA re-arms them)
+    unsigned* cnt = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(part) + align256((size_t)n * p * splits * 4));
+    return kmajor ? launch_skinny_k<Tin, RI, RJ, true>(A, B, part, C, cnt, n, m, p, kc, splits, tj, tiles, s)
+                  : launch_skinny_k<Tin, RI, RJ, false>(A, B, part, C, cnt, n, m, p, kc, splits, tj, tiles, s);
 }
 
 template <typename Tin, int RI>
@@ -596,7 +626,8 @@ size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
     size_t b = align256((size_t)m * p * 4);
     size_t part = 0;
     if (version == 2 || version == -1) {
-        if (skinny_ok(n, p, false)) part = std::max(part, (size_t)n * p * skinny_splits(n, m, p) * 4);
+        if (skinny_ok(n, p, false))  // partial tiles + one arrival counter per output tile (<= 4096)
+            part = std::max(part, align256((size_t)n * p * skinny_splits(n, m, p) * 4) + kSkinnyMaxOuts * 4);
         part = std::max(part, (size_t)n * p * simt_flat_splits(n, m, p) * 4);
         part = std::max(part, (size_t)n * p * tc_splits(n, m, p, true) * 4);
     }
