@@ -630,6 +630,7 @@ int ifl_redomap2(const void* A, const void* B, float* C, int64_t n, int64_t m, i
     const size_t esz = in_dt == IFL_BF16 ? 2 : 4;
     size_t need = ifl::redomap2_ws_bytes(n, m, p, c.version) - (((size_t)m * p * 4 + 255) & ~(size_t)255);
     if (!b_kmajor) need += ((size_t)m * p * esz + 255) & ~(size_t)255;
+    if (c.version != IFL_V_FLAT && need == ifl::kMmCntBytes) need = 0;  // the counters serve V_FLAT only
     if (need && (!ws || ws_bytes < need))
         return fail(IFL_EWORKSPACE, "ifl_redomap2: needs %zu workspace bytes, got %zu", need, ws_bytes);
     return cuda_status(ifl::launch_redomap2(c.version, a), "ifl_redomap2");

@@ -113,6 +113,8 @@ struct MmArgs {
     size_t ws_bytes;
     cudaStream_t stream;
 };
+// redomap2 workspace: [V_FLAT arrival counters: kMmCntBytes][yss^T][split-K partials]
+constexpr size_t kMmCntBytes = 16384;
 size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version);
 cudaError_t launch_redomap2(int version, const MmArgs& a);
 bool redomap2_tc_ok(const MmArgs& a);

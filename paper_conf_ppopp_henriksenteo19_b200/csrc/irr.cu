@@ -337,10 +337,38 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
     T acc = identity<OP, T>();
     int first = -1;  // segred: the thread's first segment end
     int lead = 0;    // segscan: elements before the thread's first segment start
-    // the walk as runs of elements between segment ends (a thread in one
-    // segment is one run; divergent lanes cost the longest run, not the sum
-    // of both paths)
+    if (ns * 32 > ne) {
+        // ends-dense tiles (segments shorter than ~32): branch-free walk
+        // (selects and predicated shared stores)
+        int j = j_s;
+        bool seen = false;
+        int ce = i < ie ? s_b[pd(i)] : 0x7fffffff;
+#pragma unroll
+        for (int k = 0; k < kMpItems; ++k) {
+            const bool valid = k < cnt;
+            const bool end = valid && ce <= j;
+            const bool elt = valid && !end;
+            const T nacc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j))));  // j <= ne: inside
+            if constexpr (SCAN) {
+                if (elt) X(j) = (int)to_bits<T>(nacc);
+            } else {
+                if (end) s_b[pd(i)] = (int)to_bits<T>(acc);
+                first = (end && first < 0) ? i : first;
+            }
+            seen = seen || end;
+            lead += (elt && !seen) ? 1 : 0;
+            i += end ? 1 : 0;
+            const int nc = s_b[pd(i)];  // read only when i < ie
+            ce = end ? (i < ie ? nc : 0x7fffffff) : ce;
+            acc = end ? d : (elt ? nacc : acc);
+            j += elt ? 1 : 0;
+        }
+        if constexpr (SCAN) first = seen ? 0 : -1;
+    } else
     {
+        // element-dense tiles: the walk as runs of elements between segment
+        // ends (a thread inside one segment is one run; divergent lanes cost
+        // the longest run, not both paths)
         int j = j_s, rem = cnt;
         bool seen = false;
         while (rem > 0) {

@@ -301,6 +301,8 @@ static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 constexpr int kSkinnyThreads = 256;
 constexpr int kSkinnyStageBytes = 128 * 1024;  // pipeline depth: as many stages as fit 128 KB (3..12)
 constexpr int64_t kSkinnyMaxOuts = 4096;
+constexpr size_t kSkinnyCntBytes = kMmCntBytes;  // one arrival counter per output tile
+static_assert(kMmCntBytes >= (size_t)kSkinnyMaxOuts * 4, "counter region");
 
 __device__ __forceinline__ void cp_async8(void* smem, const void* gmem) {
     asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
@@ -576,36 +578,34 @@ static cudaError_t launch_skinny_k(const Tin* A, const Tin* B, float* part, floa
 }
 
 template <typename Tin, int RI, int RJ>
-static cudaError_t launch_skinny_rr(const Tin* A, const Tin* B, float* C, float* part, int64_t n, int64_t m, int64_t p,
-                                    bool kmajor, cudaStream_t s) {
+static cudaError_t launch_skinny_rr(const Tin* A, const Tin* B, float* C, float* part, unsigned* cnt, int64_t n,
+                                    int64_t m, int64_t p, bool kmajor, cudaStream_t s) {
     const int64_t kc = skinny_kchunk(n, m, p), splits = ceil_div(m, kc);
     const int tj = (int)ceil_div(p, RJ);
     const int64_t tiles = ceil_div(n, RI) * tj;
-    // per-tile arrival counters after the partial tiles (zero at rest: the last CTA re-arms them)
-    unsigned* cnt = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(part) + align256((size_t)n * p * splits * 4));
     return kmajor ? launch_skinny_k<Tin, RI, RJ, true>(A, B, part, C, cnt, n, m, p, kc, splits, tj, tiles, s)
                   : launch_skinny_k<Tin, RI, RJ, false>(A, B, part, C, cnt, n, m, p, kc, splits, tj, tiles, s);
 }
 
 template <typename Tin, int RI>
-static cudaError_t launch_skinny_r(const Tin* A, const Tin* B, float* C, float* part, int64_t n, int64_t m, int64_t p,
-                                   bool kmajor, cudaStream_t s) {
+static cudaError_t launch_skinny_r(const Tin* A, const Tin* B, float* C, float* part, unsigned* cnt, int64_t n,
+                                   int64_t m, int64_t p, bool kmajor, cudaStream_t s) {
     switch (skinny_r(p)) {
-    case 8: return launch_skinny_rr<Tin, RI, 8>(A, B, C, part, n, m, p, kmajor, s);
-    case 4: return launch_skinny_rr<Tin, RI, 4>(A, B, C, part, n, m, p, kmajor, s);
-    case 2: return launch_skinny_rr<Tin, RI, 2>(A, B, C, part, n, m, p, kmajor, s);
-    default: return launch_skinny_rr<Tin, RI, 1>(A, B, C, part, n, m, p, kmajor, s);
+    case 8: return launch_skinny_rr<Tin, RI, 8>(A, B, C, part, cnt, n, m, p, kmajor, s);
+    case 4: return launch_skinny_rr<Tin, RI, 4>(A, B, C, part, cnt, n, m, p, kmajor, s);
+    case 2: return launch_skinny_rr<Tin, RI, 2>(A, B, C, part, cnt, n, m, p, kmajor, s);
+    default: return launch_skinny_rr<Tin, RI, 1>(A, B, C, part, cnt, n, m, p, kmajor, s);
     }
 }
 
 template <typename Tin>
-static cudaError_t launch_skinny(const Tin* A, const Tin* B, float* C, float* part, int64_t n, int64_t m, int64_t p,
-                                 bool kmajor, cudaStream_t s) {
+static cudaError_t launch_skinny(const Tin* A, const Tin* B, float* C, float* part, unsigned* cnt, int64_t n,
+                                 int64_t m, int64_t p, bool kmajor, cudaStream_t s) {
     switch (skinny_r(n)) {
-    case 8: return launch_skinny_r<Tin, 8>(A, B, C, part, n, m, p, kmajor, s);
-    case 4: return launch_skinny_r<Tin, 4>(A, B, C, part, n, m, p, kmajor, s);
-    case 2: return launch_skinny_r<Tin, 2>(A, B, C, part, n, m, p, kmajor, s);
-    default: return launch_skinny_r<Tin, 1>(A, B, C, part, n, m, p, kmajor, s);
+    case 8: return launch_skinny_r<Tin, 8>(A, B, C, part, cnt, n, m, p, kmajor, s);
+    case 4: return launch_skinny_r<Tin, 4>(A, B, C, part, cnt, n, m, p, kmajor, s);
+    case 2: return launch_skinny_r<Tin, 2>(A, B, C, part, cnt, n, m, p, kmajor, s);
+    default: return launch_skinny_r<Tin, 1>(A, B, C, part, cnt, n, m, p, kmajor, s);
     }
 }
 
@@ -626,8 +626,8 @@ size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
     size_t b = align256((size_t)m * p * 4);
     size_t part = 0;
     if (version == 2 || version == -1) {
-        if (skinny_ok(n, p, false))  // partial tiles + one arrival counter per output tile (<= 4096)
-            part = std::max(part, align256((size_t)n * p * skinny_splits(n, m, p) * 4) + kSkinnyMaxOuts * 4);
+        if (skinny_ok(n, p, false))
+            part = std::max(part, (size_t)n * p * skinny_splits(n, m, p) * 4);
         part = std::max(part, (size_t)n * p * simt_flat_splits(n, m, p) * 4);
         part = std::max(part, (size_t)n * p * tc_splits(n, m, p, true) * 4);
     }
@@ -642,7 +642,7 @@ size_t redomap2_ws_bytes(int64_t n, int64_t m, int64_t p, int version) {
         const int64_t s = std::max<int64_t>(1, std::min<int64_t>((int64_t)148 / tiles, nk / 64));
         part = std::max(part, (size_t)n * p * (size_t)ceil_div(nk, ceil_div(nk, s)) * 4);
     }
-    return b + align256(part);
+    return kSkinnyCntBytes + b + align256(part);
 }
 
 bool redomap2_tc_ok(const MmArgs& a) { return a.in_dt == 2 && tc_shape_ok(a.n, a.m, a.p, a.A, a.B); }
@@ -664,15 +664,18 @@ template <typename Tin>
 static cudaError_t run_mm(int version, const MmArgs& a) {
     const Tin* A = (const Tin*)a.A;
     const Tin* Bt = (const Tin*)a.B;
-    char* ws = (char*)a.ws;
+    // [V_FLAT skinny arrival counters][yss^T][split-K partial tiles]: the
+    // counters (zero at rest) never share bytes with the other regions
+    unsigned* cnt = (unsigned*)a.ws;
+    char* ws = a.ws ? (char*)a.ws + kSkinnyCntBytes : nullptr;
     if (version == 2 && skinny_ok(a.n, a.p, std::is_same<Tin, __nv_bfloat16>::value) && a.m > 0)
         // V_FLAT, skinny outputs: either B layout, no transposition pass
         // (yss with a single column is the same memory as its transpose)
-        return launch_skinny<Tin>(A, Bt, a.C, (float*)ws, a.n, a.m, a.p, a.b_kmajor != 0 || a.p == 1, a.stream);
+        return launch_skinny<Tin>(A, Bt, a.C, (float*)ws, cnt, a.n, a.m, a.p, a.b_kmajor != 0 || a.p == 1, a.stream);
     constexpr bool kBf16 = std::is_same<Tin, __nv_bfloat16>::value;
     // tensor cores (bf16), V_MIDDLE and the row-level leaves read yss^T; the
     // SIMT tile kernels of V_TOP / V_FLAT read either layout in place
-    const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, a.b_kmajor ? a.B : a.ws);
+    const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, a.b_kmajor ? a.B : (const void*)ws);
     const bool direct = !a.b_kmajor && (version == 0 || version == 2) && !tc;
     size_t used = 0;
     if (!a.b_kmajor && !direct) {  // yss [m][p] -> yss^T [p][m]

@@ -420,12 +420,15 @@ def test_mm_tree_guard(L):
     assert ifl.select("redomap2.f32", 4096, 64, 64).version in ("top", "middle", "flat")
     ifl.set_thresholds("redomap2.f32.row", 4096, 1 << 19)
     try:
+        # B as yss [m][p] without a workspace: the choice is reported, then
+        # IFL_EWORKSPACE (the transposition buffer) -- nothing is launched
         c = ifl.ifl_choice()
-        assert L.ifl_redomap2(256, 512, 1024, 4096, 64, 16, 1, 1, -1, None, 0, None, ctypes.byref(c)) != 0  # no ws
+        assert L.ifl_redomap2(256, 512, 1024, 4096, 64, 16, 1, 0, -1, None, 0, None, ctypes.byref(c)) == \
+            ifl.IFL_EWORKSPACE
         assert c.version == 4                                                    # ROW_TOP: n >= t_rt
-        L.ifl_redomap2(256, 512, 1024, 4095, 64, 16, 1, 1, -1, None, 0, None, ctypes.byref(c))
+        assert L.ifl_redomap2(256, 512, 1024, 4095, 64, 16, 1, 0, -1, None, 0, None, ctypes.byref(c)) != 0
         assert c.version == 5                                                    # ROW_MIDDLE: 4095*8*32 >= 2^19
-        L.ifl_redomap2(256, 512, 1024, 64, 64, 4, 1, 1, -1, None, 0, None, ctypes.byref(c))
+        assert L.ifl_redomap2(256, 512, 1024, 64, 64, 4, 1, 0, -1, None, 0, None, ctypes.byref(c)) != 0
         assert c.version in (0, 1, 2)                                            # 64*4*32 < 2^19
         assert L.ifl_redomap2(256, 512, 1024, 64, 10000, 4, 1, 1, 5, None, 0, None, None) == ifl.IFL_ENOTFIT
     finally:
