@@ -281,8 +281,9 @@ __global__ void __launch_bounds__(256) mm_tile_simt_kernel(const Tin* __restrict
 __global__ void mm_splitk_finalize(const float* __restrict__ part, float* __restrict__ C, int64_t outs, int splits);
 bool tc_shape_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* Bt);
 int tc_splits(int64_t n, int64_t m, int64_t p, bool flat);
+bool tc_mn_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* B);
 cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* part, int64_t n, int64_t m, int64_t p,
-                             int splits, cudaStream_t s);
+                             int splits, cudaStream_t s, bool b_mn = false);
 
 static size_t align256(size_t b) { return (b + 255) & ~(size_t)255; }
 
@@ -675,8 +676,11 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
     constexpr bool kBf16 = std::is_same<Tin, __nv_bfloat16>::value;
     // tensor cores (bf16), V_MIDDLE and the row-level leaves read yss^T; the
     // SIMT tile kernels of V_TOP / V_FLAT read either layout in place
-    const bool tc = kBf16 && tc_shape_ok(a.n, a.m, a.p, A, a.b_kmajor ? a.B : (const void*)ws);
-    const bool direct = !a.b_kmajor && (version == 0 || version == 2) && !tc;
+    // (the tensor-core kernel reads yss in place too when its rows have a
+    // 16-byte pitch: MN-major B operand)
+    const bool tc_mn = kBf16 && !a.b_kmajor && (version == 0 || version == 2) && tc_mn_ok(a.n, a.m, a.p, A, a.B);
+    const bool tc = kBf16 && (tc_mn || tc_shape_ok(a.n, a.m, a.p, A, a.b_kmajor ? a.B : (const void*)ws));
+    const bool direct = !a.b_kmajor && (version == 0 || version == 2) && (!tc || tc_mn);
     size_t used = 0;
     if (!a.b_kmajor && !direct) {  // yss [m][p] -> yss^T [p][m]
         Tin* t = (Tin*)ws;
@@ -702,7 +706,7 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
         // bf16: 128x256 tensor-core tiles split along k (even a mostly empty
         // tile beats SIMT here); f32: SIMT 32x32 (16x16 when skinny) tiles
         if (tc)
-            return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, true), a.stream);
+            return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, true), a.stream, tc_mn);
         const int BM = std::max(a.n, a.p) <= 16 ? 16 : kFlatTileBM;
         const int64_t s = simt_flat_splits(a.n, a.m, a.p);
         const int64_t nk = ceil_div(a.m, kFlatTileBK), kps = ceil_div(nk, s), splits = ceil_div(nk, kps);
@@ -738,7 +742,7 @@ static cudaError_t run_mm(int version, const MmArgs& a) {
         return cudaGetLastError();
     }
     // ---- V_TOP: output tiles, sequential k (tensor cores for bf16)
-    if (tc) return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, false), a.stream);
+    if (tc) return launch_mm_top_tc(A, Bt, a.C, part, a.n, a.m, a.p, tc_splits(a.n, a.m, a.p, false), a.stream, tc_mn);
     // SIMT TOP: 128x128 tiles; when fewer than half the SMs would get one, the
     // 32x32 tiles (k in chunks of >= 8 x 32, each walked sequentially) -- B200:
     // n = p = 64..512 outputs from 105-60 us down to the 32x32 engine's 11-18 us

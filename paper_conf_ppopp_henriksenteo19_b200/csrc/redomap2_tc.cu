@@ -53,6 +53,20 @@ __device__ __forceinline__ uint64_t umma_desc_sw128(uint32_t saddr) {
     return d;
 }
 
+// UMMA shared-memory descriptor for an MN-major operand (B given as yss
+// [m][p]: n contiguous), 128-byte swizzle: atoms of 64 n x 8 k (8 rows of
+// 128 B), 8-k-row groups SBO = 1024 B apart, 64-wide n blocks LBO apart (the
+// TMA boxes of one stage, 64 k-rows x 128 B = 8 KB each).
+__device__ __forceinline__ uint64_t umma_desc_mn_sw128(uint32_t saddr, uint32_t lbo) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);  // start address
+    d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;  // leading byte offset: between n blocks
+    d |= (uint64_t)(1024 >> 4) << 32;          // stride byte offset: between 8-row k groups
+    d |= (uint64_t)1 << 46;                    // descriptor version (sm_100)
+    d |= (uint64_t)2 << 61;                    // layout: SWIZZLE_128B
+    return d;
+}
+
 // instruction descriptor, kind::f16: D f32, A/B bf16, both K-major, M x N
 __host__ __device__ constexpr uint32_t umma_idesc_bf16(int M, int N) {
     return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
@@ -116,7 +130,9 @@ __device__ __forceinline__ void tma_store_3d(const CUtensorMap* map, const void*
                  : "memory");
 }
 
-template <bool TST>
+// BMN: B is yss [m][p] (MN-major, read in place: four 64-column TMA boxes per
+// stage, MN-major descriptors, the b_major bit of the instruction descriptor).
+template <bool TST, bool BMN>
 __global__ void __launch_bounds__(TC_THREADS, 1)
     mm_top_tc_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB,
                      const __grid_constant__ CUtensorMap mapC, float* C, float* part, int64_t n, int64_t m,
@@ -184,13 +200,20 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                     uint8_t* sa = smem + s * TC_STAGE_BYTES;
                     mbar_arrive_expect_tx(&full[s], TC_STAGE_BYTES);
                     tma_load_2d(sa, &mapA, (kt0 + kt) * TC_BK, m0, &full[s]);
-                    tma_load_2d(sa + TC_A_BYTES, &mapB, (kt0 + kt) * TC_BK, n0, &full[s]);
+                    if constexpr (BMN) {
+#pragma unroll
+                        for (int q = 0; q < TC_BN / 64; ++q)
+                            tma_load_2d(sa + TC_A_BYTES + q * (TC_BK * 128), &mapB, n0 + 64 * q, (kt0 + kt) * TC_BK,
+                                        &full[s]);
+                    } else {
+                        tma_load_2d(sa + TC_A_BYTES, &mapB, (kt0 + kt) * TC_BK, n0, &full[s]);
+                    }
                 }
             }
         }
     } else if (warp == 1) {
         if (lane == 0) {  // ---- MMA issuer
-            constexpr uint32_t idesc = umma_idesc_bf16(TC_BM, TC_BN);
+            constexpr uint32_t idesc = umma_idesc_bf16(TC_BM, TC_BN) | (BMN ? (1u << 16) : 0u);
             int gk = 0, li = 0;
             for (int it = blockIdx.x; it < items; it += gridDim.x, ++li) {
                 int z, m0, n0, kt0, nk;
@@ -206,9 +229,12 @@ __global__ void __launch_bounds__(TC_THREADS, 1)
                     const uint32_t sa = smem_u32(smem + s * TC_STAGE_BYTES);
                     const uint32_t sb = sa + TC_A_BYTES;
 #pragma unroll
-                    for (int kk = 0; kk < TC_BK / 16; ++kk)
-                        umma_bf16(d, umma_desc_sw128(sa + kk * 32), umma_desc_sw128(sb + kk * 32), idesc,
-                                  (kt | kk) != 0 ? 1u : 0u);
+                    for (int kk = 0; kk < TC_BK / 16; ++kk) {
+                        // K = 16 per MMA: 32 bytes along a K-major row, 16 rows (2 KB) of an MN-major box
+                        const uint64_t bd = BMN ? umma_desc_mn_sw128(sb + kk * 2048, TC_BK * 128)
+                                                : umma_desc_sw128(sb + kk * 32);
+                        umma_bf16(d, umma_desc_sw128(sa + kk * 32), bd, idesc, (kt | kk) != 0 ? 1u : 0u);
+                    }
                     umma_commit(&empty[s]);
                 }
                 umma_commit(&tfull[acc]);
@@ -306,6 +332,19 @@ static bool make_map(CUtensorMap* map, const void* base, int64_t rows, int64_t k
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+// yss [m][p] (MN-major B): 64 (n) x 64 (k) boxes, 128-byte swizzle
+static bool make_map_mn(CUtensorMap* map, const void* base, int64_t m, int64_t p) {
+    EncodeTiledFn fn = encode_fn();
+    if (!fn) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)p, (cuuint64_t)m};
+    const cuuint64_t strides[1] = {(cuuint64_t)p * 2};
+    const cuuint32_t box[2] = {64, (cuuint32_t)TC_BK};
+    const cuuint32_t estr[2] = {1, 1};
+    return fn(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
 // fp32 output [splits][n][p] as a 3-D map, 32 x 32 boxes, 128-byte swizzle
 static bool make_out_map(CUtensorMap* map, float* base, int64_t n, int64_t p, int splits) {
     EncodeTiledFn fn = encode_fn();
@@ -347,14 +386,21 @@ int tc_splits(int64_t n, int64_t m, int64_t p, bool flat) {
     return (int)ceil_div(nk, kps);
 }
 
+bool tc_mn_ok(int64_t n, int64_t m, int64_t p, const void* A, const void* B) {
+    return tc_shape_ok(n, m, p, A, B) && p % 8 == 0;  // yss rows: 16-byte pitch
+}
+
 cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* part, int64_t n, int64_t m, int64_t p,
-                             int splits, cudaStream_t s) {
+                             int splits, cudaStream_t s, bool b_mn) {
     CUtensorMap ma, mb;
-    if (!make_map(&ma, A, n, m, TC_BM) || !make_map(&mb, Bt, p, m, TC_BN)) return cudaErrorInvalidValue;
+    if (!make_map(&ma, A, n, m, TC_BM) || !(b_mn ? make_map_mn(&mb, Bt, m, p) : make_map(&mb, Bt, p, m, TC_BN)))
+        return cudaErrorInvalidValue;
     static std::once_flag once;
     std::call_once(once, [] {
-        cudaFuncSetAttribute(mm_top_tc_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
-        cudaFuncSetAttribute(mm_top_tc_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
+        cudaFuncSetAttribute(mm_top_tc_kernel<true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
+        cudaFuncSetAttribute(mm_top_tc_kernel<false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
+        cudaFuncSetAttribute(mm_top_tc_kernel<true, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
+        cudaFuncSetAttribute(mm_top_tc_kernel<false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, TC_SMEM_P);
     });
     const int nk = (int)ceil_div(m, TC_BK);
     const int kps = (int)ceil_div(nk, splits);
@@ -375,10 +421,21 @@ cudaError_t launch_mm_top_tc(const void* A, const void* Bt, float* C, float* par
     // 8192^3: 1.51 vs 1.36 PF, DRAM 1.3 vs 3.4 GB; 4096^3 is faster in row order)
     const int64_t opbytes = 2 * (n * m + p * m);
     const int group = opbytes > ((int64_t)96 << 20) ? IFL_TC_GROUP : 1;
-    if (tst)
-        mm_top_tc_kernel<true><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, mc, C, part, n, m, p, kps, splits, group);
-    else
-        mm_top_tc_kernel<false><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, ma, C, part, n, m, p, kps, splits, group);
+    if (tst) {
+        if (b_mn)
+            mm_top_tc_kernel<true, true><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, mc, C, part, n, m, p, kps, splits,
+                                                                            group);
+        else
+            mm_top_tc_kernel<true, false><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, mc, C, part, n, m, p, kps, splits,
+                                                                             group);
+    } else {
+        if (b_mn)
+            mm_top_tc_kernel<false, true><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, ma, C, part, n, m, p, kps, splits,
+                                                                             group);
+        else
+            mm_top_tc_kernel<false, false><<<grid, TC_THREADS, TC_SMEM_P, s>>>(ma, mb, ma, C, part, n, m, p, kps,
+                                                                              splits, group);
+    }
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess || splits == 1) return e;
     const int64_t outs = n * p;

@@ -153,3 +153,10 @@ def test_tc_8192_cube_first_last_tiles(ifl, orc):
     cols = [0, 255, 256, 7935, 7936, 8191]
     want, ab = orc.redomap2(bits(A), bits(Bt[cols]), b_kmajor=True, with_abs=True)
     assert (np.abs(C[:, cols].numpy().astype(np.float64) - want) <= 1e-5 * ab + 1e-30).all()
+    # B as yss [m][p] (b_kmajor = 0): the MN-major operand path, no transposition
+    C2 = ifl.redomap2(A.cuda(), Bt.t().contiguous().cuda(), b_kmajor=False, version="top").cpu()
+    rows2 = [0, 8064, 8191]
+    want, ab = orc.redomap2(bits(A[rows2]), bits(Bt), b_kmajor=True, with_abs=True)
+    assert (np.abs(C2[rows2].numpy().astype(np.float64) - want) <= 1e-5 * ab + 1e-30).all()
+    want, ab = orc.redomap2(bits(A), bits(Bt[[0, 7936, 8191]]), b_kmajor=True, with_abs=True)
+    assert (np.abs(C2[:, [0, 7936, 8191]].numpy().astype(np.float64) - want) <= 1e-5 * ab + 1e-30).all()

@@ -38,5 +38,8 @@ for q in [int(a) for a in sys.argv[1:]] or [2048, 4096, 8192]:
     ws = ifl.workspace(ifl.workspace_bytes("redomap2", q, q, q, "bf16"), "cuda", "mm")
     t = gtime(lambda: ifl.redomap2(A, Bt, out=C, ws=ws, version="top"))
     tc = gtime(lambda: torch.matmul(A, Bt.t()))
+    B = Bt.t().contiguous()  # yss [m][p]: the MN-major operand path (b_kmajor = 0)
+    trm = gtime(lambda: ifl.redomap2(A, B, b_kmajor=False, out=C, ws=ws, version="top"))
     print(json.dumps({"q": q, "us": round(t * 1e3, 1), "TFLOPs": round(2 * q**3 / t / 1e9, 1),
+                      "rowmajor_B_us": round(trm * 1e3, 1), "rowmajor_over_kmajor": round(trm / t, 3),
                       "cublas_TFLOPs": round(2 * q**3 / tc / 1e9, 1)}), flush=True)
