@@ -354,7 +354,7 @@ struct SkinnyGeom {
 template <int RI, int RJ>
 __device__ __forceinline__ void skinny_store(float v, float* __restrict__ part, float* __restrict__ C,
                                              unsigned* __restrict__ cnt, int64_t n, int64_t p, int64_t i0,
-                                             int64_t j0, int tile) {
+                                             int64_t j0, int tile, float* red) {
     __shared__ unsigned s_last;
     const int t = threadIdx.x;
     const int splits = (int)gridDim.x;
@@ -371,10 +371,22 @@ __device__ __forceinline__ void skinny_store(float v, float* __restrict__ part, 
     __syncthreads();
     if (!s_last) return;
     __threadfence();
+    // every thread sums a fixed contiguous block of the splits of one output,
+    // the blocks are added in block order: a fixed association whatever the
+    // arrival order (deterministic), with the CTA's loads in flight together
+    constexpr int NO = RI * RJ, TPO = kSkinnyThreads / NO;
+    const int o = t % NO, g = t / NO;
+    const int64_t io = i0 + o / RJ, jo = j0 + o % RJ;
+    const int chunk = (splits + TPO - 1) / TPO, q0 = g * chunk, q1 = min(splits, q0 + chunk);
+    float r = 0.f;
+    if (io < n && jo < p)
+        for (int q = q0; q < q1; ++q) r += __ldcg(part + (int64_t)q * n * p + io * p + jo);
+    red[g * NO + o] = r;
+    __syncthreads();
     if (own) {
-        float r = 0.f;
-        for (int q = 0; q < splits; ++q) r += __ldcg(part + (int64_t)q * n * p + i * p + j);
-        C[i * p + j] = r;
+        float sum = 0.f;
+        for (int q = 0; q < TPO; ++q) sum += red[q * NO + t];
+        C[i * p + j] = sum;
     }
     if (t == 0) cnt[tile] = 0u;
 }
@@ -387,7 +399,8 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __
     using Gm = SkinnyGeom<Tin, RI, RJ, KMAJ>;
     constexpr int E = Gm::E, NW = kSkinnyThreads / 32, S = Gm::S;
     extern __shared__ __align__(16) uint2 sbuf[];  // [S][WORDS][threads]
-    __shared__ float red[NW][RI * RJ];
+    constexpr int NRED = NW * RI * RJ > kSkinnyThreads ? NW * RI * RJ : kSkinnyThreads;
+    __shared__ float red[NRED];  // [NW][RI * RJ] per-warp sums, then the finalize's [TPO][RI * RJ]
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
     const int tile = blockIdx.y;
     const int64_t i0 = (int64_t)(tile / tiles_j) * RI, j0 = (int64_t)(tile % tiles_j) * RJ;
@@ -473,14 +486,15 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __
 #pragma unroll
         for (int c = 0; c < RJ; ++c) {
             const float v = warp_reduce<OP_SUM>(acc[r][c]);
-            if (lane == 0) red[w][r * RJ + c] = v;
+            if (lane == 0) red[w * RI * RJ + r * RJ + c] = v;
         }
     __syncthreads();
     float s = 0.f;
     if (t < RI * RJ)
 #pragma unroll
-        for (int q = 0; q < NW; ++q) s += red[q][t];
-    skinny_store<RI, RJ>(s, part, C, cnt, n, p, i0, j0, tile);
+        for (int q = 0; q < NW; ++q) s += red[q * RI * RJ + t];
+    __syncthreads();  // red is reused by the finalize
+    skinny_store<RI, RJ>(s, part, C, cnt, n, p, i0, j0, tile, red);
 }
 
 // Scalar form (misaligned operands or m not a multiple of the vector width).
@@ -493,7 +507,8 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const 
                                                                           int64_t m, int64_t p, int64_t kchunk,
                                                                           int tiles_j) {
     constexpr int NW = kSkinnyThreads / 32;
-    __shared__ float red[NW][RI * RJ];
+    constexpr int NRED = NW * RI * RJ > kSkinnyThreads ? NW * RI * RJ : kSkinnyThreads;
+    __shared__ float red[NRED];  // [NW][RI * RJ] per-warp sums, then the finalize's [TPO][RI * RJ]
     const int t = threadIdx.x, lane = t & 31, w = t >> 5;
     const int tile = blockIdx.y;
     const int64_t i0 = (int64_t)(tile / tiles_j) * RI, j0 = (int64_t)(tile % tiles_j) * RJ;
@@ -522,14 +537,15 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const 
 #pragma unroll
         for (int c = 0; c < RJ; ++c) {
             const float v = warp_reduce<OP_SUM>(acc[r][c]);
-            if (lane == 0) red[w][r * RJ + c] = v;
+            if (lane == 0) red[w * RI * RJ + r * RJ + c] = v;
         }
     __syncthreads();
     float s = 0.f;
     if (t < RI * RJ)
 #pragma unroll
-        for (int q = 0; q < NW; ++q) s += red[q][t];
-    skinny_store<RI, RJ>(s, part, C, cnt, n, p, i0, j0, tile);
+        for (int q = 0; q < NW; ++q) s += red[q * RI * RJ + t];
+    __syncthreads();  // red is reused by the finalize
+    skinny_store<RI, RJ>(s, part, C, cnt, n, p, i0, j0, tile, red);
 }
 
 // Where the engine is V_FLAT's form: f32 up to 4096 outputs; bf16 up to 256
@@ -538,7 +554,7 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_scalar_kernel(const 
 static bool skinny_ok(int64_t n, int64_t p, bool bf16) { return n * p <= (bf16 ? 256 : kSkinnyMaxOuts); }
 static int skinny_r(int64_t x) { return x >= 8 ? 8 : x >= 4 ? 4 : x >= 2 ? 2 : 1; }
 // k-chunks: one wave of CTAs over all output tiles (as many per SM as the
-// pipeline's shared memory allows), >= 2 vector rounds per chunk
+// pipeline's shared memory allows), >= 1 vector round per chunk
 static int64_t skinny_kchunk(int64_t n, int64_t m, int64_t p) {
     const int64_t tiles = ceil_div(n, skinny_r(n)) * ceil_div(p, skinny_r(p));
     // CTAs per SM the pipeline's shared memory allows (K-major words; >= 1, <= 4)
@@ -546,7 +562,7 @@ static int64_t skinny_kchunk(int64_t n, int64_t m, int64_t p) {
     const int S = std::min(12, std::max(3, kSkinnyStageBytes / (words * kSkinnyThreads * 8)));
     const int occ = std::min(4, std::max(1, (200 * 1024) / (S * words * kSkinnyThreads * 8)));
     const int64_t want = std::max<int64_t>(1, (int64_t)148 * occ / tiles);
-    int64_t kc = std::max<int64_t>((int64_t)kSkinnyThreads * 8, ceil_div(m, want));
+    int64_t kc = std::max<int64_t>((int64_t)kSkinnyThreads * 2, ceil_div(m, want));  // >= one 8-byte vector per thread
     return ceil_div(kc, 8) * 8;  // a multiple of every vector width
 }
 static int64_t skinny_splits(int64_t n, int64_t m, int64_t p) { return ceil_div(m, skinny_kchunk(n, m, p)); }
