@@ -391,7 +391,7 @@ __device__ __forceinline__ void skinny_store(float v, float* __restrict__ part, 
     if (t == 0) cnt[tile] = 0u;
 }
 
-template <typename Tin, int RI, int RJ, bool KMAJ>
+template <typename Tin, int RI, int RJ, bool KMAJ, bool CP>
 __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __restrict__ A, const Tin* __restrict__ B,
                                                                    float* __restrict__ part, float* __restrict__ C,
                                                                    unsigned* __restrict__ cnt, int64_t n, int64_t m,
@@ -414,16 +414,39 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __
 #pragma unroll
     for (int c = 0; c < RJ; ++c) br[c] = B + std::min(j0 + c, p - 1) * m;  // KMAJ rows of B^T
     auto slot = [&](int st, int word) -> uint2* { return sbuf + ((size_t)st * Gm::WORDS + word) * kSkinnyThreads + t; };
+    // row-major B with slices of >= 16 bytes (COOP): the warp copies its
+    // 32*E k-rows' slices lane-contiguously (coalesced 8-byte pieces) into
+    // the owners' slots; B word idx of thread t lives at slot t ^ swz(idx)
+    // so that both the copies and the owners' reads are bank-conflict-free
+    constexpr int UPR = Gm::SLICE >= 8 ? Gm::SLICE / 8 : 1, KW = E * UPR;
+    constexpr int KWS = KW <= 16 ? KW : 16;  // (a divisor of 16 whenever COOP)
+    constexpr bool COOP = CP && !KMAJ && Gm::SLICE >= 16 && Gm::UNIT == 8 && KW <= 16 && (16 % KWS) == 0;
+    auto swz = [](int idx) { return COOP ? (idx * (16 / KWS)) & 15 : 0; };
+    auto bslot = [&](int st, int idx, int owner) -> uint2* {
+        return sbuf + ((size_t)st * Gm::WORDS + RI + idx) * kSkinnyThreads + (owner ^ swz(idx));
+    };
     auto issue = [&](int it) {
         const int64_t k = k0 + (int64_t)it * stride + (int64_t)t * E;
+        const int st = it % S;
+        if constexpr (COOP) {
+            const int64_t kw = k0 + (int64_t)it * stride + (int64_t)(t & ~31) * E;
+            if (it < nit) {
+#pragma unroll
+                for (int r = 0; r < KW; ++r) {
+                    const int q = lane + 32 * r, row = q / UPR, u = q % UPR;
+                    if (kw + row < k1)
+                        cp_async8(bslot(st, (row % E) * UPR + u, (t & ~31) + row / E),
+                                  reinterpret_cast<const char*>(B + (kw + row) * p + j0) + u * 8);
+                }
+            }
+        }
         if (it < nit && k < k1) {
-            const int st = it % S;
 #pragma unroll
             for (int r = 0; r < RI; ++r) cp_async8(slot(st, r), ar[r] + k);
             if constexpr (KMAJ) {
 #pragma unroll
                 for (int c = 0; c < RJ; ++c) cp_async8(slot(st, RI + c), br[c] + k);
-            } else {
+            } else if constexpr (!COOP) {
 #pragma unroll
                 for (int e = 0; e < E; ++e) {
                     const char* src = reinterpret_cast<const char*>(B + (k + e) * p + j0);
@@ -448,15 +471,28 @@ __global__ void __launch_bounds__(kSkinnyThreads) mm_skinny_kernel(const Tin* __
 #pragma unroll
     for (int s = 0; s < S - 1; ++s) issue(s);
     for (int it = 0; it < nit; ++it) {
+        if constexpr (COOP) __syncwarp();  // the warp is done with the stage it refills now
         issue(it + S - 1);
         cp_async_wait<S - 1>();  // this thread's copies of iteration it have landed
+        if constexpr (COOP) __syncwarp();  // ... and those of the other lanes
         const int64_t k = k0 + (int64_t)it * stride + (int64_t)t * E;
         if (k >= k1) continue;
         const int st = it % S;
         float a[RI][E], b[RJ][E];
 #pragma unroll
         for (int r = 0; r < RI; ++r) unpack8<Tin>(*slot(st, r), a[r]);
-        if constexpr (KMAJ) {
+        if constexpr (COOP) {
+#pragma unroll
+            for (int e = 0; e < E; ++e)
+#pragma unroll
+                for (int c = 0; c < RJ; ++c) {
+                    const int byte = c * (int)sizeof(Tin);
+                    const uint2 wd = *bslot(st, e * UPR + byte / 8, t);
+                    const uint32_t h = (byte % 8) < 4 ? wd.x : wd.y;
+                    if constexpr (std::is_same<Tin, float>::value) b[c][e] = __uint_as_float(h);
+                    else b[c][e] = __uint_as_float((byte % 4) == 0 ? (h << 16) : (h & 0xffff0000u));
+                }
+        } else if constexpr (KMAJ) {
 #pragma unroll
             for (int c = 0; c < RJ; ++c) unpack8<Tin>(*slot(st, RI + c), b[c]);
         } else {
@@ -581,10 +617,17 @@ static cudaError_t launch_skinny_k(const Tin* A, const Tin* B, float* part, floa
     dim3 g((unsigned)splits, (unsigned)tiles);
     if (vec) {
         const size_t smem = Gm::SMEM;
-        auto k = mm_skinny_kernel<Tin, RI, RJ, KMAJ>;
+        // row-major B spread over several column tiles (p > RJ): slices are
+        // strided within the rows, copied warp-cooperatively (measured on B200:
+        // k = 25 f32 n = p = 16..64 1.44-1.56x -> 1.10-1.17x the k-major time;
+        // with one column tile a thread's own rows are contiguous already)
+        auto k = p > RJ ? mm_skinny_kernel<Tin, RI, RJ, KMAJ, true> : mm_skinny_kernel<Tin, RI, RJ, KMAJ, false>;
         static bool attr = false;
         if (!attr) {
-            cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            cudaFuncSetAttribute(mm_skinny_kernel<Tin, RI, RJ, KMAJ, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem);
+            cudaFuncSetAttribute(mm_skinny_kernel<Tin, RI, RJ, KMAJ, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)smem);
             attr = true;
         }
         k<<<g, kSkinnyThreads, smem, s>>>(A, B, part, C, cnt, n, m, p, kc, tj);
