@@ -151,14 +151,20 @@ def test_irr_empty_inspector_and_guard(ifl):
         ifl.reset_thresholds()
 
 
-def test_irr_bench_size_sampled(ifl, orc):
-    # the bench recipe at 2^26 elements: Pareto lengths, mean 64 (full oracle comparison)
-    off = gen.irregular_offsets(12, (1 << 26) // 64, 64.0)
+@pytest.mark.parametrize("mean", [1.0, 64.0, 65536.0])
+def test_irr_bench_size_sampled(ifl, orc, mean):
+    # the bench recipe at 2^26 elements: Pareto lengths, means 1 (mostly empty
+    # and unit segments), 64 and 65536 (tiles inside one segment): every
+    # output against the oracle, both operations, the merge-path V_FLAT and AUTO
+    off = gen.irregular_offsets(12, int((1 << 26) // mean), mean)
     offd = torch.from_numpy(off).cuda()
     x = gen.generate("F32_UNIT", 94, int(off[-1]))
     mx = ifl.irr_inspect(offd, int(off[-1]))
     assert mx == int(np.diff(off).max())
-    want, ab = orc.seg_irr(x.numpy(), off, False, with_absum=True)
-    for v in ("middle", "flat", "auto"):
-        got = ifl.segred_irr(x.cuda(), offd, version=v, max_len=mx).cpu().numpy()
-        assert (np.abs(got - want) <= 1e-5 * ab).all(), v
+    xd = x.cuda()
+    for scan in (False, True):
+        want, ab = orc.seg_irr(x.numpy(), off, scan, with_absum=True)
+        fn = ifl.segscan_irr if scan else ifl.segred_irr
+        for v in (("middle", "flat", "auto") if mean == 64.0 and not scan else ("flat", "auto")):
+            got = fn(xd, offd, version=v, max_len=mx).cpu().numpy()
+            assert (np.abs(got - want) <= 1e-5 * ab).all(), (v, scan)
