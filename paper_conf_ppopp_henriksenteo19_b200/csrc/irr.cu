@@ -309,30 +309,7 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
     // ---- staging
 #pragma unroll 4
     for (int k = t; k < ns; k += kMpThreads) s_b[pd(k)] = (int)(__ldg(off + i0 + 1 + k) - j0);
-    // elements: 16-byte loads from the aligned base a = j0 - R (group g holds
-    // local elements 4g - R .. 4g - R + 3; a group reaching past the array is
-    // read element by element), scattered into the padded shared array
-    const int64_t va = j0 & ~(int64_t)3;
-    const int vR = (int)(j0 - va), vG = (vR + ne + 3) >> 2;
-    if (vec) {
-#pragma unroll 4
-        for (int g = t; g < vG; g += kMpThreads) {
-            const int kb = 4 * g - vR;
-            T e[4];
-            if (va + 4 * g + 4 <= total) {
-                typename Vec4<T>::type u;
-                if constexpr (SCAN) u = __ldcs(reinterpret_cast<const typename Vec4<T>::type*>(in + va) + g);
-                else u = ldg_stream4(in + va + 4 * g);
-                unpack4<T>(u, e);
-            } else {
-#pragma unroll
-                for (int c = 0; c < 4; ++c) e[c] = (kb + c >= 0 && kb + c < ne) ? in[j0 + kb + c] : T();
-            }
-#pragma unroll
-            for (int c = 0; c < 4; ++c)
-                if (kb + c >= 0 && kb + c < ne) X(kb + c) = (int)to_bits<T>(e[c]);
-        }
-    } else if constexpr (SCAN) {
+    if constexpr (SCAN) {
 #pragma unroll 8
         for (int k = t; k < ne; k += kMpThreads) X(k) = (int)to_bits<T>(__ldcs(in + j0 + k));
     } else {
@@ -431,26 +408,8 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
                 X(j_s + k) = (int)to_bits<T>(combine<OP>(exv, from_bits<T>((uint32_t)X(j_s + k))));
         }
         __syncthreads();
-        if (vec) {  // 16-byte stores of the groups inside the tile, element stores at its two ends
-#pragma unroll 4
-            for (int g = t; g < vG; g += kMpThreads) {
-                const int kb = 4 * g - vR;
-                if (kb >= 0 && kb + 4 <= ne) {
-                    typename Vec4<T>::type u;
-                    u.x = from_bits<T>((uint32_t)X(kb));
-                    u.y = from_bits<T>((uint32_t)X(kb + 1));
-                    u.z = from_bits<T>((uint32_t)X(kb + 2));
-                    u.w = from_bits<T>((uint32_t)X(kb + 3));
-                    __stcs(reinterpret_cast<typename Vec4<T>::type*>(out + va) + g, u);
-                } else {
-#pragma unroll
-                    for (int c = 0; c < 4; ++c)
-                        if (kb + c >= 0 && kb + c < ne) __stcs(out + j0 + kb + c, from_bits<T>((uint32_t)X(kb + c)));
-                }
-            }
-        } else {
-            for (int k = t; k < ne; k += kMpThreads) __stcs(out + j0 + k, from_bits<T>((uint32_t)X(k)));
-        }
+#pragma unroll 8
+        for (int k = t; k < ne; k += kMpThreads) __stcs(out + j0 + k, from_bits<T>((uint32_t)X(k)));
     } else {
         if (first >= 0) {
             const T v = combine<OP>(exv, from_bits<T>((uint32_t)s_b[pd(first)]));
