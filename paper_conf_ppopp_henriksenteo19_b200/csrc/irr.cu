@@ -277,7 +277,8 @@ __device__ __forceinline__ void mp_elems_red(const T* __restrict__ in, int64_t j
 // (int32, relative to its first element) and elements share one padded
 // shared-memory array: ends at [0, ns), elements at [ns, ns + ne).
 // segscan: in may equal out (a tile reads and writes only its own elements;
-// coherent loads).
+// coherent loads).  Pass A scans only the elements after a thread's first
+// segment start; pass B scans the thread's lead elements from its carry.
 template <typename T, int OP, int F, bool SCAN>
 __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out, const int64_t* __restrict__ off,
                                                             int64_t n, int64_t total, T d,
@@ -350,7 +351,7 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
             const bool elt = valid && !end;
             const T nacc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j))));  // j <= ne: inside
             if constexpr (SCAN) {
-                if (elt) X(j) = (int)to_bits<T>(nacc);
+                if (elt && seen) X(j) = (int)to_bits<T>(nacc);  // lead elements are scanned in pass B
             } else {
                 if (end) s_b[pd(i)] = (int)to_bits<T>(acc);
                 first = (end && first < 0) ? i : first;
@@ -374,10 +375,15 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
         while (rem > 0) {
             const int ce = i < ie ? s_b[pd(i)] : 0x7fffffff;
             const int run = min(ce - j, rem);  // elements before the next end
+            if (SCAN && seen) {
 #pragma unroll 4
-            for (int q = 0; q < run; ++q) {
-                acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j + q))));
-                if constexpr (SCAN) X(j + q) = (int)to_bits<T>(acc);
+                for (int q = 0; q < run; ++q) {
+                    acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j + q))));
+                    X(j + q) = (int)to_bits<T>(acc);
+                }
+            } else {  // segred, or segscan's lead elements (scanned in pass B)
+#pragma unroll 4
+                for (int q = 0; q < run; ++q) acc = combine<OP>(acc, apply_map<F>(from_bits<T>((uint32_t)X(j + q))));
             }
             if (!seen) lead += run;
             j += run;
@@ -399,13 +405,20 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
     T exv, aggv;
     irr_cta_seg_scan<T, OP, kMpThreads>(first >= 0 ? 1u : 0u, acc, start_f, init_v, exf, exv, aggf, aggv, s_v, s_f);
     if constexpr (SCAN) {
+        // pass B: the elements before the thread's first segment start, scanned
+        // from the thread's carry (pass A only reduced them)
+        T a2 = exv;
         if (lead == kMpItems) {
 #pragma unroll
-            for (int k = 0; k < kMpItems; ++k)
-                X(j_s + k) = (int)to_bits<T>(combine<OP>(exv, from_bits<T>((uint32_t)X(j_s + k))));
+            for (int k = 0; k < kMpItems; ++k) {
+                a2 = combine<OP>(a2, apply_map<F>(from_bits<T>((uint32_t)X(j_s + k))));
+                X(j_s + k) = (int)to_bits<T>(a2);
+            }
         } else {
-            for (int k = 0; k < lead; ++k)
-                X(j_s + k) = (int)to_bits<T>(combine<OP>(exv, from_bits<T>((uint32_t)X(j_s + k))));
+            for (int k = 0; k < lead; ++k) {
+                a2 = combine<OP>(a2, apply_map<F>(from_bits<T>((uint32_t)X(j_s + k))));
+                X(j_s + k) = (int)to_bits<T>(a2);
+            }
         }
         __syncthreads();
 #pragma unroll 8
