@@ -131,6 +131,10 @@ constexpr int kMpThreads = 128, kMpItems = 32, kMpItemsLog2 = 5;
 static_assert(kMpThreads * kMpItems == kIrrTile && (1 << kMpItemsLog2) == kMpItems, "merge-path tile");
 __device__ __forceinline__ int pd(int k) { return k + (k >> 5); }
 
+__device__ __forceinline__ void mp_cp_async4(void* smem, const void* gmem) {
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(smem)), "l"(gmem) : "memory");
+}
+
 // CTA-wide exclusive scan of (flag, value) thread pieces under the segmented
 // operator (f1,v1).(f2,v2) = (f1|f2, f2 ? v2 : v1 (+) v2), seeded with an
 // initial piece (init_f, init_v): exf/exv = everything before the thread,
@@ -307,16 +311,16 @@ __global__ void __launch_bounds__(kMpThreads) irr_mp_kernel(const T* in, T* out,
         }
     }
     auto X = [&](int j) -> int& { return s_b[pd(ns + j)]; };
-    // ---- staging
+    // ---- staging.  Elements: asynchronous 4-byte copies, all in flight at
+    // once without registers (a register-staged loop keeps ~8 loads per
+    // thread in flight: four DRAM round trips per tile), issued first so the
+    // ends' loads overlap them
+#pragma unroll 8
+    for (int k = t; k < ne; k += kMpThreads) mp_cp_async4(&X(k), in + j0 + k);
+    asm volatile("cp.async.commit_group;" ::: "memory");
 #pragma unroll 4
     for (int k = t; k < ns; k += kMpThreads) s_b[pd(k)] = (int)(__ldg(off + i0 + 1 + k) - j0);
-    if constexpr (SCAN) {
-#pragma unroll 8
-        for (int k = t; k < ne; k += kMpThreads) X(k) = (int)to_bits<T>(__ldcs(in + j0 + k));
-    } else {
-#pragma unroll 8
-        for (int k = t; k < ne; k += kMpThreads) X(k) = (int)to_bits<T>(__ldg(in + j0 + k));
-    }
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
     if (t == 0) s_skip0 = 0;
     __syncthreads();
     const int Wt = ns + ne;
