@@ -87,6 +87,49 @@ def test_over_2_31_rows(ifl):
         torch.cuda.empty_cache()
 
 
+@pytest.mark.parametrize("dt", ["i32", "f32"])
+def test_irregular_over_2_31_elements(ifl, orc, dt):
+    """Irregular segments over 2^31 + 5 elements through the merge-path V_FLAT
+    (64-bit element and tile coordinates): 40 segments of ragged lengths with
+    empty ones between them, one of them holding element 2^31; sampled
+    segments (first, last, the one across 2^31, two more) against the oracle,
+    both operations."""
+    name = "I32_FULL" if dt == "i32" else "F32_UNIT"
+    total = 2**31 + 5
+    rng = np.random.default_rng(21)
+    w = rng.uniform(0.2, 1.8, 40)
+    lens = np.floor(w / w.sum() * total).astype(np.int64)
+    lens[-1] += total - lens.sum()
+    lens = np.insert(lens, [3, 3, 17, 30], 0)  # empty segments
+    off = np.zeros(lens.size + 1, np.int64)
+    np.cumsum(lens, out=off[1:])
+    assert off[-1] == total
+    x = gen.generate(name, 14, total, device="cuda")
+    offd = torch.from_numpy(off).cuda()
+    cross = int(np.searchsorted(off, 2**31, side="right") - 1)
+    segs = sorted({0, 3, cross, 25, lens.size - 1})
+    for scan in (False, True):
+        fn = ifl.segscan_irr if scan else ifl.segred_irr
+        got = fn(x, offd, "sum", version="flat")
+        torch.cuda.synchronize()
+        for i in segs:
+            a, b = int(off[i]), int(off[i + 1])
+            xs = x[a:b].cpu().numpy()
+            sub = np.array([0, b - a], np.int64)
+            if dt == "i32":
+                want = orc.seg_irr(xs, sub, scan)
+                g = got[a:b] if scan else got[i:i + 1]
+                np.testing.assert_array_equal(g.cpu().numpy(), want, err_msg=f"seg {i} scan={scan}")
+            else:
+                want, ab = orc.seg_irr(xs, sub, scan, with_absum=True)
+                g = (got[a:b] if scan else got[i:i + 1]).cpu().numpy().astype(np.float64)
+                assert (np.abs(g - want) <= 1e-5 * ab).all(), f"seg {i} scan={scan}"
+        del got
+        torch.cuda.empty_cache()
+    del x
+    torch.cuda.empty_cache()
+
+
 def _free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
