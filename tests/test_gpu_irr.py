@@ -168,3 +168,9 @@ def test_irr_bench_size_sampled(ifl, orc, mean):
         for v in (("middle", "flat", "auto") if mean == 64.0 and not scan else ("flat", "auto")):
             got = fn(xd, offd, version=v, max_len=mx).cpu().numpy()
             assert (np.abs(got - want) <= 1e-5 * ab).all(), (v, scan)
+    # in place at full size (every tile reads its elements before any tile writes them back)
+    xin = x.cuda()
+    got = ifl.segscan_irr(xin, offd, version="flat", out=xin)
+    assert got.data_ptr() == xin.data_ptr()
+    want, ab = orc.seg_irr(x.numpy(), off, True, with_absum=True)
+    assert (np.abs(got.cpu().numpy() - want) <= 1e-5 * ab).all(), "in place"
