@@ -630,6 +630,15 @@ def suite_dist():
         os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(s.getsockname()[1]))
         s.close()
         td.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    # the local segreds run AUTO with thresholds tuned as the bench tunes them
+    # (V_MIDDLE group size, then the 4-leaf chain on the 2^25 / 2^27 sweeps)
+    train = [(1 << k, 1 << (lg - k)) for lg in (25, 27) for k in range(lg + 1)]
+    g, _, _ = ifl.tune("segred.b4.midg", [s for s in train if s[1] <= 8192], reps=7, cost=1)
+    nb = ifl.lib().ifl_tune_scratch_bytes(b"segred.b4.tree", np.asarray(train, np.int64).ctypes.data, len(train))
+    scratch = torch.empty(nb, dtype=torch.uint8, device="cuda")
+    scratch.view(-1)[: (nb // 4) * 4].view(torch.float32).copy_(gen.generate("F32_UNIT", 4, nb // 4, device="cuda"))
+    ifl.tune("segred.b4.tree", train, reps=7, cost=1, scratch=scratch)
+    del scratch
     N = 1 << 30
     x = gen.generate("F32_UNIT", 8, N, device="cuda")
     rows = []
@@ -651,6 +660,8 @@ def suite_dist():
                      {"workload": "configs[4]: 2^30 f32 segred via dist.py over n in {1, 2^4, 2^10, 2^16, 2^20, "
                                   "2^24}, world size 1 on this box (default device-level guard)"})
     line["scaling"] = "weak"
+    line["thresholds"] = {"segred.b4": list(ifl.get_thresholds("segred.b4")),
+                          "segred.b4.cl": list(ifl.get_thresholds("segred.b4.cl")), "group_shift": g - 8}
     line["best_shape_GBps"] = round(best, 1)
     line["rows"] = rows
     line["roofline"] = {"bound": "hbm", "kernel": "segred sweep (read-only stream: the copy peak counts a read "
