@@ -26,6 +26,9 @@ namespace ifl {
 namespace {
 
 constexpr int kLvcThreads = 256;
+#ifndef IFL_LVC_CHAINS
+#define IFL_LVC_CHAINS 2  // independent scan chains per lane (2 = the half chains of round 1)
+#endif
 
 template <int IT>
 __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcSite sy, int gx, int Gx, int Gy,
@@ -78,30 +81,33 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
     //            y'_k = loc_k + P_k * p  with P_k = alpha_{j0} ... alpha_{j0+k}
     //            and p the group-exclusive prefix (the value entering the lane);
     //   backward x_j = delta_j x_{j+1} + eps_j, mirrored with suffix products.
-    // The lane's items are scanned as two independent half chains (H = IT/2
-    // items each, twice the instruction-level parallelism of one chain); the
-    // halves are joined with their slope products:
-    //   Q[k] = alpha_{j0+h0} ... alpha_{j0+k}   (h0 = 0 for the first half, H for the second)
-    //   E[k] = delta_{j0+k} ... delta_{j0+h1}   (h1 = H-1 for the first half, IT-1 for the second)
-    constexpr int H = IT / 2;
-    float Q[IT], E[IT];
-    {
+    // The lane's items are scanned as NC independent chains of C = IT / NC
+    // items (NC-fold instruction-level parallelism), joined with their slope
+    // products:
+    //   Q[k] = alpha_{chain start} ... alpha_{j0+k},  QE[c] = Q at chain c's end
+    //   E[k] = delta_{j0+k} ... delta_{chain end},    EE[c] = E at chain c's start
+    constexpr int NC = IFL_LVC_CHAINS, C = IT / NC;
+    static_assert(IT % NC == 0 && C >= 1, "chains");
+    float Q[IT], E[IT], QE[NC], EE[NC];
+#pragma unroll
+    for (int c = 0; c < NC; ++c) {
         float pr = 1.f;
 #pragma unroll
-        for (int k = 0; k < H; ++k) Q[k] = pr = pr * al[k];
+        for (int k = c * C; k < (c + 1) * C; ++k) Q[k] = pr = pr * al[k];
+        QE[c] = pr;
         pr = 1.f;
 #pragma unroll
-        for (int k = H; k < IT; ++k) Q[k] = pr = pr * al[k];
-        pr = 1.f;
-#pragma unroll
-        for (int k = IT - 1; k >= H; --k) E[k] = pr = pr * de[k];
-        pr = 1.f;
-#pragma unroll
-        for (int k = H - 1; k >= 0; --k) E[k] = pr = pr * de[k];
+        for (int k = (c + 1) * C - 1; k >= c * C; --k) E[k] = pr = pr * de[k];
+        EE[c] = pr;
     }
     float raf[5], rab[5];  // slope of the running inclusive map before each shuffle round
     {
-        float af = Q[H - 1] * Q[IT - 1], ab = E[0] * E[H];
+        float af = 1.f, ab = 1.f;
+#pragma unroll
+        for (int c = 0; c < NC; ++c) {
+            af *= QE[c];
+            ab *= EE[c];
+        }
 #pragma unroll
         for (int r = 0; r < 5; ++r) {
             const int off = 1 << r;
@@ -116,14 +122,17 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
         }
     }
     for (int64_t t = 0; t < numT; ++t) {
-        // (x) forward: half chains from 0, lane total g = gB + Q_B * gA
-        float gA = 0.f, gB = 0.f;
+        // (x) forward: chains from 0, then the lane total e = QE[c] e + g_c
+        float gc[NC];
 #pragma unroll
-        for (int k = 0; k < H; ++k) {
-            yv[k] = gA = fmaf(al[k], gA, yv[k]);
-            yv[H + k] = gB = fmaf(al[H + k], gB, yv[H + k]);
-        }
-        float g = fmaf(Q[IT - 1], gA, gB);
+        for (int c = 0; c < NC; ++c) gc[c] = 0.f;
+#pragma unroll
+        for (int k = 0; k < C; ++k)
+#pragma unroll
+            for (int c = 0; c < NC; ++c) yv[c * C + k] = gc[c] = fmaf(al[c * C + k], gc[c], yv[c * C + k]);
+        float g = gc[0];
+#pragma unroll
+        for (int c = 1; c < NC; ++c) g = fmaf(QE[c], g, gc[c]);
 #pragma unroll
         for (int r = 0; r < 5; ++r) {
             const int off = 1 << r;
@@ -134,20 +143,26 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
         }
         float p = __shfl_up_sync(0xffffffffu, g, 1, G);
         if (gl == 0) p = 0.f;
-        const float vA = fmaf(Q[H - 1], p, gA);  // y' at the end of the first half
+        float vin[NC];  // y' entering each chain
+        vin[0] = p;
 #pragma unroll
-        for (int k = 0; k < H; ++k) {
-            yv[k] = fmaf(Q[k], p, yv[k]) * ib[k];  // eps_j = y'_j / beta_j
-            yv[H + k] = fmaf(Q[H + k], vA, yv[H + k]) * ib[H + k];
-        }
-        // (.) backward: half chains from 0 (from each half's right end)
-        float hA = 0.f, hB = 0.f;
+        for (int c = 1; c < NC; ++c) vin[c] = fmaf(QE[c - 1], vin[c - 1], gc[c - 1]);
 #pragma unroll
-        for (int k = H - 1; k >= 0; --k) {
-            yv[k] = hA = fmaf(de[k], hA, yv[k]);
-            yv[H + k] = hB = fmaf(de[H + k], hB, yv[H + k]);
-        }
-        float h = fmaf(E[0], hB, hA);
+        for (int k = 0; k < C; ++k)
+#pragma unroll
+            for (int c = 0; c < NC; ++c)
+                yv[c * C + k] = fmaf(Q[c * C + k], vin[c], yv[c * C + k]) * ib[c * C + k];  // eps_j = y'_j / beta_j
+        // (.) backward: chains from 0 at their right ends, lane total from the right
+        float hc[NC];
+#pragma unroll
+        for (int c = 0; c < NC; ++c) hc[c] = 0.f;
+#pragma unroll
+        for (int k = C - 1; k >= 0; --k)
+#pragma unroll
+            for (int c = 0; c < NC; ++c) yv[c * C + k] = hc[c] = fmaf(de[c * C + k], hc[c], yv[c * C + k]);
+        float h = hc[NC - 1];
+#pragma unroll
+        for (int c = NC - 2; c >= 0; --c) h = fmaf(EE[c], h, hc[c]);
 #pragma unroll
         for (int r = 0; r < 5; ++r) {
             const int off = 1 << r;
@@ -158,12 +173,14 @@ __global__ void __launch_bounds__(kLvcThreads) lvc_outer_kernel(LvcSite sx, LvcS
         }
         float u = __shfl_down_sync(0xffffffffu, h, 1, G);
         if (gl == G - 1) u = 0.f;
-        const float xB = fmaf(E[H], u, hB);  // x at the start of the second half
+        float win[NC];  // x entering each chain from the right
+        win[NC - 1] = u;
 #pragma unroll
-        for (int k = 0; k < H; ++k) {
-            yv[H + k] = fmaf(E[H + k], u, yv[H + k]);
-            yv[k] = fmaf(E[k], xB, yv[k]);
-        }
+        for (int c = NC - 2; c >= 0; --c) win[c] = fmaf(EE[c + 1], win[c + 1], hc[c + 1]);
+#pragma unroll
+        for (int k = 0; k < C; ++k)
+#pragma unroll
+            for (int c = 0; c < NC; ++c) yv[c * C + k] = fmaf(E[c * C + k], win[c], yv[c * C + k]);
     }
     if (vec) {
 #pragma unroll
